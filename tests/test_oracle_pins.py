@@ -1,0 +1,306 @@
+"""Pins for the CPU oracle (oracle/blu_oracle.cpp) against things other than itself.
+
+Each pin is chosen so that a plausible oracle mistake (a dropped term, a wrong index, a transposed
+operand, wrong first-value handling for MIN/MAX, missing wrap) fails at least one test:
+
+  * brute force: O(N^2) nested loops in pure Python on tiny inputs (SURVEY.md §8(c) "Brute force");
+  * closed form: k(i) = decode(i mod G), v(i) = a*i + b, exact with Python big ints (§8(c));
+  * invariants: sum COUNT = N, sum SUM = column sum (wrap / exact dyadic), MIN <= AVG <= MAX,
+    row-permutation invariance (north_star "checked ... against invariants");
+  * special cases reducing to library routines: one group -> numpy column reductions; all
+    distinct -> each group is its row; N = 0 -> no groups;
+  * A11 two's-complement wrap of int64 SUM; A12 AVG rounding.
+
+The definition pinned is SQL GROUP BY with COUNT/SUM/MIN/MAX/AVG (PAPER.md P:151, P:153, P:162,
+P:176; BASELINE.json north_star). No GPU needed.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import blugen
+import oracle
+from blugen import AVG, COUNT, F64, I32, I64, MAX, MIN, SUM
+
+pytestmark = pytest.mark.filterwarnings("ignore::RuntimeWarning")
+
+
+def wrap64(x: int) -> int:
+    return ((x + (1 << 63)) % (1 << 64)) - (1 << 63)
+
+
+def brute_force(schema, key_cols, val_cols):
+    """O(N^2): for each first occurrence of a key tuple, scan every row. Pure Python."""
+    n = len(key_cols[0]) if key_cols else 0
+    K = len(schema.keys)
+    rk = [tuple(int(key_cols[k][i]) for k in range(K)) for i in range(n)]
+    pyvals = [[(float(v[i]) if d == F64 else int(v[i])) for i in range(n)] for v, d in zip(val_cols, schema.vals)]
+    out = []
+    for i in range(n):
+        g = rk[i]
+        first = True
+        for j in range(i):
+            if rk[j] == g:
+                first = False
+                break
+        if not first:
+            continue
+        members = [j for j in range(n) if rk[j] == g]
+        res = []
+        for op, col in schema.aggs:
+            if op == COUNT:
+                res.append(("i", len(members), None))
+                continue
+            vs = [pyvals[col][j] for j in members]
+            isf = schema.vals[col] == F64
+            if op in (SUM, AVG):
+                if isf:
+                    s = math.fsum(vs)
+                    sa = math.fsum(abs(x) for x in vs)
+                    res.append(("f", s if op == SUM else s / len(members), sa))
+                else:
+                    s = wrap64(sum(vs))
+                    res.append(("i", s, None) if op == SUM else ("f", float(s) / float(len(members)), None))
+            elif op == MIN:
+                res.append(("f" if isf else "i", min(vs), None))
+            else:
+                res.append(("f" if isf else "i", max(vs), None))
+        out.append((g, len(members), res))
+    out.sort(key=lambda t: t[0])
+    return out
+
+
+def assert_matches_brute(schema, kc, vc, exact_f64=True):
+    o = oracle.groupby_arrays(schema, kc, vc)
+    b = brute_force(schema, kc, vc)
+    assert o.n_groups == len(b)
+    for gi, (key, cnt, res) in enumerate(b):
+        assert tuple(int(x) for x in o.keys[gi]) == key
+        assert int(o.count[gi]) == cnt
+        for a, (kind, val, sa) in enumerate(res):
+            got = o.aggs[a][gi]
+            if kind == "i":
+                assert int(got) == val, (gi, a, got, val)
+            elif exact_f64 or sa is None:
+                assert float(got) == val, (gi, a, got, val)
+            else:
+                assert abs(float(got) - val) <= 1e-12 * max(sa, 1e-300) + 0.0, (gi, a, got, val, sa)
+
+
+def _rand_cols(rng, n, key_spec, val_dtypes, dyadic=True):
+    kc = []
+    for d, dict_size in key_spec:
+        hi = dict_size if dict_size else 7
+        arr = rng.integers(0, hi, n)
+        if not dict_size:  # sparse codes: large, spread values with collisions
+            arr = arr * 1_000_000_007 + 3
+        kc.append(arr.astype(blugen.NP_DTYPE[d]))
+    vc = []
+    for d in val_dtypes:
+        if d == I32:
+            v = rng.integers(-(2**31), 2**31, n).astype(np.int32)
+        elif d == I64:
+            v = rng.integers(-(2**62), 2**62, n).astype(np.int64)
+        else:
+            if dyadic:
+                v = (rng.integers(-(2**20), 2**20, n) / 64.0).astype(np.float64)
+            else:
+                v = (rng.random(n) - 0.5) * 1e6
+        vc.append(v)
+    return kc, vc
+
+
+ALL_AGGS = lambda nv, vdt: [(COUNT, -1)] + [(op, c) for c in range(nv) for op in (SUM, MIN, MAX, AVG)]
+
+
+@pytest.mark.parametrize("case", range(8))
+def test_brute_force_small(case):
+    rng = np.random.default_rng(1000 + case)
+    K = 1 + case % 3
+    key_spec = [([I32, I64][(case + j) % 2], [3, 5, 2, 0][(case + j) % 4]) for j in range(K)]
+    vdt = [I32, I64, F64]
+    n = [1, 2, 31, 33, 200, 500, 700, 300][case]
+    kc, vc = _rand_cols(rng, n, key_spec, vdt)
+    sch = blugen.Schema(key_spec, vdt, ALL_AGGS(3, vdt))
+    assert_matches_brute(sch, kc, vc)
+
+
+def test_brute_force_n2000():
+    rng = np.random.default_rng(7)
+    key_spec = [(I32, 9), (I64, 4)]
+    vdt = [I64, F64, I32]
+    kc, vc = _rand_cols(rng, 2000, key_spec, vdt)
+    sch = blugen.Schema(key_spec, vdt, ALL_AGGS(3, vdt))
+    assert_matches_brute(sch, kc, vc)
+
+
+def test_brute_force_general_f64_tolerance():
+    """Non-dyadic doubles: the oracle's long-double sum is within 1e-12 * sum|v| of fsum (A13)."""
+    rng = np.random.default_rng(11)
+    key_spec = [(I32, 6)]
+    vdt = [F64]
+    kc, vc = _rand_cols(rng, 1500, key_spec, vdt, dyadic=False)
+    sch = blugen.Schema(key_spec, vdt, [(COUNT, -1), (SUM, 0), (AVG, 0), (MIN, 0), (MAX, 0)])
+    assert_matches_brute(sch, kc, vc, exact_f64=False)
+
+
+def test_int64_sum_wraps_twos_complement():
+    """A11: int64 SUM wraps like the GPU's 64-bit adds; pinned by explicit big-int arithmetic."""
+    sch = blugen.Schema([(I32, 2)], [I64], [(SUM, 0), (MIN, 0), (MAX, 0), (AVG, 0)])
+    k = np.array([0, 0, 0, 1, 1], np.int32)
+    v = np.array([2**62, 2**62, 2**62, -(2**63), -1], np.int64)
+    o = oracle.groupby_arrays(sch, [k], [v])
+    assert int(o.aggs[0][0]) == wrap64(3 * 2**62) == -(2**62)
+    assert int(o.aggs[0][1]) == wrap64(-(2**63) - 1) == 2**63 - 1
+    assert int(o.aggs[1][1]) == -(2**63) and int(o.aggs[2][1]) == -1
+    assert float(o.aggs[3][0]) == float(-(2**62)) / 3.0
+
+
+def test_minmax_first_value_not_sentinel():
+    """MIN/MAX start from the first row (no sentinel can leak): all-negative MAX, all-positive MIN."""
+    sch = blugen.Schema([(I64, 0)], [I32, F64], [(MAX, 0), (MIN, 0), (MAX, 1), (MIN, 1)])
+    k = np.array([5, 5, 9], np.int64)
+    v0 = np.array([-7, -3, 2**31 - 1], np.int32)
+    v1 = np.array([-2.5, -0.5, 1e300], np.float64)
+    o = oracle.groupby_arrays(sch, [k], [v0, v1])
+    assert list(o.keys[:, 0]) == [5, 9]
+    assert list(o.aggs[0]) == [-3, 2**31 - 1] and list(o.aggs[1]) == [-7, 2**31 - 1]
+    assert list(o.aggs[2]) == [-0.5, 1e300] and list(o.aggs[3]) == [-2.5, 1e300]
+
+
+@pytest.mark.parametrize("a,b,vd,G,N", [(3, -1000, I32, 1024, 100_003), (-7919, 123456789, I64, 16, 1_000_000),
+                                       (5, 7, I64, 100_000, 250_001), (1, 0, I32, 1, 1000),
+                                       (1, -5, I64, 1, 2_000_001)])
+def test_closed_form(a, b, vd, G, N):
+    """k(i) = decode(i mod G) (mixed radix), v(i) = a*i + b. With c_g = ceil((N-g)/G):
+    COUNT_g = c_g; SUM_g = a(g c_g + G c_g (c_g-1)/2) + b c_g; MIN/MAX = a g + b and
+    a(g + G(c_g-1)) + b (swapped if a < 0); AVG = SUM/COUNT."""
+    # radices whose product is G (G = 1024 -> 32 x 32; 100000 -> 100 x 50 x 20; 16 -> 16; 1 -> 1)
+    radix = {1024: [32, 32], 16: [16], 100_000: [100, 50, 20], 1: [1]}[G]
+    strides = [int(np.prod(radix[:j])) for j in range(len(radix))]
+    w = blugen.Workload(
+        "closed", N, 0xC105ED,
+        [blugen.Col(I32, blugen.CYCLIC_DIGIT, 0, n_groups=G, stride=s, radix=r) for s, r in zip(strides, radix)],
+        [blugen.Col(vd, blugen.LINEAR, 1, lo=a, hi=b)],
+        blugen.Schema([(I32, r) for r in radix], [vd], [(COUNT, -1), (SUM, 0), (MIN, 0), (MAX, 0), (AVG, 0)]),
+        G, G)
+    o = oracle.groupby_generated(w)
+    assert o.n_groups == min(G, N)
+    for gi in range(o.n_groups):
+        g = sum(int(o.keys[gi][j]) * strides[j] for j in range(len(radix)))
+        c = -(-(N - g) // G)
+        s = a * (g * c + G * c * (c - 1) // 2) + b * c
+        lo, hi = a * g + b, a * (g + G * (c - 1)) + b
+        if a < 0:
+            lo, hi = hi, lo
+        assert int(o.count[gi]) == c
+        assert int(o.aggs[0][gi]) == c
+        assert int(o.aggs[1][gi]) == wrap64(s)
+        assert int(o.aggs[2][gi]) == lo and int(o.aggs[3][gi]) == hi
+        assert float(o.aggs[4][gi]) == float(s) / float(c)
+
+
+def _invariants(sch, kc, vc, o):
+    n = len(kc[0])
+    assert int(o.count.sum()) == n
+    for a, (op, col) in enumerate(sch.aggs):
+        if op == SUM:
+            if sch.vals[col] == F64:
+                assert float(math.fsum(o.aggs[a])) == math.fsum(vc[col].tolist())  # dyadic: exact
+            else:
+                assert wrap64(sum(int(x) for x in o.aggs[a])) == wrap64(sum(int(x) for x in vc[col]))
+    mins = {col: o.aggs[a] for a, (op, col) in enumerate(sch.aggs) if op == MIN}
+    maxs = {col: o.aggs[a] for a, (op, col) in enumerate(sch.aggs) if op == MAX}
+    for a, (op, col) in enumerate(sch.aggs):
+        if op == AVG and col in mins and col in maxs:
+            assert np.all(mins[col].astype(np.float64) <= o.aggs[a]) and np.all(o.aggs[a] <= maxs[col].astype(np.float64))
+
+
+def test_invariants_and_permutation():
+    rng = np.random.default_rng(3)
+    key_spec = [(I32, 40), (I32, 25)]
+    vdt = [I32, I64, F64]
+    n = 60_000
+    kc, vc = _rand_cols(rng, n, key_spec, vdt)
+    vc[1] = rng.integers(-(10**12), 10**12, n)
+    sch = blugen.Schema(key_spec, vdt, ALL_AGGS(3, vdt))
+    o = oracle.groupby_arrays(sch, kc, vc)
+    _invariants(sch, kc, vc, o)
+    perm = rng.permutation(n)
+    o2 = oracle.groupby_arrays(sch, [k[perm] for k in kc], [v[perm] for v in vc])
+    assert np.array_equal(o.keys, o2.keys) and np.array_equal(o.count, o2.count)
+    for x, y in zip(o.aggs, o2.aggs):
+        assert np.array_equal(x, y)
+
+
+def test_one_group_reduces_to_column_reductions():
+    rng = np.random.default_rng(5)
+    n = 10_000
+    k = np.full(n, 3, np.int32)
+    v0 = rng.integers(-(2**31), 2**31, n).astype(np.int32)
+    v1 = rng.integers(-(2**40), 2**40, n).astype(np.int64)
+    v2 = (rng.integers(-(2**20), 2**20, n) / 64.0)
+    sch = blugen.Schema([(I32, 8)], [I32, I64, F64], ALL_AGGS(3, None))
+    o = oracle.groupby_arrays(sch, [k], [v0, v1, v2])
+    assert o.n_groups == 1 and int(o.keys[0, 0]) == 3 and int(o.count[0]) == n
+    exp = []
+    for v in (v0, v1, v2):
+        s = float(np.sum(v)) if v.dtype == np.float64 else int(np.sum(v.astype(np.int64)))
+        exp += [s, v.min(), v.max(), s / n if v.dtype == np.float64 else float(s) / n]
+    got = [x[0] for x in o.aggs[1:]]
+    for g, e in zip(got, exp):
+        assert g == e
+
+
+def test_all_distinct_each_group_is_its_row():
+    rng = np.random.default_rng(6)
+    n = 5000
+    k = rng.permutation(10**6)[:n].astype(np.int64)
+    v = rng.integers(-(2**62), 2**62, n)
+    f = (rng.random(n) - 0.5) * 1e9
+    sch = blugen.Schema([(I64, 0)], [I64, F64], ALL_AGGS(2, None))
+    o = oracle.groupby_arrays(sch, [k], [v, f])
+    order = np.argsort(k)
+    assert np.array_equal(o.keys[:, 0], k[order]) and np.all(o.count == 1)
+    for a, (op, col) in enumerate(sch.aggs[1:], start=1):
+        src = [v, f][col][order]
+        if op == AVG:
+            assert np.array_equal(o.aggs[a], src.astype(np.float64))
+        else:
+            assert np.array_equal(o.aggs[a], src)
+
+
+def test_empty_input():
+    sch = blugen.Schema([(I32, 4)], [I64], [(COUNT, -1), (SUM, 0)])
+    o = oracle.groupby_arrays(sch, [np.zeros(0, np.int32)], [np.zeros(0, np.int64)])
+    assert o.n_groups == 0
+
+
+def test_slices_partition_the_result():
+    w = blugen.workload("C4", n_rows=200_000)
+    full = oracle.groupby_generated(w)
+    parts = [oracle.groupby_generated(w, slice_p=p, slice_P=5) for p in range(5)]
+    for p, r in enumerate(parts):  # slice rule (k0 + 31 k1 + 961 k2) mod P == p
+        k = r.keys.astype(np.int64)
+        assert np.all((k[:, 0] + 31 * k[:, 1] + 961 * k[:, 2]) % 5 == p)
+    u = oracle.concat(parts)
+    assert np.array_equal(u.keys, full.keys) and np.array_equal(u.count, full.count)
+    for x, y in zip(u.aggs, full.aggs):
+        assert np.array_equal(x, y)
+
+
+def test_filter_is_subset_and_generated_equals_arrays():
+    w = blugen.workload("C2", n_rows=100_000)
+    kc, vc = blugen.host_columns(w)
+    full_a = oracle.groupby_arrays(w.schema, kc, vc)
+    full_g = oracle.groupby_generated(w)
+    assert np.array_equal(full_a.keys, full_g.keys)
+    for x, y in zip(full_a.aggs, full_g.aggs):
+        assert np.array_equal(x, y)
+    pick = full_a.keys[::97]
+    sub = oracle.groupby_generated(w, filter_keys=pick)
+    idx = np.arange(0, full_a.n_groups, 97)
+    assert np.array_equal(sub.keys, pick)
+    for x, y in zip(sub.aggs, full_a.aggs):
+        assert np.array_equal(x, y[idx])
