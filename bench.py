@@ -1,0 +1,324 @@
+#!/usr/bin/env python
+"""bench.py — GROUP BY throughput of libblugby on B200 (BASELINE.json metric).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl blugby|reference]
+
+One "step" is one whole GROUP BY of one batch of synthetic fact-table rows (SURVEY.md §8(a) S0-S8:
+init, aggregate, CTA merge, compaction, the host read of n_groups; plus the NCCL merge at N > 1).
+The default workload is BASELINE.json configs[1] = C2 (100M rows, 2 i32 dictionary keys, 4 value
+columns, COUNT/SUM/MIN/MAX/AVG, path (a)). At N > 1 every rank aggregates its own 100M rows (weak
+scaling) and the dense states are combined with NCCL all-reduces.
+
+Timing: inputs generated in HBM before timing; between steps L2 is flushed (a 512 MB memset, outside
+the per-step CUDA events); each step is bracketed by CUDA events on the launching stream; K steps are
+bracketed by a barrier + synchronize; the max over ranks is reported. `--impl reference` times the
+CPU oracle (oracle/, plain single-threaded std::map) on a bounded sample of the same workload.
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "GROUP BY rows/s and HBM GB/s (% of B200 peak) at 1/2/4/8 GPUs vs CPU oracle"
+PEAKS_FALLBACK = {"hbm_gbs": 6650.0}  # B200_PROFILING.md fallback (used only if MEASURED_PEAKS.json is absent)
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
+    return PEAKS_FALLBACK["hbm_gbs"], "fallback (B200_PROFILING.md)"
+
+
+def load_traffic(config):
+    """Per-launch DRAM traffic (read + write bytes) of the aggregation kernel from the committed
+    ncu --set full summary (profiles/), or None."""
+    p = os.path.join(ROOT, "profiles", f"ncu_{config}_summary.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d.get("dram_bytes_per_launch"), d.get("rows_per_launch")
+    return None, None
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled DURING the timed region (B200_PROFILING.md)."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-i", str(self.index), "-lms", "50"], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.06)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=2)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[2:6]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def workload_for(config, rank, world):
+    import blugen
+    w = blugen.workload(config)
+    return w
+
+
+def result_bytes(res):
+    n = 0
+    for t in list(res.keys) + list(res.aggs or []):
+        n += t.numel() * t.element_size()
+    return n
+
+
+# ----------------------------------------------------------------------------------------------
+# CPU oracle leg (cpu_baseline and --impl reference)
+# ----------------------------------------------------------------------------------------------
+def oracle_rate(config, rows, row0=0):
+    import blugen
+    import oracle
+    w = blugen.workload(config)
+    t0 = time.perf_counter()
+    o = oracle.groupby_generated(w, row0=row0, n=rows)
+    dt = time.perf_counter() - t0
+    return rows / dt, dt, o.n_groups
+
+
+def cpu_baseline(config, seconds=10.0):
+    """The oracle as it stands, single-threaded, on a bounded sample (first rows of the workload)."""
+    r, dt, _ = oracle_rate(config, 200_000)
+    rows = int(min(max(r * seconds, 200_000), 10**9))
+    rows = min(rows, 50_000_000 if config in ("C1", "C2") else rows)
+    rate, dt, ng = oracle_rate(config, rows)
+    return {"value": rate, "unit": "rows/s", "cores": 1, "kind": "oracle",
+            "sample": f"{config} rows [0, {rows}) ({dt:.1f} s, {ng} groups), plain single-threaded std::map, "
+                      f"host {os.cpu_count()} cores visible"}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    import blugen
+    w = blugen.workload(args.config)
+    r0, _, _ = oracle_rate(args.config, 100_000)
+    budget = 90.0
+    rows = int(max(50_000, min(10_000_000, r0 * budget / max(1, args.steps + args.warmup))))
+    for i in range(args.warmup):
+        oracle_rate(args.config, rows, row0=i * rows)
+    times = []
+    for i in range(args.steps):
+        _, dt, _ = oracle_rate(args.config, rows, row0=(args.warmup + i) * rows % max(1, w.n_rows - rows))
+        times.append(dt)
+    tot = sum(times)
+    value = rows * args.steps / tot
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "rows/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * tot / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64+f64",
+            "data": "synthetic",
+            "config": {"workload": f"{args.config}: {w.note}", "rows_per_step": rows, "full_rows": w.n_rows},
+            "cpu_baseline": {"value": value, "unit": "rows/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{rows} rows per step of {args.config}, single-threaded std::map oracle"},
+            "e2e": {"value": value, "unit": "rows/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ----------------------------------------------------------------------------------------------
+# GPU leg
+# ----------------------------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5"])
+    ap.add_argument("--impl", default="blugby", choices=["blugby", "reference"])
+    ap.add_argument("--rows", type=int, default=None, help="override rows per rank (testing only)")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(3, args.warmup)
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    import blugen
+    from paper_conf_sigmod_merajispcksygnk16_b200 import blugby as bg
+    from paper_conf_sigmod_merajispcksygnk16_b200 import dist as bdist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    bg.blu_gby_bind_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream(dev)
+
+    w = blugen.workload(args.config, n_rows=args.rows) if args.rows else blugen.workload(args.config)
+    if args.config == "C5" and world > 1:
+        # C5 is 4B rows sharded over the GPUs (strong scaling of one query)
+        per = w.n_rows // world
+        row0, n = rank * per, (per if rank < world - 1 else w.n_rows - rank * per)
+        scaling = "strong"
+    else:
+        row0, n = rank * w.n_rows, w.n_rows  # every rank its own rows (weak scaling)
+        scaling = "weak"
+    kc = [blugen.gen_device(c, w.seed, row0, n, dev) for c in w.key_cols]
+    vc = [blugen.gen_device(c, w.seed, row0, n, dev) for c in w.val_cols]
+    torch.cuda.synchronize()
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows if scaling == "strong" else n)
+    info = plan.info()
+    flush = torch.empty(512 * 2**20, dtype=torch.uint8, device=dev)
+
+    def step():
+        if world == 1:
+            return bg.blu_gby_execute(plan, kc, vc, stream=stream)
+        res, _ = bdist.dist_execute(plan, kc, vc, stream=stream)
+        return res
+
+    bg.blu_gby_set_timing(True)
+    for _ in range(args.warmup):
+        flush.zero_()
+        r = step()
+    n_groups = r.n_groups
+    del r
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    agg_ms = []
+    sampler = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler.start()
+    time.sleep(0.15)
+    c0 = bg.blu_gby_launch_count()
+    for i in range(args.steps):
+        flush.zero_()
+        ev[i][0].record(stream)
+        r = step()
+        ev[i][1].record(stream)
+        t = bg.blu_gby_last_timing()
+        agg_ms.append(t["aggregate_ms"] / max(1, t["aggregate_launches"]))
+        del r
+    torch.cuda.synchronize()
+    launches = bg.blu_gby_launch_count() - c0
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    tot_ms = sum(step_ms)
+    if world > 1:
+        t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        tot_ms = float(t.item())
+    rows_total = (w.n_rows if scaling == "strong" else n * world) * args.steps
+    value = rows_total / (tot_ms / 1000.0)
+    bpr = w.bytes_per_row
+    input_gbs = value * bpr / 1e9
+    peak, peak_src = load_peaks()
+
+    # dominant kernel: the aggregation kernel (S5), timed with CUDA events on its launch stream
+    agg_avg_ms = statistics.mean(agg_ms)
+    rows_per_launch = n  # one aggregate launch per execute (rows < grid * 2^30)
+    achieved = rows_per_launch * bpr / (agg_avg_ms / 1000.0) / 1e9
+    traffic, traffic_rows = load_traffic(args.config)
+    if traffic is not None and traffic_rows:
+        traffic = traffic * rows_per_launch / traffic_rows
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": traffic, "kernel": "k_agg_dense_smem" if info["path"] == 0 else "k_agg_global",
+                "algorithmic_bytes_per_launch": rows_per_launch * bpr, "avg_launch_ms": agg_avg_ms,
+                "peak_source": peak_src, "share_of_step": agg_avg_ms / (tot_ms / args.steps)}
+
+    # e2e: same metric through the C ABI with pinned HOST columns (H2D + D2H inside the timed region)
+    e2e = None
+    if not args.no_e2e and world == 1:
+        hk = [k.cpu().pin_memory() for k in kc]
+        hv = [v.cpu().pin_memory() for v in vc]
+        h2d = sum(t.numel() * t.element_size() for t in hk + hv)
+        bg.blu_gby_execute_host(plan, hk, hv, stream=stream)
+        e_steps = min(3, args.steps)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        d2h = 0
+        for _ in range(e_steps):
+            res = bg.blu_gby_execute_host(plan, hk, hv, stream=stream)
+            d2h = sum(a.nbytes for a in list(res.keys) + list(res.aggs))
+        torch.cuda.synchronize()
+        dt = (time.perf_counter() - t0) / e_steps
+        e2e = {"value": n / dt, "unit": "rows/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "ms_per_step": dt * 1000, "note": "blu_gby_execute_host: pinned host columns, chunked H2D "
+                                                 "overlapped with aggregation, host result"}
+        del hk, hv
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(args.config)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "rows/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
+            "scaling": scaling, "vs_baseline": None, "dtype": "int64+f64", "data": "synthetic",
+            "config": {"workload": f"{args.config}: {w.note}", "rows_per_gpu": n, "groups": n_groups,
+                       "bytes_per_row": bpr, "path": info["path_name"], "hot_front": info["hot_front"],
+                       "grid": info["grid"], "block": info["block"], "smem_bytes": info["smem_bytes"],
+                       "parallelism": f"rows sharded x{world}" + (" + NCCL allreduce" if world > 1 and info["path"] != 1 else
+                                                                   " + NCCL all-to-all" if world > 1 else ""),
+                       "l2": "flushed between steps (512 MB memset, outside step events); inputs > L2"},
+            "input_gbs": input_gbs, "hbm_frac_input": input_gbs / peak,
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clocks,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,648 @@
+// api.cu — the execute / merge / exchange entry points of libblugby (C ABI, include/blu_gby.h).
+//
+// One execute is stream-ordered: S4 init -> S5 aggregate (one launch per input batch) -> S8
+// compaction into upper-bound-sized outputs -> ONE synchronisation that reads {flags, n_groups}.
+// If the flags report that a probe exceeded its bound (the estimate was too small, "error
+// detection code-path ... we could still process the query"), the table is regrown 4x and the
+// query rerun; a key outside its dictionary returns BLU_E_KEY_RANGE with no result.
+#include <cuda_runtime.h>
+#include <stdarg.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <functional>
+#include <mutex>
+#include <vector>
+
+#include "blu_internal.h"
+
+namespace blu {
+
+
+static thread_local bool t_timing = false;
+static thread_local blu_gby_timing_t t_last{};
+
+struct Events {
+  cudaEvent_t e[8];
+  bool ok = false;
+  void make() {
+    if (ok) return;
+    for (auto& x : e) cudaEventCreate(&x);
+    ok = true;
+  }
+};
+static thread_local Events t_ev;
+
+static uint64_t* pinned_scratch() {
+  static thread_local uint64_t* p = nullptr;
+  if (!p) {
+    if (cudaMallocHost((void**)&p, 256) != cudaSuccess) {
+      cudaGetLastError();
+      p = nullptr;
+    }
+  }
+  return p;
+}
+
+static void setup_pool() {
+  static std::once_flag once;
+  std::call_once(once, [] {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t thr = UINT64_MAX;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    cudaGetLastError();
+  });
+}
+
+static blu_status_t cuda_fail(cudaError_t e, const char* what) {
+  if (e == cudaErrorMemoryAllocation) return fail(BLU_E_OOM, "%s: %s", what, cudaGetErrorString(e));
+  return fail(BLU_E_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+#define CK(call, what)                              \
+  do {                                              \
+    cudaError_t _e = (cudaError_t)(call);           \
+    if (_e != cudaSuccess) {                        \
+      cudaGetLastError();                           \
+      return cuda_fail(_e, what);                   \
+    }                                               \
+  } while (0)
+
+// Owner record behind blu_gby_result_t::_owner.
+struct Owner {
+  std::vector<void*> dev;
+  std::vector<void*> host;
+};
+
+static size_t dtype_bytes(int dt) { return dt == BLU_I32 ? 4 : 8; }
+
+// Stream-ordered workspace that frees itself.
+struct Work {
+  cudaStream_t st;
+  std::vector<void*> ptrs;
+  explicit Work(cudaStream_t s) : st(s) {}
+  cudaError_t alloc(void** p, size_t bytes) {
+    *p = nullptr;
+    if (!bytes) return cudaSuccess;
+    cudaError_t e = cudaMallocAsync(p, bytes, st);
+    if (e == cudaSuccess) ptrs.push_back(*p);
+    return e;
+  }
+  ~Work() {
+    for (void* p : ptrs) cudaFreeAsync(p, st);
+  }
+};
+
+// What the compaction emits.
+struct OutSpec {
+  bool partial;
+  int n_out;
+  int out_kind[kMaxFields], out_field[kMaxFields], out_field2[kMaxFields], out_dtype[kMaxFields];
+};
+
+static OutSpec make_outspec(const blu_gby_plan_s* P, const Layout& lay, bool partial) {
+  OutSpec o{};
+  o.partial = partial;
+  if (partial) {
+    o.n_out = lay.n_fields;
+    for (int j = 0; j < lay.n_fields; ++j) {
+      int k = lay.f[j].kind;
+      o.out_dtype[j] = (k == FK_MINI32 || k == FK_MAXI32) ? BLU_I32 : (k == FK_SUMF || k == FK_MINF64 || k == FK_MAXF64) ? BLU_F64 : BLU_I64;
+    }
+  } else {
+    o.n_out = (int)P->amap.size();
+    for (int a = 0; a < o.n_out; ++a) {
+      const AggMap& m = P->amap[a];
+      o.out_kind[a] = m.op == BLU_AVG ? 1 : 0;
+      o.out_field[a] = m.field;
+      o.out_field2[a] = m.field2;
+      o.out_dtype[a] = m.out_dtype;
+    }
+  }
+  return o;
+}
+
+// Feeds every input batch to the aggregation kernel for one attempt. `base` carries the targets.
+using Feeder = std::function<cudaError_t(AggParams& base, uint32_t* launches)>;
+
+static bool ptr_aligned(const void* p) { return ((uintptr_t)p & 15) == 0; }
+
+// Launch the aggregation for rows [0, n) of one batch, chunked so per-CTA 32-bit shared counters
+// cannot overflow.
+static cudaError_t agg_batch(const blu_gby_plan_s* P, int path, AggParams p, const void* const* keys,
+                             const void* const* vals, uint64_t n, const RecSrc* rs, cudaStream_t st,
+                             uint32_t grid, uint32_t block, uint32_t smem, uint32_t* launches) {
+  const Layout& L = p.lay;
+  uint64_t max_rows = ((uint64_t)grid * (1ull << 30)) & ~3ull;
+  for (uint64_t r0 = 0; r0 < n; r0 += max_rows) {
+    uint64_t m = std::min(max_rows, n - r0);
+    bool vec = true;
+    if (!rs) {
+      for (int k = 0; k < L.n_keys; ++k) {
+        p.key[k] = (const uint8_t*)keys[k] + r0 * dtype_bytes(L.key_dtype[k]);
+        vec = vec && ptr_aligned(p.key[k]);
+      }
+      for (int c = 0; c < L.n_vals; ++c) {
+        p.val[c] = (const uint8_t*)vals[c] + r0 * dtype_bytes(L.val_dtype[c]);
+        vec = vec && ptr_aligned(p.val[c]);
+      }
+    }
+    p.vec_ok = vec ? 1 : 0;
+    p.n_rows = m;
+    RecSrc r{nullptr, 0};
+    if (rs) r = RecSrc{rs->rec + r0 * rs->words, rs->words};
+    int e = launch_aggregate_impl(P, path, p, r, rs != nullptr, st, grid, block, smem);
+    if (e) return (cudaError_t)e;
+    if (launches) ++*launches;
+  }
+  return cudaSuccess;
+}
+
+// The core: init -> feed -> compact -> one sync -> regrow on overflow.
+static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int path, bool front, uint64_t cap0,
+                             uint64_t total_rows, const Feeder& feed, bool partial, cudaStream_t st,
+                             blu_gby_result_t* out, bool host_out, float* h2d_ms_acc) {
+  setup_pool();
+  memset(out, 0, sizeof *out);
+  const bool dense = path != BLU_PATH_HASH_GLOBAL;
+  const uint64_t D = lay.domain;
+  uint64_t cap = dense ? D : cap0;
+  uint32_t retries = 0;
+  blu_gby_timing_t tm{};
+  if (t_timing) t_ev.make();
+  OutSpec os = make_outspec(P, lay, partial);
+
+  for (;;) {
+    Work w(st);
+    void* table = nullptr;
+    void* dense_g[4] = {nullptr, nullptr, nullptr, nullptr};
+    if (t_timing) cudaEventRecord(t_ev.e[0], st);
+    if (dense) {
+      for (int g = 0; g < 4; ++g) CK(w.alloc(&dense_g[g], (size_t)lay.n_group[g] * D * 8), "dense state alloc");
+      CK(launch_init_dense(lay, dense_g, D, st), "init dense");
+    } else {
+      CK(w.alloc(&table, (size_t)cap * lay.slot_bytes), "hash table alloc");
+      CK(launch_init_slots(lay, table, cap, st), "init slots");
+    }
+    const uint64_t n_entries = dense ? D : cap;
+    const uint64_t nb = (n_entries + 4095) / 4096;
+    void* small = nullptr;
+    CK(w.alloc(&small, 64 + 16 * std::max<uint64_t>(nb, 1)), "workspace alloc");
+    uint32_t* d_flags = (uint32_t*)small;
+    uint64_t* d_ngroups = (uint64_t*)((uint8_t*)small + 8);
+    uint64_t* d_bcounts = (uint64_t*)((uint8_t*)small + 64);
+    uint64_t* d_boffs = d_bcounts + std::max<uint64_t>(nb, 1);
+    CK(cudaMemsetAsync(small, 0, 64, st), "memset flags");
+    if (t_timing) cudaEventRecord(t_ev.e[1], st);
+
+    AggParams base{};
+    base.lay = lay;
+    base.table = table;
+    base.cap_mask = dense ? 0 : cap - 1;
+    base.max_probe = (uint32_t)std::min<uint64_t>(cap, 4096);
+    for (int g = 0; g < 4; ++g) base.dense[g] = dense_g[g];
+    base.front_slots = front ? P->front_slots : 0;
+    base.flags = d_flags;
+    uint32_t launches = 0;
+    CK(feed(base, &launches), "aggregate launch");
+    if (t_timing) cudaEventRecord(t_ev.e[2], st);
+
+    // outputs, sized by the upper bound min(entries, rows)
+    const uint64_t U = std::min<uint64_t>(n_entries, total_rows);
+    Owner* own = new Owner();
+    std::vector<void*> okeys(lay.n_keys, nullptr), ovals(os.n_out, nullptr);
+    auto free_owner = [&]() {
+      for (void* p : own->dev) cudaFreeAsync(p, st);
+      delete own;
+    };
+    cudaError_t ae = cudaSuccess;
+    for (int k = 0; k < lay.n_keys && ae == cudaSuccess; ++k) {
+      ae = U ? cudaMallocAsync(&okeys[k], U * dtype_bytes(lay.key_dtype[k]), st) : cudaSuccess;
+      if (okeys[k]) own->dev.push_back(okeys[k]);
+    }
+    for (int o = 0; o < os.n_out && ae == cudaSuccess; ++o) {
+      ae = U ? cudaMallocAsync(&ovals[o], U * dtype_bytes(os.out_dtype[o]), st) : cudaSuccess;
+      if (ovals[o]) own->dev.push_back(ovals[o]);
+    }
+    if (ae != cudaSuccess) {
+      cudaGetLastError();
+      free_owner();
+      return cuda_fail(ae, "output alloc");
+    }
+    if (U) {
+      CompactParams cp{};
+      cp.lay = lay;
+      cp.source = dense ? 1 : 0;
+      cp.table = table;
+      for (int g = 0; g < 4; ++g) cp.dense[g] = dense_g[g];
+      cp.n_entries = n_entries;
+      cp.partial = partial ? 1 : 0;
+      cp.n_out = os.n_out;
+      for (int o = 0; o < os.n_out; ++o) {
+        cp.out_kind[o] = os.out_kind[o];
+        cp.out_field[o] = os.out_field[o];
+        cp.out_field2[o] = os.out_field2[o];
+        cp.out_dtype[o] = os.out_dtype[o];
+        cp.out_vals[o] = ovals[o];
+      }
+      for (int k = 0; k < lay.n_keys; ++k) cp.out_keys[k] = okeys[k];
+      cp.block_counts = d_bcounts;
+      cp.block_offsets = d_boffs;
+      cp.n_groups = d_ngroups;
+      int ce = launch_compact(cp, st, nullptr);
+      if (ce) {
+        free_owner();
+        return cuda_fail((cudaError_t)ce, "compaction launch");
+      }
+    }
+    if (t_timing) cudaEventRecord(t_ev.e[3], st);
+    uint64_t* hs = pinned_scratch();
+    uint64_t hbuf[2] = {0, 0};
+    uint64_t* dst = hs ? hs : hbuf;
+    cudaError_t ce = cudaMemcpyAsync(dst, small, 16, cudaMemcpyDeviceToHost, st);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(st);
+    if (ce != cudaSuccess) {
+      cudaGetLastError();
+      free_owner();
+      return cuda_fail(ce, "execute");
+    }
+    uint32_t flags = (uint32_t)dst[0];
+    uint64_t ng = dst[1];
+    if (t_timing) {
+      float a = 0, b = 0, c = 0;
+      cudaEventElapsedTime(&a, t_ev.e[0], t_ev.e[1]);
+      cudaEventElapsedTime(&b, t_ev.e[1], t_ev.e[2]);
+      cudaEventElapsedTime(&c, t_ev.e[2], t_ev.e[3]);
+      tm.init_ms += a;
+      tm.aggregate_ms += b;
+      tm.compact_ms += c;
+      tm.aggregate_launches += launches;
+    }
+    if (flags & FLAG_KEY_RANGE) {
+      free_owner();
+      return fail(BLU_E_KEY_RANGE, "a key code is outside [0, dict_size) or a sparse code is negative");
+    }
+    if ((flags & FLAG_OVERFLOW) && !dense) {
+      free_owner();
+      cap *= 4;
+      ++retries;
+      if (cap > (1ull << 40)) return fail(BLU_E_OOM, "hash table regrow beyond 2^40 slots");
+      continue;
+    }
+    // success
+    P->retries_last.store(retries);
+    out->n_groups = ng;
+    out->n_keys = lay.n_keys;
+    out->is_partial = partial ? 1 : 0;
+    out->is_host = host_out ? 1 : 0;
+    void** kc = (void**)calloc(std::max(1, lay.n_keys), sizeof(void*));
+    void** vc = (void**)calloc(std::max(1, os.n_out), sizeof(void*));
+    for (int k = 0; k < lay.n_keys; ++k) kc[k] = okeys[k];
+    for (int o = 0; o < os.n_out; ++o) vc[o] = ovals[o];
+    if (host_out) {
+      // copy to host and release the device outputs
+      Owner* hown = new Owner();
+      for (int k = 0; k < lay.n_keys; ++k) {
+        size_t b = ng * dtype_bytes(lay.key_dtype[k]);
+        void* h = malloc(std::max<size_t>(b, 1));
+        if (b) cudaMemcpyAsync(h, okeys[k], b, cudaMemcpyDeviceToHost, st);
+        hown->host.push_back(h);
+        kc[k] = h;
+      }
+      for (int o = 0; o < os.n_out; ++o) {
+        size_t b = ng * dtype_bytes(os.out_dtype[o]);
+        void* h = malloc(std::max<size_t>(b, 1));
+        if (b) cudaMemcpyAsync(h, ovals[o], b, cudaMemcpyDeviceToHost, st);
+        hown->host.push_back(h);
+        vc[o] = h;
+      }
+      cudaError_t se = cudaStreamSynchronize(st);
+      free_owner();
+      own = hown;
+      if (se != cudaSuccess) {
+        for (void* h : hown->host) free(h);
+        delete hown;
+        free(kc);
+        free(vc);
+        return cuda_fail(se, "result D2H");
+      }
+    }
+    if (partial) {
+      out->n_states = os.n_out;
+      out->state_cols = vc;
+      out->agg_cols = nullptr;
+    } else {
+      out->n_aggs = os.n_out;
+      out->agg_cols = vc;
+      out->state_cols = nullptr;
+    }
+    out->key_cols = kc;
+    out->_owner = own;
+    if (t_timing) {
+      tm.retries = retries;
+      if (h2d_ms_acc) tm.h2d_ms = *h2d_ms_acc;
+      tm.total_ms = tm.init_ms + tm.aggregate_ms + tm.compact_ms;
+      t_last = tm;
+    }
+    return BLU_OK;
+  }
+}
+
+static bool nonnull_cols(const void* const* cols, int n) {
+  if (n == 0) return true;
+  if (!cols) return false;
+  for (int i = 0; i < n; ++i)
+    if (!cols[i]) return false;
+  return true;
+}
+
+// Schema column pointers -> kernel columns (the layout's value columns are the schema's).
+static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* keys, const void* const* vals,
+                                   uint64_t n, cudaStream_t st, bool partial, blu_gby_result_t* out) {
+  if (!P || !out) return fail(BLU_E_INVALID, "NULL plan or out");
+  if (n && (!nonnull_cols(keys, P->lay.n_keys) || !nonnull_cols(vals, P->lay.n_vals)))
+    return fail(BLU_E_INVALID, "NULL column pointer");
+  const Layout& L = P->lay;
+  Feeder feed = [&](AggParams& base, uint32_t* launches) -> cudaError_t {
+    return agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, launches);
+  };
+  return run_core(P, L, P->path, P->hot_front != 0, P->cap, n, feed, partial, st, out, false, nullptr);
+}
+
+}  // namespace blu
+
+using namespace blu;
+
+extern "C" {
+
+void blu_gby_set_timing(int32_t enable) { t_timing = enable != 0; }
+
+blu_status_t blu_gby_last_timing(blu_gby_timing_t* out) {
+  if (!out) return fail(BLU_E_INVALID, "NULL out");
+  *out = t_last;
+  return BLU_OK;
+}
+
+uint64_t blu_gby_launch_count(void) { return launches_total(); }
+
+blu_status_t blu_gby_execute(blu_gby_plan_t P, const void* const* key_cols, const void* const* val_cols, uint64_t n_rows,
+                             void* stream, blu_gby_result_t* out) {
+  return execute_device(P, key_cols, val_cols, n_rows, (cudaStream_t)stream, false, out);
+}
+
+blu_status_t blu_gby_execute_partial(blu_gby_plan_t P, const void* const* key_cols, const void* const* val_cols,
+                                     uint64_t n_rows, void* stream, blu_gby_result_t* out) {
+  return execute_device(P, key_cols, val_cols, n_rows, (cudaStream_t)stream, true, out);
+}
+
+blu_status_t blu_gby_execute_host(blu_gby_plan_t P, const void* const* hkeys, const void* const* hvals, uint64_t n,
+                                  void* stream, blu_gby_result_t* out) {
+  if (!P || !out) return fail(BLU_E_INVALID, "NULL plan or out");
+  if (n && (!nonnull_cols(hkeys, P->lay.n_keys) || !nonnull_cols(hvals, P->lay.n_vals)))
+    return fail(BLU_E_INVALID, "NULL column pointer");
+  cudaStream_t st = (cudaStream_t)stream;
+  const Layout& L = P->lay;
+  // chunk: ~256 MB of rows per staging buffer, a multiple of 4 rows
+  size_t row_bytes = 0;
+  for (int k = 0; k < L.n_keys; ++k) row_bytes += dtype_bytes(L.key_dtype[k]);
+  for (int c = 0; c < L.n_vals; ++c) row_bytes += dtype_bytes(L.val_dtype[c]);
+  uint64_t chunk = std::max<uint64_t>(4, ((256ull << 20) / std::max<size_t>(row_bytes, 1)) & ~3ull);
+  if (chunk > n) chunk = (n + 3) & ~3ull;
+  const int ncols = L.n_keys + L.n_vals;
+  setup_pool();
+  void* stage[2] = {nullptr, nullptr};
+  cudaStream_t cs = nullptr;
+  cudaEvent_t ready[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr}, t0 = nullptr, t1 = nullptr;
+  auto cleanup = [&]() {
+    for (int b = 0; b < 2; ++b) {
+      if (stage[b]) cudaFreeAsync(stage[b], st);
+      if (ready[b]) cudaEventDestroy(ready[b]);
+      if (freed[b]) cudaEventDestroy(freed[b]);
+    }
+    if (t0) cudaEventDestroy(t0);
+    if (t1) cudaEventDestroy(t1);
+    if (cs) {
+      cudaStreamSynchronize(cs);
+      cudaStreamDestroy(cs);
+    }
+  };
+  if (n) {
+    for (int b = 0; b < 2; ++b) {
+      if (cudaMallocAsync(&stage[b], chunk * row_bytes + 16 * ncols, st) != cudaSuccess) {
+        cudaGetLastError();
+        cleanup();
+        return fail(BLU_E_OOM, "staging buffers");
+      }
+      cudaEventCreateWithFlags(&ready[b], cudaEventDisableTiming);
+      cudaEventCreateWithFlags(&freed[b], cudaEventDisableTiming);
+    }
+    cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+    cudaEventCreate(&t0);
+    cudaEventCreate(&t1);
+  }
+  float h2d_ms = 0.f;
+  Feeder feed = [&](AggParams& base, uint32_t* launches) -> cudaError_t {
+    if (!n) return cudaSuccess;
+    cudaEventRecord(t0, st);
+    cudaStreamWaitEvent(cs, t0, 0);  // staging buffers are allocated on st
+    uint64_t nchunks = (n + chunk - 1) / chunk;
+    for (uint64_t i = 0; i < nchunks; ++i) {
+      int b = (int)(i & 1);
+      uint64_t r0 = i * chunk, m = std::min(chunk, n - r0);
+      if (i >= 2) cudaStreamWaitEvent(cs, freed[b], 0);
+      const void* dk[kMaxKeys];
+      const void* dv[kMaxVals];
+      uint8_t* ptr = (uint8_t*)stage[b];
+      for (int k = 0; k < L.n_keys; ++k) {
+        size_t eb = dtype_bytes(L.key_dtype[k]);
+        cudaMemcpyAsync(ptr, (const uint8_t*)hkeys[k] + r0 * eb, m * eb, cudaMemcpyHostToDevice, cs);
+        dk[k] = ptr;
+        ptr += (chunk * eb + 15) / 16 * 16;
+      }
+      for (int c = 0; c < L.n_vals; ++c) {
+        size_t eb = dtype_bytes(L.val_dtype[c]);
+        cudaMemcpyAsync(ptr, (const uint8_t*)hvals[c] + r0 * eb, m * eb, cudaMemcpyHostToDevice, cs);
+        dv[c] = ptr;
+        ptr += (chunk * eb + 15) / 16 * 16;
+      }
+      cudaEventRecord(ready[b], cs);
+      cudaStreamWaitEvent(st, ready[b], 0);
+      cudaError_t e = agg_batch(P, P->path, base, dk, dv, m, nullptr, st, P->grid, P->block, P->smem_bytes, launches);
+      if (e) return e;
+      cudaEventRecord(freed[b], st);
+    }
+    cudaEventRecord(t1, st);
+    return cudaGetLastError();
+  };
+  blu_status_t s = run_core(P, L, P->path, P->hot_front != 0, P->cap, n, feed, false, st, out, true, nullptr);
+  if (s == BLU_OK && n && t_timing) {
+    cudaEventElapsedTime(&h2d_ms, t0, t1);  // copy+aggregate pipeline span
+    t_last.h2d_ms = h2d_ms;
+  }
+  cleanup();
+  return s;
+}
+
+static blu_status_t merge_impl(blu_gby_plan_t P, const blu_gby_result_t* parts, int32_t np, void* stream, bool partial_out,
+                               blu_gby_result_t* out) {
+  if (!P || !out || (np > 0 && !parts) || np < 0) return fail(BLU_E_INVALID, "bad merge arguments");
+  cudaStream_t st = (cudaStream_t)stream;
+  const Layout& M = P->merge_lay;
+  uint64_t total = 0;
+  for (int i = 0; i < np; ++i) {
+    if (!parts[i].is_partial || parts[i].is_host) return fail(BLU_E_INVALID, "partial %d: not a device partial result", i);
+    if (parts[i].n_states != M.n_vals || parts[i].n_keys != M.n_keys) return fail(BLU_E_INVALID, "partial %d: schema mismatch", i);
+    total += parts[i].n_groups;
+  }
+  uint64_t est = std::max<uint64_t>(1, std::min<uint64_t>(total, std::max<uint64_t>(P->est_groups, 1)));
+  uint64_t cap = 1024;
+  while ((double)cap * 0.7 < (double)est) cap <<= 1;
+  uint32_t grid = (uint32_t)P->sms * 8, block = 256;
+  Feeder feed = [&](AggParams& base, uint32_t* launches) -> cudaError_t {
+    for (int i = 0; i < np; ++i) {
+      if (!parts[i].n_groups) continue;
+      cudaError_t e = agg_batch(P, BLU_PATH_HASH_GLOBAL, base, (const void* const*)parts[i].key_cols,
+                                (const void* const*)parts[i].state_cols, parts[i].n_groups, nullptr, st, grid, block, 0,
+                                launches);
+      if (e) return e;
+    }
+    return cudaSuccess;
+  };
+  return run_core(P, M, BLU_PATH_HASH_GLOBAL, false, cap, total, feed, partial_out, st, out, false, nullptr);
+}
+
+blu_status_t blu_gby_merge(blu_gby_plan_t P, const blu_gby_result_t* parts, int32_t np, void* stream, blu_gby_result_t* out) {
+  return merge_impl(P, parts, np, stream, false, out);
+}
+
+blu_status_t blu_gby_merge_partial(blu_gby_plan_t P, const blu_gby_result_t* parts, int32_t np, void* stream,
+                                   blu_gby_result_t* out) {
+  return merge_impl(P, parts, np, stream, true, out);
+}
+
+blu_status_t blu_gby_merge_records(blu_gby_plan_t P, const void* records, uint64_t n, void* stream, int32_t partial_out,
+                                   blu_gby_result_t* out) {
+  if (!P || !out || (n && !records)) return fail(BLU_E_INVALID, "bad merge_records arguments");
+  cudaStream_t st = (cudaStream_t)stream;
+  const Layout& M = P->merge_lay;
+  uint64_t est = std::max<uint64_t>(1, std::min<uint64_t>(n, std::max<uint64_t>(P->est_groups, 1)));
+  uint64_t cap = 1024;
+  while ((double)cap * 0.7 < (double)est) cap <<= 1;
+  uint32_t grid = (uint32_t)P->sms * 8, block = 256;
+  RecSrc rs{(const uint64_t*)records, (uint32_t)(1 + M.n_vals)};
+  Feeder feed = [&](AggParams& base, uint32_t* launches) -> cudaError_t {
+    if (!n) return cudaSuccess;
+    return agg_batch(P, BLU_PATH_HASH_GLOBAL, base, nullptr, nullptr, n, &rs, st, grid, block, 0, launches);
+  };
+  return run_core(P, M, BLU_PATH_HASH_GLOBAL, false, cap, n, feed, partial_out != 0, st, out, false, nullptr);
+}
+
+blu_status_t blu_gby_execute_dense_state(blu_gby_plan_t P, const void* const* keys, const void* const* vals, uint64_t n,
+                                         void* stream, void* const* state_arrays, int32_t init) {
+  if (!P || !state_arrays) return fail(BLU_E_INVALID, "NULL plan or state arrays");
+  if (P->path == BLU_PATH_HASH_GLOBAL) return fail(BLU_E_UNSUPPORTED, "dense state needs path a or b'");
+  if (n && (!nonnull_cols(keys, P->lay.n_keys) || !nonnull_cols(vals, P->lay.n_vals)))
+    return fail(BLU_E_INVALID, "NULL column pointer");
+  setup_pool();
+  cudaStream_t st = (cudaStream_t)stream;
+  const Layout& L = P->lay;
+  void* dg[4];
+  for (int g = 0; g < 4; ++g) {
+    dg[g] = state_arrays[g];
+    if (L.n_group[g] && !dg[g]) return fail(BLU_E_INVALID, "state array %d is NULL", g);
+  }
+  if (init) CK(launch_init_dense(L, dg, L.domain, st), "init dense");
+  Work w(st);
+  void* small = nullptr;
+  CK(w.alloc(&small, 64), "flags alloc");
+  CK(cudaMemsetAsync(small, 0, 64, st), "memset flags");
+  AggParams base{};
+  base.lay = L;
+  for (int g = 0; g < 4; ++g) base.dense[g] = dg[g];
+  base.front_slots = P->hot_front ? P->front_slots : 0;
+  base.flags = (uint32_t*)small;
+  CK(agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, nullptr), "aggregate");
+  uint64_t* hs = pinned_scratch();
+  uint64_t hb[2] = {0, 0};
+  uint64_t* dst = hs ? hs : hb;
+  CK(cudaMemcpyAsync(dst, small, 8, cudaMemcpyDeviceToHost, st), "flags D2H");
+  CK(cudaStreamSynchronize(st), "sync");
+  if ((uint32_t)dst[0] & FLAG_KEY_RANGE) return fail(BLU_E_KEY_RANGE, "a key code is outside [0, dict_size)");
+  return BLU_OK;
+}
+
+blu_status_t blu_gby_finalize_dense_state(blu_gby_plan_t P, void* const* state_arrays, void* stream, blu_gby_result_t* out) {
+  if (!P || !state_arrays || !out) return fail(BLU_E_INVALID, "NULL argument");
+  if (P->path == BLU_PATH_HASH_GLOBAL) return fail(BLU_E_UNSUPPORTED, "dense state needs path a or b'");
+  cudaStream_t st = (cudaStream_t)stream;
+  const Layout& L = P->lay;
+  // Reuse run_core with a feeder that copies the caller's state in place of init+aggregate.
+  Feeder feed = [&](AggParams& base, uint32_t*) -> cudaError_t {
+    for (int g = 0; g < 4; ++g) {
+      size_t b = (size_t)L.n_group[g] * L.domain * 8;
+      if (b) {
+        cudaError_t e = cudaMemcpyAsync(base.dense[g], state_arrays[g], b, cudaMemcpyDeviceToDevice, st);
+        if (e) return e;
+      }
+    }
+    return cudaSuccess;
+  };
+  return run_core(P, L, P->path, false, L.domain, L.domain, feed, false, st, out, false, nullptr);
+}
+
+blu_status_t blu_gby_partition(blu_gby_plan_t P, const blu_gby_result_t* partial, int32_t n_parts, void* stream, void* send_buf,
+                               uint64_t* send_counts) {
+  if (!P || !partial || !send_counts || n_parts < 1 || n_parts > 1024) return fail(BLU_E_INVALID, "bad partition arguments");
+  if (!partial->is_partial || partial->is_host) return fail(BLU_E_INVALID, "partition needs a device partial result");
+  if (partial->n_groups && !send_buf) return fail(BLU_E_INVALID, "NULL send_buf");
+  cudaStream_t st = (cudaStream_t)stream;
+  setup_pool();
+  if (!partial->n_groups) {
+    for (int i = 0; i < n_parts; ++i) send_counts[i] = 0;
+    return BLU_OK;
+  }
+  Work w(st);
+  void* tmp = nullptr;
+  CK(w.alloc(&tmp, 16 * (size_t)n_parts), "partition workspace");
+  CK(cudaMemsetAsync(tmp, 0, 16 * (size_t)n_parts, st), "memset");
+  uint64_t* d_counts = (uint64_t*)tmp;
+  uint64_t* d_offs = d_counts + n_parts;
+  CK(launch_partition(P->merge_lay, (const void* const*)partial->key_cols, (const void* const*)partial->state_cols,
+                      partial->n_groups, n_parts, send_buf, d_counts, d_offs, st),
+     "partition");
+  CK(cudaMemcpyAsync(send_counts, d_counts, 8 * (size_t)n_parts, cudaMemcpyDeviceToHost, st), "counts D2H");
+  CK(cudaStreamSynchronize(st), "sync");
+  return BLU_OK;
+}
+
+blu_status_t blu_gby_init_table(blu_gby_plan_t P, void* dev_table, uint64_t n_slots, void* stream) {
+  if (!P || (n_slots && !dev_table)) return fail(BLU_E_INVALID, "NULL plan or table");
+  CK(launch_init_slots(P->lay, dev_table, n_slots, stream), "init slots");
+  return BLU_OK;
+}
+
+blu_status_t blu_gby_bind_device(int32_t device) {
+  CK(cudaSetDevice(device), "cudaSetDevice");
+  return BLU_OK;
+}
+
+void blu_gby_result_free(blu_gby_result_t* r, void* stream) {
+  if (!r) return;
+  Owner* o = (Owner*)r->_owner;
+  if (o) {
+    for (void* p : o->dev) cudaFreeAsync(p, (cudaStream_t)stream);
+    for (void* h : o->host) free(h);
+    delete o;
+  }
+  free(r->key_cols);
+  free(r->agg_cols);
+  free(r->state_cols);
+  memset(r, 0, sizeof *r);
+}
+
+}  // extern "C"

@@ -1,0 +1,870 @@
+// kernels.cu — the sm_100a kernels of libblugby.
+//
+//   k_init_slots / k_init_dense   S4  hash-table mask copied by parallel threads (Table 1)
+//   k_agg_dense_smem<NV,R>        S5a path (a): per-CTA shared-memory dense tables, CTA -> global
+//                                     merge with native 64-bit REDs (§4.3.2)
+//   k_agg_global<NV,R,FRONT,DIRECT>
+//                                 S5b path (b): global open-addressing table, read-before-CAS
+//                                     linear probing on the 64-bit key, REDs on the aggregate
+//                                     fields (§4.3.1; §4.4 atomics);
+//                                     DIRECT = path (b'): direct-mapped dense domain;
+//                                     FRONT = shared-memory hot-key front (P:168 spill/merge)
+//   k_compact_count/scan/emit     S8  path (c): occupancy -> block counts -> exclusive scan ->
+//                                     dense output, key unpack, AVG = SUM / COUNT
+//   k_partition_*                 S10 owner bucketing of partial states for the all-to-all
+//
+// Column streams are read with 128-bit non-coherent loads that bypass L1 allocation and carry an
+// L2 evict-first policy, so the fact-table stream does not evict an L2-resident hash table.
+// No tensor cores: nothing here is a contraction.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+
+#include "blu_internal.h"
+
+namespace blu {
+
+static std::atomic<uint64_t> g_launches{0};
+void count_launch(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+uint64_t launches_total() { return g_launches.load(); }
+
+// ------------------------------------------------------------------------------------------------
+// device helpers
+// ------------------------------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t fmix64(uint64_t h) {  // Murmur3 finalizer (P:153 cites Murmur)
+  h ^= h >> 33;
+  h *= 0xff51afd7ed558ccdull;
+  h ^= h >> 33;
+  h *= 0xc4ceb9fe1a85ec53ull;
+  h ^= h >> 33;
+  return h;
+}
+
+// Order-preserving map of IEEE-754 f64 bits onto int64 (an involution).
+__device__ __forceinline__ int64_t ord_f64(uint64_t bits) {
+  int64_t b = (int64_t)bits;
+  return b ^ ((b >> 63) & 0x7FFFFFFFFFFFFFFFll);
+}
+__device__ __forceinline__ uint64_t unord_f64(int64_t o) { return (uint64_t)(o ^ ((o >> 63) & 0x7FFFFFFFFFFFFFFFll)); }
+
+__device__ __forceinline__ uint64_t evict_first_policy() {
+  uint64_t pol;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+__device__ __forceinline__ int4 ld_stream_v4(const void* p, uint64_t pol) {
+  int4 r;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], %5;"
+      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+      : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ int32_t ld_stream_s32(const void* p, uint64_t pol) {
+  int32_t r;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ uint64_t ld_stream_u64(const void* p, uint64_t pol) {
+  uint64_t r;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(r) : "l"(p), "l"(pol));
+  return r;
+}
+
+// Load rows [row, row+R) of one column as 64-bit patterns (i32 sign-extended). Rows >= n read 0.
+template <int R>
+__device__ __forceinline__ void load_rows(const void* base, int dt, uint64_t row, uint64_t n, bool vec,
+                                          uint64_t pol, uint64_t (&out)[R]) {
+  if (dt == BLU_I32) {
+    const int32_t* p = (const int32_t*)base + row;
+    if (R == 4 && vec && row + 4 <= n) {
+      int4 v = ld_stream_v4(p, pol);
+      out[0] = (uint64_t)(int64_t)v.x;
+      if (R > 1) out[1 % R] = (uint64_t)(int64_t)v.y;
+      if (R > 2) out[2 % R] = (uint64_t)(int64_t)v.z;
+      if (R > 3) out[3 % R] = (uint64_t)(int64_t)v.w;
+    } else {
+#pragma unroll
+      for (int r = 0; r < R; ++r) out[r] = row + r < n ? (uint64_t)(int64_t)ld_stream_s32(p + r, pol) : 0ull;
+    }
+  } else {
+    const uint64_t* p = (const uint64_t*)base + row;
+    if (R % 2 == 0 && vec && row + R <= n) {
+#pragma unroll
+      for (int r = 0; r < R; r += 2) {
+        int4 v = ld_stream_v4(p + r, pol);
+        out[r] = (uint64_t)(uint32_t)v.x | ((uint64_t)(uint32_t)v.y << 32);
+        out[(r + 1) % R] = (uint64_t)(uint32_t)v.z | ((uint64_t)(uint32_t)v.w << 32);
+      }
+    } else {
+#pragma unroll
+      for (int r = 0; r < R; ++r) out[r] = row + r < n ? ld_stream_u64(p + r, pol) : 0ull;
+    }
+  }
+}
+
+// Encoded value of a row for field kind k: f64 MIN/MAX through ord_f64; everything else as is.
+__device__ __forceinline__ uint64_t encode(int k, uint64_t raw) {
+  return (k == FK_MINF64 || k == FK_MAXF64) ? (uint64_t)ord_f64(raw) : raw;
+}
+
+// Identity (the mask value of P:151) of a field in its encoded 64-bit form.
+__device__ __forceinline__ uint64_t identity64(int k) {
+  switch (k) {
+    case FK_MINI32: return (uint64_t)(int64_t)INT32_MAX;
+    case FK_MAXI32: return (uint64_t)(int64_t)INT32_MIN;
+    case FK_MINI64: case FK_MINF64: return (uint64_t)INT64_MAX;
+    case FK_MAXI64: case FK_MAXF64: return (uint64_t)INT64_MIN;
+    default: return 0ull;
+  }
+}
+
+// ---- shared-memory table (path (a) and the hot-key front). SoA per field; S entries. ----------
+// Field encodings: COUNT u32; SUMI as two u32 arrays lo[S], hi[S] (32-bit native atomics with an
+// explicit carry: 64-bit shared atomics are CAS loops on sm_100a); SUMF f64;
+// MIN/MAX i32 as i32 (native ATOMS.MIN/MAX); 64-bit MIN/MAX read-before-atomic.
+__device__ __forceinline__ void smem_apply(uint8_t* base, int k, uint32_t e, uint32_t S, uint64_t x) {
+  switch (k) {
+    case FK_COUNT:
+      atomicAdd((uint32_t*)base + e, (uint32_t)x);
+      break;
+    case FK_SUMI: {
+      uint32_t lo = (uint32_t)x, hi = (uint32_t)(x >> 32);
+      uint32_t old = atomicAdd((uint32_t*)base + e, lo);
+      hi += (uint32_t)(old + lo < old);
+      if (hi) atomicAdd((uint32_t*)base + S + e, hi);
+      break;
+    }
+    case FK_SUMF:
+      atomicAdd((double*)base + e, __longlong_as_double((long long)x));
+      break;
+    case FK_MINI32: {
+      int v = (int)x;
+      int* q = (int*)base + e;
+      if (v < *(volatile int*)q) atomicMin(q, v);
+      break;
+    }
+    case FK_MAXI32: {
+      int v = (int)x;
+      int* q = (int*)base + e;
+      if (v > *(volatile int*)q) atomicMax(q, v);
+      break;
+    }
+    case FK_MINI64: case FK_MINF64: {
+      long long v = (long long)x;
+      long long* q = (long long*)base + e;
+      if (v < *(volatile long long*)q) atomicMin(q, v);
+      break;
+    }
+    default: {  // FK_MAXI64, FK_MAXF64
+      long long v = (long long)x;
+      long long* q = (long long*)base + e;
+      if (v > *(volatile long long*)q) atomicMax(q, v);
+      break;
+    }
+  }
+}
+
+__device__ __forceinline__ void smem_init_entry(uint8_t* base, int k, uint32_t e, uint32_t S) {
+  switch (k) {
+    case FK_COUNT: ((uint32_t*)base)[e] = 0u; break;
+    case FK_SUMI: ((uint32_t*)base)[e] = 0u; ((uint32_t*)base)[S + e] = 0u; break;
+    case FK_SUMF: ((uint64_t*)base)[e] = 0ull; break;
+    case FK_MINI32: ((int*)base)[e] = INT32_MAX; break;
+    case FK_MAXI32: ((int*)base)[e] = INT32_MIN; break;
+    default: ((uint64_t*)base)[e] = identity64(k); break;
+  }
+}
+
+// Read a shared-memory entry's state as the encoded 64-bit value to combine.
+__device__ __forceinline__ uint64_t smem_read(const uint8_t* base, int k, uint32_t e, uint32_t S) {
+  switch (k) {
+    case FK_COUNT: return (uint64_t)((const uint32_t*)base)[e];
+    case FK_SUMI: return (uint64_t)((const uint32_t*)base)[e] | ((uint64_t)((const uint32_t*)base)[S + e] << 32);
+    case FK_MINI32: case FK_MAXI32: return (uint64_t)(int64_t)((const int*)base)[e];
+    default: return ((const uint64_t*)base)[e];
+  }
+}
+
+// ---- global AoS slot (path b). Fire-and-forget REDs: REDG.E.ADD.64 / ADD.F64 / MIN.S64 ... ----
+__device__ __forceinline__ void slot_apply(uint8_t* slot, const Field& f, uint64_t x) {
+  uint8_t* a = slot + f.goff;
+  switch (f.kind) {
+    case FK_COUNT: case FK_SUMI: atomicAdd((unsigned long long*)a, (unsigned long long)x); break;
+    case FK_SUMF: atomicAdd((double*)a, __longlong_as_double((long long)x)); break;
+    case FK_MINI32: atomicMin((int*)a, (int)x); break;
+    case FK_MAXI32: atomicMax((int*)a, (int)x); break;
+    case FK_MINI64: case FK_MINF64: atomicMin((long long*)a, (long long)x); break;
+    default: atomicMax((long long*)a, (long long)x); break;
+  }
+}
+
+// ---- global dense state (paths a / b'): 4 groups of int64 arrays (sidx x D + g) -----------------
+__device__ __forceinline__ void dense_apply(void* const* dense, uint64_t D, const Field& f, uint64_t g, uint64_t x) {
+  uint64_t* a = (uint64_t*)dense[f.sgroup] + (uint64_t)f.sidx * D + g;
+  switch (f.kind) {
+    case FK_COUNT: case FK_SUMI: atomicAdd((unsigned long long*)a, (unsigned long long)x); break;
+    case FK_SUMF: atomicAdd((double*)a, __longlong_as_double((long long)x)); break;
+    case FK_MINI32: case FK_MINI64: case FK_MINF64: atomicMin((long long*)a, (long long)x); break;
+    default: atomicMax((long long*)a, (long long)x); break;
+  }
+}
+
+// Linear probing from fmix64(key) & mask; read-before-CAS; keys are write-once (EMPTY -> key), so
+// a stale read can only show EMPTY and the CAS resolves it ("next empty slot").
+__device__ __forceinline__ bool hash_locate(uint8_t* table, uint64_t mask, uint32_t sb, uint64_t key,
+                                            uint64_t first, uint64_t idx, uint32_t max_probe, uint64_t& out) {
+  uint64_t cur = first;
+  for (uint32_t p = 0; p < max_probe; ++p) {
+    unsigned long long* kp = (unsigned long long*)(table + idx * sb);
+    if (p) cur = __ldcg(kp);
+    if (cur == key) { out = idx; return true; }
+    if (cur == kEmpty) {
+      unsigned long long old = atomicCAS(kp, (unsigned long long)kEmpty, (unsigned long long)key);
+      if (old == kEmpty || old == key) { out = idx; return true; }
+    }
+    idx = (idx + 1) & mask;
+  }
+  return false;
+}
+
+// Pack the key columns of rows [row, row+R) (S1, CCAT P:111): sparse -> code; dense -> mixed radix
+// sum code_j * stride_j. Invalid codes raise FLAG_KEY_RANGE; rows >= n are not valid.
+template <int R>
+__device__ __forceinline__ uint32_t pack_keys(const AggParams& p, uint64_t row, uint64_t n, uint64_t pol,
+                                              uint64_t (&key)[R]) {
+  uint32_t valid = 0;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    key[r] = 0;
+    if (row + r < n) valid |= 1u << r;
+  }
+  uint32_t bad = 0;
+  if (p.lay.sparse) {
+    uint64_t c[R];
+    load_rows<R>(p.key[0], p.lay.key_dtype[0], row, n, p.vec_ok, pol, c);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      key[r] = c[r];
+      if ((int64_t)c[r] < 0) bad |= 1u << r;
+    }
+  } else {
+    for (int k = 0; k < p.lay.n_keys; ++k) {
+      uint64_t c[R];
+      load_rows<R>(p.key[k], p.lay.key_dtype[k], row, n, p.vec_ok, pol, c);
+      const uint64_t d = p.lay.dict[k], s = p.lay.stride[k];
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        if (c[r] >= d) bad |= 1u << r;  // unsigned: negatives are huge
+        key[r] += c[r] * s;
+      }
+    }
+  }
+  bad &= valid;
+  if (bad) atomicOr(p.flags, FLAG_KEY_RANGE);
+  return valid & ~bad;
+}
+
+
+// Field-column masks: bit j set if field j reads column c; cnt: fields counting the constant 1.
+struct ColMasks {
+  uint32_t col[kMaxVals > kMaxFields ? kMaxVals : kMaxFields];
+  uint32_t cnt;
+};
+
+__device__ __forceinline__ void build_masks(const Layout& L, ColMasks& m) {
+  for (int c = 0; c < kMaxFields; ++c) m.col[c] = 0;
+  m.cnt = 0;
+  for (int j = 0; j < L.n_fields; ++j) {
+    if (L.f[j].col < 0) m.cnt |= 1u << j;
+    else m.col[L.f[j].col] |= 1u << j;
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// S4: table initialisation — the mask row copied by parallel threads with 16-byte stores
+// ------------------------------------------------------------------------------------------------
+struct SlotTemplate {
+  uint64_t w[32];  // up to 256-byte slots
+  uint32_t words;  // slot_bytes / 8
+};
+
+__global__ void __launch_bounds__(256) k_init_slots(SlotTemplate t, uint64_t* table, uint64_t n_words2) {
+  // n_words2 = number of 16-byte chunks; slot_bytes is a multiple of 16
+  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  uint32_t pairs = t.words / 2;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_words2; i += stride) {
+    uint32_t w = (uint32_t)(i % pairs) * 2;
+    ulonglong2 v = make_ulonglong2(t.w[w], t.w[w + 1]);
+    reinterpret_cast<ulonglong2*>(table)[i] = v;
+  }
+}
+
+__global__ void __launch_bounds__(256) k_fill_u64(uint64_t* a, uint64_t n, uint64_t v) {
+  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) a[i] = v;
+}
+
+// ------------------------------------------------------------------------------------------------
+// S5a: path (a) dense shared-memory aggregation (§4.3.2)
+// ------------------------------------------------------------------------------------------------
+struct SmemOffsets {
+  uint32_t off[kMaxFields];
+  uint32_t key_off;  // front only
+};
+
+__device__ __forceinline__ void smem_offsets(const Layout& L, uint32_t S, bool with_keys, SmemOffsets& so) {
+  uint32_t o = 0;
+  if (with_keys) { so.key_off = 0; o = S * 8; }
+  for (int j = 0; j < L.n_fields; ++j) {
+    so.off[j] = o;
+    o += (S * L.f[j].ssize + 15) / 16 * 16;
+  }
+}
+
+template <int NV, int R>
+__global__ void __launch_bounds__(512) k_agg_dense_smem(AggParams p) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  const Layout& L = p.lay;
+  const uint32_t D = (uint32_t)L.domain;
+  SmemOffsets so;
+  smem_offsets(L, D, false, so);
+  for (int j = 0; j < L.n_fields; ++j)
+    for (uint32_t e = threadIdx.x; e < D; e += blockDim.x) smem_init_entry(sm + so.off[j], L.f[j].kind, e, D);
+  ColMasks cm;
+  build_masks(L, cm);
+  __syncthreads();
+
+  const uint64_t pol = evict_first_policy();
+  const uint64_t n = p.n_rows;
+  const uint64_t tile = (uint64_t)blockDim.x * R;
+  const uint64_t ntiles = (n + tile - 1) / tile;
+  uint32_t flag_seen = 0;
+  for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    if (flag_seen) break;
+    flag_seen = *(volatile uint32_t*)p.flags;  // checked at the next tile (latency hidden)
+    const uint64_t row = t * tile + (uint64_t)threadIdx.x * R;
+    if (row >= n) continue;
+    uint64_t key[R];
+    uint32_t valid = pack_keys<R>(p, row, n, pol, key);
+    uint64_t v[NV][R];
+#pragma unroll
+    for (int c = 0; c < NV; ++c)
+      if (c < L.n_vals) load_rows<R>(p.val[c], L.val_dtype[c], row, n, p.vec_ok, pol, v[c]);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!(valid >> r & 1)) continue;
+      const uint32_t e = (uint32_t)key[r];
+      for (uint32_t m = cm.cnt; m; m &= m - 1) {
+        int j = __ffs(m) - 1;
+        smem_apply(sm + so.off[j], L.f[j].kind, e, D, 1ull);
+      }
+#pragma unroll
+      for (int c = 0; c < NV; ++c) {
+        if (c >= L.n_vals) break;
+        for (uint32_t m = cm.col[c]; m; m &= m - 1) {
+          int j = __ffs(m) - 1;
+          int k = L.f[j].kind;
+          smem_apply(sm + so.off[j], k, e, D, encode(k, v[c][r]));
+        }
+      }
+    }
+  }
+  __syncthreads();
+  // S7: CTA -> global merge with native 64-bit REDs ("the small hash tables in shared memory
+  // are merged to a global hash table in device memory").
+  const int cf = L.count_field;
+  for (uint32_t e = threadIdx.x; e < D; e += blockDim.x) {
+    if (smem_read(sm + so.off[cf], L.f[cf].kind, e, D) == 0) continue;
+    for (int j = 0; j < L.n_fields; ++j)
+      dense_apply(p.dense, L.domain, L.f[j], e, smem_read(sm + so.off[j], L.f[j].kind, e, D));
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// S5b: path (b) global hash table / path (b') direct-mapped, optional shared-memory hot-key front
+// ------------------------------------------------------------------------------------------------
+template <bool DIRECT>
+__device__ __forceinline__ bool global_apply_row(const AggParams& p, const ColMasks& cm, uint64_t key,
+                                                 uint64_t first, uint64_t idx, const uint64_t* vals /*NV*/,
+                                                 int nv) {
+  const Layout& L = p.lay;
+  if (DIRECT) {
+    for (uint32_t m = cm.cnt; m; m &= m - 1) dense_apply(p.dense, L.domain, L.f[__ffs(m) - 1], key, 1ull);
+    for (int c = 0; c < nv; ++c)
+      for (uint32_t m = cm.col[c]; m; m &= m - 1) {
+        const Field& f = L.f[__ffs(m) - 1];
+        dense_apply(p.dense, L.domain, f, key, encode(f.kind, vals[c]));
+      }
+    return true;
+  } else {
+    uint64_t slot;
+    if (!hash_locate((uint8_t*)p.table, p.cap_mask, L.slot_bytes, key, first, idx, p.max_probe, slot)) return false;
+    uint8_t* s = (uint8_t*)p.table + slot * L.slot_bytes;
+    for (uint32_t m = cm.cnt; m; m &= m - 1) slot_apply(s, L.f[__ffs(m) - 1], 1ull);
+    for (int c = 0; c < nv; ++c)
+      for (uint32_t m = cm.col[c]; m; m &= m - 1) {
+        const Field& f = L.f[__ffs(m) - 1];
+        slot_apply(s, f, encode(f.kind, vals[c]));
+      }
+    return true;
+  }
+}
+
+template <int NV, int R, bool FRONT, bool DIRECT, bool RECORDS>
+__global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  const Layout& L = p.lay;
+  const uint32_t S = p.front_slots;
+  SmemOffsets so;
+  if (FRONT) {
+    smem_offsets(L, S, true, so);
+    for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) ((uint64_t*)(sm + so.key_off))[e] = kEmpty;
+    for (int j = 0; j < L.n_fields; ++j)
+      for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) smem_init_entry(sm + so.off[j], L.f[j].kind, e, S);
+    __syncthreads();
+  }
+  ColMasks cm;
+  build_masks(L, cm);
+  const uint64_t pol = evict_first_policy();
+  const uint64_t n = p.n_rows;
+  const uint64_t tile = (uint64_t)blockDim.x * R;
+  const uint64_t ntiles = (n + tile - 1) / tile;
+  uint32_t flag_seen = 0;
+  for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    if (flag_seen) break;
+    flag_seen = *(volatile uint32_t*)p.flags;
+    const uint64_t row = t * tile + (uint64_t)threadIdx.x * R;
+    if (row >= n) continue;
+    uint64_t key[R];
+    uint64_t v[NV][R];
+    uint32_t valid;
+    if (RECORDS) {
+      valid = 0;
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        if (row + r >= n) { key[r] = 0; continue; }
+        const uint64_t* rec = rs.rec + (row + r) * rs.words;
+        key[r] = __ldg((const unsigned long long*)rec);
+        valid |= 1u << r;
+#pragma unroll
+        for (int c = 0; c < NV; ++c)
+          if (c < L.n_vals) {
+            uint64_t w = __ldg((const unsigned long long*)rec + 1 + c);
+            v[c][r] = L.val_dtype[c] == BLU_I32 ? (uint64_t)(int64_t)(int32_t)(uint32_t)w : w;
+          }
+      }
+    } else {
+      valid = pack_keys<R>(p, row, n, pol, key);
+#pragma unroll
+      for (int c = 0; c < NV; ++c)
+        if (c < L.n_vals) load_rows<R>(p.val[c], L.val_dtype[c], row, n, p.vec_ok, pol, v[c]);
+    }
+    // probe: issue the first key load of every row before resolving any (memory-level parallelism)
+    uint64_t idx[R], first[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      idx[r] = 0;
+      first[r] = 0;
+      if (!DIRECT && (valid >> r & 1)) {
+        idx[r] = fmix64(key[r]) & p.cap_mask;
+        first[r] = __ldcg((const unsigned long long*)((const uint8_t*)p.table + idx[r] * L.slot_bytes));
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!(valid >> r & 1)) continue;
+      if (FRONT) {
+        uint64_t* fk = (uint64_t*)(sm + so.key_off);
+        uint32_t s = (uint32_t)(fmix64(key[r] ^ 0x5bd1e995ull) >> 40) & (S - 1);
+        bool hit = false;
+#pragma unroll 1
+        for (int q = 0; q < 8; ++q) {
+          uint64_t cur = *(volatile uint64_t*)(fk + s);
+          if (cur == key[r]) { hit = true; break; }
+          if (cur == kEmpty) {
+            unsigned long long old = atomicCAS((unsigned long long*)(fk + s), (unsigned long long)kEmpty,
+                                               (unsigned long long)key[r]);
+            if (old == kEmpty || old == key[r]) { hit = true; break; }
+          }
+          s = (s + 1) & (S - 1);
+        }
+        if (hit) {
+          for (uint32_t m = cm.cnt; m; m &= m - 1) {
+            int j = __ffs(m) - 1;
+            smem_apply(sm + so.off[j], L.f[j].kind, s, S, 1ull);
+          }
+#pragma unroll
+          for (int c = 0; c < NV; ++c) {
+            if (c >= L.n_vals) break;
+            for (uint32_t m = cm.col[c]; m; m &= m - 1) {
+              int j = __ffs(m) - 1;
+              int k = L.f[j].kind;
+              smem_apply(sm + so.off[j], k, s, S, encode(k, v[c][r]));
+            }
+          }
+          continue;
+        }
+        if (!DIRECT) first[r] = __ldcg((const unsigned long long*)((const uint8_t*)p.table + idx[r] * L.slot_bytes));
+      }
+      uint64_t vals[NV];
+#pragma unroll
+      for (int c = 0; c < NV; ++c) vals[c] = v[c][r];
+      if (!global_apply_row<DIRECT>(p, cm, key[r], first[r], idx[r], vals, NV < L.n_vals ? NV : L.n_vals)) {
+        atomicOr(p.flags, FLAG_OVERFLOW);
+        flag_seen = 1;
+        break;
+      }
+    }
+  }
+  if (FRONT) {
+    // merge the front into the global table
+    __syncthreads();
+    uint64_t* fk = (uint64_t*)(sm + so.key_off);
+    for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) {
+      uint64_t key = fk[e];
+      if (key == kEmpty) continue;
+      if (DIRECT) {
+        for (int j = 0; j < L.n_fields; ++j)
+          dense_apply(p.dense, L.domain, L.f[j], key, smem_read(sm + so.off[j], L.f[j].kind, e, S));
+      } else {
+        uint64_t idx = fmix64(key) & p.cap_mask, slot;
+        uint64_t first = __ldcg((const unsigned long long*)((const uint8_t*)p.table + idx * L.slot_bytes));
+        if (!hash_locate((uint8_t*)p.table, p.cap_mask, L.slot_bytes, key, first, idx, p.max_probe, slot)) {
+          atomicOr(p.flags, FLAG_OVERFLOW);
+          continue;
+        }
+        uint8_t* s = (uint8_t*)p.table + slot * L.slot_bytes;
+        for (int j = 0; j < L.n_fields; ++j) slot_apply(s, L.f[j], smem_read(sm + so.off[j], L.f[j].kind, e, S));
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// S8: compaction (path (c))
+// ------------------------------------------------------------------------------------------------
+constexpr int kCT = 256;        // threads
+constexpr int kCRounds = 16;    // entries per thread
+constexpr uint64_t kCB = (uint64_t)kCT * kCRounds;
+
+__device__ __forceinline__ bool occupied(const CompactParams& p, uint64_t e) {
+  if (p.source == 0)
+    return __ldg((const unsigned long long*)((const uint8_t*)p.table + e * p.lay.slot_bytes)) != kEmpty;
+  const Field& cf = p.lay.f[p.lay.count_field];
+  return __ldg((const long long*)p.dense[cf.sgroup] + (uint64_t)cf.sidx * p.n_entries + e) > 0;
+}
+
+// field j of entry e as the encoded 64-bit value
+__device__ __forceinline__ uint64_t read_field(const CompactParams& p, int j, uint64_t e) {
+  const Field& f = p.lay.f[j];
+  if (p.source == 0) {
+    const uint8_t* a = (const uint8_t*)p.table + e * p.lay.slot_bytes + f.goff;
+    if (f.gsize == 4) return (uint64_t)(int64_t)__ldg((const int*)a);
+    return __ldg((const unsigned long long*)a);
+  }
+  return __ldg((const unsigned long long*)p.dense[f.sgroup] + (uint64_t)f.sidx * p.n_entries + e);
+}
+
+__device__ __forceinline__ void store_as(void* out, uint64_t pos, int dtype, uint64_t bits) {
+  if (dtype == BLU_I32) ((int32_t*)out)[pos] = (int32_t)(uint32_t)bits;
+  else ((uint64_t*)out)[pos] = bits;
+}
+
+__global__ void __launch_bounds__(kCT) k_compact_count(CompactParams p) {
+  uint64_t base = (uint64_t)blockIdx.x * kCB;
+  uint32_t c = 0;
+  for (int i = 0; i < kCRounds; ++i) {
+    uint64_t e = base + (uint64_t)i * kCT + threadIdx.x;
+    if (e < p.n_entries && occupied(p, e)) ++c;
+  }
+  __shared__ uint32_t ws[kCT / 32];
+  for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+  if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = c;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint64_t t = 0;
+    for (int w = 0; w < kCT / 32; ++w) t += ws[w];
+    p.block_counts[blockIdx.x] = t;
+  }
+}
+
+__global__ void __launch_bounds__(1024) k_compact_scan(uint64_t* counts, uint64_t* offsets, uint64_t nb, uint64_t* total) {
+  __shared__ uint64_t ws[32];
+  __shared__ uint64_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  for (uint64_t base = 0; base < nb; base += 1024) {
+    uint64_t i = base + threadIdx.x;
+    uint64_t x = i < nb ? counts[i] : 0;
+    uint64_t inc = x;
+    for (int o = 1; o < 32; o <<= 1) {
+      uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+      if ((threadIdx.x & 31) >= (unsigned)o) inc += y;
+    }
+    if ((threadIdx.x & 31) == 31) ws[threadIdx.x >> 5] = inc;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+      uint64_t w = ws[threadIdx.x], wi = w;
+      for (int o = 1; o < 32; o <<= 1) {
+        uint64_t y = __shfl_up_sync(0xffffffffu, wi, o);
+        if (threadIdx.x >= (unsigned)o) wi += y;
+      }
+      ws[threadIdx.x] = wi - w;  // exclusive warp offsets
+    }
+    __syncthreads();
+    uint64_t excl = carry + ws[threadIdx.x >> 5] + inc - x;
+    if (i < nb) offsets[i] = excl;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry = excl + x;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *total = carry;
+}
+
+__global__ void __launch_bounds__(kCT) k_compact_emit(CompactParams p) {
+  __shared__ uint32_t ws[kCT / 32];
+  const uint64_t base = (uint64_t)blockIdx.x * kCB;
+  uint64_t out_pos = p.block_offsets[blockIdx.x];
+  const Layout& L = p.lay;
+  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int i = 0; i < kCRounds; ++i) {
+    uint64_t e = base + (uint64_t)i * kCT + threadIdx.x;
+    bool occ = e < p.n_entries && occupied(p, e);
+    unsigned bal = __ballot_sync(0xffffffffu, occ);
+    if (lane == 0) ws[warp] = __popc(bal);
+    __syncthreads();
+    uint32_t before = 0, tot = 0;
+    for (unsigned w = 0; w < kCT / 32; ++w) {
+      if (w < warp) before += ws[w];
+      tot += ws[w];
+    }
+    before += __popc(bal & ((1u << lane) - 1u));
+    if (occ) {
+      uint64_t pos = out_pos + before;
+      uint64_t key = p.source == 0 ? __ldg((const unsigned long long*)((const uint8_t*)p.table + e * L.slot_bytes)) : e;
+      for (int k = 0; k < L.n_keys; ++k) {
+        uint64_t code = L.sparse ? key : (key / L.stride[k]) % L.dict[k];
+        store_as(p.out_keys[k], pos, L.key_dtype[k], code);
+      }
+      if (p.partial) {
+        for (int j = 0; j < L.n_fields; ++j) {
+          uint64_t x = read_field(p, j, e);
+          int k = L.f[j].kind;
+          if (k == FK_MINF64 || k == FK_MAXF64) x = unord_f64((int64_t)x);
+          int dt = (k == FK_MINI32 || k == FK_MAXI32) ? BLU_I32 : BLU_I64;
+          store_as(p.out_vals[j], pos, dt, x);
+        }
+      } else {
+        for (int o = 0; o < p.n_out; ++o) {
+          int j = p.out_field[o];
+          uint64_t x = read_field(p, j, e);
+          int k = L.f[j].kind;
+          if (p.out_kind[o] == 1) {  // AVG = (double)SUM / (double)COUNT (reading A12)
+            uint64_t cnt = read_field(p, p.out_field2[o], e);
+            double s = k == FK_SUMF ? __longlong_as_double((long long)x) : (double)(long long)x;
+            double a = s / (double)(long long)cnt;
+            x = (uint64_t)__double_as_longlong(a);
+          } else if (k == FK_MINF64 || k == FK_MAXF64) {
+            x = unord_f64((int64_t)x);
+          }
+          store_as(p.out_vals[o], pos, p.out_dtype[o], x);
+        }
+      }
+    }
+    __syncthreads();
+    out_pos += tot;
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// S10: owner partition of partial states for the all-to-all
+// ------------------------------------------------------------------------------------------------
+struct PartParams {
+  Layout lay;  // merge layout (state columns)
+  const void* key[kMaxKeys];
+  const void* st[kMaxFields];
+  uint64_t n;
+  int32_t n_parts;
+  uint64_t* counts;   // n_parts (histogram, then cursor)
+  uint64_t* offsets;  // n_parts
+  uint64_t* out;
+  uint32_t words;
+};
+
+__device__ __forceinline__ uint64_t pack_row(const PartParams& p, uint64_t i) {
+  const Layout& L = p.lay;
+  if (L.sparse) {
+    return L.key_dtype[0] == BLU_I32 ? (uint64_t)(int64_t)((const int32_t*)p.key[0])[i] : ((const uint64_t*)p.key[0])[i];
+  }
+  uint64_t key = 0;
+  for (int k = 0; k < L.n_keys; ++k) {
+    uint64_t c = L.key_dtype[k] == BLU_I32 ? (uint64_t)(int64_t)((const int32_t*)p.key[k])[i] : ((const uint64_t*)p.key[k])[i];
+    key += c * L.stride[k];
+  }
+  return key;
+}
+
+__device__ __forceinline__ uint32_t owner_of(uint64_t key, int32_t P) { return (uint32_t)__umul64hi(fmix64(key), (uint64_t)P); }
+
+__global__ void __launch_bounds__(256) k_partition_hist(PartParams p) {
+  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.n; i += stride)
+    atomicAdd((unsigned long long*)&p.counts[owner_of(pack_row(p, i), p.n_parts)], 1ull);
+}
+
+__global__ void __launch_bounds__(256) k_partition_scatter(PartParams p) {
+  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.n; i += stride) {
+    uint64_t key = pack_row(p, i);
+    uint32_t o = owner_of(key, p.n_parts);
+    uint64_t pos = p.offsets[o] + atomicAdd((unsigned long long*)&p.counts[o], 1ull);
+    uint64_t* rec = p.out + pos * p.words;
+    rec[0] = key;
+    for (int j = 0; j < p.lay.n_vals; ++j) {
+      uint64_t w = p.lay.val_dtype[j] == BLU_I32 ? (uint64_t)(int64_t)((const int32_t*)p.st[j])[i] : ((const uint64_t*)p.st[j])[i];
+      rec[1 + j] = w;
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// launchers
+// ------------------------------------------------------------------------------------------------
+static int grid_for(uint64_t n, int threads, int max_blocks) {
+  uint64_t b = (n + threads - 1) / threads;
+  if (b > (uint64_t)max_blocks) b = max_blocks;
+  return (int)(b ? b : 1);
+}
+
+int launch_init_slots(const Layout& lay, void* table, uint64_t n_slots, void* stream) {
+  if (!n_slots) return 0;
+  SlotTemplate t{};
+  uint8_t buf[256];
+  build_slot_template(lay, buf);
+  memcpy(t.w, buf, lay.slot_bytes);
+  t.words = lay.slot_bytes / 8;
+  uint64_t chunks = n_slots * (lay.slot_bytes / 16);
+  k_init_slots<<<grid_for(chunks, 256, 148 * 16), 256, 0, (cudaStream_t)stream>>>(t, (uint64_t*)table, chunks);
+  count_launch(1);
+  return (int)cudaGetLastError();
+}
+
+static uint64_t identity_host(int k) {
+  switch (k) {
+    case FK_MINI32: return (uint64_t)(int64_t)INT32_MAX;
+    case FK_MAXI32: return (uint64_t)(int64_t)INT32_MIN;
+    case FK_MINI64: case FK_MINF64: return (uint64_t)INT64_MAX;
+    case FK_MAXI64: case FK_MAXF64: return (uint64_t)INT64_MIN;
+    default: return 0ull;
+  }
+}
+
+int launch_init_dense(const Layout& lay, void* const dense[4], uint64_t D, void* stream) {
+  // Dense state groups: ISUM/FSUM -> 0; MIN -> INT64_MAX (covers widened i32 and ordered f64);
+  // MAX -> INT64_MIN. Each group is one contiguous array.
+  for (int g = 0; g < 4; ++g) {
+    uint64_t n = (uint64_t)lay.n_group[g] * D;
+    if (!n) continue;
+    uint64_t v = g == SG_MIN ? (uint64_t)INT64_MAX : g == SG_MAX ? (uint64_t)INT64_MIN : 0ull;
+    k_fill_u64<<<grid_for(n, 256, 148 * 16), 256, 0, (cudaStream_t)stream>>>((uint64_t*)dense[g], n, v);
+    count_launch(1);
+  }
+  (void)identity_host;
+  return (int)cudaGetLastError();
+}
+
+template <int NV, int R>
+static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, const RecSrc& rs, bool records,
+                         void* stream, uint32_t grid, uint32_t block, uint32_t smem) {
+  cudaStream_t st = (cudaStream_t)stream;
+  cudaError_t e = cudaSuccess;
+  if (path == BLU_PATH_DENSE_SMEM) {
+    if constexpr (NV > 16) {
+      return (int)cudaErrorInvalidValue;
+    } else {
+      auto k = k_agg_dense_smem<NV, R>;
+      if (smem > 48 * 1024) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+      if (e) return (int)e;
+      k<<<grid, block, smem, st>>>(p);
+    }
+  } else {
+    void (*k)(AggParams, RecSrc);
+    bool front = p.front_slots > 0;
+    bool direct = path == BLU_PATH_DIRECT_GLOBAL;
+    if constexpr (NV > 16) {  // merges of wide states: no front, no records
+      if (records || front || direct) return (int)cudaErrorInvalidValue;
+      k = k_agg_global<NV, R, false, false, false>;
+    } else {
+      if (records) k = k_agg_global<NV, R, false, false, true>;
+      else if (direct) k = front ? k_agg_global<NV, R, true, true, false> : k_agg_global<NV, R, false, true, false>;
+      else k = front ? k_agg_global<NV, R, true, false, false> : k_agg_global<NV, R, false, false, false>;
+    }
+    if (smem > 48 * 1024) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e) return (int)e;
+    k<<<grid, block, smem, st>>>(p, rs);
+  }
+  count_launch(1);
+  return (int)cudaGetLastError();
+}
+
+int launch_aggregate_impl(const blu_gby_plan_s* P, int path, const AggParams& p, const RecSrc& rs, bool records,
+                          void* stream, uint32_t grid, uint32_t block, uint32_t smem) {
+  int nv = p.lay.n_vals;
+  if (nv <= 1) return launch_agg_nv<1, 4>(P, path, p, rs, records, stream, grid, block, smem);
+  if (nv <= 2) return launch_agg_nv<2, 4>(P, path, p, rs, records, stream, grid, block, smem);
+  if (nv <= 4) return launch_agg_nv<4, 4>(P, path, p, rs, records, stream, grid, block, smem);
+  if (nv <= 8) return launch_agg_nv<8, 2>(P, path, p, rs, records, stream, grid, block, smem);
+  if (nv <= 16) return launch_agg_nv<16, 1>(P, path, p, rs, records, stream, grid, block, smem);
+  return launch_agg_nv<24, 1>(P, path, p, rs, records, stream, grid, block, smem);
+}
+
+int launch_compact(const CompactParams& p, void* stream, uint32_t* launches) {
+  cudaStream_t st = (cudaStream_t)stream;
+  uint64_t nb = (p.n_entries + kCB - 1) / kCB;
+  if (nb == 0) {
+    cudaMemsetAsync(p.n_groups, 0, 8, st);
+    return (int)cudaGetLastError();
+  }
+  k_compact_count<<<(unsigned)nb, kCT, 0, st>>>(p);
+  k_compact_scan<<<1, 1024, 0, st>>>(p.block_counts, p.block_offsets, nb, p.n_groups);
+  k_compact_emit<<<(unsigned)nb, kCT, 0, st>>>(p);
+  count_launch(3);
+  if (launches) *launches += 3;
+  return (int)cudaGetLastError();
+}
+
+int launch_partition(const Layout& lay, const void* const* key_cols, const void* const* state_cols, uint64_t n,
+                     int32_t n_parts, void* send_buf, uint64_t* d_counts, uint64_t* d_offsets, void* stream) {
+  // two-phase: histogram -> (host) offsets -> scatter. The caller passes d_counts zeroed; this
+  // launcher runs the histogram, copies counts to the host, scans, uploads offsets, re-zeroes the
+  // cursors and scatters.
+  cudaStream_t st = (cudaStream_t)stream;
+  PartParams p{};
+  p.lay = lay;
+  for (int k = 0; k < lay.n_keys; ++k) p.key[k] = key_cols[k];
+  for (int j = 0; j < lay.n_vals; ++j) p.st[j] = state_cols[j];
+  p.n = n;
+  p.n_parts = n_parts;
+  p.counts = d_counts;
+  p.offsets = d_offsets;
+  p.out = (uint64_t*)send_buf;
+  p.words = 1 + lay.n_vals;
+  int grid = grid_for(n, 256, 148 * 8);
+  k_partition_hist<<<grid, 256, 0, st>>>(p);
+  count_launch(1);
+  uint64_t h_counts[1024];
+  cudaMemcpyAsync(h_counts, d_counts, sizeof(uint64_t) * n_parts, cudaMemcpyDeviceToHost, st);
+  cudaStreamSynchronize(st);
+  uint64_t h_off[1024];
+  uint64_t acc = 0;
+  for (int i = 0; i < n_parts; ++i) { h_off[i] = acc; acc += h_counts[i]; }
+  cudaMemcpyAsync(d_offsets, h_off, sizeof(uint64_t) * n_parts, cudaMemcpyHostToDevice, st);
+  cudaMemsetAsync(d_counts, 0, sizeof(uint64_t) * n_parts, st);
+  k_partition_scatter<<<grid, 256, 0, st>>>(p);
+  count_launch(1);
+  cudaStreamSynchronize(st);
+  return (int)cudaGetLastError();
+}
+
+}  // namespace blu

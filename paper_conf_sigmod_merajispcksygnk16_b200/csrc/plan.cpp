@@ -1,0 +1,394 @@
+// plan.cpp — the planner ("GPU moderator") and plan-level C ABI.
+//
+// Host only: blu_gby_plan never launches work. It turns (schema, est_groups, n_rows) — the
+// metadata the DB2 runtime hands the GPU runtime — into a frozen plan:
+//   * state fields and the slot layout (key + one field per payload/aggregate, padded so
+//     the row is 1/2/4/8/16-byte aligned; Table 1 P:155-160 is the 32-byte example);
+//   * the kernel path (number of rows, estimated groups, number of aggregates):
+//       (a) dense shared-memory tables when the whole dictionary domain fits in shared memory
+//           ("Second Kernel: Small Number of Groups", §4.3.2);
+//       (b') direct-mapped global table when the dense domain is small enough to allocate
+//           (the paper's "mod hash" with a table at least as large as the domain);
+//       (b) global open-addressing hash table sized from est_groups ("First Kernel", §4.3.1,
+//           P:149-162): cap = next_pow2(ceil(max(est,1)/0.7)), >= 1024 (reading A5);
+//   * the shared-memory hot-key front for (b)/(b') when rows/groups is high (the moderator's
+//     "ratio of rows to number of groups"; "if it gets full ... merge into a global
+//     hash table");
+//   * shared memory and launch shape.
+#include <cuda_runtime.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <mutex>
+
+#include "blu_internal.h"
+
+namespace blu {
+
+thread_local std::string g_last_error;
+
+blu_status_t fail(blu_status_t s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return s;
+}
+
+static uint64_t next_pow2(uint64_t x) {
+  uint64_t p = 1;
+  while (p < x) p <<= 1;
+  return p;
+}
+
+// Planner constants (SURVEY.md §5 "Config / flags"; reading A16: the paper gives no values).
+constexpr uint32_t kSmemDenseMax = 96 * 1024;   // path (a): D x entry bytes, 2 CTAs/SM
+constexpr double kMaxLoad = 0.7;                // A5
+constexpr uint64_t kMinCap = 1024;
+constexpr uint64_t kFrontRatio = 1000;          // rows/groups above which the front pays off
+constexpr uint32_t kFrontBudget = 110 * 1024;
+constexpr uint64_t kDirectMin = 1ull << 20;
+
+static int32_t field_gsize(int kind) { return (kind == FK_MINI32 || kind == FK_MAXI32) ? 4 : 8; }
+static int32_t field_ssize(int kind) {
+  return (kind == FK_COUNT || kind == FK_MINI32 || kind == FK_MAXI32) ? 4 : 8;
+}
+static int32_t field_group(int kind) {
+  switch (kind) {
+    case FK_COUNT: case FK_SUMI: return SG_ISUM;
+    case FK_SUMF: return SG_FSUM;
+    case FK_MINI32: case FK_MINI64: case FK_MINF64: return SG_MIN;
+    default: return SG_MAX;
+  }
+}
+
+uint32_t smem_entry_bytes(const Layout& lay) {
+  uint32_t b = 0;
+  for (int j = 0; j < lay.n_fields; ++j) b += lay.f[j].ssize;
+  return b;
+}
+
+// Assign AoS offsets (natural alignment, in field order after the 8-byte key) and dense groups.
+static void finish_layout(Layout& L) {
+  uint32_t off = 8;
+  int32_t gcount[4] = {0, 0, 0, 0};
+  for (int j = 0; j < L.n_fields; ++j) {
+    Field& f = L.f[j];
+    f.gsize = field_gsize(f.kind);
+    f.ssize = field_ssize(f.kind);
+    off = (off + f.gsize - 1) / f.gsize * f.gsize;
+    f.goff = (int32_t)off;
+    off += f.gsize;
+    f.sgroup = field_group(f.kind);
+    f.sidx = gcount[f.sgroup]++;
+  }
+  for (int g = 0; g < 4; ++g) L.n_group[g] = gcount[g];
+  uint32_t raw = (off + 7) / 8 * 8;
+  uint32_t sb = 16;
+  while (sb < raw && sb < 128) sb <<= 1;
+  if (sb < raw) sb = (raw + 63) / 64 * 64;
+  L.slot_bytes = sb;
+  L.smem_entry_bytes = smem_entry_bytes(L);
+}
+
+static int add_field(Layout& L, int kind, int col, int is_count) {
+  for (int j = 0; j < L.n_fields; ++j)
+    if (L.f[j].kind == kind && L.f[j].col == col) return j;
+  Field f{};
+  f.kind = kind;
+  f.col = col;
+  f.is_count = is_count;
+  L.f[L.n_fields] = f;
+  if (is_count) L.count_field = L.n_fields;
+  return L.n_fields++;
+}
+
+static int device_sms() {
+  static int sms = -1;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    int n = 0;
+    if (cudaGetDeviceCount(&n) == cudaSuccess && n > 0) {
+      int dev = 0, v = 0;
+      cudaGetDevice(&dev);
+      if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess) sms = v;
+    } else {
+      cudaGetLastError();
+    }
+    if (sms <= 0) sms = 148;  // B200
+  });
+  return sms;
+}
+
+static const char* env(const char* k) {
+  const char* v = getenv(k);
+  return (v && *v) ? v : nullptr;
+}
+
+void build_slot_template(const Layout& L, uint8_t* out) {
+  memset(out, 0, L.slot_bytes);
+  uint64_t key = kEmpty;
+  memcpy(out, &key, 8);
+  for (int j = 0; j < L.n_fields; ++j) {
+    const Field& f = L.f[j];
+    uint8_t* p = out + f.goff;
+    int64_t v64 = 0;
+    int32_t v32 = 0;
+    switch (f.kind) {
+      case FK_MINI32: v32 = INT32_MAX; memcpy(p, &v32, 4); break;
+      case FK_MAXI32: v32 = INT32_MIN; memcpy(p, &v32, 4); break;
+      case FK_MINI64: case FK_MINF64: v64 = INT64_MAX; memcpy(p, &v64, 8); break;
+      case FK_MAXI64: case FK_MAXF64: v64 = INT64_MIN; memcpy(p, &v64, 8); break;
+      default: memcpy(p, &v64, 8); break;  // COUNT, SUM: 0
+    }
+  }
+}
+
+}  // namespace blu
+
+using namespace blu;
+
+extern "C" {
+
+const char* blu_gby_status_str(blu_status_t s) {
+  switch (s) {
+    case BLU_OK: return "BLU_OK";
+    case BLU_E_INVALID: return "BLU_E_INVALID";
+    case BLU_E_UNSUPPORTED: return "BLU_E_UNSUPPORTED";
+    case BLU_E_KEY_RANGE: return "BLU_E_KEY_RANGE";
+    case BLU_E_OOM: return "BLU_E_OOM";
+    case BLU_E_CUDA: return "BLU_E_CUDA";
+  }
+  return "BLU_E_UNKNOWN";
+}
+
+const char* blu_gby_last_error(void) { return g_last_error.c_str(); }
+
+blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64_t n_rows,
+                          blu_gby_plan_t* out_plan) {
+  if (!s || !out_plan) return fail(BLU_E_INVALID, "NULL schema or out_plan");
+  *out_plan = nullptr;
+  if (s->n_keys < 1 || s->n_keys > kMaxKeys || !s->keys)
+    return fail(BLU_E_INVALID, "n_keys must be 1..%d (got %d)", kMaxKeys, s->n_keys);
+  if (s->n_vals < 0 || s->n_vals > kMaxVals || (s->n_vals > 0 && !s->vals))
+    return fail(BLU_E_INVALID, "n_vals must be 0..%d (got %d)", kMaxVals, s->n_vals);
+  if (s->n_aggs < 1 || s->n_aggs > kMaxAggs || !s->aggs)
+    return fail(BLU_E_INVALID, "n_aggs must be 1..%d (got %d)", kMaxAggs, s->n_aggs);
+  for (int k = 0; k < s->n_keys; ++k)
+    if (s->keys[k].dtype != BLU_I32 && s->keys[k].dtype != BLU_I64)
+      return fail(BLU_E_INVALID, "key %d: dtype must be BLU_I32 or BLU_I64", k);
+  for (int c = 0; c < s->n_vals; ++c)
+    if (s->vals[c] != BLU_I32 && s->vals[c] != BLU_I64 && s->vals[c] != BLU_F64)
+      return fail(BLU_E_INVALID, "value %d: bad dtype %d", c, (int)s->vals[c]);
+  for (int a = 0; a < s->n_aggs; ++a) {
+    int op = s->aggs[a].op;
+    if (op < BLU_COUNT || op > BLU_AVG) return fail(BLU_E_INVALID, "agg %d: bad op %d", a, op);
+    if (op != BLU_COUNT && (s->aggs[a].val_col < 0 || s->aggs[a].val_col >= s->n_vals))
+      return fail(BLU_E_INVALID, "agg %d: val_col %d out of range", a, s->aggs[a].val_col);
+  }
+  bool sparse = false;
+  for (int k = 0; k < s->n_keys; ++k)
+    if (s->keys[k].dict_size == 0) sparse = true;
+  if (sparse && s->n_keys > 1)
+    return fail(BLU_E_UNSUPPORTED, "a sparse key (dict_size 0) must be the only key column (wide keys: NEXT-2)");
+
+  auto* P = new blu_gby_plan_s();
+  P->keys.assign(s->keys, s->keys + s->n_keys);
+  P->vals.assign(s->vals, s->vals + s->n_vals);
+  P->aggs.assign(s->aggs, s->aggs + s->n_aggs);
+  P->n_rows = n_rows;
+  P->est_groups = std::max<uint64_t>(1, std::min<uint64_t>(est_groups, std::max<uint64_t>(n_rows, 1)));
+
+  Layout& L = P->lay;
+  memset(&L, 0, sizeof L);
+  L.n_keys = s->n_keys;
+  L.sparse = sparse ? 1 : 0;
+  L.count_field = -1;
+  uint64_t D = 1;
+  for (int k = 0; k < s->n_keys; ++k) {
+    L.key_dtype[k] = s->keys[k].dtype;
+    L.dict[k] = s->keys[k].dict_size;
+    L.stride[k] = D;
+    if (!sparse) {
+      uint64_t d = s->keys[k].dict_size;
+      if (s->keys[k].dtype == BLU_I32 && d > (1ull << 31)) {
+        delete P;
+        return fail(BLU_E_INVALID, "key %d: dict_size %llu exceeds the i32 code range", k, (unsigned long long)d);
+      }
+      if (D > ((1ull << 62) / d)) {
+        delete P;
+        return fail(BLU_E_UNSUPPORTED, "dense key domain >= 2^62 (wide keys: NEXT-2)");
+      }
+      D *= d;
+    }
+  }
+  L.domain = sparse ? 0 : D;
+  L.n_vals = s->n_vals;
+  for (int c = 0; c < s->n_vals; ++c) L.val_dtype[c] = s->vals[c];
+
+  P->amap.resize(s->n_aggs);
+  for (int a = 0; a < s->n_aggs; ++a) {
+    int op = s->aggs[a].op, col = s->aggs[a].val_col;
+    AggMap& m = P->amap[a];
+    m.op = op;
+    m.val_col = col;
+    m.field2 = -1;
+    int dt = op == BLU_COUNT ? BLU_I64 : s->vals[col];
+    if (op == BLU_COUNT) {
+      m.field = add_field(L, FK_COUNT, -1, 1);
+      m.out_dtype = BLU_I64;
+    } else if (op == BLU_SUM || op == BLU_AVG) {
+      m.field = add_field(L, dt == BLU_F64 ? FK_SUMF : FK_SUMI, col, 0);
+      if (op == BLU_AVG) m.field2 = add_field(L, FK_COUNT, -1, 1);
+      m.out_dtype = op == BLU_AVG ? BLU_F64 : (dt == BLU_F64 ? BLU_F64 : BLU_I64);
+    } else if (op == BLU_MIN) {
+      m.field = add_field(L, dt == BLU_I32 ? FK_MINI32 : dt == BLU_I64 ? FK_MINI64 : FK_MINF64, col, 0);
+      m.out_dtype = dt;
+    } else {
+      m.field = add_field(L, dt == BLU_I32 ? FK_MAXI32 : dt == BLU_I64 ? FK_MAXI64 : FK_MAXF64, col, 0);
+      m.out_dtype = dt;
+    }
+  }
+  finish_layout(L);
+
+  // ---- moderator: pick the path ---------------------------------------------
+  uint64_t cap_est = std::max<uint64_t>(kMinCap, next_pow2((uint64_t)((double)P->est_groups / kMaxLoad + 0.999999)));
+  uint32_t entry_with_count = L.smem_entry_bytes + (L.count_field < 0 ? 4u : 0u);
+  int path;
+  if (!sparse && D * (uint64_t)entry_with_count <= kSmemDenseMax) path = BLU_PATH_DENSE_SMEM;
+  else if (!sparse && D <= std::max<uint64_t>(2 * cap_est, kDirectMin)) path = BLU_PATH_DIRECT_GLOBAL;
+  else path = BLU_PATH_HASH_GLOBAL;
+  if (const char* fp = env("BLU_GBY_FORCE_PATH")) {
+    int want = fp[0] == 'a' ? BLU_PATH_DENSE_SMEM : fp[0] == 'd' ? BLU_PATH_DIRECT_GLOBAL : BLU_PATH_HASH_GLOBAL;
+    if (want == BLU_PATH_DENSE_SMEM && (sparse || D * (uint64_t)entry_with_count > 200 * 1024)) {
+      delete P;
+      return fail(BLU_E_UNSUPPORTED, "BLU_GBY_FORCE_PATH=a: dense domain does not fit in shared memory");
+    }
+    if (want == BLU_PATH_DIRECT_GLOBAL && sparse) {
+      delete P;
+      return fail(BLU_E_UNSUPPORTED, "BLU_GBY_FORCE_PATH=d: needs dictionary-encoded keys");
+    }
+    path = want;
+  }
+  P->path = path;
+  if (path != BLU_PATH_HASH_GLOBAL && L.count_field < 0) {  // dense occupancy = COUNT > 0
+    add_field(L, FK_COUNT, -1, 1);
+    finish_layout(L);
+  }
+  P->cap = path == BLU_PATH_HASH_GLOBAL ? cap_est : D;
+
+  // hot-key front (path b / b')
+  P->hot_front = 0;
+  P->front_slots = 0;
+  if (path != BLU_PATH_DENSE_SMEM) {
+    bool on = n_rows >= kFrontRatio * P->est_groups;
+    if (const char* hf = env("BLU_GBY_HOT_FRONT")) on = hf[0] == '1';
+    if (on) {
+      uint32_t per = 8 + L.smem_entry_bytes;
+      uint32_t budget = kFrontBudget;
+      uint32_t S = 4096;
+      if (const char* fs = env("BLU_GBY_FRONT_SLOTS")) S = (uint32_t)atoi(fs);
+      while (S > 64 && S * per > budget) S >>= 1;
+      if (S * per <= 200 * 1024) {
+        P->hot_front = 1;
+        P->front_slots = S;
+      }
+    }
+  }
+
+  // shared memory and launch shape
+  P->sms = device_sms();
+  if (path == BLU_PATH_DENSE_SMEM) {
+    uint32_t b = 0;
+    for (int j = 0; j < L.n_fields; ++j) b += (uint32_t)((D * L.f[j].ssize + 15) / 16 * 16);
+    P->smem_bytes = b;
+    P->block = 512;
+  } else if (P->hot_front) {
+    uint32_t b = P->front_slots * 8;
+    for (int j = 0; j < L.n_fields; ++j) b += (P->front_slots * L.f[j].ssize + 15) / 16 * 16;
+    P->smem_bytes = b;
+    P->block = 512;
+  } else {
+    P->smem_bytes = 0;
+    P->block = 256;
+  }
+  if (const char* bs = env("BLU_GBY_BLOCK")) P->block = (uint32_t)atoi(bs);
+  uint32_t per_sm_threads = 2048;
+  uint32_t by_threads = per_sm_threads / P->block;
+  uint32_t by_smem = P->smem_bytes ? std::max<uint32_t>(1, (227 * 1024) / (P->smem_bytes + 1024)) : 32;
+  uint32_t ctas = std::max<uint32_t>(1, std::min(by_threads, by_smem));
+  if (const char* cs = env("BLU_GBY_CTAS_PER_SM")) ctas = (uint32_t)atoi(cs);
+  P->grid = (uint32_t)P->sms * ctas;
+
+  // merge layout: rows are (keys, one column per state field); COUNT becomes SUM of counts.
+  Layout& M = P->merge_lay;
+  M = L;
+  M.n_vals = L.n_fields;
+  for (int j = 0; j < L.n_fields; ++j) {
+    int k = L.f[j].kind;
+    M.val_dtype[j] = (k == FK_MINI32 || k == FK_MAXI32) ? BLU_I32
+                     : (k == FK_SUMF || k == FK_MINF64 || k == FK_MAXF64) ? BLU_F64 : BLU_I64;
+    M.f[j].col = j;
+    if (k == FK_COUNT) M.f[j].kind = FK_SUMI;  // is_count stays 1
+  }
+  finish_layout(M);
+
+  *out_plan = P;
+  return BLU_OK;
+}
+
+blu_status_t blu_gby_plan_info(blu_gby_plan_t P, int32_t* path, uint64_t* capacity, uint32_t* smem_bytes,
+                               uint32_t* retries_last) {
+  if (!P) return fail(BLU_E_INVALID, "NULL plan");
+  if (path) *path = P->path;
+  if (capacity) *capacity = P->cap;
+  if (smem_bytes) *smem_bytes = P->smem_bytes;
+  if (retries_last) *retries_last = P->retries_last.load();
+  return BLU_OK;
+}
+
+blu_status_t blu_gby_plan_info2(blu_gby_plan_t P, uint32_t* slot_bytes, int32_t* hot_front, int32_t* n_states,
+                                int32_t* state_dtypes, uint32_t* grid, uint32_t* block) {
+  if (!P) return fail(BLU_E_INVALID, "NULL plan");
+  if (slot_bytes) *slot_bytes = P->lay.slot_bytes;
+  if (hot_front) *hot_front = P->hot_front;
+  if (n_states) *n_states = P->lay.n_fields;
+  if (state_dtypes)
+    for (int j = 0; j < P->lay.n_fields; ++j) state_dtypes[j] = P->merge_lay.val_dtype[j];
+  if (grid) *grid = P->grid;
+  if (block) *block = P->block;
+  return BLU_OK;
+}
+
+blu_status_t blu_gby_dense_state_shape(blu_gby_plan_t P, int32_t* n_isum, int32_t* n_fsum, int32_t* n_min,
+                                       int32_t* n_max, uint64_t* domain) {
+  if (!P) return fail(BLU_E_INVALID, "NULL plan");
+  if (P->path == BLU_PATH_HASH_GLOBAL) return fail(BLU_E_UNSUPPORTED, "dense state needs path a or b'");
+  if (n_isum) *n_isum = P->lay.n_group[SG_ISUM];
+  if (n_fsum) *n_fsum = P->lay.n_group[SG_FSUM];
+  if (n_min) *n_min = P->lay.n_group[SG_MIN];
+  if (n_max) *n_max = P->lay.n_group[SG_MAX];
+  if (domain) *domain = P->lay.domain;
+  return BLU_OK;
+}
+
+uint32_t blu_gby_record_bytes(blu_gby_plan_t P) { return P ? 8u * (1u + (uint32_t)P->lay.n_fields) : 0u; }
+
+blu_status_t blu_gby_slot_template(blu_gby_plan_t P, void* out, uint32_t cap, uint32_t* slot_bytes) {
+  if (!P) return fail(BLU_E_INVALID, "NULL plan");
+  if (slot_bytes) *slot_bytes = P->lay.slot_bytes;
+  if (out) {
+    if (cap < P->lay.slot_bytes) return fail(BLU_E_INVALID, "template buffer too small (%u < %u)", cap, P->lay.slot_bytes);
+    build_slot_template(P->lay, (uint8_t*)out);
+  }
+  return BLU_OK;
+}
+
+void blu_gby_plan_destroy(blu_gby_plan_t P) { delete P; }
+
+}  // extern "C"

@@ -1,0 +1,70 @@
+"""Multi-GPU GROUP BY over torch.distributed (NCCL over NVLink / NVSwitch; gloo for CPU tests).
+
+One process per GPU; each rank aggregates its contiguous row range (the paper's range
+partitioning, "the input data is partitioned ... sent to some number of available
+GPU devices ... The results are then merged together in the final step"). The merge is chosen by
+the plan's path:
+
+  * dense state (paths a / b'): every rank holds the same D x fields state arrays; four
+    all-reduces (int64 SUM, f64 SUM, int64 MIN, int64 MAX) combine them; every rank finalizes the
+    same replicated result;
+  * hash path (b): each rank emits per-group partial states, buckets them by owner rank
+    (mulhi(fmix64(key), P), bits independent of the slot bits), exchanges them with an
+    all-to-all-v and merges what it owns; the result is distributed by key range.
+
+The collective orchestration (`allreduce_dense_state`, `alltoallv_records`) only moves tensors; all
+GROUP BY arithmetic stays in libblugby.
+"""
+from __future__ import annotations
+
+from typing import List, Sequence
+
+import torch
+import torch.distributed as dist
+
+
+def allreduce_dense_state(state_arrays: Sequence[torch.Tensor], group=None) -> None:
+    """[int64 SUM group, f64 SUM group, int64 MIN group, int64 MAX group] in place."""
+    ops = (dist.ReduceOp.SUM, dist.ReduceOp.SUM, dist.ReduceOp.MIN, dist.ReduceOp.MAX)
+    for t, op in zip(state_arrays, ops):
+        if t.numel():
+            dist.all_reduce(t, op=op, group=group)
+
+
+def alltoallv_records(send: torch.Tensor, send_counts: List[int], words: int, group=None) -> torch.Tensor:
+    """Exchange variable-size buckets of fixed-width records (int64 words). send holds the buckets
+    for ranks 0..P-1 back to back; send_counts[p] records go to rank p. Returns the received records
+    (concatenated in source-rank order) as a 1-D int64 tensor of words."""
+    P = dist.get_world_size(group)
+    dev = send.device
+    sc = torch.tensor(send_counts, dtype=torch.int64, device=dev)
+    rc = torch.empty(P, dtype=torch.int64, device=dev)
+    dist.all_to_all_single(rc, sc, group=group)
+    recv_counts = [int(x) for x in rc.cpu().tolist()]
+    recv = torch.empty(max(1, sum(recv_counts)) * words, dtype=torch.int64, device=dev)
+    dist.all_to_all_single(recv[: sum(recv_counts) * words], send[: sum(send_counts) * words],
+                           output_split_sizes=[c * words for c in recv_counts],
+                           input_split_sizes=[c * words for c in send_counts], group=group)
+    return recv[: sum(recv_counts) * words]
+
+
+def dist_execute(plan, key_cols, val_cols, group=None, stream=None):
+    """Whole-job GROUP BY of this rank's rows; returns (result, mode). Dense paths: replicated
+    finalized result; hash path: this rank's owned groups."""
+    from . import blugby as bg
+    P = dist.get_world_size(group)
+    info = plan.info()
+    if info["path"] != bg.BLU_PATH_HASH_GLOBAL:
+        st = bg.dense_state_arrays(plan, device=key_cols[0].device)
+        bg.blu_gby_execute_dense_state(plan, key_cols, val_cols, st, init=True, stream=stream)
+        if P > 1:
+            allreduce_dense_state(st, group)
+        return bg.blu_gby_finalize_dense_state(plan, st, stream=stream), "allreduce"
+    part = bg.blu_gby_execute_partial(plan, key_cols, val_cols, stream=stream)
+    if P == 1:
+        return bg.blu_gby_merge(plan, [part], stream=stream), "local"
+    words = plan.record_bytes // 8
+    send = torch.empty(max(1, part.n_groups) * words, dtype=torch.int64, device=key_cols[0].device)
+    counts = bg.blu_gby_partition(plan, part, P, send, stream=stream)
+    recv = alltoallv_records(send, counts, words, group)
+    return bg.blu_gby_merge_records(plan, recv, recv.numel() // words, stream=stream), "alltoall"

@@ -1,0 +1,145 @@
+"""Host-side tests of libblugby's C ABI: the library loads, exports every symbol the header declares,
+and the planner (host only, no GPU) makes the documented decisions. No GPU needed."""
+import ctypes
+import json
+import os
+import re
+import struct
+
+import pytest
+
+import blugen
+from blugen import AVG, COUNT, F64, I32, I64, MAX, MIN, SUM
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def bg():
+    from paper_conf_sigmod_merajispcksygnk16_b200 import blugby
+    return blugby
+
+
+def test_library_exports_every_header_symbol(bg):
+    hdr = open(os.path.join(ROOT, "include", "blu_gby.h")).read()
+    names = set(re.findall(r"\b(blu_gby_[a-z_0-9]+)\s*\(", hdr))
+    assert len(names) >= 20
+    lib = ctypes.CDLL(bg.LIB_PATH)
+    missing = [n for n in sorted(names) if not hasattr(lib, n)]
+    assert not missing, missing
+
+
+def test_generator_library_exports():
+    hdr = open(os.path.join(ROOT, "include", "blu_gen.h")).read()
+    names = set(re.findall(r"^(?:int|void)\s+(blu_gen_[a-z_0-9]+)\s*\(", hdr, re.M))
+    lib = ctypes.CDLL(blugen.LIB_PATH)
+    assert names and all(hasattr(lib, n) for n in names)
+
+
+def test_status_strings(bg):
+    for s, name in bg.STATUS_NAMES.items():
+        assert bg.lib.blu_gby_status_str(s).decode() == name
+
+
+def test_table1_mask_matches_paper(bg):
+    """S4 template == PAPER.md Table 1: SUM(C1), MAX(C2), MIN(C3) group by C1."""
+    g = json.load(open(os.path.join(ROOT, "tests", "golden", "table1_mask.json")))
+    dt = {"i32": I32, "i64": I64, "f64": F64}
+    ops = {"COUNT": COUNT, "SUM": SUM, "MIN": MIN, "MAX": MAX, "AVG": AVG}
+    keys = [(dt[d], n) for d, n in g["schema"]["keys"]]
+    vals = [dt[d] for d in g["schema"]["vals"]]
+    aggs = [(ops[o], c) for o, c in g["schema"]["aggs"]]
+    plan = bg.blu_gby_plan(keys, vals, aggs, est_groups=1000, n_rows=10**6)
+    assert plan.info()["path"] == bg.BLU_PATH_HASH_GLOBAL
+    t = plan.slot_template()
+    assert len(t) == g["row_bytes"] == 32
+    for f in g["fields"]:
+        raw = t[f["offset"]:f["offset"] + f["bytes"]]
+        if "value_hex" in f:
+            assert raw.hex().upper() == f["value_hex"]
+        else:
+            fmt = "<q" if f["bytes"] == 8 else "<i"
+            assert struct.unpack(fmt, raw)[0] == f["value"], f["name"]
+
+
+def _plan(bg, w, **kw):
+    est = kw.pop("est", w.est_groups)
+    return bg.plan_for(w.schema, est, kw.pop("n_rows", w.n_rows))
+
+
+def test_planner_paths_for_the_five_configs(bg):
+    """The moderator: small dense domain -> (a); dense 1e5 domain with a high
+    rows/groups ratio -> direct-mapped (b') + hot-key front; sparse keys -> hash (b)."""
+    c1 = _plan(bg, blugen.workload("C1")).info()
+    c2 = _plan(bg, blugen.workload("C2")).info()
+    c3 = _plan(bg, blugen.workload("C3")).info()
+    c4 = _plan(bg, blugen.workload("C4")).info()
+    c5 = _plan(bg, blugen.workload("C5")).info()
+    assert c1["path"] == c2["path"] == bg.BLU_PATH_DENSE_SMEM
+    assert c1["capacity"] == 16 and c2["capacity"] == 1024
+    assert c3["path"] == bg.BLU_PATH_HASH_GLOBAL and c3["capacity"] == 2**24 and c3["slot_bytes"] == 32
+    assert c3["hot_front"] == 0
+    assert c4["path"] == bg.BLU_PATH_DIRECT_GLOBAL and c4["capacity"] == 100_000 and c4["hot_front"] == 1
+    assert c5["path"] == bg.BLU_PATH_HASH_GLOBAL and c5["capacity"] == 2**27
+
+
+@pytest.mark.parametrize("est,cap", [(1, 1024), (700, 1024), (716, 1024), (717, 2048), (10_000_000, 2**24),
+                                     (50_000_000, 2**27)])
+def test_capacity_rounding(bg, est, cap):
+    """cap = next_pow2(ceil(max(est,1)/0.7)), >= 1024 ("slightly larger", reading A5)."""
+    p = bg.blu_gby_plan([(I64, 0)], [I64], [(SUM, 0)], est, 10**10)
+    assert p.info()["capacity"] == cap
+
+
+def test_est_clamped_to_rows(bg):
+    p = bg.blu_gby_plan([(I64, 0)], [I64], [(SUM, 0)], 10**9, 5000)
+    assert p.info()["capacity"] == 8192
+
+
+def test_state_fields_and_slot_sizes(bg):
+    p = bg.plan_for(blugen.workload("C3").schema, 10**7, 10**9)
+    i = p.info()
+    # COUNT, SUM(v0) i64, SUM(v1) f64 (AVG shares COUNT + SUM): key 8 + 3 x 8 = 32 B
+    assert i["n_states"] == 3 and i["state_dtypes"] == [I64, I64, F64] and i["slot_bytes"] == 32
+    p4 = bg.plan_for(blugen.workload("C4").schema, 10**5, 10**9)
+    i4 = p4.info()
+    # COUNT, SUM v0, SUM v1 (+AVG v1), SUM v2, MIN v2, MAX v2
+    assert i4["n_states"] == 6 and i4["slot_bytes"] == 64
+    assert p4.dense_state_shape() == (4, 0, 1, 1, 100_000)
+
+
+def test_schema_validation(bg):
+    with pytest.raises(bg.BluError) as e:
+        bg.blu_gby_plan([], [I64], [(SUM, 0)], 1, 1)
+    assert e.value.status == bg.BLU_E_INVALID
+    with pytest.raises(bg.BluError) as e:
+        bg.blu_gby_plan([(I32, 4)], [I64], [(SUM, 3)], 1, 1)
+    assert e.value.status == bg.BLU_E_INVALID
+    with pytest.raises(bg.BluError) as e:
+        bg.blu_gby_plan([(F64, 4)], [I64], [(SUM, 0)], 1, 1)
+    assert e.value.status == bg.BLU_E_INVALID
+    with pytest.raises(bg.BluError) as e:  # sparse key with another key column: NEXT-2
+        bg.blu_gby_plan([(I64, 0), (I32, 4)], [I64], [(SUM, 0)], 1, 1)
+    assert e.value.status == bg.BLU_E_UNSUPPORTED
+    with pytest.raises(bg.BluError) as e:  # dense domain >= 2^62
+        bg.blu_gby_plan([(I64, 2**40), (I64, 2**30)], [I64], [(SUM, 0)], 1, 1)
+    assert e.value.status == bg.BLU_E_UNSUPPORTED
+    with pytest.raises(bg.BluError) as e:
+        bg.blu_gby_plan([(I32, 4)], [I64], [(7, 0)], 1, 1)
+    assert e.value.status == bg.BLU_E_INVALID
+
+
+def test_forced_path_env(bg, monkeypatch):
+    w = blugen.workload("C2")
+    monkeypatch.setenv("BLU_GBY_FORCE_PATH", "b")
+    assert _plan(bg, w).info()["path"] == bg.BLU_PATH_HASH_GLOBAL
+    monkeypatch.setenv("BLU_GBY_FORCE_PATH", "d")
+    assert _plan(bg, w).info()["path"] == bg.BLU_PATH_DIRECT_GLOBAL
+    monkeypatch.setenv("BLU_GBY_FORCE_PATH", "a")
+    with pytest.raises(bg.BluError):
+        _plan(bg, blugen.workload("C3"))
+
+
+def test_record_bytes(bg):
+    p = bg.plan_for(blugen.workload("C3").schema, 10**7, 10**9)
+    assert p.record_bytes == 8 * (1 + 3)

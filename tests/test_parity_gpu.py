@@ -1,0 +1,315 @@
+"""GPU parity: libblugby (through its C ABI) vs the CPU oracle on the same seeded inputs.
+
+Sizes span many tiles and CTAs with ragged tails; configs C1..C5 are scaled down so the oracle
+finishes in seconds (full-size checks live in test_fullsize_gpu.py). Integers, keys and the dyadic
+f64 columns are compared bit-exactly (north_star; readings A12/A13)."""
+import os
+
+import numpy as np
+import pytest
+
+import blugen
+import oracle
+from blugen import AVG, COUNT, F64, I32, I64, MAX, MIN, REAL, SUM
+from parity_util import assert_parity, gpu_sorted, host_sorted
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def bg():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sigmod_merajispcksygnk16_b200 import blugby
+    return blugby
+
+
+SCALED = {
+    "C1": dict(n_rows=1_000_003),
+    "C2": dict(n_rows=2_000_011),
+    "C3": dict(n_rows=2_000_003, n_groups=60_000),
+    "C4": dict(n_rows=3_000_017),
+    "C5": dict(n_rows=2_500_001, n_groups=150_000),
+}
+
+
+def run_gpu(bg, w, est=None, **env):
+    kc, vc = blugen.device_columns(w)
+    plan = bg.plan_for(w.schema, w.est_groups if est is None else est, w.n_rows)
+    res = bg.blu_gby_execute(plan, kc, vc)
+    return plan, res
+
+
+@pytest.fixture(scope="module")
+def oracles():
+    cache = {}
+
+    def get(name):
+        if name not in cache:
+            w = blugen.workload(name, **SCALED[name])
+            cache[name] = (w, oracle.groupby_generated(w))
+        return cache[name]
+    return get
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C4", "C5"])
+def test_config_parity(bg, oracles, name):
+    w, o = oracles(name)
+    plan, res = run_gpu(bg, w)
+    assert res.n_groups == o.n_groups
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
+@pytest.mark.parametrize("name,paths", [("C1", "abd"), ("C2", "abd"), ("C4", "bd"), ("C3", "b")])
+@pytest.mark.parametrize("front", ["0", "1"])
+def test_forced_paths_identical(bg, oracles, monkeypatch, name, paths, front):
+    """Forced path (a) vs (b) vs (b'), hot-key front on/off: all equal the oracle."""
+    w, o = oracles(name)
+    kc, vc = blugen.device_columns(w)
+    monkeypatch.setenv("BLU_GBY_HOT_FRONT", front)
+    for p in paths:
+        monkeypatch.setenv("BLU_GBY_FORCE_PATH", p)
+        plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+        res = bg.blu_gby_execute(plan, kc, vc)
+        gk, ga = gpu_sorted(res, w.schema)
+        assert_parity(gk, ga, o, w.schema)
+
+
+@pytest.mark.parametrize("est", [1, 1000, 60_000, 2_000_003])
+def test_est_groups_invariance_and_regrow(bg, oracles, est):
+    """Under-estimates take the error path: regrow and rerun, same exact result."""
+    w, o = oracles("C3")
+    plan, res = run_gpu(bg, w, est=est)
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+    if est == 1:
+        assert plan.info()["retries_last"] >= 1
+
+
+def _mk(keys_np, vals_np):
+    return [torch.from_numpy(k).cuda() for k in keys_np], [torch.from_numpy(v).cuda() for v in vals_np]
+
+
+ALL = lambda nv: [(COUNT, -1)] + [(op, c) for c in range(nv) for op in (SUM, MIN, MAX, AVG)]
+
+
+@pytest.mark.parametrize("n", [0, 1, 3, 31, 33, 4095, 4097, 65_537])
+@pytest.mark.parametrize("path", ["a", "b", "d"])
+def test_small_and_ragged(bg, monkeypatch, n, path):
+    rng = np.random.default_rng(n + 7)
+    sch = blugen.Schema([(I32, 13), (I64, 7)], [I32, I64, F64], ALL(3))
+    kc = [rng.integers(0, 13, n).astype(np.int32), rng.integers(0, 7, n).astype(np.int64)]
+    vc = [rng.integers(-(2**31), 2**31, n).astype(np.int32), rng.integers(-(2**62), 2**62, n).astype(np.int64),
+          rng.integers(-(2**20), 2**20, n) / 64.0]
+    o = oracle.groupby_arrays(sch, kc, vc)
+    monkeypatch.setenv("BLU_GBY_FORCE_PATH", path)
+    plan = bg.plan_for(sch, 91, n)
+    dk, dv = _mk(kc, vc)
+    res = bg.blu_gby_execute(plan, dk, dv, n_rows=n)
+    gk, ga = gpu_sorted(res, sch)
+    assert_parity(gk, ga, o, sch)
+
+
+def test_single_group_and_all_distinct(bg):
+    n = 300_001
+    rng = np.random.default_rng(1)
+    sch = blugen.Schema([(I64, 0)], [I64, F64, I32], ALL(3))
+    v = [rng.integers(-(2**40), 2**40, n), rng.integers(-(2**20), 2**20, n) / 64.0,
+         rng.integers(-(2**31), 2**31, n).astype(np.int32)]
+    for kc in ([np.full(n, 12345, np.int64)], [rng.permutation(10**7)[:n].astype(np.int64)]):
+        o = oracle.groupby_arrays(sch, kc, v)
+        dk, dv = _mk(kc, v)
+        plan = bg.plan_for(sch, 1 if kc[0][0] == kc[0][1] else n, n)
+        res = bg.blu_gby_execute(plan, dk, dv)
+        gk, ga = gpu_sorted(res, sch)
+        assert_parity(gk, ga, o, sch)
+
+
+def test_key_range_errors(bg):
+    sch = blugen.Schema([(I32, 10)], [I64], [(SUM, 0)])
+    plan = bg.plan_for(sch, 10, 1000)
+    k = torch.arange(1000, dtype=torch.int32, device="cuda") % 10
+    v = torch.ones(1000, dtype=torch.int64, device="cuda")
+    for bad in (10, -1):
+        k2 = k.clone()
+        k2[777] = bad
+        with pytest.raises(bg.BluError) as e:
+            bg.blu_gby_execute(plan, [k2], [v])
+        assert e.value.status == bg.BLU_E_KEY_RANGE
+    sp = bg.plan_for(blugen.Schema([(I64, 0)], [I64], [(SUM, 0)]), 10, 1000)
+    ks = torch.arange(1000, dtype=torch.int64, device="cuda")
+    ks[5] = -3
+    with pytest.raises(bg.BluError) as e:
+        bg.blu_gby_execute(sp, [ks], [v])
+    assert e.value.status == bg.BLU_E_KEY_RANGE
+    # the valid maximum code dict_size - 1 is accepted
+    k3 = k.clone()
+    k3[:] = 9
+    r = bg.blu_gby_execute(plan, [k3], [v])
+    assert r.n_groups == 1 and int(r.aggs[0][0]) == 1000
+
+
+def test_general_f64_within_tolerance(bg):
+    """Non-dyadic doubles: SUM/AVG within 1e-12 * sum|v| of the oracle (reading A13)."""
+    n = 1_000_003
+    w = blugen.Workload("real", n, 77, [blugen.Col(I32, blugen.UNIFORM, 0, 0, 500)],
+                        [blugen.Col(F64, REAL, 1, lo=10**6)],
+                        blugen.Schema([(I32, 500)], [F64], [(COUNT, -1), (SUM, 0), (AVG, 0), (MIN, 0), (MAX, 0)]),
+                        500, 500)
+    o = oracle.groupby_generated(w)
+    for p in "ab":
+        os.environ["BLU_GBY_FORCE_PATH"] = p
+        try:
+            plan, res = run_gpu(bg, w)
+        finally:
+            del os.environ["BLU_GBY_FORCE_PATH"]
+        gk, ga = gpu_sorted(res, w.schema)
+        assert_parity(gk, ga, o, w.schema, f64_tol=1e-12)
+
+
+def test_misaligned_columns_scalar_path(bg, oracles):
+    w, _ = oracles("C2")
+    kc, vc = blugen.device_columns(w)
+    # drop the first row: every column pointer is 4 or 8 bytes past a 16-byte boundary
+    kc1, vc1 = [k[1:] for k in kc], [v[1:] for v in vc]
+    hk, hv = blugen.host_columns(w)
+    o = oracle.groupby_arrays(w.schema, [k[1:] for k in hk], [v[1:] for v in hv])
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows - 1)
+    res = bg.blu_gby_execute(plan, kc1, vc1)
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
+@pytest.mark.parametrize("name", ["C2", "C3", "C4"])
+def test_partial_merge_equals_full(bg, oracles, name):
+    """S9: execute_partial on 3 row shards, then merge (P:68 range partitions merged at the end)."""
+    w, o = oracles(name)
+    kc, vc = blugen.device_columns(w)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    cuts = [0, w.n_rows // 3 + 1, 2 * w.n_rows // 3 + 5, w.n_rows]
+    parts = [bg.blu_gby_execute_partial(plan, [k[a:b] for k in kc], [v[a:b] for v in vc])
+             for a, b in zip(cuts[:-1], cuts[1:])]
+    res = bg.blu_gby_merge(plan, parts)
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+    # merge_partial then merge again is still exact
+    mp = bg.blu_gby_merge_partial(plan, parts[:2])
+    res2 = bg.blu_gby_merge(plan, [mp, parts[2]])
+    gk, ga = gpu_sorted(res2, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
+@pytest.mark.parametrize("name", ["C3", "C2"])
+def test_partition_records_exchange(bg, oracles, name):
+    """S10 simulated on one GPU: each of P 'ranks' partitions its partial by owner; each owner merges
+    the records it would receive. The union of owners' results equals the full result."""
+    w, o = oracles(name)
+    kc, vc = blugen.device_columns(w)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    P = 4
+    cuts = np.linspace(0, w.n_rows, P + 1).astype(int)
+    rb = plan.record_bytes
+    inbox = [[] for _ in range(P)]
+    for r in range(P):
+        part = bg.blu_gby_execute_partial(plan, [k[cuts[r]:cuts[r + 1]] for k in kc],
+                                          [v[cuts[r]:cuts[r + 1]] for v in vc])
+        buf = torch.empty(max(1, part.n_groups) * rb // 8, dtype=torch.int64, device="cuda")
+        counts = bg.blu_gby_partition(plan, part, P, buf)
+        assert sum(counts) == part.n_groups
+        off = 0
+        for dst in range(P):
+            inbox[dst].append(buf[off * rb // 8:(off + counts[dst]) * rb // 8])
+            off += counts[dst]
+    keys, aggs = [], []
+    for dst in range(P):
+        recs = torch.cat(inbox[dst])
+        res = bg.blu_gby_merge_records(plan, recs, recs.numel() * 8 // rb)
+        gk, ga = gpu_sorted(res, w.schema)
+        keys.append(gk)
+        aggs.append(ga)
+    allk = np.concatenate(keys)
+    order = np.lexsort(allk.T[::-1])
+    assert_parity(allk[order], [np.concatenate([a[i] for a in aggs])[order] for i in range(len(w.schema.aggs))],
+                  o, w.schema)
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C4"])
+def test_dense_state_accumulate_and_finalize(bg, oracles, name):
+    """Path (a)/(b') multi-GPU helpers on one GPU: 3 shards accumulate into one dense state."""
+    w, o = oracles(name)
+    kc, vc = blugen.device_columns(w)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    st = bg.dense_state_arrays(plan)
+    cuts = [0, 1000, w.n_rows // 2, w.n_rows]
+    for i, (a, b) in enumerate(zip(cuts[:-1], cuts[1:])):
+        bg.blu_gby_execute_dense_state(plan, [k[a:b] for k in kc], [v[a:b] for v in vc], st, init=(i == 0))
+    res = bg.blu_gby_finalize_dense_state(plan, st)
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
+@pytest.mark.parametrize("name", ["C1", "C3"])
+def test_execute_host_columns(bg, oracles, name):
+    """Host columns in (chunked H2D overlapped with aggregation), host result out."""
+    w, o = oracles(name)
+    hk, hv = blugen.host_columns(w)
+    hk = [torch.from_numpy(k).pin_memory() for k in hk]
+    hv = [torch.from_numpy(v).pin_memory() for v in hv]
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    res = bg.blu_gby_execute_host(plan, hk, hv)
+    gk, ga = host_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
+def test_init_table_matches_table1(bg):
+    """S4 on the device: every slot equals the Table 1 mask."""
+    plan = bg.blu_gby_plan([(I64, 0)], [I64, I64, I32], [(SUM, 0), (MAX, 1), (MIN, 2)], 1000, 10**6)
+    t = plan.slot_template()
+    n = 4099
+    buf = torch.zeros(n * len(t), dtype=torch.uint8, device="cuda")
+    bg.blu_gby_init_table(plan, buf, n)
+    torch.cuda.synchronize()
+    got = buf.cpu().numpy().reshape(n, len(t))
+    want = np.frombuffer(t, np.uint8)
+    assert np.all(got == want[None, :])
+    assert t[:8] == b"\xff" * 8 and int.from_bytes(t[16:24], "little", signed=True) == -(2**63)
+    assert int.from_bytes(t[24:28], "little", signed=True) == 2**31 - 1
+
+
+def test_cross_check_against_torch_library(bg):
+    """Second reference independent of both libblugby and the oracle: torch.unique + scatter_reduce."""
+    w = blugen.workload("C2", n_rows=20_000_000)
+    kc, vc = blugen.device_columns(w)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    res = bg.blu_gby_execute(plan, kc, vc)
+    packed = kc[0].long() + 32 * kc[1].long()
+    uq, inv, cnt = torch.unique(packed, return_inverse=True, return_counts=True)
+    G = uq.numel()
+    s0 = torch.zeros(G, dtype=torch.int64, device="cuda").scatter_add_(0, inv, vc[0].long())
+    mn = torch.full((G,), 2**62, dtype=torch.int64, device="cuda").scatter_reduce_(0, inv, vc[1], "amin")
+    mx = torch.full((G,), -(2**62), dtype=torch.int64, device="cuda").scatter_reduce_(0, inv, vc[2], "amax")
+    s3 = torch.zeros(G, dtype=torch.float64, device="cuda").scatter_add_(0, inv, vc[3])
+    gp = res.keys[0].long() + 32 * res.keys[1].long()
+    order = torch.argsort(gp)
+    assert res.n_groups == G and torch.equal(gp[order], uq)
+    assert torch.equal(res.aggs[0][order], cnt)
+    assert torch.equal(res.aggs[1][order], s0)
+    assert torch.equal(res.aggs[2][order], mn) and torch.equal(res.aggs[3][order], mx)
+    assert torch.equal(res.aggs[4][order], s3 / cnt.double())
+
+
+def test_launch_count_and_timing(bg):
+    w = blugen.workload("C1", n_rows=100_000)
+    kc, vc = blugen.device_columns(w)
+    plan = bg.plan_for(w.schema, 16, w.n_rows)
+    bg.blu_gby_set_timing(True)
+    c0 = bg.blu_gby_launch_count()
+    bg.blu_gby_execute(plan, kc, vc)
+    c1 = bg.blu_gby_launch_count()
+    t = bg.blu_gby_last_timing()
+    bg.blu_gby_set_timing(False)
+    assert c1 - c0 >= 4  # init, aggregate, compact x3
+    assert t["aggregate_ms"] > 0 and t["aggregate_launches"] == 1
