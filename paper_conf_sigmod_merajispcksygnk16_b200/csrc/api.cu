@@ -55,6 +55,11 @@ static void setup_pool() {
       uint64_t thr = UINT64_MAX;
       cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
     }
+    // L2 fetch granularity for the random slot traffic of path (b) (a hint; 0 keeps the default)
+    if (const char* g = getenv("BLU_GBY_L2_FETCH")) {
+      int v = atoi(g);
+      if (v > 0) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)v);
+    }
     cudaGetLastError();
   });
 }
@@ -208,6 +213,7 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     for (int g = 0; g < 4; ++g) base.dense[g] = dense_g[g];
     base.front_slots = front ? P->front_slots : 0;
     base.flags = d_flags;
+    fill_smem_layout(base, path == BLU_PATH_DENSE_SMEM ? (uint32_t)D : base.front_slots, base.front_slots > 0);
     uint32_t launches = 0;
     CK(feed(base, &launches), "aggregate launch");
     if (t_timing) cudaEventRecord(t_ev.e[2], st);
@@ -566,6 +572,7 @@ blu_status_t blu_gby_execute_dense_state(blu_gby_plan_t P, const void* const* ke
   for (int g = 0; g < 4; ++g) base.dense[g] = dg[g];
   base.front_slots = P->hot_front ? P->front_slots : 0;
   base.flags = (uint32_t*)small;
+  fill_smem_layout(base, P->path == BLU_PATH_DENSE_SMEM ? (uint32_t)L.domain : base.front_slots, base.front_slots > 0);
   CK(agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, nullptr), "aggregate");
   uint64_t* hs = pinned_scratch();
   uint64_t hb[2] = {0, 0};

@@ -114,7 +114,16 @@ struct AggParams {
   void* dense[4];        // paths a / b': dense state groups (SG_*), each n_group[g] x D int64
   uint32_t front_slots;  // shared-memory front entries (power of two) or 0
   uint32_t* flags;       // bit 0: overflow (probe bound), bit 1: key out of range
+  // shared-memory table layout (path a: S = D; front: S = front_slots), filled by the host
+  uint32_t S;
+  uint32_t key_off;              // front keys (S x u64)
+  uint32_t soff[kMaxFields];     // per field: byte offset of its SoA array
+  uint32_t colmask[kMaxFields];  // per kernel value column: bit j = field j reads it
+  uint32_t cntmask;              // fields that count the constant 1
 };
+
+// Fill S / key_off / soff / colmask / cntmask of p for a shared-memory table of S entries.
+void fill_smem_layout(AggParams& p, uint32_t S, bool with_keys);
 
 enum : uint32_t { FLAG_OVERFLOW = 1u, FLAG_KEY_RANGE = 2u };
 

@@ -71,41 +71,97 @@ __device__ __forceinline__ uint64_t ld_stream_u64(const void* p, uint64_t pol) {
   return r;
 }
 
-// Load rows [row, row+R) of one column as 64-bit patterns (i32 sign-extended). Rows >= n read 0.
-template <int R>
-__device__ __forceinline__ void load_rows(const void* base, int dt, uint64_t row, uint64_t n, bool vec,
-                                          uint64_t pol, uint64_t (&out)[R]) {
-  if (dt == BLU_I32) {
-    const int32_t* p = (const int32_t*)base + row;
-    if (R == 4 && vec && row + 4 <= n) {
-      int4 v = ld_stream_v4(p, pol);
-      out[0] = (uint64_t)(int64_t)v.x;
-      if (R > 1) out[1 % R] = (uint64_t)(int64_t)v.y;
-      if (R > 2) out[2 % R] = (uint64_t)(int64_t)v.z;
-      if (R > 3) out[3 % R] = (uint64_t)(int64_t)v.w;
-    } else {
-#pragma unroll
-      for (int r = 0; r < R; ++r) out[r] = row + r < n ? (uint64_t)(int64_t)ld_stream_s32(p + r, pol) : 0ull;
-    }
-  } else {
-    const uint64_t* p = (const uint64_t*)base + row;
-    if (R % 2 == 0 && vec && row + R <= n) {
-#pragma unroll
-      for (int r = 0; r < R; r += 2) {
-        int4 v = ld_stream_v4(p + r, pol);
-        out[r] = (uint64_t)(uint32_t)v.x | ((uint64_t)(uint32_t)v.y << 32);
-        out[(r + 1) % R] = (uint64_t)(uint32_t)v.z | ((uint64_t)(uint32_t)v.w << 32);
-      }
-    } else {
-#pragma unroll
-      for (int r = 0; r < R; ++r) out[r] = row + r < n ? ld_stream_u64(p + r, pol) : 0ull;
-    }
-  }
+// Row mapping: a warp owns 32*R consecutive rows; lane l owns rows lb + (r>>1)*64 + (r&1) for
+// R = 4 (pairs 2l, 2l+1 and 64+2l, 65+2l), lb + r for R = 2, lb for R = 1, with lb the lane base
+// below. Every load instruction of a warp then covers one contiguous span (256 B for i32 pairs,
+// 512 B for 8-byte pairs): whole 32-byte sectors, no half-sector re-requests.
+template <int R, bool PAIR = true>
+__device__ __forceinline__ uint64_t lane_base(uint64_t tile_row0, unsigned warp, unsigned lane) {
+  if (!PAIR) return tile_row0 + ((uint64_t)warp * 32 + lane) * R;  // quad: R consecutive rows
+  return tile_row0 + (uint64_t)warp * 32 * R + (R >= 2 ? 2 * lane : lane);
+}
+template <int R, bool PAIR = true>
+__device__ __forceinline__ uint64_t row_of(uint64_t lb, int r) {
+  if (!PAIR) return lb + r;
+  return R == 4 ? lb + (uint64_t)(r >> 1) * 64 + (r & 1) : lb + r;
 }
 
-// Encoded value of a row for field kind k: f64 MIN/MAX through ord_f64; everything else as is.
-__device__ __forceinline__ uint64_t encode(int k, uint64_t raw) {
-  return (k == FK_MINF64 || k == FK_MAXF64) ? (uint64_t)ord_f64(raw) : raw;
+__device__ __forceinline__ int2 ld_stream_v2(const void* p, uint64_t pol) {
+  int2 r;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.s32 {%0,%1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(p), "l"(pol));
+  return r;
+}
+
+// Load this lane's R rows of one column as 64-bit patterns (i32 sign-extended). Rows >= n read 0.
+template <int R, bool PAIR = true>
+__device__ __forceinline__ void load_rows(const void* base, int dt, uint64_t lb, uint64_t n, bool vec,
+                                          uint64_t pol, uint64_t (&out)[R]) {
+  if (!PAIR && R == 4) {  // quad mapping: rows lb..lb+3 (path (a): one 16-byte load per i32 column)
+    if (dt == BLU_I32) {
+      const int32_t* p = (const int32_t*)base + lb;
+      if (vec && lb + 4 <= n) {
+        int4 v = ld_stream_v4(p, pol);
+        out[0] = (uint64_t)(int64_t)v.x;
+        out[1 % R] = (uint64_t)(int64_t)v.y;
+        out[2 % R] = (uint64_t)(int64_t)v.z;
+        out[3 % R] = (uint64_t)(int64_t)v.w;
+      } else {
+#pragma unroll
+        for (int r = 0; r < R; ++r) out[r] = lb + r < n ? (uint64_t)(int64_t)ld_stream_s32(p + r, pol) : 0ull;
+      }
+    } else {
+      const uint64_t* p = (const uint64_t*)base + lb;
+      if (vec && lb + 4 <= n) {
+#pragma unroll
+        for (int r = 0; r < R; r += 2) {
+          int4 v = ld_stream_v4(p + r, pol);
+          out[r] = (uint64_t)(uint32_t)v.x | ((uint64_t)(uint32_t)v.y << 32);
+          out[(r + 1) % R] = (uint64_t)(uint32_t)v.z | ((uint64_t)(uint32_t)v.w << 32);
+        }
+      } else {
+#pragma unroll
+        for (int r = 0; r < R; ++r) out[r] = lb + r < n ? ld_stream_u64(p + r, pol) : 0ull;
+      }
+    }
+    return;
+  }
+  if (dt == BLU_I32) {
+    const int32_t* p = (const int32_t*)base;
+    if (R >= 2) {
+#pragma unroll
+      for (int h = 0; h < R / 2; ++h) {
+        const uint64_t r0 = lb + (uint64_t)h * 64;
+        if (vec && r0 + 1 < n) {
+          int2 v = ld_stream_v2(p + r0, pol);
+          out[2 * h] = (uint64_t)(int64_t)v.x;
+          out[(2 * h + 1) % R] = (uint64_t)(int64_t)v.y;
+        } else {
+          out[2 * h] = r0 < n ? (uint64_t)(int64_t)ld_stream_s32(p + r0, pol) : 0ull;
+          out[(2 * h + 1) % R] = r0 + 1 < n ? (uint64_t)(int64_t)ld_stream_s32(p + r0 + 1, pol) : 0ull;
+        }
+      }
+    } else {
+      out[0] = lb < n ? (uint64_t)(int64_t)ld_stream_s32(p + lb, pol) : 0ull;
+    }
+  } else {
+    const uint64_t* p = (const uint64_t*)base;
+    if (R >= 2) {
+#pragma unroll
+      for (int h = 0; h < R / 2; ++h) {
+        const uint64_t r0 = lb + (uint64_t)h * 64;
+        if (vec && r0 + 1 < n) {
+          int4 v = ld_stream_v4(p + r0, pol);
+          out[2 * h] = (uint64_t)(uint32_t)v.x | ((uint64_t)(uint32_t)v.y << 32);
+          out[(2 * h + 1) % R] = (uint64_t)(uint32_t)v.z | ((uint64_t)(uint32_t)v.w << 32);
+        } else {
+          out[2 * h] = r0 < n ? ld_stream_u64(p + r0, pol) : 0ull;
+          out[(2 * h + 1) % R] = r0 + 1 < n ? ld_stream_u64(p + r0 + 1, pol) : 0ull;
+        }
+      }
+    } else {
+      out[0] = lb < n ? ld_stream_u64(p + lb, pol) : 0ull;
+    }
+  }
 }
 
 // Identity (the mask value of P:151) of a field in its encoded 64-bit form.
@@ -119,49 +175,69 @@ __device__ __forceinline__ uint64_t identity64(int k) {
   }
 }
 
-// ---- shared-memory table (path (a) and the hot-key front). SoA per field; S entries. ----------
-// Field encodings: COUNT u32; SUMI as two u32 arrays lo[S], hi[S] (32-bit native atomics with an
-// explicit carry: 64-bit shared atomics are CAS loops on sm_100a); SUMF f64;
-// MIN/MAX i32 as i32 (native ATOMS.MIN/MAX); 64-bit MIN/MAX read-before-atomic.
-__device__ __forceinline__ void smem_apply(uint8_t* base, int k, uint32_t e, uint32_t S, uint64_t x) {
-  switch (k) {
-    case FK_COUNT:
-      atomicAdd((uint32_t*)base + e, (uint32_t)x);
-      break;
-    case FK_SUMI: {
-      uint32_t lo = (uint32_t)x, hi = (uint32_t)(x >> 32);
-      uint32_t old = atomicAdd((uint32_t*)base + e, lo);
-      hi += (uint32_t)(old + lo < old);
-      if (hi) atomicAdd((uint32_t*)base + S + e, hi);
-      break;
-    }
-    case FK_SUMF:
-      atomicAdd((double*)base + e, __longlong_as_double((long long)x));
-      break;
-    case FK_MINI32: {
-      int v = (int)x;
-      int* q = (int*)base + e;
-      if (v < *(volatile int*)q) atomicMin(q, v);
-      break;
-    }
-    case FK_MAXI32: {
-      int v = (int)x;
-      int* q = (int*)base + e;
-      if (v > *(volatile int*)q) atomicMax(q, v);
-      break;
-    }
-    case FK_MINI64: case FK_MINF64: {
-      long long v = (long long)x;
-      long long* q = (long long*)base + e;
-      if (v < *(volatile long long*)q) atomicMin(q, v);
-      break;
-    }
-    default: {  // FK_MAXI64, FK_MAXF64
-      long long v = (long long)x;
-      long long* q = (long long*)base + e;
-      if (v > *(volatile long long*)q) atomicMax(q, v);
-      break;
-    }
+// ---- per-field update primitives, specialised on the field kind at compile time ----------------
+// The kind of every field is warp-uniform, so kernels dispatch ONCE per field per tile (a uniform
+// switch) and then run straight-line updates for all R rows of the tile.
+template <int K>
+struct KC {
+  static constexpr int v = K;
+};
+
+template <class Fn>
+__device__ __forceinline__ void dispatch_kind(int kind, Fn&& fn) {
+  switch (kind) {
+    case FK_COUNT: fn(KC<FK_COUNT>{}); break;
+    case FK_SUMI: fn(KC<FK_SUMI>{}); break;
+    case FK_SUMF: fn(KC<FK_SUMF>{}); break;
+    case FK_MINI32: fn(KC<FK_MINI32>{}); break;
+    case FK_MAXI32: fn(KC<FK_MAXI32>{}); break;
+    case FK_MINI64: fn(KC<FK_MINI64>{}); break;
+    case FK_MAXI64: fn(KC<FK_MAXI64>{}); break;
+    case FK_MINF64: fn(KC<FK_MINF64>{}); break;
+    default: fn(KC<FK_MAXF64>{}); break;
+  }
+}
+
+// Encoded value of a field: f64 MIN/MAX through ord_f64 (RAW row values only).
+template <int K, bool RAW>
+__device__ __forceinline__ uint64_t enc(uint64_t x) {
+  if (RAW && (K == FK_MINF64 || K == FK_MAXF64)) return (uint64_t)ord_f64(x);
+  return x;
+}
+
+// Shared-memory table (path (a) and the hot-key front): SoA per field, S entries per field.
+// Encodings: COUNT u32; SUMI as two u32 arrays lo[S], hi[S] — native 32-bit ATOMS with an explicit
+// carry (64-bit shared atomics are CAS loops on sm_100a); SUMF f64 (CAS loop);
+// MIN/MAX i32 native ATOMS.MIN/MAX; 64-bit MIN/MAX read first, atomic only if it improves (after
+// warm-up a running min/max almost never changes, so almost every row costs one LDS).
+template <int K, bool RAW>
+__device__ __forceinline__ void s_upd(uint8_t* base, uint32_t e, uint32_t S, uint64_t x) {
+  x = enc<K, RAW>(x);
+  if constexpr (K == FK_COUNT) {
+    atomicAdd((uint32_t*)base + e, (uint32_t)x);
+  } else if constexpr (K == FK_SUMI) {
+    uint32_t lo = (uint32_t)x, hi = (uint32_t)(x >> 32);
+    uint32_t old = atomicAdd((uint32_t*)base + e, lo);
+    hi += (uint32_t)(old + lo < old);
+    if (hi) atomicAdd((uint32_t*)base + S + e, hi);
+  } else if constexpr (K == FK_SUMF) {
+    atomicAdd((double*)base + e, __longlong_as_double((long long)x));
+  } else if constexpr (K == FK_MINI32) {
+    int v = (int)x;
+    int* q = (int*)base + e;
+    if (v < *(volatile int*)q) atomicMin(q, v);
+  } else if constexpr (K == FK_MAXI32) {
+    int v = (int)x;
+    int* q = (int*)base + e;
+    if (v > *(volatile int*)q) atomicMax(q, v);
+  } else if constexpr (K == FK_MINI64 || K == FK_MINF64) {
+    long long v = (long long)x;
+    long long* q = (long long*)base + e;
+    if (v < *(volatile long long*)q) atomicMin(q, v);
+  } else {
+    long long v = (long long)x;
+    long long* q = (long long*)base + e;
+    if (v > *(volatile long long*)q) atomicMax(q, v);
   }
 }
 
@@ -176,38 +252,41 @@ __device__ __forceinline__ void smem_init_entry(uint8_t* base, int k, uint32_t e
   }
 }
 
-// Read a shared-memory entry's state as the encoded 64-bit value to combine.
-__device__ __forceinline__ uint64_t smem_read(const uint8_t* base, int k, uint32_t e, uint32_t S) {
-  switch (k) {
-    case FK_COUNT: return (uint64_t)((const uint32_t*)base)[e];
-    case FK_SUMI: return (uint64_t)((const uint32_t*)base)[e] | ((uint64_t)((const uint32_t*)base)[S + e] << 32);
-    case FK_MINI32: case FK_MAXI32: return (uint64_t)(int64_t)((const int*)base)[e];
-    default: return ((const uint64_t*)base)[e];
-  }
+// A shared-memory entry's state as the encoded 64-bit value to combine into global memory.
+template <int K>
+__device__ __forceinline__ uint64_t s_read(const uint8_t* base, uint32_t e, uint32_t S) {
+  if constexpr (K == FK_COUNT) return (uint64_t)((const uint32_t*)base)[e];
+  else if constexpr (K == FK_SUMI)
+    return (uint64_t)((const uint32_t*)base)[e] | ((uint64_t)((const uint32_t*)base)[S + e] << 32);
+  else if constexpr (K == FK_MINI32 || K == FK_MAXI32) return (uint64_t)(int64_t)((const int*)base)[e];
+  else return ((const uint64_t*)base)[e];
 }
 
-// ---- global AoS slot (path b). Fire-and-forget REDs: REDG.E.ADD.64 / ADD.F64 / MIN.S64 ... ----
-__device__ __forceinline__ void slot_apply(uint8_t* slot, const Field& f, uint64_t x) {
-  uint8_t* a = slot + f.goff;
-  switch (f.kind) {
-    case FK_COUNT: case FK_SUMI: atomicAdd((unsigned long long*)a, (unsigned long long)x); break;
-    case FK_SUMF: atomicAdd((double*)a, __longlong_as_double((long long)x)); break;
-    case FK_MINI32: atomicMin((int*)a, (int)x); break;
-    case FK_MAXI32: atomicMax((int*)a, (int)x); break;
-    case FK_MINI64: case FK_MINF64: atomicMin((long long*)a, (long long)x); break;
-    default: atomicMax((long long*)a, (long long)x); break;
-  }
+// Global AoS slot field (path b): fire-and-forget reductions REDG.E.ADD.64 / ADD.F64 / MIN.S64 ...
+template <int K, bool RAW>
+__device__ __forceinline__ void g_upd(uint8_t* a, uint64_t x) {
+  x = enc<K, RAW>(x);
+  if constexpr (K == FK_COUNT || K == FK_SUMI) atomicAdd((unsigned long long*)a, (unsigned long long)x);
+  else if constexpr (K == FK_SUMF) atomicAdd((double*)a, __longlong_as_double((long long)x));
+  else if constexpr (K == FK_MINI32) atomicMin((int*)a, (int)x);
+  else if constexpr (K == FK_MAXI32) atomicMax((int*)a, (int)x);
+  else if constexpr (K == FK_MINI64 || K == FK_MINF64) atomicMin((long long*)a, (long long)x);
+  else atomicMax((long long*)a, (long long)x);
 }
 
-// ---- global dense state (paths a / b'): 4 groups of int64 arrays (sidx x D + g) -----------------
-__device__ __forceinline__ void dense_apply(void* const* dense, uint64_t D, const Field& f, uint64_t g, uint64_t x) {
-  uint64_t* a = (uint64_t*)dense[f.sgroup] + (uint64_t)f.sidx * D + g;
-  switch (f.kind) {
-    case FK_COUNT: case FK_SUMI: atomicAdd((unsigned long long*)a, (unsigned long long)x); break;
-    case FK_SUMF: atomicAdd((double*)a, __longlong_as_double((long long)x)); break;
-    case FK_MINI32: case FK_MINI64: case FK_MINF64: atomicMin((long long*)a, (long long)x); break;
-    default: atomicMax((long long*)a, (long long)x); break;
-  }
+// Global dense state field (paths a / b'): every field 8 bytes (i32 MIN/MAX widened).
+template <int K, bool RAW>
+__device__ __forceinline__ void d_upd(uint64_t* a, uint64_t x) {
+  x = enc<K, RAW>(x);
+  if constexpr (K == FK_COUNT || K == FK_SUMI) atomicAdd((unsigned long long*)a, (unsigned long long)x);
+  else if constexpr (K == FK_SUMF) atomicAdd((double*)a, __longlong_as_double((long long)x));
+  else if constexpr (K == FK_MINI32 || K == FK_MINI64 || K == FK_MINF64) atomicMin((long long*)a, (long long)x);
+  else atomicMax((long long*)a, (long long)x);
+}
+
+__device__ __forceinline__ uint64_t* dense_addr(const AggParams& p, int j, uint64_t g) {
+  const Field& f = p.lay.f[j];
+  return (uint64_t*)p.dense[f.sgroup] + (uint64_t)f.sidx * p.lay.domain + g;
 }
 
 // Linear probing from fmix64(key) & mask; read-before-CAS; keys are write-once (EMPTY -> key), so
@@ -230,19 +309,19 @@ __device__ __forceinline__ bool hash_locate(uint8_t* table, uint64_t mask, uint3
 
 // Pack the key columns of rows [row, row+R) (S1, CCAT P:111): sparse -> code; dense -> mixed radix
 // sum code_j * stride_j. Invalid codes raise FLAG_KEY_RANGE; rows >= n are not valid.
-template <int R>
+template <int R, bool PAIR = true>
 __device__ __forceinline__ uint32_t pack_keys(const AggParams& p, uint64_t row, uint64_t n, uint64_t pol,
                                               uint64_t (&key)[R]) {
   uint32_t valid = 0;
 #pragma unroll
   for (int r = 0; r < R; ++r) {
     key[r] = 0;
-    if (row + r < n) valid |= 1u << r;
+    if (row_of<R, PAIR>(row, r) < n) valid |= 1u << r;
   }
   uint32_t bad = 0;
   if (p.lay.sparse) {
     uint64_t c[R];
-    load_rows<R>(p.key[0], p.lay.key_dtype[0], row, n, p.vec_ok, pol, c);
+    load_rows<R, PAIR>(p.key[0], p.lay.key_dtype[0], row, n, p.vec_ok, pol, c);
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       key[r] = c[r];
@@ -251,7 +330,7 @@ __device__ __forceinline__ uint32_t pack_keys(const AggParams& p, uint64_t row, 
   } else {
     for (int k = 0; k < p.lay.n_keys; ++k) {
       uint64_t c[R];
-      load_rows<R>(p.key[k], p.lay.key_dtype[k], row, n, p.vec_ok, pol, c);
+      load_rows<R, PAIR>(p.key[k], p.lay.key_dtype[k], row, n, p.vec_ok, pol, c);
       const uint64_t d = p.lay.dict[k], s = p.lay.stride[k];
 #pragma unroll
       for (int r = 0; r < R; ++r) {
@@ -265,19 +344,63 @@ __device__ __forceinline__ uint32_t pack_keys(const AggParams& p, uint64_t row, 
   return valid & ~bad;
 }
 
+// Apply every field to the rows in `mask` of a shared-memory table at entries e[r].
+template <int NV, int R>
+__device__ __forceinline__ void smem_apply_rows(const AggParams& p, uint8_t* sm, const uint32_t (&e)[R],
+                                                uint32_t mask, const uint64_t (&v)[NV][R]) {
+  const uint32_t S = p.S;
+  for (uint32_t m = p.cntmask; m; m &= m - 1) {
+    uint8_t* b = sm + p.soff[__ffs(m) - 1];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (mask >> r & 1) s_upd<FK_COUNT, true>(b, e[r], S, 1ull);
+  }
+#pragma unroll
+  for (int c = 0; c < NV; ++c) {
+    if (c >= p.lay.n_vals) break;
+    for (uint32_t m = p.colmask[c]; m; m &= m - 1) {
+      const int j = __ffs(m) - 1;
+      uint8_t* b = sm + p.soff[j];
+      dispatch_kind(p.lay.f[j].kind, [&](auto kc) {
+        constexpr int K = decltype(kc)::v;
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+          if (mask >> r & 1) s_upd<K, true>(b, e[r], S, v[c][r]);
+      });
+    }
+  }
+}
 
-// Field-column masks: bit j set if field j reads column c; cnt: fields counting the constant 1.
-struct ColMasks {
-  uint32_t col[kMaxVals > kMaxFields ? kMaxVals : kMaxFields];
-  uint32_t cnt;
-};
-
-__device__ __forceinline__ void build_masks(const Layout& L, ColMasks& m) {
-  for (int c = 0; c < kMaxFields; ++c) m.col[c] = 0;
-  m.cnt = 0;
-  for (int j = 0; j < L.n_fields; ++j) {
-    if (L.f[j].col < 0) m.cnt |= 1u << j;
-    else m.col[L.f[j].col] |= 1u << j;
+// Apply every field to the rows in `mask` of the global target: AoS slots (hash) or dense state.
+template <int NV, int R, bool DIRECT>
+__device__ __forceinline__ void global_apply_rows(const AggParams& p, const uint64_t (&slot)[R], uint32_t mask,
+                                                  const uint64_t (&v)[NV][R]) {
+  const Layout& L = p.lay;
+  uint8_t* tb = (uint8_t*)p.table;
+  for (uint32_t m = p.cntmask; m; m &= m - 1) {
+    const int j = __ffs(m) - 1;
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (mask >> r & 1) {
+        if (DIRECT) d_upd<FK_COUNT, true>(dense_addr(p, j, slot[r]), 1ull);
+        else g_upd<FK_COUNT, true>(tb + slot[r] * L.slot_bytes + L.f[j].goff, 1ull);
+      }
+  }
+#pragma unroll
+  for (int c = 0; c < NV; ++c) {
+    if (c >= L.n_vals) break;
+    for (uint32_t m = p.colmask[c]; m; m &= m - 1) {
+      const int j = __ffs(m) - 1;
+      dispatch_kind(L.f[j].kind, [&](auto kc) {
+        constexpr int K = decltype(kc)::v;
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+          if (mask >> r & 1) {
+            if (DIRECT) d_upd<K, true>(dense_addr(p, j, slot[r]), v[c][r]);
+            else g_upd<K, true>(tb + slot[r] * L.slot_bytes + L.f[j].goff, v[c][r]);
+          }
+      });
+    }
   }
 }
 
@@ -308,31 +431,13 @@ __global__ void __launch_bounds__(256) k_fill_u64(uint64_t* a, uint64_t n, uint6
 // ------------------------------------------------------------------------------------------------
 // S5a: path (a) dense shared-memory aggregation (§4.3.2)
 // ------------------------------------------------------------------------------------------------
-struct SmemOffsets {
-  uint32_t off[kMaxFields];
-  uint32_t key_off;  // front only
-};
-
-__device__ __forceinline__ void smem_offsets(const Layout& L, uint32_t S, bool with_keys, SmemOffsets& so) {
-  uint32_t o = 0;
-  if (with_keys) { so.key_off = 0; o = S * 8; }
-  for (int j = 0; j < L.n_fields; ++j) {
-    so.off[j] = o;
-    o += (S * L.f[j].ssize + 15) / 16 * 16;
-  }
-}
-
 template <int NV, int R>
 __global__ void __launch_bounds__(512) k_agg_dense_smem(AggParams p) {
   extern __shared__ __align__(16) uint8_t sm[];
   const Layout& L = p.lay;
-  const uint32_t D = (uint32_t)L.domain;
-  SmemOffsets so;
-  smem_offsets(L, D, false, so);
+  const uint32_t D = p.S;
   for (int j = 0; j < L.n_fields; ++j)
-    for (uint32_t e = threadIdx.x; e < D; e += blockDim.x) smem_init_entry(sm + so.off[j], L.f[j].kind, e, D);
-  ColMasks cm;
-  build_masks(L, cm);
+    for (uint32_t e = threadIdx.x; e < D; e += blockDim.x) smem_init_entry(sm + p.soff[j], L.f[j].kind, e, D);
   __syncthreads();
 
   const uint64_t pol = evict_first_policy();
@@ -342,100 +447,59 @@ __global__ void __launch_bounds__(512) k_agg_dense_smem(AggParams p) {
   uint32_t flag_seen = 0;
   for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
     if (flag_seen) break;
-    flag_seen = *(volatile uint32_t*)p.flags;  // checked at the next tile (latency hidden)
-    const uint64_t row = t * tile + (uint64_t)threadIdx.x * R;
-    if (row >= n) continue;
+    flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);  // warp-uniform, seen next tile
+    const uint64_t row = lane_base<R, false>(t * tile, threadIdx.x >> 5, threadIdx.x & 31);
     uint64_t key[R];
-    uint32_t valid = pack_keys<R>(p, row, n, pol, key);
+    const uint32_t valid = pack_keys<R, false>(p, row, n, pol, key);
     uint64_t v[NV][R];
 #pragma unroll
     for (int c = 0; c < NV; ++c)
-      if (c < L.n_vals) load_rows<R>(p.val[c], L.val_dtype[c], row, n, p.vec_ok, pol, v[c]);
+      if (c < L.n_vals) load_rows<R, false>(p.val[c], L.val_dtype[c], row, n, p.vec_ok, pol, v[c]);
+    uint32_t e[R];
 #pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (!(valid >> r & 1)) continue;
-      const uint32_t e = (uint32_t)key[r];
-      for (uint32_t m = cm.cnt; m; m &= m - 1) {
-        int j = __ffs(m) - 1;
-        smem_apply(sm + so.off[j], L.f[j].kind, e, D, 1ull);
-      }
-#pragma unroll
-      for (int c = 0; c < NV; ++c) {
-        if (c >= L.n_vals) break;
-        for (uint32_t m = cm.col[c]; m; m &= m - 1) {
-          int j = __ffs(m) - 1;
-          int k = L.f[j].kind;
-          smem_apply(sm + so.off[j], k, e, D, encode(k, v[c][r]));
-        }
-      }
-    }
+    for (int r = 0; r < R; ++r) e[r] = (uint32_t)key[r];
+    smem_apply_rows<NV, R>(p, sm, e, valid, v);
   }
   __syncthreads();
   // S7: CTA -> global merge with native 64-bit REDs ("the small hash tables in shared memory
   // are merged to a global hash table in device memory").
-  const int cf = L.count_field;
+  const uint8_t* cnt = sm + p.soff[L.count_field];
   for (uint32_t e = threadIdx.x; e < D; e += blockDim.x) {
-    if (smem_read(sm + so.off[cf], L.f[cf].kind, e, D) == 0) continue;
-    for (int j = 0; j < L.n_fields; ++j)
-      dense_apply(p.dense, L.domain, L.f[j], e, smem_read(sm + so.off[j], L.f[j].kind, e, D));
+    if (((const uint32_t*)cnt)[e] == 0) continue;
+    for (int j = 0; j < L.n_fields; ++j) {
+      uint8_t* b = sm + p.soff[j];
+      dispatch_kind(L.f[j].kind, [&](auto kc) {
+        constexpr int K = decltype(kc)::v;
+        d_upd<K, false>(dense_addr(p, j, e), s_read<K>(b, e, D));
+      });
+    }
   }
 }
 
 // ------------------------------------------------------------------------------------------------
 // S5b: path (b) global hash table / path (b') direct-mapped, optional shared-memory hot-key front
 // ------------------------------------------------------------------------------------------------
-template <bool DIRECT>
-__device__ __forceinline__ bool global_apply_row(const AggParams& p, const ColMasks& cm, uint64_t key,
-                                                 uint64_t first, uint64_t idx, const uint64_t* vals /*NV*/,
-                                                 int nv) {
-  const Layout& L = p.lay;
-  if (DIRECT) {
-    for (uint32_t m = cm.cnt; m; m &= m - 1) dense_apply(p.dense, L.domain, L.f[__ffs(m) - 1], key, 1ull);
-    for (int c = 0; c < nv; ++c)
-      for (uint32_t m = cm.col[c]; m; m &= m - 1) {
-        const Field& f = L.f[__ffs(m) - 1];
-        dense_apply(p.dense, L.domain, f, key, encode(f.kind, vals[c]));
-      }
-    return true;
-  } else {
-    uint64_t slot;
-    if (!hash_locate((uint8_t*)p.table, p.cap_mask, L.slot_bytes, key, first, idx, p.max_probe, slot)) return false;
-    uint8_t* s = (uint8_t*)p.table + slot * L.slot_bytes;
-    for (uint32_t m = cm.cnt; m; m &= m - 1) slot_apply(s, L.f[__ffs(m) - 1], 1ull);
-    for (int c = 0; c < nv; ++c)
-      for (uint32_t m = cm.col[c]; m; m &= m - 1) {
-        const Field& f = L.f[__ffs(m) - 1];
-        slot_apply(s, f, encode(f.kind, vals[c]));
-      }
-    return true;
-  }
-}
-
 template <int NV, int R, bool FRONT, bool DIRECT, bool RECORDS>
 __global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
   extern __shared__ __align__(16) uint8_t sm[];
   const Layout& L = p.lay;
-  const uint32_t S = p.front_slots;
-  SmemOffsets so;
+  const uint32_t S = p.S;
   if (FRONT) {
-    smem_offsets(L, S, true, so);
-    for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) ((uint64_t*)(sm + so.key_off))[e] = kEmpty;
+    for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) ((uint64_t*)(sm + p.key_off))[e] = kEmpty;
     for (int j = 0; j < L.n_fields; ++j)
-      for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) smem_init_entry(sm + so.off[j], L.f[j].kind, e, S);
+      for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) smem_init_entry(sm + p.soff[j], L.f[j].kind, e, S);
     __syncthreads();
   }
-  ColMasks cm;
-  build_masks(L, cm);
   const uint64_t pol = evict_first_policy();
   const uint64_t n = p.n_rows;
   const uint64_t tile = (uint64_t)blockDim.x * R;
   const uint64_t ntiles = (n + tile - 1) / tile;
+  uint8_t* tb = (uint8_t*)p.table;
   uint32_t flag_seen = 0;
   for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
     if (flag_seen) break;
-    flag_seen = *(volatile uint32_t*)p.flags;
-    const uint64_t row = t * tile + (uint64_t)threadIdx.x * R;
-    if (row >= n) continue;
+    flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);  // warp-uniform abort
+    const uint64_t row = lane_base<R>(t * tile, threadIdx.x >> 5, threadIdx.x & 31);
     uint64_t key[R];
     uint64_t v[NV][R];
     uint32_t valid;
@@ -443,8 +507,12 @@ __global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
       valid = 0;
 #pragma unroll
       for (int r = 0; r < R; ++r) {
-        if (row + r >= n) { key[r] = 0; continue; }
-        const uint64_t* rec = rs.rec + (row + r) * rs.words;
+        key[r] = 0;
+#pragma unroll
+        for (int c = 0; c < NV; ++c) v[c][r] = 0;
+        const uint64_t rr = row_of<R>(row, r);
+        if (rr >= n) continue;
+        const uint64_t* rec = rs.rec + rr * rs.words;
         key[r] = __ldg((const unsigned long long*)rec);
         valid |= 1u << r;
 #pragma unroll
@@ -460,82 +528,84 @@ __global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
       for (int c = 0; c < NV; ++c)
         if (c < L.n_vals) load_rows<R>(p.val[c], L.val_dtype[c], row, n, p.vec_ok, pol, v[c]);
     }
-    // probe: issue the first key load of every row before resolving any (memory-level parallelism)
-    uint64_t idx[R], first[R];
+    uint32_t miss = valid;
+    if (FRONT) {
+      // hot-key front: small open-addressing table per CTA in shared memory
+      uint64_t* fk = (uint64_t*)(sm + p.key_off);
+      uint32_t fe[R];
+      uint32_t hit = 0;
 #pragma unroll
-    for (int r = 0; r < R; ++r) {
-      idx[r] = 0;
-      first[r] = 0;
-      if (!DIRECT && (valid >> r & 1)) {
-        idx[r] = fmix64(key[r]) & p.cap_mask;
-        first[r] = __ldcg((const unsigned long long*)((const uint8_t*)p.table + idx[r] * L.slot_bytes));
-      }
-    }
-#pragma unroll
-    for (int r = 0; r < R; ++r) {
-      if (!(valid >> r & 1)) continue;
-      if (FRONT) {
-        uint64_t* fk = (uint64_t*)(sm + so.key_off);
+      for (int r = 0; r < R; ++r) {
+        fe[r] = 0;
+        if (!(valid >> r & 1)) continue;
         uint32_t s = (uint32_t)(fmix64(key[r] ^ 0x5bd1e995ull) >> 40) & (S - 1);
-        bool hit = false;
 #pragma unroll 1
         for (int q = 0; q < 8; ++q) {
           uint64_t cur = *(volatile uint64_t*)(fk + s);
-          if (cur == key[r]) { hit = true; break; }
+          if (cur == key[r]) { hit |= 1u << r; break; }
           if (cur == kEmpty) {
             unsigned long long old = atomicCAS((unsigned long long*)(fk + s), (unsigned long long)kEmpty,
                                                (unsigned long long)key[r]);
-            if (old == kEmpty || old == key[r]) { hit = true; break; }
+            if (old == kEmpty || old == key[r]) { hit |= 1u << r; break; }
           }
           s = (s + 1) & (S - 1);
         }
-        if (hit) {
-          for (uint32_t m = cm.cnt; m; m &= m - 1) {
-            int j = __ffs(m) - 1;
-            smem_apply(sm + so.off[j], L.f[j].kind, s, S, 1ull);
-          }
-#pragma unroll
-          for (int c = 0; c < NV; ++c) {
-            if (c >= L.n_vals) break;
-            for (uint32_t m = cm.col[c]; m; m &= m - 1) {
-              int j = __ffs(m) - 1;
-              int k = L.f[j].kind;
-              smem_apply(sm + so.off[j], k, s, S, encode(k, v[c][r]));
-            }
-          }
-          continue;
-        }
-        if (!DIRECT) first[r] = __ldcg((const unsigned long long*)((const uint8_t*)p.table + idx[r] * L.slot_bytes));
+        fe[r] = s;
       }
-      uint64_t vals[NV];
-#pragma unroll
-      for (int c = 0; c < NV; ++c) vals[c] = v[c][r];
-      if (!global_apply_row<DIRECT>(p, cm, key[r], first[r], idx[r], vals, NV < L.n_vals ? NV : L.n_vals)) {
-        atomicOr(p.flags, FLAG_OVERFLOW);
-        flag_seen = 1;
-        break;
-      }
+      __syncwarp();  // reconverge after the data-dependent probe loops (independent thread scheduling)
+      smem_apply_rows<NV, R>(p, sm, fe, hit, v);
+      miss = valid & ~hit;
     }
+    uint64_t slot[R];
+    if (DIRECT) {
+#pragma unroll
+      for (int r = 0; r < R; ++r) slot[r] = key[r];
+    } else {
+      // issue the first key load of every row before resolving any (memory-level parallelism)
+      uint64_t first[R];
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        slot[r] = fmix64(key[r]) & p.cap_mask;
+        first[r] = (miss >> r & 1) ? __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes)) : 0ull;
+      }
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        if (!(miss >> r & 1)) continue;
+        uint64_t s;
+        if (hash_locate(tb, p.cap_mask, L.slot_bytes, key[r], first[r], slot[r], p.max_probe, s)) {
+          slot[r] = s;
+        } else {
+          miss &= ~(1u << r);
+          atomicOr(p.flags, FLAG_OVERFLOW);
+        }
+      }
+      __syncwarp();  // reconverge before the field reductions so each RED instruction is warp-wide
+    }
+    global_apply_rows<NV, R, DIRECT>(p, slot, miss, v);
   }
   if (FRONT) {
     // merge the front into the global table
     __syncthreads();
-    uint64_t* fk = (uint64_t*)(sm + so.key_off);
+    const uint64_t* fk = (const uint64_t*)(sm + p.key_off);
     for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) {
-      uint64_t key = fk[e];
+      const uint64_t key = fk[e];
       if (key == kEmpty) continue;
-      if (DIRECT) {
-        for (int j = 0; j < L.n_fields; ++j)
-          dense_apply(p.dense, L.domain, L.f[j], key, smem_read(sm + so.off[j], L.f[j].kind, e, S));
-      } else {
-        uint64_t idx = fmix64(key) & p.cap_mask, slot;
-        uint64_t first = __ldcg((const unsigned long long*)((const uint8_t*)p.table + idx * L.slot_bytes));
-        if (!hash_locate((uint8_t*)p.table, p.cap_mask, L.slot_bytes, key, first, idx, p.max_probe, slot)) {
+      uint64_t s = key;
+      if (!DIRECT) {
+        uint64_t idx = fmix64(key) & p.cap_mask;
+        uint64_t first = __ldcg((const unsigned long long*)(tb + idx * L.slot_bytes));
+        if (!hash_locate(tb, p.cap_mask, L.slot_bytes, key, first, idx, p.max_probe, s)) {
           atomicOr(p.flags, FLAG_OVERFLOW);
           continue;
         }
-        uint8_t* s = (uint8_t*)p.table + slot * L.slot_bytes;
-        for (int j = 0; j < L.n_fields; ++j) slot_apply(s, L.f[j], smem_read(sm + so.off[j], L.f[j].kind, e, S));
+      }
+      for (int j = 0; j < L.n_fields; ++j) {
+        const uint8_t* b = sm + p.soff[j];
+        dispatch_kind(L.f[j].kind, [&](auto kc) {
+          constexpr int K = decltype(kc)::v;
+          if (DIRECT) d_upd<K, false>(dense_addr(p, j, s), s_read<K>(b, e, S));
+          else g_upd<K, false>(tb + s * L.slot_bytes + L.f[j].goff, s_read<K>(b, e, S));
+        });
       }
     }
   }

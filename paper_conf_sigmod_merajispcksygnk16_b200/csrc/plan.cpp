@@ -149,6 +149,24 @@ void build_slot_template(const Layout& L, uint8_t* out) {
   }
 }
 
+void fill_smem_layout(AggParams& p, uint32_t S, bool with_keys) {
+  const Layout& L = p.lay;
+  uint32_t o = 0;
+  p.S = S;
+  p.key_off = 0;
+  if (with_keys) o = S * 8;
+  for (int j = 0; j < L.n_fields; ++j) {
+    p.soff[j] = o;
+    o += (S * (uint32_t)L.f[j].ssize + 15) / 16 * 16;
+  }
+  for (int c = 0; c < kMaxFields; ++c) p.colmask[c] = 0;
+  p.cntmask = 0;
+  for (int j = 0; j < L.n_fields; ++j) {
+    if (L.f[j].col < 0) p.cntmask |= 1u << j;
+    else p.colmask[L.f[j].col] |= 1u << j;
+  }
+}
+
 }  // namespace blu
 
 using namespace blu;
