@@ -367,6 +367,100 @@ static bool nonnull_cols(const void* const* cols, int n) {
   return true;
 }
 
+// Partitioned path (b): per chunk of rows, pass 1 scatters rows into P->parts buckets (partition
+// buffers in HBM), pass 2 aggregates bucket by bucket (one persistent launch). If any bucket
+// overflows its capacity (heavily skewed keys), a device-side gate skips pass 2 and runs the
+// one-pass kernel over the chunk's original rows instead. No host synchronisation.
+static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, const void* const* keys,
+                                    const void* const* vals, uint64_t n, cudaStream_t st, uint32_t* launches,
+                                    Work& w) {
+  const Layout& L = P->lay;
+  const uint32_t B = P->parts;
+  size_t row_bytes = 8;
+  for (int c = 0; c < L.n_vals; ++c) row_bytes += dtype_bytes(L.val_dtype[c]);
+  size_t free_b = 0, total_b = 0;
+  cudaMemGetInfo(&free_b, &total_b);
+  uint64_t budget_rows = (uint64_t)((double)free_b * 0.6 / (double)row_bytes / 1.03);
+  uint64_t M = std::min<uint64_t>(n, std::max<uint64_t>(budget_rows, 1ull << 22));
+  if (const char* cr = getenv("BLU_GBY_PART_CHUNK")) M = std::min<uint64_t>(n, std::max<uint64_t>(1024, strtoull(cr, 0, 10)));
+  uint64_t seg_cap = ((uint64_t)((double)((M + B - 1) / B) * 1.03) + 4096 + 63) & ~63ull;
+  uint64_t rows_alloc = seg_cap * B;
+  void* kbuf = nullptr;
+  void* vbuf[kMaxVals] = {};
+  void* meta = nullptr;
+  cudaError_t e = w.alloc(&kbuf, rows_alloc * 8);
+  for (int c = 0; c < L.n_vals && e == cudaSuccess; ++c) e = w.alloc(&vbuf[c], rows_alloc * dtype_bytes(L.val_dtype[c]));
+  if (e == cudaSuccess) e = w.alloc(&meta, (size_t)B * 16 + 64);
+  if (e != cudaSuccess) return e;
+  uint64_t* d_seg_base = (uint64_t*)meta;
+  uint64_t* d_cursor = d_seg_base + B;
+  uint32_t* d_gate = (uint32_t*)(d_cursor + B);
+  std::vector<uint64_t> hb(B);
+  for (uint32_t b = 0; b < B; ++b) hb[b] = (uint64_t)b * seg_cap;
+  e = cudaMemcpyAsync(d_seg_base, hb.data(), (size_t)B * 8, cudaMemcpyHostToDevice, st);
+  if (e) return e;
+  uint32_t scatter_grid = (uint32_t)P->sms * 2;
+  Layout L2 = L;  // pass 2 reads the packed u64 key as a single sparse key column
+  L2.n_keys = 1;
+  L2.sparse = 1;
+  L2.key_dtype[0] = BLU_I64;
+  for (uint64_t r0 = 0; r0 < n; r0 += M) {
+    const uint64_t m = std::min(M, n - r0);
+    if ((e = cudaMemsetAsync(d_cursor, 0, (size_t)B * 8 + 8, st))) return e;
+    AggParams p1 = base;
+    bool vec = true;
+    for (int k = 0; k < L.n_keys; ++k) {
+      p1.key[k] = (const uint8_t*)keys[k] + r0 * dtype_bytes(L.key_dtype[k]);
+      vec = vec && ptr_aligned(p1.key[k]);
+    }
+    for (int c = 0; c < L.n_vals; ++c) {
+      p1.val[c] = (const uint8_t*)vals[c] + r0 * dtype_bytes(L.val_dtype[c]);
+      vec = vec && ptr_aligned(p1.val[c]);
+    }
+    p1.vec_ok = vec;
+    p1.n_rows = m;
+    ScatterParams sp{};
+    sp.B = B;
+    {  // bucket = top log2(B) bits of the slot index of the CURRENT table (it may have regrown)
+      uint32_t lc = (uint32_t)__builtin_popcountll(base.cap_mask), lb = 0;
+      while ((1u << lb) < B) ++lb;
+      sp.shift = lc > lb ? lc - lb : 0;
+    }
+    sp.seg_base = d_seg_base;
+    sp.cursor = d_cursor;
+    sp.seg_cap = seg_cap;
+    sp.out_key = (uint64_t*)kbuf;
+    for (int c = 0; c < L.n_vals; ++c) sp.out_val[c] = vbuf[c];
+    sp.gate = d_gate;
+    int le = launch_scatter(p1, sp, st, scatter_grid);
+    if (le) return (cudaError_t)le;
+    // pass 2 (runs if no bucket overflowed)
+    AggParams p2 = base;
+    p2.lay = L2;
+    p2.key[0] = kbuf;
+    for (int c = 0; c < L.n_vals; ++c) p2.val[c] = vbuf[c];
+    p2.vec_ok = 1;
+    p2.n_rows = 0;
+    p2.seg_base = d_seg_base;
+    p2.seg_count = d_cursor;
+    p2.n_segs = B;
+    p2.gate = d_gate;
+    p2.gate_run_if = 0;
+    p2.front_slots = 0;
+    le = launch_aggregate_impl(P, BLU_PATH_HASH_GLOBAL, p2, RecSrc{nullptr, 0}, false, st, P->grid, P->block, 0);
+    if (le) return (cudaError_t)le;
+    // fallback one-pass over the chunk's rows (runs only if a bucket overflowed)
+    AggParams p3 = p1;
+    p3.gate = d_gate;
+    p3.gate_run_if = 1;
+    le = launch_aggregate_impl(P, BLU_PATH_HASH_GLOBAL, p3, RecSrc{nullptr, 0}, false, st, P->grid, P->block,
+                               P->smem_bytes);
+    if (le) return (cudaError_t)le;
+    if (launches) *launches += 3;
+  }
+  return cudaSuccess;
+}
+
 // Schema column pointers -> kernel columns (the layout's value columns are the schema's).
 static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* keys, const void* const* vals,
                                    uint64_t n, cudaStream_t st, bool partial, blu_gby_result_t* out) {
@@ -375,6 +469,10 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
     return fail(BLU_E_INVALID, "NULL column pointer");
   const Layout& L = P->lay;
   Feeder feed = [&](AggParams& base, uint32_t* launches) -> cudaError_t {
+    if (P->path == BLU_PATH_HASH_GLOBAL && P->parts > 1 && n >= 4096 * (uint64_t)P->parts) {
+      Work pw(st);
+      return partitioned_feed(P, base, keys, vals, n, st, launches, pw);
+    }
     return agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, launches);
   };
   return run_core(P, L, P->path, P->hot_front != 0, P->cap, n, feed, partial, st, out, false, nullptr);

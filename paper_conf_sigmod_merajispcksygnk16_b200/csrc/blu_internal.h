@@ -93,6 +93,8 @@ struct blu_gby_plan_s {
   uint32_t smem_bytes;    // dynamic shared memory of the aggregation kernel
   uint32_t grid, block;
   int32_t sms;
+  uint32_t parts;         // path b: buckets of the partitioned two-pass mode (1 = one pass)
+  uint32_t part_shift;    // log2(cap) - log2(parts)
   mutable std::atomic<uint32_t> retries_last{0};
 };
 
@@ -120,6 +122,25 @@ struct AggParams {
   uint32_t soff[kMaxFields];     // per field: byte offset of its SoA array
   uint32_t colmask[kMaxFields];  // per kernel value column: bit j = field j reads it
   uint32_t cntmask;              // fields that count the constant 1
+  // partitioned pass 2 (segments mode): rows of segment b are [seg_base[b], seg_base[b] + seg_count[b])
+  const uint64_t* seg_base;
+  const uint64_t* seg_count;
+  uint32_t n_segs;
+  // device-side gate: the kernel runs only if ((*gate != 0) == gate_run_if); NULL = always
+  const uint32_t* gate;
+  uint32_t gate_run_if;
+};
+
+// Pass 1 of the partitioned path (b): scatter rows into B buckets by the top bits of their slot.
+struct ScatterParams {
+  uint32_t B;
+  uint32_t shift;            // bucket = (fmix64(key) & cap_mask) >> shift
+  const uint64_t* seg_base;  // B: first row of each bucket in the partition buffers
+  uint64_t* cursor;          // B: rows appended so far (zeroed per chunk)
+  uint64_t seg_cap;          // rows per bucket
+  uint64_t* out_key;         // packed keys (u64)
+  void* out_val[kMaxVals];   // value columns, input dtypes
+  uint32_t* gate;            // set to 1 if any bucket overflows (pass 2 then falls back)
 };
 
 // Fill S / key_off / soff / colmask / cntmask of p for a shared-memory table of S entries.
@@ -157,6 +178,7 @@ struct RecSrc {
 int launch_aggregate_impl(const blu_gby_plan_s* P, int path, const AggParams& p, const RecSrc& rs, bool records,
                           void* stream, uint32_t grid, uint32_t block, uint32_t smem);
 uint64_t launches_total();
+int launch_scatter(const AggParams& p, const ScatterParams& s, void* stream, uint32_t grid);
 blu_status_t fail(blu_status_t s, const char* fmt, ...);
 int launch_init_slots(const Layout& lay, void* table, uint64_t n_slots, void* stream);
 int launch_init_dense(const Layout& lay, void* const dense[4], uint64_t D, void* stream);

@@ -479,11 +479,36 @@ __global__ void __launch_bounds__(512) k_agg_dense_smem(AggParams p) {
 // ------------------------------------------------------------------------------------------------
 // S5b: path (b) global hash table / path (b') direct-mapped, optional shared-memory hot-key front
 // ------------------------------------------------------------------------------------------------
-template <int NV, int R, bool FRONT, bool DIRECT, bool RECORDS>
+// MODE 0: rows from columns; 1: records (merge of exchanged partials); 2: segments (pass 2 of the
+// partitioned mode: tiles enumerate the buckets in order, so at any moment all CTAs work inside
+// one bucket whose slice of the table is L2-resident).
+template <int NV, int R, bool FRONT, bool DIRECT, int MODE>
 __global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
   extern __shared__ __align__(16) uint8_t sm[];
+  constexpr bool RECORDS = MODE == 1;
+  constexpr bool SEG = MODE == 2;
+  if (p.gate && ((*(volatile const uint32_t*)p.gate != 0) != (p.gate_run_if != 0))) return;
   const Layout& L = p.lay;
   const uint32_t S = p.S;
+  __shared__ uint64_t tpre[SEG ? 1025 : 1];
+  if constexpr (SEG) {  // tile prefix over the buckets (warp 0)
+    if (threadIdx.x < 32) {
+      const uint64_t tile = (uint64_t)blockDim.x * R;
+      uint64_t carry = 0;
+      for (uint32_t b0 = 0; b0 < p.n_segs; b0 += 32) {
+        uint32_t b = b0 + threadIdx.x;
+        uint64_t x = b < p.n_segs ? (p.seg_count[b] + tile - 1) / tile : 0, inc = x;
+        for (int o = 1; o < 32; o <<= 1) {
+          uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+          if ((int)threadIdx.x >= o) inc += y;
+        }
+        if (b < p.n_segs) tpre[b] = carry + inc - x;
+        carry += __shfl_sync(0xffffffffu, inc, 31);
+      }
+      if (threadIdx.x == 0) tpre[p.n_segs] = carry;
+    }
+    __syncthreads();
+  }
   if (FRONT) {
     for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) ((uint64_t*)(sm + p.key_off))[e] = kEmpty;
     for (int j = 0; j < L.n_fields; ++j)
@@ -491,15 +516,24 @@ __global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
     __syncthreads();
   }
   const uint64_t pol = evict_first_policy();
-  const uint64_t n = p.n_rows;
   const uint64_t tile = (uint64_t)blockDim.x * R;
-  const uint64_t ntiles = (n + tile - 1) / tile;
+  const uint64_t ntiles = SEG ? tpre[p.n_segs] : (p.n_rows + tile - 1) / tile;
   uint8_t* tb = (uint8_t*)p.table;
   uint32_t flag_seen = 0;
   for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
     if (flag_seen) break;
     flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);  // warp-uniform abort
-    const uint64_t row = lane_base<R>(t * tile, threadIdx.x >> 5, threadIdx.x & 31);
+    uint64_t n = p.n_rows, row0 = t * tile;
+    if constexpr (SEG) {  // bucket of tile t: largest b with tpre[b] <= t
+      uint32_t lo = 0, hi = p.n_segs - 1;
+      while (lo < hi) {
+        uint32_t mid = (lo + hi + 1) >> 1;
+        if (tpre[mid] <= t) lo = mid; else hi = mid - 1;
+      }
+      row0 = p.seg_base[lo] + (t - tpre[lo]) * tile;
+      n = p.seg_base[lo] + p.seg_count[lo];
+    }
+    const uint64_t row = lane_base<R>(row0, threadIdx.x >> 5, threadIdx.x & 31);
     uint64_t key[R];
     uint64_t v[NV][R];
     uint32_t valid;
@@ -609,6 +643,133 @@ __global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
       }
     }
   }
+}
+
+// ------------------------------------------------------------------------------------------------
+// Partitioned path (b), pass 1: radix scatter of rows into B buckets by the top bits of their slot.
+// Per tile: shared-memory counting sort by bucket, one global cursor reservation per (tile,
+// bucket), then coalesced writes of each bucket's contiguous segment (packed u64 key + values).
+// ------------------------------------------------------------------------------------------------
+__device__ __forceinline__ void block_excl_scan_512(uint32_t* a, uint32_t* out, uint32_t B, uint32_t* warp_tot,
+                                                    uint32_t* total) {
+  // exclusive scan of a[0..B) (B <= 2 * blockDim.x, blockDim.x == 512) into out
+  const unsigned t = threadIdx.x, lane = t & 31, w = t >> 5;
+  uint32_t x0 = 2 * t < B ? a[2 * t] : 0, x1 = 2 * t + 1 < B ? a[2 * t + 1] : 0;
+  uint32_t sum = x0 + x1, inc = sum;
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+    if ((int)lane >= o) inc += y;
+  }
+  if (lane == 31) warp_tot[w] = inc;
+  __syncthreads();
+  if (w == 0) {
+    uint32_t v = lane < blockDim.x / 32 ? warp_tot[lane] : 0, vi = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(0xffffffffu, vi, o);
+      if ((int)lane >= o) vi += y;
+    }
+    if (lane < blockDim.x / 32) warp_tot[lane] = vi - v;
+    if (lane == 31) *total = vi;
+  }
+  __syncthreads();
+  uint32_t excl = warp_tot[w] + inc - sum;
+  if (2 * t < B) out[2 * t] = excl;
+  if (2 * t + 1 < B) out[2 * t + 1] = excl + x0;
+}
+
+template <int NV, int R>
+__global__ void __launch_bounds__(512) k_scatter(AggParams p, ScatterParams sp) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  const Layout& L = p.lay;
+  const uint32_t B = sp.B;
+  const uint32_t TILE = blockDim.x * R;
+  uint64_t* skey = (uint64_t*)sm;                       // TILE
+  uint64_t* sval = skey + TILE;                         // NV x TILE
+  uint64_t* gpos = sval + (size_t)NV * TILE;            // B
+  uint32_t* hist = (uint32_t*)(gpos + B);               // B
+  uint32_t* lstart = hist + B;                          // B
+  uint32_t* wtot = lstart + B;                          // 32
+  uint32_t* total = wtot + 32;                          // 1
+  uint16_t* sbid = (uint16_t*)(total + 4);              // TILE
+  const uint64_t pol = evict_first_policy();
+  const uint64_t n = p.n_rows;
+  const uint64_t ntiles = (n + TILE - 1) / TILE;
+  for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
+    __syncthreads();
+    const uint64_t row = lane_base<R>(t * TILE, threadIdx.x >> 5, threadIdx.x & 31);
+    uint64_t key[R];
+    const uint32_t valid = pack_keys<R>(p, row, n, pol, key);
+    uint64_t v[NV][R];
+#pragma unroll
+    for (int c = 0; c < NV; ++c)
+      if (c < L.n_vals) load_rows<R>(p.val[c], L.val_dtype[c], row, n, p.vec_ok, pol, v[c]);
+    uint32_t bb[R], pos[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      bb[r] = (uint32_t)((fmix64(key[r]) & p.cap_mask) >> sp.shift);
+      pos[r] = (valid >> r & 1) ? atomicAdd(&hist[bb[r]], 1u) : 0u;
+    }
+    __syncthreads();
+    block_excl_scan_512(hist, lstart, B, wtot, total);
+    for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
+      uint32_t h = hist[b];
+      if (h) {
+        uint64_t g = atomicAdd((unsigned long long*)&sp.cursor[b], (unsigned long long)h);
+        gpos[b] = g;
+        if (g + h > sp.seg_cap) atomicExch(sp.gate, 1u);
+      }
+    }
+    __syncthreads();  // lstart and gpos visible to every thread
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (valid >> r & 1) {
+        uint32_t e = lstart[bb[r]] + pos[r];
+        skey[e] = key[r];
+        sbid[e] = (uint16_t)bb[r];
+#pragma unroll
+        for (int c = 0; c < NV; ++c) sval[(size_t)c * TILE + e] = v[c][r];
+      }
+    __syncthreads();
+    const uint32_t tot = *total;
+    for (uint32_t e = threadIdx.x; e < tot; e += blockDim.x) {
+      const uint32_t b = sbid[e];
+      const uint64_t g = gpos[b] + (e - lstart[b]);
+      if (g >= sp.seg_cap) continue;
+      const uint64_t idx = sp.seg_base[b] + g;
+      sp.out_key[idx] = skey[e];
+#pragma unroll
+      for (int c = 0; c < NV; ++c)
+        if (c < L.n_vals) {
+          const uint64_t x = sval[(size_t)c * TILE + e];
+          if (L.val_dtype[c] == BLU_I32) ((int32_t*)sp.out_val[c])[idx] = (int32_t)(uint32_t)x;
+          else ((uint64_t*)sp.out_val[c])[idx] = x;
+        }
+    }
+    __syncthreads();
+  }
+}
+
+template <int NV, int R>
+static int launch_scatter_nv(const AggParams& p, const ScatterParams& sp, cudaStream_t st, uint32_t grid) {
+  const uint32_t TILE = 512 * R;
+  size_t smem = (size_t)TILE * 8 * (1 + NV) + (size_t)sp.B * 16 + 36 * 4 + 16 + (size_t)TILE * 2;
+  auto k = k_scatter<NV, R>;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e) return (int)e;
+  k<<<grid, 512, smem, st>>>(p, sp);
+  count_launch(1);
+  return (int)cudaGetLastError();
+}
+
+int launch_scatter(const AggParams& p, const ScatterParams& sp, void* stream, uint32_t grid) {
+  cudaStream_t st = (cudaStream_t)stream;
+  int nv = p.lay.n_vals;
+  if (nv <= 1) return launch_scatter_nv<1, 4>(p, sp, st, grid);
+  if (nv <= 2) return launch_scatter_nv<2, 4>(p, sp, st, grid);
+  if (nv <= 4) return launch_scatter_nv<4, 4>(p, sp, st, grid);
+  if (nv <= 8) return launch_scatter_nv<8, 2>(p, sp, st, grid);
+  return launch_scatter_nv<16, 1>(p, sp, st, grid);
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -864,11 +1025,12 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
     bool direct = path == BLU_PATH_DIRECT_GLOBAL;
     if constexpr (NV > 16) {  // merges of wide states: no front, no records
       if (records || front || direct) return (int)cudaErrorInvalidValue;
-      k = k_agg_global<NV, R, false, false, false>;
+      k = k_agg_global<NV, R, false, false, 0>;
     } else {
-      if (records) k = k_agg_global<NV, R, false, false, true>;
-      else if (direct) k = front ? k_agg_global<NV, R, true, true, false> : k_agg_global<NV, R, false, true, false>;
-      else k = front ? k_agg_global<NV, R, true, false, false> : k_agg_global<NV, R, false, false, false>;
+      if (records) k = k_agg_global<NV, R, false, false, 1>;
+      else if (p.seg_base) k = k_agg_global<NV, R, false, false, 2>;
+      else if (direct) k = front ? k_agg_global<NV, R, true, true, 0> : k_agg_global<NV, R, false, true, 0>;
+      else k = front ? k_agg_global<NV, R, true, false, 0> : k_agg_global<NV, R, false, false, 0>;
     }
     if (smem > 48 * 1024) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e) return (int)e;

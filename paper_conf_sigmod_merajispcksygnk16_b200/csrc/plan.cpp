@@ -53,6 +53,7 @@ constexpr uint64_t kMinCap = 1024;
 constexpr uint64_t kFrontRatio = 1000;          // rows/groups above which the front pays off
 constexpr uint32_t kFrontBudget = 110 * 1024;
 constexpr uint64_t kDirectMin = 1ull << 20;
+constexpr uint32_t kPartBudgetMB = 48;          // L2 slice per bucket (126 MB L2)
 
 static int32_t field_gsize(int kind) { return (kind == FK_MINI32 || kind == FK_MAXI32) ? 4 : 8; }
 static int32_t field_ssize(int kind) {
@@ -159,6 +160,11 @@ void fill_smem_layout(AggParams& p, uint32_t S, bool with_keys) {
     p.soff[j] = o;
     o += (S * (uint32_t)L.f[j].ssize + 15) / 16 * 16;
   }
+  p.seg_base = nullptr;
+  p.seg_count = nullptr;
+  p.n_segs = 0;
+  p.gate = nullptr;
+  p.gate_run_if = 0;
   for (int c = 0; c < kMaxFields; ++c) p.colmask[c] = 0;
   p.cntmask = 0;
   for (int j = 0; j < L.n_fields; ++j) {
@@ -299,6 +305,25 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     finish_layout(L);
   }
   P->cap = path == BLU_PATH_HASH_GLOBAL ? cap_est : D;
+
+  // Partitioned two-pass mode for path (b) when the table exceeds an L2-sized budget: rows are
+  // first scattered into B buckets by the top bits of their slot, then aggregated bucket by bucket
+  // so each bucket's slice of the table stays L2-resident (126 MB L2).
+  P->parts = 1;
+  P->part_shift = 0;
+  if (path == BLU_PATH_HASH_GLOBAL) {
+    uint64_t budget = (uint64_t)kPartBudgetMB << 20;
+    if (const char* pm = env("BLU_GBY_PART_MB")) budget = (uint64_t)atoi(pm) << 20;
+    uint64_t tbytes = P->cap * (uint64_t)L.slot_bytes;
+    uint64_t B = 1;
+    while (budget && B < 1024 && tbytes / B > budget && B < P->cap / 1024) B <<= 1;
+    if (const char* pp = env("BLU_GBY_PARTS")) B = std::max(1, atoi(pp));
+    P->parts = (uint32_t)B;
+    uint32_t lc = 0, lb = 0;
+    while ((1ull << lc) < P->cap) ++lc;
+    while ((1u << lb) < P->parts) ++lb;
+    P->part_shift = lc - lb;
+  }
 
   // hot-key front (path b / b')
   P->hot_front = 0;

@@ -313,3 +313,44 @@ def test_launch_count_and_timing(bg):
     bg.blu_gby_set_timing(False)
     assert c1 - c0 >= 4  # init, aggregate, compact x3
     assert t["aggregate_ms"] > 0 and t["aggregate_launches"] == 1
+
+
+@pytest.mark.parametrize("parts,chunk", [("8", None), ("16", "300000"), ("64", "1000003")])
+def test_partitioned_two_pass(bg, oracles, monkeypatch, parts, chunk):
+    """Path (b) partitioned mode: scatter into buckets by slot bits, then bucket-by-bucket
+    aggregation; several chunks; identical to the oracle."""
+    w, o = oracles("C3")
+    kc, vc = blugen.device_columns(w)
+    monkeypatch.setenv("BLU_GBY_PARTS", parts)
+    if chunk:
+        monkeypatch.setenv("BLU_GBY_PART_CHUNK", chunk)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    res = bg.blu_gby_execute(plan, kc, vc)
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
+def test_partitioned_skew_falls_back(bg, monkeypatch):
+    """A bucket overflow (every row in one bucket) takes the device-side fallback: still exact."""
+    n = 600_000
+    rng = np.random.default_rng(3)
+    sch = blugen.Schema([(I64, 0)], [I64, F64], [(COUNT, -1), (SUM, 0), (AVG, 1), (MIN, 0), (MAX, 1)])
+    k = np.where(rng.random(n) < 0.9, 77, rng.integers(0, 5000, n)).astype(np.int64)
+    v = [rng.integers(-(2**40), 2**40, n), rng.integers(-(2**20), 2**20, n) / 64.0]
+    o = oracle.groupby_arrays(sch, [k], v)
+    monkeypatch.setenv("BLU_GBY_PARTS", "16")
+    dk, dv = _mk([k], v)
+    plan = bg.plan_for(sch, 5000, n)
+    res = bg.blu_gby_execute(plan, dk, dv)
+    gk, ga = gpu_sorted(res, sch)
+    assert_parity(gk, ga, o, sch)
+
+
+def test_partitioned_with_regrow(bg, oracles, monkeypatch):
+    w, o = oracles("C5")
+    kc, vc = blugen.device_columns(w)
+    monkeypatch.setenv("BLU_GBY_PARTS", "4")
+    plan = bg.plan_for(w.schema, 1000, w.n_rows)  # under-estimate: partitioned + regrow
+    res = bg.blu_gby_execute(plan, kc, vc)
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
