@@ -380,6 +380,17 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   for (int c = 0; c < L.n_vals; ++c) row_bytes += dtype_bytes(L.val_dtype[c]);
   size_t free_b = 0, total_b = 0;
   cudaMemGetInfo(&free_b, &total_b);
+  {  // memory cached by the stream-ordered pool (reserved, not in use) is available too
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaMemPool_t pool;
+    uint64_t reserved = 0, used = 0;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess &&
+        cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved) == cudaSuccess &&
+        cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used) == cudaSuccess && reserved > used)
+      free_b += (size_t)(reserved - used);
+    cudaGetLastError();
+  }
   uint64_t budget_rows = (uint64_t)((double)free_b * 0.6 / (double)row_bytes / 1.03);
   uint64_t M = std::min<uint64_t>(n, std::max<uint64_t>(budget_rows, 1ull << 22));
   if (const char* cr = getenv("BLU_GBY_PART_CHUNK")) M = std::min<uint64_t>(n, std::max<uint64_t>(1024, strtoull(cr, 0, 10)));
