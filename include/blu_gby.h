@@ -122,9 +122,22 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* schema, uint64_t est_groups, u
  * (P:141 error path); hot_front: 1 if path (b) uses a per-CTA shared-memory hot-key front. */
 blu_status_t blu_gby_plan_info(blu_gby_plan_t plan, int32_t* path, uint64_t* capacity,
                                uint32_t* smem_bytes, uint32_t* retries_last);
-blu_status_t blu_gby_plan_info2(blu_gby_plan_t plan, uint32_t* slot_bytes, int32_t* hot_front,
-                                int32_t* n_states, int32_t* state_dtypes /* n_states, may be NULL */,
-                                uint32_t* grid, uint32_t* block);
+/* Full plan description (all fields filled). */
+typedef struct {
+    int32_t path;            /* blu_path_t                                                         */
+    uint64_t capacity;       /* hash slots (b) or dense domain D (a, b')                           */
+    uint64_t est_groups;     /* the clamped estimate the plan was sized from                      */
+    uint32_t slot_bytes;     /* global AoS slot (key + state fields, padded)                      */
+    uint32_t smem_bytes;     /* dynamic shared memory of the aggregation kernel                   */
+    int32_t hot_front;       /* 1: shared-memory hot-key front (b, b')                            */
+    uint32_t front_slots;
+    uint32_t partitions;     /* (b): buckets of the partitioned two-pass mode (1 = one pass)      */
+    int32_t n_states;        /* state fields (partial results / records)                         */
+    int32_t state_dtypes[32];/* blu_dtype_t of each state field                                   */
+    uint32_t grid, block;    /* aggregation launch shape                                          */
+    uint32_t retries_last;
+} blu_gby_plan_desc_t;
+blu_status_t blu_gby_plan_describe(blu_gby_plan_t plan, blu_gby_plan_desc_t* out);
 
 /* ---- execute -------------------------------------------------------------------------------
  * key_cols: n_keys DEVICE arrays of n_rows elements (dtype per schema); val_cols: n_vals DEVICE

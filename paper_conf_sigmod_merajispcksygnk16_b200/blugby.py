@@ -51,6 +51,14 @@ class ResultC(ctypes.Structure):
                 ("state_cols", ctypes.POINTER(ctypes.c_void_p)), ("_owner", ctypes.c_void_p)]
 
 
+class PlanDescC(ctypes.Structure):
+    _fields_ = [("path", ctypes.c_int32), ("capacity", ctypes.c_uint64), ("est_groups", ctypes.c_uint64),
+                ("slot_bytes", ctypes.c_uint32), ("smem_bytes", ctypes.c_uint32), ("hot_front", ctypes.c_int32),
+                ("front_slots", ctypes.c_uint32), ("partitions", ctypes.c_uint32), ("n_states", ctypes.c_int32),
+                ("state_dtypes", ctypes.c_int32 * 32), ("grid", ctypes.c_uint32), ("block", ctypes.c_uint32),
+                ("retries_last", ctypes.c_uint32)]
+
+
 class TimingC(ctypes.Structure):
     _fields_ = [("init_ms", ctypes.c_float), ("aggregate_ms", ctypes.c_float), ("compact_ms", ctypes.c_float),
                 ("h2d_ms", ctypes.c_float), ("total_ms", ctypes.c_float),
@@ -66,7 +74,7 @@ def _load():
     sigs = {
         "blu_gby_plan": ([P(SchemaC), u64, u64, P(vp)], i32),
         "blu_gby_plan_info": ([vp, P(i32), P(u64), P(u32), P(u32)], i32),
-        "blu_gby_plan_info2": ([vp, P(u32), P(i32), P(i32), P(i32), P(u32), P(u32)], i32),
+        "blu_gby_plan_describe": ([vp, P(PlanDescC)], i32),
         "blu_gby_execute": ([vp, P(vp), P(vp), u64, vp, P(ResultC)], i32),
         "blu_gby_execute_host": ([vp, P(vp), P(vp), u64, vp, P(ResultC)], i32),
         "blu_gby_execute_partial": ([vp, P(vp), P(vp), u64, vp, P(ResultC)], i32),
@@ -151,17 +159,12 @@ class Plan:
                 pass
 
     def info(self) -> dict:
-        path, cap, smem, retries = ctypes.c_int32(), ctypes.c_uint64(), ctypes.c_uint32(), ctypes.c_uint32()
-        _check(lib.blu_gby_plan_info(self.handle, ctypes.byref(path), ctypes.byref(cap), ctypes.byref(smem),
-                                     ctypes.byref(retries)))
-        sb, hf, ns, grid, block = (ctypes.c_uint32(), ctypes.c_int32(), ctypes.c_int32(), ctypes.c_uint32(),
-                                   ctypes.c_uint32())
-        sd = (ctypes.c_int32 * 32)()
-        _check(lib.blu_gby_plan_info2(self.handle, ctypes.byref(sb), ctypes.byref(hf), ctypes.byref(ns), sd,
-                                      ctypes.byref(grid), ctypes.byref(block)))
-        return dict(path=path.value, path_name=PATH_NAMES[path.value], capacity=cap.value, smem_bytes=smem.value,
-                    retries_last=retries.value, slot_bytes=sb.value, hot_front=hf.value, n_states=ns.value,
-                    state_dtypes=[sd[i] for i in range(ns.value)], grid=grid.value, block=block.value)
+        d = PlanDescC()
+        _check(lib.blu_gby_plan_describe(self.handle, ctypes.byref(d)))
+        out = {k: getattr(d, k) for k, _ in PlanDescC._fields_ if k != "state_dtypes"}
+        out["state_dtypes"] = [d.state_dtypes[i] for i in range(d.n_states)]
+        out["path_name"] = PATH_NAMES[d.path]
+        return out
 
     def dense_state_shape(self) -> Tuple[int, int, int, int, int]:
         a, b, c, d, D = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32(), ctypes.c_uint64()

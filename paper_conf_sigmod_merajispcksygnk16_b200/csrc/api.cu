@@ -86,7 +86,75 @@ struct Owner {
 
 static size_t dtype_bytes(int dt) { return dt == BLU_I32 ? 4 : 8; }
 
-// Stream-ordered workspace that frees itself.
+// Workspace cache (per process, per device): the hash table, dense state and partition buffers of
+// an execute come from blocks that are cudaMalloc'd once and reused by later executes — the B200
+// counterpart of the paper's "single large memory segment" registered up front and sub-allocated
+// per call. Re-mapping tens of GB of stream-ordered pool memory per query stalls the GPU.
+// A block is handed back only after the stream that used it has been synchronised (every entry
+// point synchronises before returning).
+struct CacheBlock {
+  void* p;
+  size_t bytes;
+  int dev;
+  bool busy;
+};
+static std::mutex g_cache_mu;
+static std::vector<CacheBlock> g_cache;
+
+static cudaError_t cache_get(void** out, size_t bytes) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  bytes = (bytes + (2u << 20) - 1) & ~(size_t)((2u << 20) - 1);
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  int best = -1;
+  for (int i = 0; i < (int)g_cache.size(); ++i) {
+    const CacheBlock& b = g_cache[i];
+    if (b.busy || b.dev != dev || b.bytes < bytes || b.bytes > 2 * bytes + (64u << 20)) continue;
+    if (best < 0 || b.bytes < g_cache[best].bytes) best = i;
+  }
+  if (best >= 0) {
+    g_cache[best].busy = true;
+    *out = g_cache[best].p;
+    return cudaSuccess;
+  }
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, bytes);
+  if (e == cudaErrorMemoryAllocation) {  // give idle cached blocks back and retry once
+    cudaGetLastError();
+    for (auto it = g_cache.begin(); it != g_cache.end();) {
+      if (!it->busy && it->dev == dev) {
+        cudaFree(it->p);
+        it = g_cache.erase(it);
+      } else {
+        ++it;
+      }
+    }
+    e = cudaMalloc(&p, bytes);
+  }
+  if (e != cudaSuccess) return e;
+  g_cache.push_back(CacheBlock{p, bytes, dev, true});
+  *out = p;
+  return cudaSuccess;
+}
+
+static size_t cache_idle_bytes() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  size_t t = 0;
+  for (auto& b : g_cache)
+    if (!b.busy && b.dev == dev) t += b.bytes;
+  return t;
+}
+
+static void cache_put(void* p) {
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  for (auto& b : g_cache)
+    if (b.p == p) b.busy = false;
+}
+
+// Scratch of one execute; released (to the cache) when destroyed, after the stream has been
+// synchronised by the caller.
 struct Work {
   cudaStream_t st;
   std::vector<void*> ptrs;
@@ -94,12 +162,12 @@ struct Work {
   cudaError_t alloc(void** p, size_t bytes) {
     *p = nullptr;
     if (!bytes) return cudaSuccess;
-    cudaError_t e = cudaMallocAsync(p, bytes, st);
+    cudaError_t e = cache_get(p, bytes);
     if (e == cudaSuccess) ptrs.push_back(*p);
     return e;
   }
   ~Work() {
-    for (void* p : ptrs) cudaFreeAsync(p, st);
+    for (void* p : ptrs) cache_put(p);
   }
 };
 
@@ -133,7 +201,7 @@ static OutSpec make_outspec(const blu_gby_plan_s* P, const Layout& lay, bool par
 }
 
 // Feeds every input batch to the aggregation kernel for one attempt. `base` carries the targets.
-using Feeder = std::function<cudaError_t(AggParams& base, uint32_t* launches)>;
+using Feeder = std::function<cudaError_t(AggParams& base, uint32_t* launches, Work& w)>;
 
 static bool ptr_aligned(const void* p) { return ((uintptr_t)p & 15) == 0; }
 
@@ -215,7 +283,7 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     base.flags = d_flags;
     fill_smem_layout(base, path == BLU_PATH_DENSE_SMEM ? (uint32_t)D : base.front_slots, base.front_slots > 0);
     uint32_t launches = 0;
-    CK(feed(base, &launches), "aggregate launch");
+    CK(feed(base, &launches, w), "aggregate launch");
     if (t_timing) cudaEventRecord(t_ev.e[2], st);
 
     // outputs, sized by the upper bound min(entries, rows)
@@ -391,6 +459,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       free_b += (size_t)(reserved - used);
     cudaGetLastError();
   }
+  free_b += cache_idle_bytes();  // idle workspace blocks are reusable
   uint64_t budget_rows = (uint64_t)((double)free_b * 0.6 / (double)row_bytes / 1.03);
   uint64_t M = std::min<uint64_t>(n, std::max<uint64_t>(budget_rows, 1ull << 22));
   if (const char* cr = getenv("BLU_GBY_PART_CHUNK")) M = std::min<uint64_t>(n, std::max<uint64_t>(1024, strtoull(cr, 0, 10)));
@@ -417,7 +486,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   L2.key_dtype[0] = BLU_I64;
   for (uint64_t r0 = 0; r0 < n; r0 += M) {
     const uint64_t m = std::min(M, n - r0);
-    if ((e = cudaMemsetAsync(d_cursor, 0, (size_t)B * 8 + 8, st))) return e;
+    if ((e = cudaMemsetAsync(d_cursor, 0, (size_t)B * 8 + 16, st))) return e;
     AggParams p1 = base;
     bool vec = true;
     for (int k = 0; k < L.n_keys; ++k) {
@@ -455,6 +524,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     p2.seg_base = d_seg_base;
     p2.seg_count = d_cursor;
     p2.n_segs = B;
+    p2.tile_ctr = getenv("BLU_GBY_DYN") && atoi(getenv("BLU_GBY_DYN")) == 0 ? nullptr : (uint64_t*)(d_cursor + B + 1);
     p2.gate = d_gate;
     p2.gate_run_if = 0;
     p2.front_slots = 0;
@@ -479,11 +549,9 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
   if (n && (!nonnull_cols(keys, P->lay.n_keys) || !nonnull_cols(vals, P->lay.n_vals)))
     return fail(BLU_E_INVALID, "NULL column pointer");
   const Layout& L = P->lay;
-  Feeder feed = [&](AggParams& base, uint32_t* launches) -> cudaError_t {
-    if (P->path == BLU_PATH_HASH_GLOBAL && P->parts > 1 && n >= 4096 * (uint64_t)P->parts) {
-      Work pw(st);
-      return partitioned_feed(P, base, keys, vals, n, st, launches, pw);
-    }
+  Feeder feed = [&](AggParams& base, uint32_t* launches, Work& w) -> cudaError_t {
+    if (P->path == BLU_PATH_HASH_GLOBAL && P->parts > 1 && n >= 4096 * (uint64_t)P->parts)
+      return partitioned_feed(P, base, keys, vals, n, st, launches, w);
     return agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, launches);
   };
   return run_core(P, L, P->path, P->hot_front != 0, P->cap, n, feed, partial, st, out, false, nullptr);
@@ -561,7 +629,7 @@ blu_status_t blu_gby_execute_host(blu_gby_plan_t P, const void* const* hkeys, co
     cudaEventCreate(&t1);
   }
   float h2d_ms = 0.f;
-  Feeder feed = [&](AggParams& base, uint32_t* launches) -> cudaError_t {
+  Feeder feed = [&](AggParams& base, uint32_t* launches, Work&) -> cudaError_t {
     if (!n) return cudaSuccess;
     cudaEventRecord(t0, st);
     cudaStreamWaitEvent(cs, t0, 0);  // staging buffers are allocated on st
@@ -618,7 +686,7 @@ static blu_status_t merge_impl(blu_gby_plan_t P, const blu_gby_result_t* parts, 
   uint64_t cap = 1024;
   while ((double)cap * 0.7 < (double)est) cap <<= 1;
   uint32_t grid = (uint32_t)P->sms * 8, block = 256;
-  Feeder feed = [&](AggParams& base, uint32_t* launches) -> cudaError_t {
+  Feeder feed = [&](AggParams& base, uint32_t* launches, Work&) -> cudaError_t {
     for (int i = 0; i < np; ++i) {
       if (!parts[i].n_groups) continue;
       cudaError_t e = agg_batch(P, BLU_PATH_HASH_GLOBAL, base, (const void* const*)parts[i].key_cols,
@@ -650,7 +718,7 @@ blu_status_t blu_gby_merge_records(blu_gby_plan_t P, const void* records, uint64
   while ((double)cap * 0.7 < (double)est) cap <<= 1;
   uint32_t grid = (uint32_t)P->sms * 8, block = 256;
   RecSrc rs{(const uint64_t*)records, (uint32_t)(1 + M.n_vals)};
-  Feeder feed = [&](AggParams& base, uint32_t* launches) -> cudaError_t {
+  Feeder feed = [&](AggParams& base, uint32_t* launches, Work&) -> cudaError_t {
     if (!n) return cudaSuccess;
     return agg_batch(P, BLU_PATH_HASH_GLOBAL, base, nullptr, nullptr, n, &rs, st, grid, block, 0, launches);
   };
@@ -698,7 +766,7 @@ blu_status_t blu_gby_finalize_dense_state(blu_gby_plan_t P, void* const* state_a
   cudaStream_t st = (cudaStream_t)stream;
   const Layout& L = P->lay;
   // Reuse run_core with a feeder that copies the caller's state in place of init+aggregate.
-  Feeder feed = [&](AggParams& base, uint32_t*) -> cudaError_t {
+  Feeder feed = [&](AggParams& base, uint32_t*, Work&) -> cudaError_t {
     for (int g = 0; g < 4; ++g) {
       size_t b = (size_t)L.n_group[g] * L.domain * 8;
       if (b) {

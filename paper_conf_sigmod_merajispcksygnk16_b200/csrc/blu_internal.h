@@ -126,6 +126,7 @@ struct AggParams {
   const uint64_t* seg_base;
   const uint64_t* seg_count;
   uint32_t n_segs;
+  uint64_t* tile_ctr;            // segments mode: dynamic warp-tile counter (zeroed per launch)
   // device-side gate: the kernel runs only if ((*gate != 0) == gate_run_if); NULL = always
   const uint32_t* gate;
   uint32_t gate_run_if;

@@ -491,9 +491,9 @@ __global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
   const Layout& L = p.lay;
   const uint32_t S = p.S;
   __shared__ uint64_t tpre[SEG ? 1025 : 1];
-  if constexpr (SEG) {  // tile prefix over the buckets (warp 0)
+  if constexpr (SEG) {  // warp-tile prefix over the buckets (warp 0)
     if (threadIdx.x < 32) {
-      const uint64_t tile = (uint64_t)blockDim.x * R;
+      const uint64_t tile = 32ull * R;
       uint64_t carry = 0;
       for (uint32_t b0 = 0; b0 < p.n_segs; b0 += 32) {
         uint32_t b = b0 + threadIdx.x;
@@ -516,15 +516,42 @@ __global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
     __syncthreads();
   }
   const uint64_t pol = evict_first_policy();
-  const uint64_t tile = (uint64_t)blockDim.x * R;
+  // SEG: warp tiles (32*R rows) handed out in bucket order by a global counter, so every warp of
+  // the grid stays inside the same one or two buckets (their table slices L2-resident); static
+  // grid-stride assignment lets CTAs drift several buckets apart and thrash L2.
+  const uint64_t tile = SEG ? 32ull * R : (uint64_t)blockDim.x * R;
   const uint64_t ntiles = SEG ? tpre[p.n_segs] : (p.n_rows + tile - 1) / tile;
+  const unsigned lane = threadIdx.x & 31;
   uint8_t* tb = (uint8_t*)p.table;
   uint32_t flag_seen = 0;
-  for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+  // SEG: a warp claims kGrab consecutive warp tiles per atomic (one counter for the whole grid)
+  constexpr uint32_t kGrab = 16;
+  uint64_t t = blockIdx.x, chunk = 0, chunk_next = 0;
+  uint32_t k_in = 0;
+  const bool dyn = SEG && p.tile_ctr != nullptr;
+  if (SEG && !dyn) t = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);  // static warp tiles
+  if (dyn) {
+    chunk = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;
+    chunk = __shfl_sync(0xffffffffu, chunk, 0);
+    chunk_next = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;  // prefetched
+    t = chunk * kGrab;
+  }
+  while (t < ntiles) {
     if (flag_seen) break;
     flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);  // warp-uniform abort
-    uint64_t n = p.n_rows, row0 = t * tile;
-    if constexpr (SEG) {  // bucket of tile t: largest b with tpre[b] <= t
+    uint64_t n = p.n_rows, row0 = t * tile, t_next = t + gridDim.x;
+    uint64_t row;
+    if constexpr (SEG) {  // bucket of warp tile t: largest b with tpre[b] <= t
+      if (!dyn) {
+        t_next = t + (uint64_t)gridDim.x * (blockDim.x >> 5);
+      } else if (++k_in < kGrab) {
+        t_next = t + 1;
+      } else {
+        k_in = 0;
+        chunk = __shfl_sync(0xffffffffu, chunk_next, 0);
+        t_next = chunk * kGrab;
+        chunk_next = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;
+      }
       uint32_t lo = 0, hi = p.n_segs - 1;
       while (lo < hi) {
         uint32_t mid = (lo + hi + 1) >> 1;
@@ -532,8 +559,10 @@ __global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
       }
       row0 = p.seg_base[lo] + (t - tpre[lo]) * tile;
       n = p.seg_base[lo] + p.seg_count[lo];
+      row = lane_base<R>(row0, 0, lane);
+    } else {
+      row = lane_base<R>(row0, threadIdx.x >> 5, lane);
     }
-    const uint64_t row = lane_base<R>(row0, threadIdx.x >> 5, threadIdx.x & 31);
     uint64_t key[R];
     uint64_t v[NV][R];
     uint32_t valid;
@@ -595,27 +624,59 @@ __global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
 #pragma unroll
       for (int r = 0; r < R; ++r) slot[r] = key[r];
     } else {
-      // issue the first key load of every row before resolving any (memory-level parallelism)
-      uint64_t first[R];
+      // Convergent multi-row probe: every pending row of the lane advances one slot per iteration
+      // and all their key loads are issued together (memory-level parallelism); the warp stays
+      // converged (__any_sync), so the REDs that follow are warp-wide.
+      uint64_t cur[R];
 #pragma unroll
       for (int r = 0; r < R; ++r) {
         slot[r] = fmix64(key[r]) & p.cap_mask;
-        first[r] = (miss >> r & 1) ? __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes)) : 0ull;
+        cur[r] = (miss >> r & 1) ? __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes)) : 0ull;
       }
+      uint32_t pending = miss;
+      for (uint32_t it = 0;; ++it) {
 #pragma unroll
-      for (int r = 0; r < R; ++r) {
-        if (!(miss >> r & 1)) continue;
-        uint64_t s;
-        if (hash_locate(tb, p.cap_mask, L.slot_bytes, key[r], first[r], slot[r], p.max_probe, s)) {
-          slot[r] = s;
-        } else {
-          miss &= ~(1u << r);
-          atomicOr(p.flags, FLAG_OVERFLOW);
+        for (int r = 0; r < R; ++r) {
+          if (!(pending >> r & 1)) continue;
+          if (cur[r] == key[r]) {
+            pending &= ~(1u << r);
+          } else {
+            if (cur[r] == kEmpty) {
+              unsigned long long old = atomicCAS((unsigned long long*)(tb + slot[r] * L.slot_bytes),
+                                                 (unsigned long long)kEmpty, (unsigned long long)key[r]);
+              if (old == kEmpty || old == key[r]) {
+                pending &= ~(1u << r);
+                continue;
+              }
+            }
+            slot[r] = (slot[r] + 1) & p.cap_mask;
+          }
         }
+        if (!__any_sync(0xffffffffu, pending)) break;
+        if (it + 1 >= 4) {
+          // long tails (a few rows per warp): finish them one lane at a time, then reconverge
+#pragma unroll
+          for (int r = 0; r < R; ++r) {
+            if (!(pending >> r & 1)) continue;
+            uint64_t sl;
+            const uint64_t c = __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes));
+            if (hash_locate(tb, p.cap_mask, L.slot_bytes, key[r], c, slot[r], p.max_probe, sl)) {
+              slot[r] = sl;
+            } else {  // the estimate was too small: flag, regrow, rerun
+              miss &= ~(1u << r);
+              atomicOr(p.flags, FLAG_OVERFLOW);
+            }
+          }
+          break;
+        }
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+          if (pending >> r & 1) cur[r] = __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes));
       }
       __syncwarp();  // reconverge before the field reductions so each RED instruction is warp-wide
     }
     global_apply_rows<NV, R, DIRECT>(p, slot, miss, v);
+    t = t_next;
   }
   if (FRONT) {
     // merge the front into the global table

@@ -49,6 +49,7 @@ static uint64_t next_pow2(uint64_t x) {
 // Planner constants (SURVEY.md §5 "Config / flags"; reading A16: the paper gives no values).
 constexpr uint32_t kSmemDenseMax = 96 * 1024;   // path (a): D x entry bytes, 2 CTAs/SM
 constexpr double kMaxLoad = 0.7;                // A5
+constexpr double kMaxLoadPart = 0.5;            // partitioned mode (buckets are L2-resident)
 constexpr uint64_t kMinCap = 1024;
 constexpr uint64_t kFrontRatio = 1000;          // rows/groups above which the front pays off
 constexpr uint32_t kFrontBudget = 110 * 1024;
@@ -318,6 +319,15 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     uint64_t B = 1;
     while (budget && B < 1024 && tbytes / B > budget && B < P->cap / 1024) B <<= 1;
     if (const char* pp = env("BLU_GBY_PARTS")) B = std::max(1, atoi(pp));
+    if (B > 1 && !env("BLU_GBY_PARTS")) {
+      // partitioned tables live in L2 one bucket at a time: trade HBM footprint for short probes
+      uint64_t cap2 = std::max<uint64_t>(kMinCap, next_pow2((uint64_t)((double)P->est_groups / kMaxLoadPart + 0.999999)));
+      if (cap2 > P->cap) {
+        P->cap = cap2;
+        tbytes = P->cap * (uint64_t)L.slot_bytes;
+        while (budget && B < 1024 && tbytes / B > budget && B < P->cap / 1024) B <<= 1;
+      }
+    }
     P->parts = (uint32_t)B;
     uint32_t lc = 0, lb = 0;
     while ((1ull << lc) < P->cap) ++lc;
@@ -395,16 +405,22 @@ blu_status_t blu_gby_plan_info(blu_gby_plan_t P, int32_t* path, uint64_t* capaci
   return BLU_OK;
 }
 
-blu_status_t blu_gby_plan_info2(blu_gby_plan_t P, uint32_t* slot_bytes, int32_t* hot_front, int32_t* n_states,
-                                int32_t* state_dtypes, uint32_t* grid, uint32_t* block) {
-  if (!P) return fail(BLU_E_INVALID, "NULL plan");
-  if (slot_bytes) *slot_bytes = P->lay.slot_bytes;
-  if (hot_front) *hot_front = P->hot_front;
-  if (n_states) *n_states = P->lay.n_fields;
-  if (state_dtypes)
-    for (int j = 0; j < P->lay.n_fields; ++j) state_dtypes[j] = P->merge_lay.val_dtype[j];
-  if (grid) *grid = P->grid;
-  if (block) *block = P->block;
+blu_status_t blu_gby_plan_describe(blu_gby_plan_t P, blu_gby_plan_desc_t* o) {
+  if (!P || !o) return fail(BLU_E_INVALID, "NULL plan or out");
+  memset(o, 0, sizeof *o);
+  o->path = P->path;
+  o->capacity = P->cap;
+  o->est_groups = P->est_groups;
+  o->slot_bytes = P->lay.slot_bytes;
+  o->smem_bytes = P->smem_bytes;
+  o->hot_front = P->hot_front;
+  o->front_slots = P->front_slots;
+  o->partitions = P->parts;
+  o->n_states = P->lay.n_fields;
+  for (int j = 0; j < P->lay.n_fields && j < 32; ++j) o->state_dtypes[j] = P->merge_lay.val_dtype[j];
+  o->grid = P->grid;
+  o->block = P->block;
+  o->retries_last = P->retries_last.load();
   return BLU_OK;
 }
 

@@ -77,18 +77,27 @@ def test_planner_paths_for_the_five_configs(bg):
     c5 = _plan(bg, blugen.workload("C5")).info()
     assert c1["path"] == c2["path"] == bg.BLU_PATH_DENSE_SMEM
     assert c1["capacity"] == 16 and c2["capacity"] == 1024
-    assert c3["path"] == bg.BLU_PATH_HASH_GLOBAL and c3["capacity"] == 2**24 and c3["slot_bytes"] == 32
+    # C3: 537 MB at load 0.6 exceeds the L2 budget -> partitioned mode, sized at load <= 0.5
+    assert c3["path"] == bg.BLU_PATH_HASH_GLOBAL and c3["capacity"] == 2**25 and c3["slot_bytes"] == 32
+    assert c3["partitions"] >= 16 and c3["capacity"] * 32 // c3["partitions"] <= 48 * 2**20
     assert c3["hot_front"] == 0
     assert c4["path"] == bg.BLU_PATH_DIRECT_GLOBAL and c4["capacity"] == 100_000 and c4["hot_front"] == 1
-    assert c5["path"] == bg.BLU_PATH_HASH_GLOBAL and c5["capacity"] == 2**27
+    assert c5["path"] == bg.BLU_PATH_HASH_GLOBAL and c5["capacity"] == 2**27 and c5["partitions"] >= 64
+    assert c1["partitions"] == c2["partitions"] == c4["partitions"] == 1
 
 
 @pytest.mark.parametrize("est,cap", [(1, 1024), (700, 1024), (716, 1024), (717, 2048), (10_000_000, 2**24),
                                      (50_000_000, 2**27)])
-def test_capacity_rounding(bg, est, cap):
-    """cap = next_pow2(ceil(max(est,1)/0.7)), >= 1024 ("slightly larger", reading A5)."""
+def test_capacity_rounding(bg, monkeypatch, est, cap):
+    """cap = next_pow2(ceil(max(est,1)/0.7)), >= 1024 (P:151 "slightly larger", reading A5);
+    one-pass mode (the partitioned mode sizes its L2-resident buckets at load <= 0.5)."""
+    monkeypatch.setenv("BLU_GBY_PART_MB", "0")
     p = bg.blu_gby_plan([(I64, 0)], [I64], [(SUM, 0)], est, 10**10)
-    assert p.info()["capacity"] == cap
+    assert p.info()["capacity"] == cap and p.info()["partitions"] == 1
+    monkeypatch.delenv("BLU_GBY_PART_MB")
+    p2 = bg.blu_gby_plan([(I64, 0)], [I64], [(SUM, 0)], est, 10**10)
+    if p2.info()["partitions"] > 1:
+        assert p2.info()["capacity"] >= 2 * est
 
 
 def test_est_clamped_to_rows(bg):

@@ -11,10 +11,10 @@ torch.cuda.synchronize()
 plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
 print(json.dumps(plan.info()))
 bg.blu_gby_set_timing(True)
-for i in range(4):
+for i in range(int(os.environ.get('ITERS', '4'))):
     t0 = time.perf_counter()
     r = bg.blu_gby_execute(plan, kc, vc)
     t1 = time.perf_counter()
     t = bg.blu_gby_last_timing()
-    print(f"wall {1000*(t1-t0):8.2f} ms  init {t['init_ms']:.2f} agg {t['aggregate_ms']:.2f} compact {t['compact_ms']:.2f} launches {t['aggregate_launches']} groups {r.n_groups}")
+    print(f"wall {1000*(t1-t0):8.2f} ms  init {t['init_ms']:.2f} agg {t['aggregate_ms']:.2f} compact {t['compact_ms']:.2f} launches {t['aggregate_launches']} retries {t['retries']} groups {r.n_groups}")
     del r
