@@ -532,6 +532,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     if (le) return (cudaError_t)le;
     // fallback one-pass over the chunk's rows (runs only if a bucket overflowed)
     AggParams p3 = p1;
+    p3.jit_ok = 0;  // gated fallback, normally a no-op: keep the precompiled kernel
     p3.gate = d_gate;
     p3.gate_run_if = 1;
     le = launch_aggregate_impl(P, BLU_PATH_HASH_GLOBAL, p3, RecSrc{nullptr, 0}, false, st, P->grid, P->block,
@@ -550,6 +551,7 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
     return fail(BLU_E_INVALID, "NULL column pointer");
   const Layout& L = P->lay;
   Feeder feed = [&](AggParams& base, uint32_t* launches, Work& w) -> cudaError_t {
+    base.jit_ok = 1;
     if (P->path == BLU_PATH_HASH_GLOBAL && P->parts > 1 && n >= 4096 * (uint64_t)P->parts)
       return partitioned_feed(P, base, keys, vals, n, st, launches, w);
     return agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, launches);
@@ -631,6 +633,7 @@ blu_status_t blu_gby_execute_host(blu_gby_plan_t P, const void* const* hkeys, co
   float h2d_ms = 0.f;
   Feeder feed = [&](AggParams& base, uint32_t* launches, Work&) -> cudaError_t {
     if (!n) return cudaSuccess;
+    base.jit_ok = 1;
     cudaEventRecord(t0, st);
     cudaStreamWaitEvent(cs, t0, 0);  // staging buffers are allocated on st
     uint64_t nchunks = (n + chunk - 1) / chunk;
@@ -750,6 +753,7 @@ blu_status_t blu_gby_execute_dense_state(blu_gby_plan_t P, const void* const* ke
   base.front_slots = P->hot_front ? P->front_slots : 0;
   base.flags = (uint32_t*)small;
   fill_smem_layout(base, P->path == BLU_PATH_DENSE_SMEM ? (uint32_t)L.domain : base.front_slots, base.front_slots > 0);
+  base.jit_ok = 1;
   CK(agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, nullptr), "aggregate");
   uint64_t* hs = pinned_scratch();
   uint64_t hb[2] = {0, 0};

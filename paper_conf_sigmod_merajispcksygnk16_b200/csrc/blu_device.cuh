@@ -1,0 +1,853 @@
+// blu_device.cuh — libblugby's device code: helpers and the bodies of the hot kernels.
+//
+// Compiled twice: ahead of time by nvcc into libblugby.so with GenericSpec (the schema is read from
+// the kernel parameters at run time), and at run time by NVRTC with a per-plan JitSpec whose key
+// dtypes, dictionary strides, value dtypes and state-field program are compile-time constants
+// (jit.cpp). The same source therefore produces both the generic kernels and the specialised,
+// straight-line ones. No host headers: under NVRTC the integer typedefs come from the JIT preamble.
+#pragma once
+
+#ifndef BLU_JIT
+#include "blu_params.h"
+#endif
+
+namespace blu {
+
+// Schema read from AggParams::lay at run time.
+struct GenericSpec {
+  static constexpr bool kStatic = false;
+};
+
+// ------------------------------------------------------------------------------------------------
+// device helpers
+// ------------------------------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t fmix64(uint64_t h) {  // Murmur3 finalizer (P:153 cites Murmur)
+  h ^= h >> 33;
+  h *= 0xff51afd7ed558ccdull;
+  h ^= h >> 33;
+  h *= 0xc4ceb9fe1a85ec53ull;
+  h ^= h >> 33;
+  return h;
+}
+
+// Order-preserving map of IEEE-754 f64 bits onto int64 (an involution).
+__device__ __forceinline__ int64_t ord_f64(uint64_t bits) {
+  int64_t b = (int64_t)bits;
+  return b ^ ((b >> 63) & 0x7FFFFFFFFFFFFFFFll);
+}
+__device__ __forceinline__ uint64_t unord_f64(int64_t o) { return (uint64_t)(o ^ ((o >> 63) & 0x7FFFFFFFFFFFFFFFll)); }
+
+__device__ __forceinline__ uint64_t evict_first_policy() {
+  uint64_t pol;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+__device__ __forceinline__ int4 ld_stream_v4(const void* p, uint64_t pol) {
+  int4 r;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], %5;"
+      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+      : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ int32_t ld_stream_s32(const void* p, uint64_t pol) {
+  int32_t r;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ uint64_t ld_stream_u64(const void* p, uint64_t pol) {
+  uint64_t r;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(r) : "l"(p), "l"(pol));
+  return r;
+}
+
+// Row mapping: a warp owns 32*R consecutive rows; lane l owns rows lb + (r>>1)*64 + (r&1) for
+// R = 4 (pairs 2l, 2l+1 and 64+2l, 65+2l), lb + r for R = 2, lb for R = 1, with lb the lane base
+// below. Every load instruction of a warp then covers one contiguous span (256 B for i32 pairs,
+// 512 B for 8-byte pairs): whole 32-byte sectors, no half-sector re-requests.
+template <int R, bool PAIR = true>
+__device__ __forceinline__ uint64_t lane_base(uint64_t tile_row0, unsigned warp, unsigned lane) {
+  if (!PAIR) return tile_row0 + ((uint64_t)warp * 32 + lane) * R;  // quad: R consecutive rows
+  return tile_row0 + (uint64_t)warp * 32 * R + (R >= 2 ? 2 * lane : lane);
+}
+template <int R, bool PAIR = true>
+__device__ __forceinline__ uint64_t row_of(uint64_t lb, int r) {
+  if (!PAIR) return lb + r;
+  return R == 4 ? lb + (uint64_t)(r >> 1) * 64 + (r & 1) : lb + r;
+}
+
+__device__ __forceinline__ int2 ld_stream_v2(const void* p, uint64_t pol) {
+  int2 r;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.s32 {%0,%1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(p), "l"(pol));
+  return r;
+}
+
+// Load this lane's R rows of one column as 64-bit patterns (i32 sign-extended). Rows >= n read 0.
+template <int R, bool PAIR = true>
+__device__ __forceinline__ void load_rows(const void* base, int dt, uint64_t lb, uint64_t n, bool vec,
+                                          uint64_t pol, uint64_t (&out)[R]) {
+  if (!PAIR && R == 4) {  // quad mapping: rows lb..lb+3 (path (a): one 16-byte load per i32 column)
+    if (dt == BLU_I32) {
+      const int32_t* p = (const int32_t*)base + lb;
+      if (vec && lb + 4 <= n) {
+        int4 v = ld_stream_v4(p, pol);
+        out[0] = (uint64_t)(int64_t)v.x;
+        out[1 % R] = (uint64_t)(int64_t)v.y;
+        out[2 % R] = (uint64_t)(int64_t)v.z;
+        out[3 % R] = (uint64_t)(int64_t)v.w;
+      } else {
+#pragma unroll
+        for (int r = 0; r < R; ++r) out[r] = lb + r < n ? (uint64_t)(int64_t)ld_stream_s32(p + r, pol) : 0ull;
+      }
+    } else {
+      const uint64_t* p = (const uint64_t*)base + lb;
+      if (vec && lb + 4 <= n) {
+#pragma unroll
+        for (int r = 0; r < R; r += 2) {
+          int4 v = ld_stream_v4(p + r, pol);
+          out[r] = (uint64_t)(uint32_t)v.x | ((uint64_t)(uint32_t)v.y << 32);
+          out[(r + 1) % R] = (uint64_t)(uint32_t)v.z | ((uint64_t)(uint32_t)v.w << 32);
+        }
+      } else {
+#pragma unroll
+        for (int r = 0; r < R; ++r) out[r] = lb + r < n ? ld_stream_u64(p + r, pol) : 0ull;
+      }
+    }
+    return;
+  }
+  if (dt == BLU_I32) {
+    const int32_t* p = (const int32_t*)base;
+    if (R >= 2) {
+#pragma unroll
+      for (int h = 0; h < R / 2; ++h) {
+        const uint64_t r0 = lb + (uint64_t)h * 64;
+        if (vec && r0 + 1 < n) {
+          int2 v = ld_stream_v2(p + r0, pol);
+          out[2 * h] = (uint64_t)(int64_t)v.x;
+          out[(2 * h + 1) % R] = (uint64_t)(int64_t)v.y;
+        } else {
+          out[2 * h] = r0 < n ? (uint64_t)(int64_t)ld_stream_s32(p + r0, pol) : 0ull;
+          out[(2 * h + 1) % R] = r0 + 1 < n ? (uint64_t)(int64_t)ld_stream_s32(p + r0 + 1, pol) : 0ull;
+        }
+      }
+    } else {
+      out[0] = lb < n ? (uint64_t)(int64_t)ld_stream_s32(p + lb, pol) : 0ull;
+    }
+  } else {
+    const uint64_t* p = (const uint64_t*)base;
+    if (R >= 2) {
+#pragma unroll
+      for (int h = 0; h < R / 2; ++h) {
+        const uint64_t r0 = lb + (uint64_t)h * 64;
+        if (vec && r0 + 1 < n) {
+          int4 v = ld_stream_v4(p + r0, pol);
+          out[2 * h] = (uint64_t)(uint32_t)v.x | ((uint64_t)(uint32_t)v.y << 32);
+          out[(2 * h + 1) % R] = (uint64_t)(uint32_t)v.z | ((uint64_t)(uint32_t)v.w << 32);
+        } else {
+          out[2 * h] = r0 < n ? ld_stream_u64(p + r0, pol) : 0ull;
+          out[(2 * h + 1) % R] = r0 + 1 < n ? ld_stream_u64(p + r0 + 1, pol) : 0ull;
+        }
+      }
+    } else {
+      out[0] = lb < n ? ld_stream_u64(p + lb, pol) : 0ull;
+    }
+  }
+}
+
+// Identity (the mask value of P:151) of a field in its encoded 64-bit form.
+__device__ __forceinline__ uint64_t identity64(int k) {
+  switch (k) {
+    case FK_MINI32: return (uint64_t)(int64_t)INT32_MAX;
+    case FK_MAXI32: return (uint64_t)(int64_t)INT32_MIN;
+    case FK_MINI64: case FK_MINF64: return (uint64_t)INT64_MAX;
+    case FK_MAXI64: case FK_MAXF64: return (uint64_t)INT64_MIN;
+    default: return 0ull;
+  }
+}
+
+// ---- per-field update primitives, specialised on the field kind at compile time ----------------
+// The kind of every field is warp-uniform, so kernels dispatch ONCE per field per tile (a uniform
+// switch) and then run straight-line updates for all R rows of the tile.
+template <int K>
+struct KC {
+  static constexpr int v = K;
+};
+
+// Compile-time loop: f(KC<I>{}) for I in [B, E).
+template <int B, int E, class F>
+__device__ __forceinline__ void sfor(F&& f) {
+  if constexpr (B < E) {
+    f(KC<B>{});
+    sfor<B + 1, E>(f);
+  }
+}
+
+template <class Fn>
+__device__ __forceinline__ void dispatch_kind(int kind, Fn&& fn) {
+  switch (kind) {
+    case FK_COUNT: fn(KC<FK_COUNT>{}); break;
+    case FK_SUMI: fn(KC<FK_SUMI>{}); break;
+    case FK_SUMF: fn(KC<FK_SUMF>{}); break;
+    case FK_MINI32: fn(KC<FK_MINI32>{}); break;
+    case FK_MAXI32: fn(KC<FK_MAXI32>{}); break;
+    case FK_MINI64: fn(KC<FK_MINI64>{}); break;
+    case FK_MAXI64: fn(KC<FK_MAXI64>{}); break;
+    case FK_MINF64: fn(KC<FK_MINF64>{}); break;
+    default: fn(KC<FK_MAXF64>{}); break;
+  }
+}
+
+// Encoded value of a field: f64 MIN/MAX through ord_f64 (RAW row values only).
+template <int K, bool RAW>
+__device__ __forceinline__ uint64_t enc(uint64_t x) {
+  if (RAW && (K == FK_MINF64 || K == FK_MAXF64)) return (uint64_t)ord_f64(x);
+  return x;
+}
+
+// Shared-memory table (path (a) and the hot-key front): SoA per field, S entries per field.
+// Encodings: COUNT u32; SUMI as two u32 arrays lo[S], hi[S] — native 32-bit ATOMS with an explicit
+// carry (64-bit shared atomics are CAS loops on sm_100a); SUMF f64 (CAS loop);
+// MIN/MAX i32 native ATOMS.MIN/MAX; 64-bit MIN/MAX read first, atomic only if it improves (after
+// warm-up a running min/max almost never changes, so almost every row costs one LDS).
+template <int K, bool RAW>
+__device__ __forceinline__ void s_upd(uint8_t* base, uint32_t e, uint32_t S, uint64_t x) {
+  x = enc<K, RAW>(x);
+  if constexpr (K == FK_COUNT) {
+    atomicAdd((uint32_t*)base + e, (uint32_t)x);
+  } else if constexpr (K == FK_SUMI) {
+    uint32_t lo = (uint32_t)x, hi = (uint32_t)(x >> 32);
+    uint32_t old = atomicAdd((uint32_t*)base + e, lo);
+    hi += (uint32_t)(old + lo < old);
+    if (hi) atomicAdd((uint32_t*)base + S + e, hi);
+  } else if constexpr (K == FK_SUMF) {
+    atomicAdd((double*)base + e, __longlong_as_double((long long)x));
+  } else if constexpr (K == FK_MINI32) {
+    int v = (int)x;
+    int* q = (int*)base + e;
+    if (v < *(volatile int*)q) atomicMin(q, v);
+  } else if constexpr (K == FK_MAXI32) {
+    int v = (int)x;
+    int* q = (int*)base + e;
+    if (v > *(volatile int*)q) atomicMax(q, v);
+  } else if constexpr (K == FK_MINI64 || K == FK_MINF64) {
+    long long v = (long long)x;
+    long long* q = (long long*)base + e;
+    if (v < *(volatile long long*)q) atomicMin(q, v);
+  } else {
+    long long v = (long long)x;
+    long long* q = (long long*)base + e;
+    if (v > *(volatile long long*)q) atomicMax(q, v);
+  }
+}
+
+__device__ __forceinline__ void smem_init_entry(uint8_t* base, int k, uint32_t e, uint32_t S) {
+  switch (k) {
+    case FK_COUNT: ((uint32_t*)base)[e] = 0u; break;
+    case FK_SUMI: ((uint32_t*)base)[e] = 0u; ((uint32_t*)base)[S + e] = 0u; break;
+    case FK_SUMF: ((uint64_t*)base)[e] = 0ull; break;
+    case FK_MINI32: ((int*)base)[e] = INT32_MAX; break;
+    case FK_MAXI32: ((int*)base)[e] = INT32_MIN; break;
+    default: ((uint64_t*)base)[e] = identity64(k); break;
+  }
+}
+
+// A shared-memory entry's state as the encoded 64-bit value to combine into global memory.
+template <int K>
+__device__ __forceinline__ uint64_t s_read(const uint8_t* base, uint32_t e, uint32_t S) {
+  if constexpr (K == FK_COUNT) return (uint64_t)((const uint32_t*)base)[e];
+  else if constexpr (K == FK_SUMI)
+    return (uint64_t)((const uint32_t*)base)[e] | ((uint64_t)((const uint32_t*)base)[S + e] << 32);
+  else if constexpr (K == FK_MINI32 || K == FK_MAXI32) return (uint64_t)(int64_t)((const int*)base)[e];
+  else return ((const uint64_t*)base)[e];
+}
+
+// Global AoS slot field (path b): fire-and-forget reductions REDG.E.ADD.64 / ADD.F64 / MIN.S64 ...
+template <int K, bool RAW>
+__device__ __forceinline__ void g_upd(uint8_t* a, uint64_t x) {
+  x = enc<K, RAW>(x);
+  if constexpr (K == FK_COUNT || K == FK_SUMI) atomicAdd((unsigned long long*)a, (unsigned long long)x);
+  else if constexpr (K == FK_SUMF) atomicAdd((double*)a, __longlong_as_double((long long)x));
+  else if constexpr (K == FK_MINI32) atomicMin((int*)a, (int)x);
+  else if constexpr (K == FK_MAXI32) atomicMax((int*)a, (int)x);
+  else if constexpr (K == FK_MINI64 || K == FK_MINF64) atomicMin((long long*)a, (long long)x);
+  else atomicMax((long long*)a, (long long)x);
+}
+
+// Global dense state field (paths a / b'): every field 8 bytes (i32 MIN/MAX widened).
+template <int K, bool RAW>
+__device__ __forceinline__ void d_upd(uint64_t* a, uint64_t x) {
+  x = enc<K, RAW>(x);
+  if constexpr (K == FK_COUNT || K == FK_SUMI) atomicAdd((unsigned long long*)a, (unsigned long long)x);
+  else if constexpr (K == FK_SUMF) atomicAdd((double*)a, __longlong_as_double((long long)x));
+  else if constexpr (K == FK_MINI32 || K == FK_MINI64 || K == FK_MINF64) atomicMin((long long*)a, (long long)x);
+  else atomicMax((long long*)a, (long long)x);
+}
+
+__device__ __forceinline__ uint64_t* dense_addr(const AggParams& p, int j, uint64_t g) {
+  const Field& f = p.lay.f[j];
+  return (uint64_t*)p.dense[f.sgroup] + (uint64_t)f.sidx * p.lay.domain + g;
+}
+
+// Linear probing from fmix64(key) & mask; read-before-CAS; keys are write-once (EMPTY -> key), so
+// a stale read can only show EMPTY and the CAS resolves it ("next empty slot").
+__device__ __forceinline__ bool hash_locate(uint8_t* table, uint64_t mask, uint32_t sb, uint64_t key,
+                                            uint64_t first, uint64_t idx, uint32_t max_probe, uint64_t& out) {
+  uint64_t cur = first;
+  for (uint32_t p = 0; p < max_probe; ++p) {
+    unsigned long long* kp = (unsigned long long*)(table + idx * sb);
+    if (p) cur = __ldcg(kp);
+    if (cur == key) { out = idx; return true; }
+    if (cur == kEmpty) {
+      unsigned long long old = atomicCAS(kp, (unsigned long long)kEmpty, (unsigned long long)key);
+      if (old == kEmpty || old == key) { out = idx; return true; }
+    }
+    idx = (idx + 1) & mask;
+  }
+  return false;
+}
+
+// Pack the key columns of rows [row, row+R) (S1, CCAT P:111): sparse -> code; dense -> mixed radix
+// sum code_j * stride_j. Invalid codes raise FLAG_KEY_RANGE; rows >= n are not valid.
+template <class SP, int R, bool PAIR = true>
+__device__ __forceinline__ uint32_t pack_keys(const AggParams& p, uint64_t row, uint64_t n, uint64_t pol,
+                                              uint64_t (&key)[R]) {
+  uint32_t valid = 0;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    key[r] = 0;
+    if (row_of<R, PAIR>(row, r) < n) valid |= 1u << r;
+  }
+  uint32_t bad = 0;
+  if constexpr (SP::kStatic) {  // JIT: key dtypes, dictionary sizes and strides are constants
+    if constexpr (SP::SPARSE) {
+      uint64_t c[R];
+      constexpr int dt = SP::KDT[0];
+      load_rows<R, PAIR>(p.key[0], dt, row, n, p.vec_ok, pol, c);
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        key[r] = c[r];
+        if ((int64_t)c[r] < 0) bad |= 1u << r;
+      }
+    } else {
+      sfor<0, SP::NK>([&](auto kc) {
+        constexpr int k = decltype(kc)::v;
+        constexpr int dt = SP::KDT[k];
+        constexpr uint64_t d = SP::DICT[k], st = SP::STRIDE[k];
+        uint64_t c[R];
+        load_rows<R, PAIR>(p.key[k], dt, row, n, p.vec_ok, pol, c);
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (c[r] >= d) bad |= 1u << r;
+          key[r] += c[r] * st;
+        }
+      });
+    }
+  } else if (p.lay.sparse) {
+    uint64_t c[R];
+    load_rows<R, PAIR>(p.key[0], p.lay.key_dtype[0], row, n, p.vec_ok, pol, c);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      key[r] = c[r];
+      if ((int64_t)c[r] < 0) bad |= 1u << r;
+    }
+  } else {
+    for (int k = 0; k < p.lay.n_keys; ++k) {
+      uint64_t c[R];
+      load_rows<R, PAIR>(p.key[k], p.lay.key_dtype[k], row, n, p.vec_ok, pol, c);
+      const uint64_t d = p.lay.dict[k], s = p.lay.stride[k];
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        if (c[r] >= d) bad |= 1u << r;  // unsigned: negatives are huge
+        key[r] += c[r] * s;
+      }
+    }
+  }
+  bad &= valid;
+  if (bad) atomicOr(p.flags, FLAG_KEY_RANGE);
+  return valid & ~bad;
+}
+
+// Load this lane's rows of every value column (JIT: dtypes are constants).
+template <class SP, int NV, int R, bool PAIR = true>
+__device__ __forceinline__ void load_vals(const AggParams& p, uint64_t row, uint64_t n, uint64_t pol,
+                                          uint64_t (&v)[NV][R]) {
+  if constexpr (SP::kStatic) {
+    sfor<0, SP::NV>([&](auto cc) {
+      constexpr int c = decltype(cc)::v;
+      constexpr int dt = SP::VDT[c];
+      load_rows<R, PAIR>(p.val[c], dt, row, n, p.vec_ok, pol, v[c]);
+    });
+  } else {
+#pragma unroll
+    for (int c = 0; c < NV; ++c)
+      if (c < p.lay.n_vals) load_rows<R, PAIR>(p.val[c], p.lay.val_dtype[c], row, n, p.vec_ok, pol, v[c]);
+  }
+}
+
+// Apply every field to the rows in `mask` of a shared-memory table at entries e[r].
+template <class SP, int NV, int R>
+__device__ __forceinline__ void smem_apply_rows(const AggParams& p, uint8_t* sm, const uint32_t (&e)[R],
+                                                uint32_t mask, const uint64_t (&v)[NV][R]) {
+  const uint32_t S = p.S;
+  if constexpr (SP::kStatic) {  // JIT: one straight-line update per (field, row)
+    sfor<0, SP::NF>([&](auto jc) {
+      constexpr int j = decltype(jc)::v;
+      constexpr int K = SP::KIND[j], c = SP::COL[j];
+      uint8_t* b = sm + p.soff[j];
+#pragma unroll
+      for (int r = 0; r < R; ++r)
+        if (mask >> r & 1) {
+          if constexpr (c < 0) s_upd<FK_COUNT, true>(b, e[r], S, 1ull);
+          else s_upd<K, true>(b, e[r], S, v[c][r]);
+        }
+    });
+    return;
+  }
+  for (uint32_t m = p.cntmask; m; m &= m - 1) {
+    uint8_t* b = sm + p.soff[__ffs(m) - 1];
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (mask >> r & 1) s_upd<FK_COUNT, true>(b, e[r], S, 1ull);
+  }
+#pragma unroll
+  for (int c = 0; c < NV; ++c) {
+    if (c >= p.lay.n_vals) break;
+    for (uint32_t m = p.colmask[c]; m; m &= m - 1) {
+      const int j = __ffs(m) - 1;
+      uint8_t* b = sm + p.soff[j];
+      dispatch_kind(p.lay.f[j].kind, [&](auto kc) {
+        constexpr int K = decltype(kc)::v;
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+          if (mask >> r & 1) s_upd<K, true>(b, e[r], S, v[c][r]);
+      });
+    }
+  }
+}
+
+// Apply every field to the rows in `mask` of the global target: AoS slots (hash) or dense state.
+template <class SP, int NV, int R, bool DIRECT>
+__device__ __forceinline__ void global_apply_rows(const AggParams& p, const uint64_t (&slot)[R], uint32_t mask,
+                                                  const uint64_t (&v)[NV][R]) {
+  const Layout& L = p.lay;
+  uint8_t* tb = (uint8_t*)p.table;
+  if constexpr (SP::kStatic) {  // JIT: slot size, field offsets and dense groups are constants
+    sfor<0, SP::NF>([&](auto jc) {
+      constexpr int j = decltype(jc)::v;
+      constexpr int K = SP::KIND[j], c = SP::COL[j], KK = c < 0 ? FK_COUNT : K;
+      constexpr int sg = SP::SGROUP[j], goff = SP::GOFF[j];
+      constexpr uint64_t base = (uint64_t)SP::SIDX[j] * SP::DOMAIN, slot_b = SP::SLOT;
+#pragma unroll
+      for (int r = 0; r < R; ++r)
+        if (mask >> r & 1) {
+          const uint64_t x = c < 0 ? 1ull : v[c < 0 ? 0 : c][r];
+          if constexpr (DIRECT) d_upd<KK, true>((uint64_t*)p.dense[sg] + base + slot[r], x);
+          else g_upd<KK, true>(tb + slot[r] * slot_b + goff, x);
+        }
+    });
+    return;
+  }
+  for (uint32_t m = p.cntmask; m; m &= m - 1) {
+    const int j = __ffs(m) - 1;
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (mask >> r & 1) {
+        if (DIRECT) d_upd<FK_COUNT, true>(dense_addr(p, j, slot[r]), 1ull);
+        else g_upd<FK_COUNT, true>(tb + slot[r] * L.slot_bytes + L.f[j].goff, 1ull);
+      }
+  }
+#pragma unroll
+  for (int c = 0; c < NV; ++c) {
+    if (c >= L.n_vals) break;
+    for (uint32_t m = p.colmask[c]; m; m &= m - 1) {
+      const int j = __ffs(m) - 1;
+      dispatch_kind(L.f[j].kind, [&](auto kc) {
+        constexpr int K = decltype(kc)::v;
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+          if (mask >> r & 1) {
+            if (DIRECT) d_upd<K, true>(dense_addr(p, j, slot[r]), v[c][r]);
+            else g_upd<K, true>(tb + slot[r] * L.slot_bytes + L.f[j].goff, v[c][r]);
+          }
+      });
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// S5a: path (a) dense shared-memory aggregation (§4.3.2)
+// ------------------------------------------------------------------------------------------------
+template <class SP, int NV, int R>
+__device__ __forceinline__ void dense_body(const AggParams& p) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  const Layout& L = p.lay;
+  const uint32_t D = p.S;
+  for (int j = 0; j < L.n_fields; ++j)
+    for (uint32_t e = threadIdx.x; e < D; e += blockDim.x) smem_init_entry(sm + p.soff[j], L.f[j].kind, e, D);
+  __syncthreads();
+
+  const uint64_t pol = evict_first_policy();
+  const uint64_t n = p.n_rows;
+  const uint64_t tile = (uint64_t)blockDim.x * R;
+  const uint64_t ntiles = (n + tile - 1) / tile;
+  uint32_t flag_seen = 0;
+  for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    if (flag_seen) break;
+    flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);  // warp-uniform, seen next tile
+    const uint64_t row = lane_base<R, false>(t * tile, threadIdx.x >> 5, threadIdx.x & 31);
+    uint64_t key[R];
+    const uint32_t valid = pack_keys<SP, R, false>(p, row, n, pol, key);
+    uint64_t v[NV][R];
+    load_vals<SP, NV, R, false>(p, row, n, pol, v);
+    uint32_t e[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) e[r] = (uint32_t)key[r];
+    smem_apply_rows<SP, NV, R>(p, sm, e, valid, v);
+  }
+  __syncthreads();
+  // S7: CTA -> global merge with native 64-bit REDs ("the small hash tables in shared memory
+  // are merged to a global hash table in device memory").
+  const uint8_t* cnt = sm + p.soff[L.count_field];
+  for (uint32_t e = threadIdx.x; e < D; e += blockDim.x) {
+    if (((const uint32_t*)cnt)[e] == 0) continue;
+    for (int j = 0; j < L.n_fields; ++j) {
+      uint8_t* b = sm + p.soff[j];
+      dispatch_kind(L.f[j].kind, [&](auto kc) {
+        constexpr int K = decltype(kc)::v;
+        d_upd<K, false>(dense_addr(p, j, e), s_read<K>(b, e, D));
+      });
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// S5b: path (b) global hash table / path (b') direct-mapped, optional shared-memory hot-key front
+// ------------------------------------------------------------------------------------------------
+// MODE 0: rows from columns; 1: records (merge of exchanged partials); 2: segments (pass 2 of the
+// partitioned mode: tiles enumerate the buckets in order, so at any moment all CTAs work inside
+// one bucket whose slice of the table is L2-resident).
+template <class SP, int NV, int R, bool FRONT, bool DIRECT, int MODE>
+__device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  constexpr bool RECORDS = MODE == 1;
+  constexpr bool SEG = MODE == 2;
+  if (p.gate && ((*(volatile const uint32_t*)p.gate != 0) != (p.gate_run_if != 0))) return;
+  const Layout& L = p.lay;
+  const uint32_t S = p.S;
+  __shared__ uint64_t tpre[SEG ? 1025 : 1];
+  if constexpr (SEG) {  // warp-tile prefix over the buckets (warp 0)
+    if (threadIdx.x < 32) {
+      const uint64_t tile = 32ull * R;
+      uint64_t carry = 0;
+      for (uint32_t b0 = 0; b0 < p.n_segs; b0 += 32) {
+        uint32_t b = b0 + threadIdx.x;
+        uint64_t x = b < p.n_segs ? (p.seg_count[b] + tile - 1) / tile : 0, inc = x;
+        for (int o = 1; o < 32; o <<= 1) {
+          uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+          if ((int)threadIdx.x >= o) inc += y;
+        }
+        if (b < p.n_segs) tpre[b] = carry + inc - x;
+        carry += __shfl_sync(0xffffffffu, inc, 31);
+      }
+      if (threadIdx.x == 0) tpre[p.n_segs] = carry;
+    }
+    __syncthreads();
+  }
+  if (FRONT) {
+    for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) ((uint64_t*)(sm + p.key_off))[e] = kEmpty;
+    for (int j = 0; j < L.n_fields; ++j)
+      for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) smem_init_entry(sm + p.soff[j], L.f[j].kind, e, S);
+    __syncthreads();
+  }
+  const uint64_t pol = evict_first_policy();
+  // SEG: warp tiles (32*R rows) handed out in bucket order by a global counter, so every warp of
+  // the grid stays inside the same one or two buckets (their table slices L2-resident); static
+  // grid-stride assignment lets CTAs drift several buckets apart and thrash L2.
+  const uint64_t tile = SEG ? 32ull * R : (uint64_t)blockDim.x * R;
+  const uint64_t ntiles = SEG ? tpre[p.n_segs] : (p.n_rows + tile - 1) / tile;
+  const unsigned lane = threadIdx.x & 31;
+  uint8_t* tb = (uint8_t*)p.table;
+  uint32_t flag_seen = 0;
+  // SEG: a warp claims kGrab consecutive warp tiles per atomic (one counter for the whole grid)
+  constexpr uint32_t kGrab = 16;
+  uint64_t t = blockIdx.x, chunk = 0, chunk_next = 0;
+  uint32_t k_in = 0;
+  const bool dyn = SEG && p.tile_ctr != nullptr;
+  if (SEG && !dyn) t = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);  // static warp tiles
+  if (dyn) {
+    chunk = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;
+    chunk = __shfl_sync(0xffffffffu, chunk, 0);
+    chunk_next = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;  // prefetched
+    t = chunk * kGrab;
+  }
+  while (t < ntiles) {
+    if (flag_seen) break;
+    flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);  // warp-uniform abort
+    uint64_t n = p.n_rows, row0 = t * tile, t_next = t + gridDim.x;
+    uint64_t row;
+    if constexpr (SEG) {  // bucket of warp tile t: largest b with tpre[b] <= t
+      if (!dyn) {
+        t_next = t + (uint64_t)gridDim.x * (blockDim.x >> 5);
+      } else if (++k_in < kGrab) {
+        t_next = t + 1;
+      } else {
+        k_in = 0;
+        chunk = __shfl_sync(0xffffffffu, chunk_next, 0);
+        t_next = chunk * kGrab;
+        chunk_next = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;
+      }
+      uint32_t lo = 0, hi = p.n_segs - 1;
+      while (lo < hi) {
+        uint32_t mid = (lo + hi + 1) >> 1;
+        if (tpre[mid] <= t) lo = mid; else hi = mid - 1;
+      }
+      row0 = p.seg_base[lo] + (t - tpre[lo]) * tile;
+      n = p.seg_base[lo] + p.seg_count[lo];
+      row = lane_base<R>(row0, 0, lane);
+    } else {
+      row = lane_base<R>(row0, threadIdx.x >> 5, lane);
+    }
+    uint64_t key[R];
+    uint64_t v[NV][R];
+    uint32_t valid;
+    if (RECORDS) {
+      valid = 0;
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        key[r] = 0;
+#pragma unroll
+        for (int c = 0; c < NV; ++c) v[c][r] = 0;
+        const uint64_t rr = row_of<R>(row, r);
+        if (rr >= n) continue;
+        const uint64_t* rec = rs.rec + rr * rs.words;
+        key[r] = __ldg((const unsigned long long*)rec);
+        valid |= 1u << r;
+#pragma unroll
+        for (int c = 0; c < NV; ++c)
+          if (c < L.n_vals) {
+            uint64_t w = __ldg((const unsigned long long*)rec + 1 + c);
+            v[c][r] = L.val_dtype[c] == BLU_I32 ? (uint64_t)(int64_t)(int32_t)(uint32_t)w : w;
+          }
+      }
+    } else {
+      valid = pack_keys<SP, R>(p, row, n, pol, key);
+      load_vals<SP, NV, R>(p, row, n, pol, v);
+    }
+    uint32_t miss = valid;
+    if (FRONT) {
+      // hot-key front: small open-addressing table per CTA in shared memory
+      uint64_t* fk = (uint64_t*)(sm + p.key_off);
+      uint32_t fe[R];
+      uint32_t hit = 0;
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        fe[r] = 0;
+        if (!(valid >> r & 1)) continue;
+        uint32_t s = (uint32_t)(fmix64(key[r] ^ 0x5bd1e995ull) >> 40) & (S - 1);
+#pragma unroll 1
+        for (int q = 0; q < 8; ++q) {
+          uint64_t cur = *(volatile uint64_t*)(fk + s);
+          if (cur == key[r]) { hit |= 1u << r; break; }
+          if (cur == kEmpty) {
+            unsigned long long old = atomicCAS((unsigned long long*)(fk + s), (unsigned long long)kEmpty,
+                                               (unsigned long long)key[r]);
+            if (old == kEmpty || old == key[r]) { hit |= 1u << r; break; }
+          }
+          s = (s + 1) & (S - 1);
+        }
+        fe[r] = s;
+      }
+      __syncwarp();  // reconverge after the data-dependent probe loops (independent thread scheduling)
+      smem_apply_rows<SP, NV, R>(p, sm, fe, hit, v);
+      miss = valid & ~hit;
+    }
+    uint64_t slot[R];
+    if (DIRECT) {
+#pragma unroll
+      for (int r = 0; r < R; ++r) slot[r] = key[r];
+    } else {
+      // Convergent multi-row probe: every pending row of the lane advances one slot per iteration
+      // and all their key loads are issued together (memory-level parallelism); the warp stays
+      // converged (__any_sync), so the REDs that follow are warp-wide.
+      uint64_t cur[R];
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        slot[r] = fmix64(key[r]) & p.cap_mask;
+        cur[r] = (miss >> r & 1) ? __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes)) : 0ull;
+      }
+      uint32_t pending = miss;
+      for (uint32_t it = 0;; ++it) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (!(pending >> r & 1)) continue;
+          if (cur[r] == key[r]) {
+            pending &= ~(1u << r);
+          } else {
+            if (cur[r] == kEmpty) {
+              unsigned long long old = atomicCAS((unsigned long long*)(tb + slot[r] * L.slot_bytes),
+                                                 (unsigned long long)kEmpty, (unsigned long long)key[r]);
+              if (old == kEmpty || old == key[r]) {
+                pending &= ~(1u << r);
+                continue;
+              }
+            }
+            slot[r] = (slot[r] + 1) & p.cap_mask;
+          }
+        }
+        if (!__any_sync(0xffffffffu, pending)) break;
+        if (it + 1 >= 4) {
+          // long tails (a few rows per warp): finish them one lane at a time, then reconverge
+#pragma unroll
+          for (int r = 0; r < R; ++r) {
+            if (!(pending >> r & 1)) continue;
+            uint64_t sl;
+            const uint64_t c = __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes));
+            if (hash_locate(tb, p.cap_mask, L.slot_bytes, key[r], c, slot[r], p.max_probe, sl)) {
+              slot[r] = sl;
+            } else {  // the estimate was too small: flag, regrow, rerun
+              miss &= ~(1u << r);
+              atomicOr(p.flags, FLAG_OVERFLOW);
+            }
+          }
+          break;
+        }
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+          if (pending >> r & 1) cur[r] = __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes));
+      }
+      __syncwarp();  // reconverge before the field reductions so each RED instruction is warp-wide
+    }
+    global_apply_rows<SP, NV, R, DIRECT>(p, slot, miss, v);
+    t = t_next;
+  }
+  if (FRONT) {
+    // merge the front into the global table
+    __syncthreads();
+    const uint64_t* fk = (const uint64_t*)(sm + p.key_off);
+    for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) {
+      const uint64_t key = fk[e];
+      if (key == kEmpty) continue;
+      uint64_t s = key;
+      if (!DIRECT) {
+        uint64_t idx = fmix64(key) & p.cap_mask;
+        uint64_t first = __ldcg((const unsigned long long*)(tb + idx * L.slot_bytes));
+        if (!hash_locate(tb, p.cap_mask, L.slot_bytes, key, first, idx, p.max_probe, s)) {
+          atomicOr(p.flags, FLAG_OVERFLOW);
+          continue;
+        }
+      }
+      for (int j = 0; j < L.n_fields; ++j) {
+        const uint8_t* b = sm + p.soff[j];
+        dispatch_kind(L.f[j].kind, [&](auto kc) {
+          constexpr int K = decltype(kc)::v;
+          if (DIRECT) d_upd<K, false>(dense_addr(p, j, s), s_read<K>(b, e, S));
+          else g_upd<K, false>(tb + s * L.slot_bytes + L.f[j].goff, s_read<K>(b, e, S));
+        });
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
+// Partitioned path (b), pass 1: radix scatter of rows into B buckets by the top bits of their slot.
+// Per tile: shared-memory counting sort by bucket, one global cursor reservation per (tile,
+// bucket), then coalesced writes of each bucket's contiguous segment (packed u64 key + values).
+// ------------------------------------------------------------------------------------------------
+__device__ __forceinline__ void block_excl_scan_512(uint32_t* a, uint32_t* out, uint32_t B, uint32_t* warp_tot,
+                                                    uint32_t* total) {
+  // exclusive scan of a[0..B) (B <= 2 * blockDim.x, blockDim.x == 512) into out
+  const unsigned t = threadIdx.x, lane = t & 31, w = t >> 5;
+  uint32_t x0 = 2 * t < B ? a[2 * t] : 0, x1 = 2 * t + 1 < B ? a[2 * t + 1] : 0;
+  uint32_t sum = x0 + x1, inc = sum;
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+    if ((int)lane >= o) inc += y;
+  }
+  if (lane == 31) warp_tot[w] = inc;
+  __syncthreads();
+  if (w == 0) {
+    uint32_t v = lane < blockDim.x / 32 ? warp_tot[lane] : 0, vi = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(0xffffffffu, vi, o);
+      if ((int)lane >= o) vi += y;
+    }
+    if (lane < blockDim.x / 32) warp_tot[lane] = vi - v;
+    if (lane == 31) *total = vi;
+  }
+  __syncthreads();
+  uint32_t excl = warp_tot[w] + inc - sum;
+  if (2 * t < B) out[2 * t] = excl;
+  if (2 * t + 1 < B) out[2 * t + 1] = excl + x0;
+}
+
+template <class SP, int NV, int R>
+__device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterParams& sp) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  const Layout& L = p.lay;
+  const uint32_t B = sp.B;
+  const uint32_t TILE = blockDim.x * R;
+  uint64_t* skey = (uint64_t*)sm;                       // TILE
+  uint64_t* sval = skey + TILE;                         // NV x TILE
+  uint64_t* gpos = sval + (size_t)NV * TILE;            // B
+  uint32_t* hist = (uint32_t*)(gpos + B);               // B
+  uint32_t* lstart = hist + B;                          // B
+  uint32_t* wtot = lstart + B;                          // 32
+  uint32_t* total = wtot + 32;                          // 1
+  uint16_t* sbid = (uint16_t*)(total + 4);              // TILE
+  const uint64_t pol = evict_first_policy();
+  const uint64_t n = p.n_rows;
+  const uint64_t ntiles = (n + TILE - 1) / TILE;
+  for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
+    __syncthreads();
+    const uint64_t row = lane_base<R>(t * TILE, threadIdx.x >> 5, threadIdx.x & 31);
+    uint64_t key[R];
+    const uint32_t valid = pack_keys<SP, R>(p, row, n, pol, key);
+    uint64_t v[NV][R];
+    load_vals<SP, NV, R>(p, row, n, pol, v);
+    uint32_t bb[R], pos[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      bb[r] = (uint32_t)((fmix64(key[r]) & p.cap_mask) >> sp.shift);
+      pos[r] = (valid >> r & 1) ? atomicAdd(&hist[bb[r]], 1u) : 0u;
+    }
+    __syncthreads();
+    block_excl_scan_512(hist, lstart, B, wtot, total);
+    for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
+      uint32_t h = hist[b];
+      if (h) {
+        uint64_t g = atomicAdd((unsigned long long*)&sp.cursor[b], (unsigned long long)h);
+        gpos[b] = g;
+        if (g + h > sp.seg_cap) atomicExch(sp.gate, 1u);
+      }
+    }
+    __syncthreads();  // lstart and gpos visible to every thread
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (valid >> r & 1) {
+        uint32_t e = lstart[bb[r]] + pos[r];
+        skey[e] = key[r];
+        sbid[e] = (uint16_t)bb[r];
+#pragma unroll
+        for (int c = 0; c < NV; ++c) sval[(size_t)c * TILE + e] = v[c][r];
+      }
+    __syncthreads();
+    const uint32_t tot = *total;
+    for (uint32_t e = threadIdx.x; e < tot; e += blockDim.x) {
+      const uint32_t b = sbid[e];
+      const uint64_t g = gpos[b] + (e - lstart[b]);
+      if (g >= sp.seg_cap) continue;
+      const uint64_t idx = sp.seg_base[b] + g;
+      sp.out_key[idx] = skey[e];
+#pragma unroll
+      for (int c = 0; c < NV; ++c)
+        if (c < L.n_vals) {
+          const uint64_t x = sval[(size_t)c * TILE + e];
+          if (L.val_dtype[c] == BLU_I32) ((int32_t*)sp.out_val[c])[idx] = (int32_t)(uint32_t)x;
+          else ((uint64_t*)sp.out_val[c])[idx] = x;
+        }
+    }
+    __syncthreads();
+  }
+}
+
+}  // namespace blu

@@ -9,61 +9,13 @@
 #include <vector>
 
 #include "blu_gby.h"
+#include "blu_params.h"
 
 namespace blu {
 
-constexpr int kMaxKeys = 8;
-constexpr int kMaxVals = 16;
-constexpr int kMaxAggs = 16;
-constexpr int kMaxFields = 24;
-constexpr uint64_t kEmpty = ~0ull;  // key portion of the mask: M/4 Fs (Table 1)
 
-// State-field kinds. Each aggregate maps to one or two fields (AVG = SUM field + COUNT field);
-// fields are deduplicated per (kind, column) so SUM(v) and AVG(v) share one SUM field.
-enum FieldKind : int32_t {
-  FK_COUNT = 0,   // += 1 per row (COUNT(*)), 64-bit
-  FK_SUMI = 1,    // int64 sum with two's-complement wrap (i32/i64 inputs widened)
-  FK_SUMF = 2,    // f64 sum
-  FK_MINI32 = 3,  // MIN over i32 (32-bit field in the slot, init INT32_MAX as in Table 1)
-  FK_MAXI32 = 4,  // MAX over i32 (init INT32_MIN)
-  FK_MINI64 = 5,  // MIN over i64 (init INT64_MAX)
-  FK_MAXI64 = 6,  // MAX over i64 (init INT64_MIN, Table 1)
-  FK_MINF64 = 7,  // MIN over f64 through the order-preserving int64 map (init +INT64_MAX)
-  FK_MAXF64 = 8,  // MAX over f64 (init INT64_MIN)
-};
 
-// Where the dense state of a field lives in the 4 allreduce groups (blu_gby.h execute_dense_state).
-enum StateGroup : int32_t { SG_ISUM = 0, SG_FSUM = 1, SG_MIN = 2, SG_MAX = 3 };
 
-struct Field {
-  int32_t kind;    // FieldKind
-  int32_t col;     // value column (-1: COUNT from the constant 1)
-  int32_t gsize;   // bytes in the global AoS slot (4 or 8)
-  int32_t goff;    // byte offset in the global AoS slot
-  int32_t sgroup;  // StateGroup for dense global state
-  int32_t sidx;    // index within its group
-  int32_t ssize;   // bytes per entry in a shared-memory table (4 or 8)
-  int32_t is_count;
-};
-
-// Everything a kernel needs to know about the row format and the fields.
-struct Layout {
-  int32_t n_keys;
-  int32_t key_dtype[kMaxKeys];
-  uint64_t dict[kMaxKeys];
-  uint64_t stride[kMaxKeys];  // mixed radix: stride_0 = 1, stride_j = prod_{i<j} dict_i
-  int32_t sparse;             // 1: single sparse key column (code itself is the packed key)
-  uint64_t domain;            // D = prod dict (dense keys only)
-
-  int32_t n_vals;                // value columns the kernel reads (schema columns or states)
-  int32_t val_dtype[kMaxVals];
-  int32_t n_fields;
-  Field f[kMaxFields];
-  int32_t count_field;           // index of the COUNT field or -1
-  uint32_t slot_bytes;           // global AoS slot (key + fields, padded)
-  int32_t n_group[4];            // fields per StateGroup
-  uint32_t smem_entry_bytes;     // per entry of a shared-memory table (no key)
-};
 
 struct AggMap {
   int32_t op;
@@ -100,80 +52,13 @@ struct blu_gby_plan_s {
 
 namespace blu {
 
-// ---------------------------------------------------------------------------------------------
-// Kernel parameter blocks (passed by value; < 4 KB)
-// ---------------------------------------------------------------------------------------------
-struct AggParams {
-  Layout lay;
-  const void* key[kMaxKeys];
-  const void* val[kMaxVals];
-  uint64_t n_rows;
-  int32_t vec_ok;        // all column pointers 16-byte aligned
-  // targets
-  void* table;           // path b: AoS slots (cap x slot_bytes)
-  uint64_t cap_mask;     // cap - 1 (power of two)
-  uint32_t max_probe;
-  void* dense[4];        // paths a / b': dense state groups (SG_*), each n_group[g] x D int64
-  uint32_t front_slots;  // shared-memory front entries (power of two) or 0
-  uint32_t* flags;       // bit 0: overflow (probe bound), bit 1: key out of range
-  // shared-memory table layout (path a: S = D; front: S = front_slots), filled by the host
-  uint32_t S;
-  uint32_t key_off;              // front keys (S x u64)
-  uint32_t soff[kMaxFields];     // per field: byte offset of its SoA array
-  uint32_t colmask[kMaxFields];  // per kernel value column: bit j = field j reads it
-  uint32_t cntmask;              // fields that count the constant 1
-  // partitioned pass 2 (segments mode): rows of segment b are [seg_base[b], seg_base[b] + seg_count[b])
-  const uint64_t* seg_base;
-  const uint64_t* seg_count;
-  uint32_t n_segs;
-  uint64_t* tile_ctr;            // segments mode: dynamic warp-tile counter (zeroed per launch)
-  // device-side gate: the kernel runs only if ((*gate != 0) == gate_run_if); NULL = always
-  const uint32_t* gate;
-  uint32_t gate_run_if;
-};
 
-// Pass 1 of the partitioned path (b): scatter rows into B buckets by the top bits of their slot.
-struct ScatterParams {
-  uint32_t B;
-  uint32_t shift;            // bucket = (fmix64(key) & cap_mask) >> shift
-  const uint64_t* seg_base;  // B: first row of each bucket in the partition buffers
-  uint64_t* cursor;          // B: rows appended so far (zeroed per chunk)
-  uint64_t seg_cap;          // rows per bucket
-  uint64_t* out_key;         // packed keys (u64)
-  void* out_val[kMaxVals];   // value columns, input dtypes
-  uint32_t* gate;            // set to 1 if any bucket overflows (pass 2 then falls back)
-};
 
 // Fill S / key_off / soff / colmask / cntmask of p for a shared-memory table of S entries.
 void fill_smem_layout(AggParams& p, uint32_t S, bool with_keys);
 
-enum : uint32_t { FLAG_OVERFLOW = 1u, FLAG_KEY_RANGE = 2u };
 
-struct CompactParams {
-  Layout lay;
-  int32_t source;        // 0: AoS hash table, 1: dense state (occupancy = COUNT > 0)
-  const void* table;
-  const void* dense[4];
-  uint64_t n_entries;    // cap or D
-  int32_t partial;       // 1: emit state fields, 0: finalized aggregates
-  int32_t n_out;         // output value columns
-  // finalized: per output column (aggregate) which field(s) and dtype
-  int32_t out_kind[kMaxFields];   // 0 field as stored, 1 AVG
-  int32_t out_field[kMaxFields];
-  int32_t out_field2[kMaxFields];
-  int32_t out_dtype[kMaxFields];
-  void* out_keys[kMaxKeys];
-  void* out_vals[kMaxFields];
-  uint64_t* block_counts;
-  uint64_t* block_offsets;
-  uint64_t* n_groups;    // device
-};
 
-// Records-mode input for merges of exchanged partials: rows of `words` u64 (key, states).
-struct RecSrc {
-  const uint64_t* rec;
-  uint32_t words;
-};
 
 // Launchers (kernels.cu). All return cudaError_t as int.
 int launch_aggregate_impl(const blu_gby_plan_s* P, int path, const AggParams& p, const RecSrc& rs, bool records,
@@ -189,6 +74,11 @@ int launch_partition(const Layout& lay, const void* const* key_cols, const void*
                      void* stream);
 
 void count_launch(uint64_t n);
+
+// NVRTC specialisation (jit.cpp)
+bool jit_enabled();
+const void* jit_kernel(const std::string& spec_src, const std::string& entry_src, const char* entry);
+std::string jit_spec(const char* name, const Layout& L);
 
 // Planner helpers (plan.cpp)
 uint32_t smem_entry_bytes(const Layout& lay);

@@ -54,8 +54,11 @@ def oracles():
     return get
 
 
+@pytest.mark.parametrize("jit", ["1", "0"])
 @pytest.mark.parametrize("name", ["C1", "C2", "C3", "C4", "C5"])
-def test_config_parity(bg, oracles, name):
+def test_config_parity(bg, oracles, monkeypatch, name, jit):
+    """Both the NVRTC-specialised kernels (default) and the precompiled generic ones."""
+    monkeypatch.setenv("BLU_GBY_JIT", jit)
     w, o = oracles(name)
     plan, res = run_gpu(bg, w)
     assert res.n_groups == o.n_groups
