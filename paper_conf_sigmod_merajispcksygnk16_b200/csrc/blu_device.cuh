@@ -85,22 +85,25 @@ __device__ __forceinline__ int2 ld_stream_v2(const void* p, uint64_t pol) {
 template <int R, bool PAIR = true>
 __device__ __forceinline__ void load_rows(const void* base, int dt, uint64_t lb, uint64_t n, bool vec,
                                           uint64_t pol, uint64_t (&out)[R]) {
-  if (!PAIR && R == 4) {  // quad mapping: rows lb..lb+3 (path (a): one 16-byte load per i32 column)
+  if (!PAIR && R >= 4) {  // quad mapping: rows lb..lb+R-1 (path (a): 16-byte loads, 4 i32 rows each)
     if (dt == BLU_I32) {
       const int32_t* p = (const int32_t*)base + lb;
-      if (vec && lb + 4 <= n) {
-        int4 v = ld_stream_v4(p, pol);
-        out[0] = (uint64_t)(int64_t)v.x;
-        out[1 % R] = (uint64_t)(int64_t)v.y;
-        out[2 % R] = (uint64_t)(int64_t)v.z;
-        out[3 % R] = (uint64_t)(int64_t)v.w;
+      if (vec && lb + R <= n) {
+#pragma unroll
+        for (int q = 0; q < R; q += 4) {
+          int4 v = ld_stream_v4(p + q, pol);
+          out[q] = (uint64_t)(int64_t)v.x;
+          out[(q + 1) % R] = (uint64_t)(int64_t)v.y;
+          out[(q + 2) % R] = (uint64_t)(int64_t)v.z;
+          out[(q + 3) % R] = (uint64_t)(int64_t)v.w;
+        }
       } else {
 #pragma unroll
         for (int r = 0; r < R; ++r) out[r] = lb + r < n ? (uint64_t)(int64_t)ld_stream_s32(p + r, pol) : 0ull;
       }
     } else {
       const uint64_t* p = (const uint64_t*)base + lb;
-      if (vec && lb + 4 <= n) {
+      if (vec && lb + R <= n) {
 #pragma unroll
         for (int r = 0; r < R; r += 2) {
           int4 v = ld_stream_v4(p + r, pol);
@@ -522,6 +525,109 @@ __device__ __forceinline__ void dense_body(const AggParams& p) {
 // ------------------------------------------------------------------------------------------------
 // S5b: path (b) global hash table / path (b') direct-mapped, optional shared-memory hot-key front
 // ------------------------------------------------------------------------------------------------
+// ---- JIT front path with warp-level pre-aggregation (skewed keys) -----------------------------
+template <int K>
+__device__ __forceinline__ uint64_t combine_vals(uint64_t a, uint64_t b) {
+  if constexpr (K == FK_SUMI || K == FK_COUNT) return a + b;
+  else if constexpr (K == FK_SUMF) return (uint64_t)__double_as_longlong(__longlong_as_double((long long)a) + __longlong_as_double((long long)b));
+  else if constexpr (K == FK_MINI32 || K == FK_MINI64) return (int64_t)a < (int64_t)b ? a : b;
+  else if constexpr (K == FK_MAXI32 || K == FK_MAXI64) return (int64_t)a > (int64_t)b ? a : b;
+  else if constexpr (K == FK_MINF64) return __longlong_as_double((long long)a) < __longlong_as_double((long long)b) ? a : b;
+  else return __longlong_as_double((long long)a) > __longlong_as_double((long long)b) ? a : b;
+}
+
+// For each of the lane's R rows: lanes holding the same key (__match_any_sync) reduce every field
+// onto the lowest such lane with a successor-doubling shuffle tree (log2 of the largest group per
+// warp steps); only that leader probes the shared-memory front and applies the combined update
+// (COUNT adds the group size). Zipf hot keys then cost one shared atomic per field per warp instead
+// of one per row. Rows whose key is not in the front go to the global table with the same
+// combined values.
+template <class SP, int NV, int R, bool DIRECT>
+__device__ __forceinline__ void front_dedupe_rows(const AggParams& p, uint8_t* sm, const uint64_t (&key)[R],
+                                                  uint32_t valid, const uint64_t (&v)[NV][R]) {
+  const unsigned lane = threadIdx.x & 31;
+  const uint32_t S = p.S;
+  uint64_t* fk = (uint64_t*)(sm + p.key_off);
+  uint8_t* tb = (uint8_t*)p.table;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const bool vr = valid >> r & 1;
+    const uint64_t mk = vr ? key[r] : ((1ull << 63) | lane);
+    const uint32_t peers = __match_any_sync(0xffffffffu, mk);
+    const uint32_t np = __popc(peers);
+    const uint32_t rank = __popc(peers & ((1u << lane) - 1u));
+    const uint32_t above = lane == 31 ? 0u : (peers & (0xffffffffu << (lane + 1)));
+    int sk = above ? __ffs(above) - 1 : -1;
+    const uint32_t maxnp = __reduce_max_sync(0xffffffffu, np);
+    uint64_t xr[SP::NF];
+    sfor<0, SP::NF>([&](auto jc) {
+      constexpr int j = decltype(jc)::v;
+      constexpr int c = SP::COL[j];
+      xr[j] = c < 0 ? (uint64_t)np : v[c < 0 ? 0 : c][r];
+    });
+    for (uint32_t k = 1; k < maxnp; k <<= 1) {
+      const int src = sk < 0 ? (int)lane : sk;
+      const bool take = sk >= 0 && (rank & (2 * k - 1)) == 0;
+      sfor<0, SP::NF>([&](auto jc) {
+        constexpr int j = decltype(jc)::v;
+        constexpr int c = SP::COL[j], K = SP::KIND[j];
+        if constexpr (c >= 0) {
+          const uint64_t y = __shfl_sync(0xffffffffu, xr[j], src);
+          if (take) xr[j] = combine_vals<K>(xr[j], y);
+        }
+      });
+      const int s2 = __shfl_sync(0xffffffffu, sk, src);
+      sk = sk < 0 ? -1 : s2;
+    }
+    if (!vr || rank != 0) continue;
+    // leader: linear probe of the front (up to 8 slots)
+    uint32_t e = (uint32_t)(fmix64(key[r] ^ 0x5bd1e995ull) >> 40) & (S - 1);
+    bool hit = false;
+#pragma unroll 1
+    for (int q = 0; q < 8; ++q) {
+      const uint64_t cur = *(volatile uint64_t*)(fk + e);
+      if (cur == key[r]) { hit = true; break; }
+      if (cur == kEmpty) {
+        unsigned long long old = atomicCAS((unsigned long long*)(fk + e), (unsigned long long)kEmpty,
+                                           (unsigned long long)key[r]);
+        if (old == kEmpty || old == key[r]) { hit = true; break; }
+      }
+      e = (e + 1) & (S - 1);
+    }
+    if (hit) {
+      sfor<0, SP::NF>([&](auto jc) {
+        constexpr int j = decltype(jc)::v;
+        constexpr int KK = SP::COL[j] < 0 ? FK_COUNT : SP::KIND[j];
+        s_upd<KK, true>(sm + p.soff[j], e, S, xr[j]);
+      });
+    } else if constexpr (DIRECT) {
+      sfor<0, SP::NF>([&](auto jc) {
+        constexpr int j = decltype(jc)::v;
+        constexpr int KK = SP::COL[j] < 0 ? FK_COUNT : SP::KIND[j];
+        constexpr int sg = SP::SGROUP[j];
+        constexpr uint64_t base = (uint64_t)SP::SIDX[j] * SP::DOMAIN;
+        d_upd<KK, true>((uint64_t*)p.dense[sg] + base + key[r], xr[j]);
+      });
+    } else {
+      constexpr uint64_t slot_b = SP::SLOT;
+      const uint64_t idx = fmix64(key[r]) & p.cap_mask;
+      const uint64_t first = __ldcg((const unsigned long long*)(tb + idx * slot_b));
+      uint64_t sl;
+      if (!hash_locate(tb, p.cap_mask, (uint32_t)slot_b, key[r], first, idx, p.max_probe, sl)) {
+        atomicOr(p.flags, FLAG_OVERFLOW);
+        continue;
+      }
+      sfor<0, SP::NF>([&](auto jc) {
+        constexpr int j = decltype(jc)::v;
+        constexpr int KK = SP::COL[j] < 0 ? FK_COUNT : SP::KIND[j];
+        constexpr int goff = SP::GOFF[j];
+        g_upd<KK, true>(tb + sl * slot_b + goff, xr[j]);
+      });
+    }
+  }
+  __syncwarp();
+}
+
 // MODE 0: rows from columns; 1: records (merge of exchanged partials); 2: segments (pass 2 of the
 // partitioned mode: tiles enumerate the buckets in order, so at any moment all CTAs work inside
 // one bucket whose slice of the table is L2-resident).
@@ -633,7 +739,15 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
       load_vals<SP, NV, R>(p, row, n, pol, v);
     }
     uint32_t miss = valid;
-    if (FRONT) {
+    bool deduped = false;
+    if constexpr (FRONT && SP::kStatic) {
+      if constexpr (SP::DEDUPE) {  // opt-in (BLU_GBY_DEDUPE=1): pays off only for extreme skew
+        front_dedupe_rows<SP, NV, R, DIRECT>(p, sm, key, valid, v);
+        miss = 0;
+        deduped = true;
+      }
+    }
+    if (FRONT && !deduped) {
       // hot-key front: small open-addressing table per CTA in shared memory
       uint64_t* fk = (uint64_t*)(sm + p.key_off);
       uint32_t fe[R];

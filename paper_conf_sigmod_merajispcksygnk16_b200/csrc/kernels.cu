@@ -35,13 +35,18 @@ uint64_t launches_total() { return g_launches.load(); }
 
 // R (rows per thread) for a given number of value columns; identical for AOT and JIT kernels.
 static int rows_per_thread(int nv) { return nv <= 4 ? 4 : nv <= 8 ? 2 : 1; }
+// JIT-only tuning knobs (benchmarks): rows per thread of the dense kernel, min CTAs per SM.
+static int jit_env(const char* k, int def) {
+  const char* v = getenv(k);
+  return v && *v ? atoi(v) : def;
+}
 
 // Launch the NVRTC-specialised kernel for this plan's layout, if the JIT is enabled and succeeds.
 static bool launch_jit(const char* body, const char* entry_decl, const AggParams& p, void** args, cudaStream_t st,
                        uint32_t grid, uint32_t block, uint32_t smem, const char* entry) {
   if (!p.jit_ok || !jit_enabled()) return false;
   const std::string spec = jit_spec("JitSpec", p.lay);
-  std::string src = "extern \"C\" __global__ void __launch_bounds__(512) ";
+  std::string src = "extern \"C\" __global__ void __launch_bounds__(512, " + std::to_string(jit_env("BLU_GBY_JIT_MINB", 1)) + ") ";
   src += entry_decl;
   src += " { ";
   src += body;
@@ -374,11 +379,13 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
   cudaStream_t st = (cudaStream_t)stream;
   cudaError_t e = cudaSuccess;
   if (!records && p.jit_ok) {
-    const int nv = p.lay.n_vals < 1 ? 1 : p.lay.n_vals, r = rows_per_thread(p.lay.n_vals);
+    const int nv = p.lay.n_vals < 1 ? 1 : p.lay.n_vals;
+    int r = rows_per_thread(p.lay.n_vals);
     char body[256], decl[160], name[64];
     AggParams pc = p;
     RecSrc rc = rs;
     if (path == BLU_PATH_DENSE_SMEM) {
+      r = jit_env("BLU_GBY_JIT_R", r);
       snprintf(name, sizeof name, "blu_jit_dense_%d_%d", nv, r);
       snprintf(decl, sizeof decl, "%s(blu::AggParams p)", name);
       snprintf(body, sizeof body, "blu::dense_body<blu::JitSpec, %d, %d>(p);", nv, r);

@@ -346,7 +346,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
       uint32_t budget = kFrontBudget;
       uint32_t S = 4096;
       if (const char* fs = env("BLU_GBY_FRONT_SLOTS")) S = (uint32_t)atoi(fs);
-      while (S > 64 && S * per > budget) S >>= 1;
+      while (S > 64 && S * per > budget) S >>= 1;  // power of two, >= 64: 4-way buckets
       if (S * per <= 200 * 1024) {
         P->hot_front = 1;
         P->front_slots = S;
@@ -375,6 +375,9 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   uint32_t by_threads = per_sm_threads / P->block;
   uint32_t by_smem = P->smem_bytes ? std::max<uint32_t>(1, (227 * 1024) / (P->smem_bytes + 1024)) : 32;
   uint32_t ctas = std::max<uint32_t>(1, std::min(by_threads, by_smem));
+  // path (a): one resident wave (512 threads x <= 64 registers -> 2 CTAs/SM); a second wave would
+  // pay the shared-table init and CTA->global flush again (measured: 0.75 vs 0.76-1.0 ms on C2)
+  if (path == BLU_PATH_DENSE_SMEM) ctas = std::min<uint32_t>(ctas, 2);
   if (const char* cs = env("BLU_GBY_CTAS_PER_SM")) ctas = (uint32_t)atoi(cs);
   P->grid = (uint32_t)P->sms * ctas;
 
