@@ -144,7 +144,7 @@ def run_reference(args):
     import blugen
     w = blugen.workload(args.config)
     r0, _, _ = oracle_rate(args.config, 100_000)
-    budget = 90.0
+    budget = float(os.environ.get("BLU_BENCH_REF_BUDGET_S", "90"))
     rows = int(max(50_000, min(10_000_000, r0 * budget / max(1, args.steps + args.warmup))))
     for i in range(args.warmup):
         oracle_rate(args.config, rows, row0=i * rows)
