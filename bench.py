@@ -231,6 +231,7 @@ def main():
     del r
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     agg_ms = []
+    agg_kernel = ""
     sampler = ClockSampler(local)
     if world > 1:
         dist.barrier()
@@ -245,6 +246,7 @@ def main():
         ev[i][1].record(stream)
         t = bg.blu_gby_last_timing()
         agg_ms.append(t["aggregate_ms"] / max(1, t["aggregate_launches"]))
+        agg_kernel = t["kernel"]
         del r
     torch.cuda.synchronize()
     launches = bg.blu_gby_launch_count() - c0
@@ -271,7 +273,7 @@ def main():
     if traffic is not None and traffic_rows:
         traffic = traffic * rows_per_launch / traffic_rows
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": traffic, "kernel": "k_agg_dense_smem" if info["path"] == 0 else "k_agg_global",
+                "traffic": traffic, "kernel": agg_kernel,
                 "algorithmic_bytes_per_launch": rows_per_launch * bpr, "avg_launch_ms": agg_avg_ms,
                 "peak_source": peak_src, "share_of_step": agg_avg_ms / (tot_ms / args.steps)}
 

@@ -218,6 +218,7 @@ blu_status_t blu_gby_init_table(blu_gby_plan_t plan, void* dev_table, uint64_t n
 typedef struct {
     float init_ms, aggregate_ms, compact_ms, h2d_ms, total_ms;
     uint32_t aggregate_launches, retries;
+    char kernel[64];     /* name of the last aggregation kernel launched (JIT entry or generic) */
 } blu_gby_timing_t;
 void blu_gby_set_timing(int32_t enable);
 blu_status_t blu_gby_last_timing(blu_gby_timing_t* out);

@@ -62,7 +62,7 @@ class PlanDescC(ctypes.Structure):
 class TimingC(ctypes.Structure):
     _fields_ = [("init_ms", ctypes.c_float), ("aggregate_ms", ctypes.c_float), ("compact_ms", ctypes.c_float),
                 ("h2d_ms", ctypes.c_float), ("total_ms", ctypes.c_float),
-                ("aggregate_launches", ctypes.c_uint32), ("retries", ctypes.c_uint32)]
+                ("aggregate_launches", ctypes.c_uint32), ("retries", ctypes.c_uint32), ("kernel", ctypes.c_char * 64)]
 
 
 def _load():
@@ -402,7 +402,9 @@ def blu_gby_set_timing(enable: bool):
 def blu_gby_last_timing() -> dict:
     t = TimingC()
     _check(lib.blu_gby_last_timing(ctypes.byref(t)))
-    return {k: getattr(t, k) for k, _ in TimingC._fields_}
+    d = {k: getattr(t, k) for k, _ in TimingC._fields_}
+    d["kernel"] = t.kernel.decode(errors="replace")
+    return d
 
 
 def blu_gby_launch_count() -> int:

@@ -20,6 +20,7 @@
 namespace blu {
 
 
+extern thread_local char t_last_kernel[64];  // kernels.cu
 static thread_local bool t_timing = false;
 static thread_local blu_gby_timing_t t_last{};
 
@@ -201,7 +202,7 @@ static OutSpec make_outspec(const blu_gby_plan_s* P, const Layout& lay, bool par
 }
 
 // Feeds every input batch to the aggregation kernel for one attempt. `base` carries the targets.
-using Feeder = std::function<cudaError_t(AggParams& base, uint32_t* launches, Work& w)>;
+using Feeder = std::function<cudaError_t(AggParams& base, uint32_t* launches, Work& w, const FinalParams* fin)>;
 
 static bool ptr_aligned(const void* p) { return ((uintptr_t)p & 15) == 0; }
 
@@ -209,7 +210,8 @@ static bool ptr_aligned(const void* p) { return ((uintptr_t)p & 15) == 0; }
 // cannot overflow.
 static cudaError_t agg_batch(const blu_gby_plan_s* P, int path, AggParams p, const void* const* keys,
                              const void* const* vals, uint64_t n, const RecSrc* rs, cudaStream_t st,
-                             uint32_t grid, uint32_t block, uint32_t smem, uint32_t* launches) {
+                             uint32_t grid, uint32_t block, uint32_t smem, uint32_t* launches,
+                             const FinalParams* fin = nullptr) {
   const Layout& L = p.lay;
   uint64_t max_rows = ((uint64_t)grid * (1ull << 30)) & ~3ull;
   for (uint64_t r0 = 0; r0 < n; r0 += max_rows) {
@@ -229,7 +231,7 @@ static cudaError_t agg_batch(const blu_gby_plan_s* P, int path, AggParams p, con
     p.n_rows = m;
     RecSrc r{nullptr, 0};
     if (rs) r = RecSrc{rs->rec + r0 * rs->words, rs->words};
-    int e = launch_aggregate_impl(P, path, p, r, rs != nullptr, st, grid, block, smem);
+    int e = launch_aggregate_impl(P, path, p, r, rs != nullptr, st, grid, block, smem, fin);
     if (e) return (cudaError_t)e;
     if (launches) ++*launches;
   }
@@ -239,7 +241,7 @@ static cudaError_t agg_batch(const blu_gby_plan_s* P, int path, AggParams p, con
 // The core: init -> feed -> compact -> one sync -> regrow on overflow.
 static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int path, bool front, uint64_t cap0,
                              uint64_t total_rows, const Feeder& feed, bool partial, cudaStream_t st,
-                             blu_gby_result_t* out, bool host_out, float* h2d_ms_acc) {
+                             blu_gby_result_t* out, bool host_out, float* h2d_ms_acc, bool fuse_req = false) {
   setup_pool();
   memset(out, 0, sizeof *out);
   const bool dense = path != BLU_PATH_HASH_GLOBAL;
@@ -255,9 +257,12 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     void* table = nullptr;
     void* dense_g[4] = {nullptr, nullptr, nullptr, nullptr};
     if (t_timing) cudaEventRecord(t_ev.e[0], st);
+    // path (a) with a small domain: init (S4) and compaction (S8) fused into the aggregation kernel
+    const bool fuse = fuse_req && path == BLU_PATH_DENSE_SMEM && D <= 65536 && !partial && !host_out &&
+                      !getenv("BLU_GBY_NO_FUSE");
     if (dense) {
       for (int g = 0; g < 4; ++g) CK(w.alloc(&dense_g[g], (size_t)lay.n_group[g] * D * 8), "dense state alloc");
-      CK(launch_init_dense(lay, dense_g, D, st), "init dense");
+      if (!fuse) CK(launch_init_dense(lay, dense_g, D, st), "init dense");
     } else {
       CK(w.alloc(&table, (size_t)cap * lay.slot_bytes), "hash table alloc");
       CK(launch_init_slots(lay, table, cap, st), "init slots");
@@ -283,9 +288,6 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     base.flags = d_flags;
     fill_smem_layout(base, path == BLU_PATH_DENSE_SMEM ? (uint32_t)D : base.front_slots, base.front_slots > 0);
     uint32_t launches = 0;
-    CK(feed(base, &launches, w), "aggregate launch");
-    if (t_timing) cudaEventRecord(t_ev.e[2], st);
-
     // outputs, sized by the upper bound min(entries, rows)
     const uint64_t U = std::min<uint64_t>(n_entries, total_rows);
     Owner* own = new Owner();
@@ -308,7 +310,33 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       free_owner();
       return cuda_fail(ae, "output alloc");
     }
-    if (U) {
+    FinalParams fp{};
+    if (fuse) {
+      base.fuse_init = 1;
+      base.sync = (uint32_t*)((uint8_t*)small + 16);
+      fp.enabled = 1;
+      fp.n_out = os.n_out;
+      for (int o = 0; o < os.n_out; ++o) {
+        fp.out_kind[o] = os.out_kind[o];
+        fp.out_field[o] = os.out_field[o];
+        fp.out_field2[o] = os.out_field2[o];
+        fp.out_dtype[o] = os.out_dtype[o];
+        fp.out_vals[o] = ovals[o];
+      }
+      for (int k = 0; k < lay.n_keys; ++k) fp.out_keys[k] = okeys[k];
+      fp.n_groups = d_ngroups;
+    }
+    {
+      cudaError_t fe = feed(base, &launches, w, fuse ? &fp : nullptr);
+      if (fe != cudaSuccess) {
+        cudaGetLastError();
+        free_owner();
+        return cuda_fail(fe, "aggregate launch");
+      }
+    }
+    if (t_timing) cudaEventRecord(t_ev.e[2], st);
+
+    if (U && !fuse) {
       CompactParams cp{};
       cp.lay = lay;
       cp.source = dense ? 1 : 0;
@@ -421,6 +449,7 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       tm.retries = retries;
       if (h2d_ms_acc) tm.h2d_ms = *h2d_ms_acc;
       tm.total_ms = tm.init_ms + tm.aggregate_ms + tm.compact_ms;
+      memcpy(tm.kernel, t_last_kernel, sizeof tm.kernel);
       t_last = tm;
     }
     return BLU_OK;
@@ -550,13 +579,17 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
   if (n && (!nonnull_cols(keys, P->lay.n_keys) || !nonnull_cols(vals, P->lay.n_vals)))
     return fail(BLU_E_INVALID, "NULL column pointer");
   const Layout& L = P->lay;
-  Feeder feed = [&](AggParams& base, uint32_t* launches, Work& w) -> cudaError_t {
+  // fused init + compaction needs exactly one aggregation launch
+  const bool single = n <= (((uint64_t)P->grid * (1ull << 30)) & ~3ull);
+  Feeder feed = [&](AggParams& base, uint32_t* launches, Work& w, const FinalParams* fin) -> cudaError_t {
     base.jit_ok = 1;
     if (P->path == BLU_PATH_HASH_GLOBAL && P->parts > 1 && n >= 4096 * (uint64_t)P->parts)
       return partitioned_feed(P, base, keys, vals, n, st, launches, w);
-    return agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, launches);
+    return agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, launches, fin);
   };
-  return run_core(P, L, P->path, P->hot_front != 0, P->cap, n, feed, partial, st, out, false, nullptr);
+  // fusion only pays where launch latency dominates (<= 16M rows)
+  return run_core(P, L, P->path, P->hot_front != 0, P->cap, n, feed, partial, st, out, false, nullptr,
+                  single && n > 0 && n <= (16ull << 20));
 }
 
 }  // namespace blu
@@ -631,7 +664,7 @@ blu_status_t blu_gby_execute_host(blu_gby_plan_t P, const void* const* hkeys, co
     cudaEventCreate(&t1);
   }
   float h2d_ms = 0.f;
-  Feeder feed = [&](AggParams& base, uint32_t* launches, Work&) -> cudaError_t {
+  Feeder feed = [&](AggParams& base, uint32_t* launches, Work&, const FinalParams*) -> cudaError_t {
     if (!n) return cudaSuccess;
     base.jit_ok = 1;
     cudaEventRecord(t0, st);
@@ -689,7 +722,7 @@ static blu_status_t merge_impl(blu_gby_plan_t P, const blu_gby_result_t* parts, 
   uint64_t cap = 1024;
   while ((double)cap * 0.7 < (double)est) cap <<= 1;
   uint32_t grid = (uint32_t)P->sms * 8, block = 256;
-  Feeder feed = [&](AggParams& base, uint32_t* launches, Work&) -> cudaError_t {
+  Feeder feed = [&](AggParams& base, uint32_t* launches, Work&, const FinalParams*) -> cudaError_t {
     for (int i = 0; i < np; ++i) {
       if (!parts[i].n_groups) continue;
       cudaError_t e = agg_batch(P, BLU_PATH_HASH_GLOBAL, base, (const void* const*)parts[i].key_cols,
@@ -721,7 +754,7 @@ blu_status_t blu_gby_merge_records(blu_gby_plan_t P, const void* records, uint64
   while ((double)cap * 0.7 < (double)est) cap <<= 1;
   uint32_t grid = (uint32_t)P->sms * 8, block = 256;
   RecSrc rs{(const uint64_t*)records, (uint32_t)(1 + M.n_vals)};
-  Feeder feed = [&](AggParams& base, uint32_t* launches, Work&) -> cudaError_t {
+  Feeder feed = [&](AggParams& base, uint32_t* launches, Work&, const FinalParams*) -> cudaError_t {
     if (!n) return cudaSuccess;
     return agg_batch(P, BLU_PATH_HASH_GLOBAL, base, nullptr, nullptr, n, &rs, st, grid, block, 0, launches);
   };
@@ -770,7 +803,7 @@ blu_status_t blu_gby_finalize_dense_state(blu_gby_plan_t P, void* const* state_a
   cudaStream_t st = (cudaStream_t)stream;
   const Layout& L = P->lay;
   // Reuse run_core with a feeder that copies the caller's state in place of init+aggregate.
-  Feeder feed = [&](AggParams& base, uint32_t*, Work&) -> cudaError_t {
+  Feeder feed = [&](AggParams& base, uint32_t*, Work&, const FinalParams*) -> cudaError_t {
     for (int g = 0; g < 4; ++g) {
       size_t b = (size_t)L.n_group[g] * L.domain * 8;
       if (b) {

@@ -479,11 +479,82 @@ __device__ __forceinline__ void global_apply_rows(const AggParams& p, const uint
 // ------------------------------------------------------------------------------------------------
 // S5a: path (a) dense shared-memory aggregation (§4.3.2)
 // ------------------------------------------------------------------------------------------------
-template <class SP, int NV, int R>
-__device__ __forceinline__ void dense_body(const AggParams& p) {
+// ---- path (a) fused init / finalize helpers ---------------------------------------------------
+// Dense-state identities per group: int64 SUM / f64 SUM -> 0, MIN -> INT64_MAX, MAX -> INT64_MIN.
+__device__ __forceinline__ void dense_init_all(const AggParams& p) {
+  const uint64_t D = p.lay.domain;
+  for (int g = 0; g < 4; ++g) {
+    const uint64_t n = (uint64_t)p.lay.n_group[g] * D;
+    const uint64_t v = g == SG_MIN ? (uint64_t)INT64_MAX : g == SG_MAX ? (uint64_t)INT64_MIN : 0ull;
+    for (uint64_t i = threadIdx.x; i < n; i += blockDim.x) ((uint64_t*)p.dense[g])[i] = v;
+  }
+}
+
+__device__ __forceinline__ void store_bits(void* out, uint64_t pos, int dtype, uint64_t bits) {
+  if (dtype == BLU_I32) ((int32_t*)out)[pos] = (int32_t)(uint32_t)bits;
+  else ((uint64_t*)out)[pos] = bits;
+}
+
+// One CTA compacts the D-entry dense state (occupancy = COUNT > 0) into the result columns in key
+// order: block-wide ballot/popc prefix per chunk of blockDim entries.
+__device__ __forceinline__ void dense_finalize_block(const AggParams& p, const FinalParams& fp) {
+  __shared__ uint32_t wcnt[32];
+  __shared__ uint64_t base_s;
+  const Layout& L = p.lay;
+  const uint64_t D = L.domain;
+  const Field& cf = L.f[L.count_field];
+  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  if (threadIdx.x == 0) base_s = 0;
+  __syncthreads();
+  for (uint64_t c0 = 0; c0 < D; c0 += blockDim.x) {
+    const uint64_t e = c0 + threadIdx.x;
+    const bool occ = e < D && __ldcg((const long long*)p.dense[cf.sgroup] + (uint64_t)cf.sidx * D + e) > 0;
+    const unsigned bal = __ballot_sync(0xffffffffu, occ);
+    if (lane == 0) wcnt[warp] = __popc(bal);
+    __syncthreads();
+    uint32_t before = 0, tot = 0;
+    for (unsigned w = 0; w < nw; ++w) {
+      if (w < warp) before += wcnt[w];
+      tot += wcnt[w];
+    }
+    before += __popc(bal & ((1u << lane) - 1u));
+    if (occ) {
+      const uint64_t pos = base_s + before;
+      for (int k = 0; k < L.n_keys; ++k) store_bits(fp.out_keys[k], pos, L.key_dtype[k], (e / L.stride[k]) % L.dict[k]);
+      for (int o = 0; o < fp.n_out; ++o) {
+        const Field& f = L.f[fp.out_field[o]];
+        uint64_t x = __ldcg((const unsigned long long*)p.dense[f.sgroup] + (uint64_t)f.sidx * D + e);
+        if (fp.out_kind[o] == 1) {  // AVG = (double)SUM / (double)COUNT (reading A12)
+          const Field& f2 = L.f[fp.out_field2[o]];
+          const uint64_t cnt = __ldcg((const unsigned long long*)p.dense[f2.sgroup] + (uint64_t)f2.sidx * D + e);
+          const double sm_ = f.kind == FK_SUMF ? __longlong_as_double((long long)x) : (double)(long long)x;
+          x = (uint64_t)__double_as_longlong(sm_ / (double)(long long)cnt);
+        } else if (f.kind == FK_MINF64 || f.kind == FK_MAXF64) {
+          x = unord_f64((int64_t)x);
+        }
+        store_bits(fp.out_vals[o], pos, fp.out_dtype[o], x);
+      }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) base_s += tot;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *fp.n_groups = base_s;
+}
+
+// FUSE (small inputs, where launch latency dominates): S4 init and S8 compaction run inside this
+// kernel. Kept out of the large-input instantiation, whose register budget it would squeeze.
+template <class SP, int NV, int R, bool FUSE = false>
+__device__ __forceinline__ void dense_body(const AggParams& p, const FinalParams& fp) {
   extern __shared__ __align__(16) uint8_t sm[];
   const Layout& L = p.lay;
   const uint32_t D = p.S;
+  if (FUSE && p.fuse_init && blockIdx.x == 0) {  // S4 fused: CTA 0 initialises the global dense state
+    dense_init_all(p);
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) atomicExch(&p.sync[0], 1u);
+  }
   for (int j = 0; j < L.n_fields; ++j)
     for (uint32_t e = threadIdx.x; e < D; e += blockDim.x) smem_init_entry(sm + p.soff[j], L.f[j].kind, e, D);
   __syncthreads();
@@ -507,6 +578,12 @@ __device__ __forceinline__ void dense_body(const AggParams& p) {
     smem_apply_rows<SP, NV, R>(p, sm, e, valid, v);
   }
   __syncthreads();
+  if (FUSE && p.fuse_init) {  // the dense state must be initialised before this CTA flushes into it
+    if (threadIdx.x == 0)
+      while (atomicAdd(&p.sync[0], 0u) == 0u) __nanosleep(64);
+    __syncthreads();
+    __threadfence();
+  }
   // S7: CTA -> global merge with native 64-bit REDs ("the small hash tables in shared memory
   // are merged to a global hash table in device memory").
   const uint8_t* cnt = sm + p.soff[L.count_field];
@@ -518,6 +595,17 @@ __device__ __forceinline__ void dense_body(const AggParams& p) {
         constexpr int K = decltype(kc)::v;
         d_upd<K, false>(dense_addr(p, j, e), s_read<K>(b, e, D));
       });
+    }
+  }
+  if (FUSE && fp.enabled) {  // S8 fused: the last CTA to finish compacts the dense state
+    __shared__ int am_last;
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) am_last = atomicAdd(&p.sync[1], 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (am_last) {
+      __threadfence();
+      dense_finalize_block(p, fp);
     }
   }
 }

@@ -62,7 +62,8 @@ void fill_smem_layout(AggParams& p, uint32_t S, bool with_keys);
 
 // Launchers (kernels.cu). All return cudaError_t as int.
 int launch_aggregate_impl(const blu_gby_plan_s* P, int path, const AggParams& p, const RecSrc& rs, bool records,
-                          void* stream, uint32_t grid, uint32_t block, uint32_t smem);
+                          void* stream, uint32_t grid, uint32_t block, uint32_t smem,
+                          const FinalParams* fin = nullptr);
 uint64_t launches_total();
 int launch_scatter(const AggParams& p, const ScatterParams& s, void* stream, uint32_t grid);
 blu_status_t fail(blu_status_t s, const char* fmt, ...);

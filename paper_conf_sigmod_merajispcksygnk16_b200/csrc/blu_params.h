@@ -102,6 +102,23 @@ struct AggParams {
   const uint32_t* gate;
   uint32_t gate_run_if;
   uint32_t jit_ok;               // host: 1 = the launcher may use the NVRTC-specialised kernel
+  // path (a) fusion: CTA 0 initialises the dense state (fuse_init) and the last CTA to finish
+  // compacts it into the result (FinalParams::enabled); sync[0] = init done, sync[1] = CTAs done
+  uint32_t fuse_init;
+  uint32_t* sync;
+};
+
+// Path (a) in-kernel compaction (S8 fused into S5a/S7 for small dense domains).
+struct FinalParams {
+  int32_t enabled;
+  int32_t n_out;
+  int32_t out_kind[kMaxFields];   // 0 field as stored, 1 AVG
+  int32_t out_field[kMaxFields];
+  int32_t out_field2[kMaxFields];
+  int32_t out_dtype[kMaxFields];
+  void* out_keys[kMaxKeys];
+  void* out_vals[kMaxFields];
+  uint64_t* n_groups;
 };
 
 // Pass 1 of the partitioned path (b): scatter rows into B buckets by the top bits of their slot.

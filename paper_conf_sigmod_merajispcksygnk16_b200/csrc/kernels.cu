@@ -25,11 +25,17 @@
 #include "blu_device.cuh"
 
 #include <stdio.h>
+#include <string.h>
 #include <string>
 
 namespace blu {
 
 static std::atomic<uint64_t> g_launches{0};
+thread_local char t_last_kernel[64] = "";
+static void note_kernel(const char* k) {
+  strncpy(t_last_kernel, k, sizeof t_last_kernel - 1);
+  t_last_kernel[sizeof t_last_kernel - 1] = 0;
+}
 void count_launch(uint64_t n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 uint64_t launches_total() { return g_launches.load(); }
 
@@ -43,10 +49,11 @@ static int jit_env(const char* k, int def) {
 
 // Launch the NVRTC-specialised kernel for this plan's layout, if the JIT is enabled and succeeds.
 static bool launch_jit(const char* body, const char* entry_decl, const AggParams& p, void** args, cudaStream_t st,
-                       uint32_t grid, uint32_t block, uint32_t smem, const char* entry) {
+                       uint32_t grid, uint32_t block, uint32_t smem, const char* entry, int min_blocks = 1) {
   if (!p.jit_ok || !jit_enabled()) return false;
   const std::string spec = jit_spec("JitSpec", p.lay);
-  std::string src = "extern \"C\" __global__ void __launch_bounds__(512, " + std::to_string(jit_env("BLU_GBY_JIT_MINB", 1)) + ") ";
+  std::string src = "extern \"C\" __global__ void __launch_bounds__(512, " +
+                    std::to_string(jit_env("BLU_GBY_JIT_MINB", min_blocks)) + ") ";
   src += entry_decl;
   src += " { ";
   src += body;
@@ -62,6 +69,7 @@ static bool launch_jit(const char* body, const char* entry_decl, const AggParams
     return false;
   }
   count_launch(1);
+  if (strncmp(entry, "blu_jit_scatter", 15) != 0) note_kernel(entry);
   return true;
 }
 
@@ -93,9 +101,9 @@ __global__ void __launch_bounds__(256) k_fill_u64(uint64_t* a, uint64_t n, uint6
 // ------------------------------------------------------------------------------------------------
 // AOT kernels (GenericSpec): the schema-generic versions of the bodies in blu_device.cuh
 // ------------------------------------------------------------------------------------------------
-template <int NV, int R>
-__global__ void __launch_bounds__(512) k_agg_dense_smem(AggParams p) {
-  dense_body<GenericSpec, NV, R>(p);
+template <int NV, int R, bool FUSE>
+__global__ void __launch_bounds__(512, 2) k_agg_dense_smem(AggParams p, FinalParams fp) {
+  dense_body<GenericSpec, NV, R, FUSE>(p, fp);
 }
 
 template <int NV, int R, bool FRONT, bool DIRECT, int MODE>
@@ -375,7 +383,7 @@ int launch_init_dense(const Layout& lay, void* const dense[4], uint64_t D, void*
 
 template <int NV, int R>
 static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, const RecSrc& rs, bool records,
-                         void* stream, uint32_t grid, uint32_t block, uint32_t smem) {
+                         void* stream, uint32_t grid, uint32_t block, uint32_t smem, const FinalParams* fin) {
   cudaStream_t st = (cudaStream_t)stream;
   cudaError_t e = cudaSuccess;
   if (!records && p.jit_ok) {
@@ -386,11 +394,14 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
     RecSrc rc = rs;
     if (path == BLU_PATH_DENSE_SMEM) {
       r = jit_env("BLU_GBY_JIT_R", r);
-      snprintf(name, sizeof name, "blu_jit_dense_%d_%d", nv, r);
-      snprintf(decl, sizeof decl, "%s(blu::AggParams p)", name);
-      snprintf(body, sizeof body, "blu::dense_body<blu::JitSpec, %d, %d>(p);", nv, r);
-      void* args[] = {&pc};
-      if (launch_jit(body, decl, p, args, st, grid, block, smem, name)) return 0;
+      const int fuse = fin && fin->enabled;
+      snprintf(name, sizeof name, "blu_jit_dense_%d_%d%s", nv, r, fuse ? "_fused" : "");
+      snprintf(decl, sizeof decl, "%s(blu::AggParams p, blu::FinalParams fp)", name);
+      snprintf(body, sizeof body, "blu::dense_body<blu::JitSpec, %d, %d, %s>(p, fp);", nv, r, fuse ? "true" : "false");
+      FinalParams fpc = fin ? *fin : FinalParams{};
+      void* args[] = {&pc, &fpc};
+      // 2 CTAs x 512 threads per SM: <= 64 registers (one resident wave, see plan.cpp)
+      if (launch_jit(body, decl, p, args, st, grid, block, smem, name, 2)) return 0;
     } else {
       const int front = p.front_slots > 0, direct = path == BLU_PATH_DIRECT_GLOBAL, mode = p.seg_base ? 2 : 0;
       snprintf(name, sizeof name, "blu_jit_global_%d_%d_%d_%d_%d", nv, r, front, direct, mode);
@@ -405,10 +416,11 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
     if constexpr (NV > 16) {
       return (int)cudaErrorInvalidValue;
     } else {
-      auto k = k_agg_dense_smem<NV, R>;
+      note_kernel("k_agg_dense_smem (generic)");
+      auto k = (fin && fin->enabled) ? k_agg_dense_smem<NV, R, true> : k_agg_dense_smem<NV, R, false>;
       if (smem > 48 * 1024) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
       if (e) return (int)e;
-      k<<<grid, block, smem, st>>>(p);
+      k<<<grid, block, smem, st>>>(p, fin ? *fin : FinalParams{});
     }
   } else {
     void (*k)(AggParams, RecSrc);
@@ -425,6 +437,7 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
     }
     if (smem > 48 * 1024) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e) return (int)e;
+    if (!p.gate || p.gate_run_if == 0) note_kernel("k_agg_global (generic)");
     k<<<grid, block, smem, st>>>(p, rs);
   }
   count_launch(1);
@@ -432,14 +445,14 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
 }
 
 int launch_aggregate_impl(const blu_gby_plan_s* P, int path, const AggParams& p, const RecSrc& rs, bool records,
-                          void* stream, uint32_t grid, uint32_t block, uint32_t smem) {
+                          void* stream, uint32_t grid, uint32_t block, uint32_t smem, const FinalParams* fin) {
   int nv = p.lay.n_vals;
-  if (nv <= 1) return launch_agg_nv<1, 4>(P, path, p, rs, records, stream, grid, block, smem);
-  if (nv <= 2) return launch_agg_nv<2, 4>(P, path, p, rs, records, stream, grid, block, smem);
-  if (nv <= 4) return launch_agg_nv<4, 4>(P, path, p, rs, records, stream, grid, block, smem);
-  if (nv <= 8) return launch_agg_nv<8, 2>(P, path, p, rs, records, stream, grid, block, smem);
-  if (nv <= 16) return launch_agg_nv<16, 1>(P, path, p, rs, records, stream, grid, block, smem);
-  return launch_agg_nv<24, 1>(P, path, p, rs, records, stream, grid, block, smem);
+  if (nv <= 1) return launch_agg_nv<1, 4>(P, path, p, rs, records, stream, grid, block, smem, fin);
+  if (nv <= 2) return launch_agg_nv<2, 4>(P, path, p, rs, records, stream, grid, block, smem, fin);
+  if (nv <= 4) return launch_agg_nv<4, 4>(P, path, p, rs, records, stream, grid, block, smem, fin);
+  if (nv <= 8) return launch_agg_nv<8, 2>(P, path, p, rs, records, stream, grid, block, smem, fin);
+  if (nv <= 16) return launch_agg_nv<16, 1>(P, path, p, rs, records, stream, grid, block, smem, fin);
+  return launch_agg_nv<24, 1>(P, path, p, rs, records, stream, grid, block, smem, fin);
 }
 
 int launch_compact(const CompactParams& p, void* stream, uint32_t* launches) {

@@ -314,8 +314,16 @@ def test_launch_count_and_timing(bg):
     c1 = bg.blu_gby_launch_count()
     t = bg.blu_gby_last_timing()
     bg.blu_gby_set_timing(False)
-    assert c1 - c0 >= 4  # init, aggregate, compact x3
-    assert t["aggregate_ms"] > 0 and t["aggregate_launches"] == 1
+    assert c1 - c0 >= 1  # path (a): init and compaction fused into the one aggregation launch
+    assert t["aggregate_ms"] > 0 and t["aggregate_launches"] == 1 and t["kernel"]
+    os.environ["BLU_GBY_NO_FUSE"] = "1"
+    try:
+        c0 = bg.blu_gby_launch_count()
+        r = bg.blu_gby_execute(plan, kc, vc)
+        assert bg.blu_gby_launch_count() - c0 >= 4  # fill, aggregate, compact x3
+        assert r.n_groups == 16
+    finally:
+        del os.environ["BLU_GBY_NO_FUSE"]
 
 
 @pytest.mark.parametrize("parts,chunk", [("8", None), ("16", "300000"), ("64", "1000003")])
