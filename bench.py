@@ -60,6 +60,8 @@ class ClockSampler:
         self.lines = []
 
     def start(self):
+        if self.index < 0:
+            return
         try:
             self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
                                           "-i", str(self.index), "-lms", "50"], stdout=subprocess.PIPE,
@@ -179,6 +181,7 @@ def main():
     ap.add_argument("--rows", type=int, default=None, help="override rows per rank (testing only)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-clocks", action="store_true", help="do not sample nvidia-smi (diagnostics)")
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
@@ -232,7 +235,7 @@ def main():
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     agg_ms = []
     agg_kernel = ""
-    sampler = ClockSampler(local)
+    sampler = ClockSampler(local if not args.no_clocks else -1)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()

@@ -215,10 +215,31 @@ def _torch_dtype(dt):
     return _TORCH_DT[dt]
 
 
-class _DevArray:
-    """__cuda_array_interface__ provider that keeps its Result alive while a tensor views it."""
+class _Owner:
+    """Owns one library result (blu_gby_result_t) and frees it when the last reference goes away.
+    Result objects and every zero-copy tensor view reference the owner — never the other way round —
+    so no reference cycle delays the free until a garbage-collection pass."""
 
-    def __init__(self, owner, ptr: int, n: int, dt: int):
+    def __init__(self, rc: ResultC, stream: int):
+        self.rc = rc
+        self.stream = stream
+
+    def free(self):
+        rc, self.rc = self.rc, None
+        if rc is not None and rc._owner:
+            try:
+                lib.blu_gby_result_free(ctypes.byref(rc), self.stream)
+            except Exception:
+                pass
+
+    def __del__(self):
+        self.free()
+
+
+class _DevArray:
+    """__cuda_array_interface__ provider that keeps the result's owner alive while a tensor views it."""
+
+    def __init__(self, owner: _Owner, ptr: int, n: int, dt: int):
         typestr = {BLU_I32: "<i4", BLU_I64: "<i8", BLU_F64: "<f8"}[dt]
         self._owner = owner
         self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr if n else 0, False),
@@ -230,8 +251,7 @@ class Result:
     arrays (host results). Library memory is released when this object and every view are gone."""
 
     def __init__(self, rc: ResultC, key_dtypes: List[int], out_dtypes: List[int], stream: int, device=None):
-        self._rc = rc
-        self._stream = stream
+        self._owner = _Owner(rc, stream)
         self.n_groups = int(rc.n_groups)
         self.is_partial = bool(rc.is_partial)
         self.is_host = bool(rc.is_host)
@@ -256,22 +276,15 @@ class Result:
         import torch
         if n == 0:
             return torch.zeros(0, dtype=_torch_dtype(dt), device=device or "cuda")
-        return torch.as_tensor(_DevArray(self, ptr, n, dt), device=device or "cuda")
+        return torch.as_tensor(_DevArray(self._owner, ptr, n, dt), device=device or "cuda")
 
     @property
     def c(self) -> ResultC:
-        return self._rc
+        return self._owner.rc
 
     def free(self):
-        rc, self._rc = getattr(self, "_rc", None), None
-        if rc is not None and rc._owner:
-            try:
-                lib.blu_gby_result_free(ctypes.byref(rc), self._stream)
-            except Exception:
-                pass
-
-    def __del__(self):
-        self.free()
+        """Release the library memory now (views become invalid)."""
+        self._owner.free()
 
 
 def _out_dtypes(plan: Plan, partial: bool) -> List[int]:

@@ -11,6 +11,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <chrono>
 #include <functional>
 #include <mutex>
 #include <vector>
@@ -297,6 +298,7 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       delete own;
     };
     cudaError_t ae = cudaSuccess;
+    auto t_oa = std::chrono::steady_clock::now();
     for (int k = 0; k < lay.n_keys && ae == cudaSuccess; ++k) {
       ae = U ? cudaMallocAsync(&okeys[k], U * dtype_bytes(lay.key_dtype[k]), st) : cudaSuccess;
       if (okeys[k]) own->dev.push_back(okeys[k]);
@@ -305,6 +307,10 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       ae = U ? cudaMallocAsync(&ovals[o], U * dtype_bytes(os.out_dtype[o]), st) : cudaSuccess;
       if (ovals[o]) own->dev.push_back(ovals[o]);
     }
+    if (getenv("BLU_GBY_DEBUG_HOST"))
+      fprintf(stderr, "[blugby host] output alloc %.3f ms (%llu rows)\n",
+              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_oa).count(),
+              (unsigned long long)U);
     if (ae != cudaSuccess) {
       cudaGetLastError();
       free_owner();
@@ -366,8 +372,13 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     uint64_t* hs = pinned_scratch();
     uint64_t hbuf[2] = {0, 0};
     uint64_t* dst = hs ? hs : hbuf;
+    static const bool hdbg = getenv("BLU_GBY_DEBUG_HOST") != nullptr;
+    auto t_sync0 = std::chrono::steady_clock::now();
     cudaError_t ce = cudaMemcpyAsync(dst, small, 16, cudaMemcpyDeviceToHost, st);
     if (ce == cudaSuccess) ce = cudaStreamSynchronize(st);
+    if (hdbg)
+      fprintf(stderr, "[blugby host] final sync waited %.3f ms\n",
+              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_sync0).count());
     if (ce != cudaSuccess) {
       cudaGetLastError();
       free_owner();
@@ -471,26 +482,36 @@ static bool nonnull_cols(const void* const* cols, int n) {
 static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, const void* const* keys,
                                     const void* const* vals, uint64_t n, cudaStream_t st, uint32_t* launches,
                                     Work& w) {
+  static const bool hdbg = getenv("BLU_GBY_DEBUG_HOST") != nullptr;
+  auto now = [] { return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count(); };
+  const double h0 = now();
   const Layout& L = P->lay;
   const uint32_t B = P->parts;
   size_t row_bytes = 8;
   for (int c = 0; c < L.n_vals; ++c) row_bytes += dtype_bytes(L.val_dtype[c]);
-  size_t free_b = 0, total_b = 0;
-  cudaMemGetInfo(&free_b, &total_b);
-  {  // memory cached by the stream-ordered pool (reserved, not in use) is available too
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaMemPool_t pool;
-    uint64_t reserved = 0, used = 0;
-    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess &&
-        cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved) == cudaSuccess &&
-        cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used) == cudaSuccess && reserved > used)
-      free_b += (size_t)(reserved - used);
-    cudaGetLastError();
+  // Chunk rows: decided once per plan from the free memory (cudaMemGetInfo and the pool queries are
+  // host-side calls that would otherwise sit between this query's launches every time).
+  uint64_t M = P->part_chunk.load();
+  if (M == 0) {
+    size_t free_b = 0, total_b = 0;
+    cudaMemGetInfo(&free_b, &total_b);
+    {  // memory cached by the stream-ordered pool (reserved, not in use) is available too
+      int dev = 0;
+      cudaGetDevice(&dev);
+      cudaMemPool_t pool;
+      uint64_t reserved = 0, used = 0;
+      if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess &&
+          cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved) == cudaSuccess &&
+          cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used) == cudaSuccess && reserved > used)
+        free_b += (size_t)(reserved - used);
+      cudaGetLastError();
+    }
+    free_b += cache_idle_bytes();  // idle workspace blocks are reusable
+    uint64_t budget_rows = (uint64_t)((double)free_b * 0.6 / (double)row_bytes / 1.03);
+    M = std::max<uint64_t>(budget_rows, 1ull << 22);
+    P->part_chunk.store(M);
   }
-  free_b += cache_idle_bytes();  // idle workspace blocks are reusable
-  uint64_t budget_rows = (uint64_t)((double)free_b * 0.6 / (double)row_bytes / 1.03);
-  uint64_t M = std::min<uint64_t>(n, std::max<uint64_t>(budget_rows, 1ull << 22));
+  M = std::min<uint64_t>(n, M);
   if (const char* cr = getenv("BLU_GBY_PART_CHUNK")) M = std::min<uint64_t>(n, std::max<uint64_t>(1024, strtoull(cr, 0, 10)));
   uint64_t seg_cap = ((uint64_t)((double)((M + B - 1) / B) * 1.03) + 4096 + 63) & ~63ull;
   uint64_t rows_alloc = seg_cap * B;
@@ -501,13 +522,9 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   for (int c = 0; c < L.n_vals && e == cudaSuccess; ++c) e = w.alloc(&vbuf[c], rows_alloc * dtype_bytes(L.val_dtype[c]));
   if (e == cudaSuccess) e = w.alloc(&meta, (size_t)B * 16 + 64);
   if (e != cudaSuccess) return e;
-  uint64_t* d_seg_base = (uint64_t*)meta;
-  uint64_t* d_cursor = d_seg_base + B;
+  const double h1 = now();
+  uint64_t* d_cursor = (uint64_t*)meta;
   uint32_t* d_gate = (uint32_t*)(d_cursor + B);
-  std::vector<uint64_t> hb(B);
-  for (uint32_t b = 0; b < B; ++b) hb[b] = (uint64_t)b * seg_cap;
-  e = cudaMemcpyAsync(d_seg_base, hb.data(), (size_t)B * 8, cudaMemcpyHostToDevice, st);
-  if (e) return e;
   uint32_t scatter_grid = (uint32_t)P->sms * 2;
   Layout L2 = L;  // pass 2 reads the packed u64 key as a single sparse key column
   L2.n_keys = 1;
@@ -535,14 +552,21 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       while ((1u << lb) < B) ++lb;
       sp.shift = lc > lb ? lc - lb : 0;
     }
-    sp.seg_base = d_seg_base;
+    sp.seg_stride = seg_cap;
     sp.cursor = d_cursor;
     sp.seg_cap = seg_cap;
     sp.out_key = (uint64_t*)kbuf;
     for (int c = 0; c < L.n_vals; ++c) sp.out_val[c] = vbuf[c];
     sp.gate = d_gate;
+    static const bool dbg = getenv("BLU_GBY_DEBUG_PART") != nullptr;
+    cudaEvent_t ev[4];
+    if (dbg) {
+      for (auto& x : ev) cudaEventCreate(&x);
+      cudaEventRecord(ev[0], st);
+    }
     int le = launch_scatter(p1, sp, st, scatter_grid);
     if (le) return (cudaError_t)le;
+    if (dbg) cudaEventRecord(ev[1], st);
     // pass 2 (runs if no bucket overflowed)
     AggParams p2 = base;
     p2.lay = L2;
@@ -550,7 +574,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     for (int c = 0; c < L.n_vals; ++c) p2.val[c] = vbuf[c];
     p2.vec_ok = 1;
     p2.n_rows = 0;
-    p2.seg_base = d_seg_base;
+    p2.seg_stride = seg_cap;
     p2.seg_count = d_cursor;
     p2.n_segs = B;
     p2.tile_ctr = getenv("BLU_GBY_DYN") && atoi(getenv("BLU_GBY_DYN")) == 0 ? nullptr : (uint64_t*)(d_cursor + B + 1);
@@ -564,11 +588,26 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     p3.jit_ok = 0;  // gated fallback, normally a no-op: keep the precompiled kernel
     p3.gate = d_gate;
     p3.gate_run_if = 1;
+    if (dbg) cudaEventRecord(ev[2], st);
     le = launch_aggregate_impl(P, BLU_PATH_HASH_GLOBAL, p3, RecSrc{nullptr, 0}, false, st, P->grid, P->block,
                                P->smem_bytes);
     if (le) return (cudaError_t)le;
+    if (dbg) {
+      cudaEventRecord(ev[3], st);
+      cudaEventSynchronize(ev[3]);
+      float a = 0, b = 0, c = 0;
+      cudaEventElapsedTime(&a, ev[0], ev[1]);
+      cudaEventElapsedTime(&b, ev[1], ev[2]);
+      cudaEventElapsedTime(&c, ev[2], ev[3]);
+      uint32_t gate = 0;
+      cudaMemcpy(&gate, d_gate, 4, cudaMemcpyDeviceToHost);
+      fprintf(stderr, "[blugby part] chunk rows %llu B %u seg_cap %llu: scatter %.2f ms pass2 %.2f ms fallback %.2f ms gate %u\n",
+              (unsigned long long)m, B, (unsigned long long)seg_cap, a, b, c, gate);
+      for (auto& x : ev) cudaEventDestroy(x);
+    }
     if (launches) *launches += 3;
   }
+  if (hdbg) fprintf(stderr, "[blugby host] feed: alloc %.3f ms, launches %.3f ms\n", h1 - h0, now() - h1);
   return cudaSuccess;
 }
 

@@ -794,8 +794,8 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
         uint32_t mid = (lo + hi + 1) >> 1;
         if (tpre[mid] <= t) lo = mid; else hi = mid - 1;
       }
-      row0 = p.seg_base[lo] + (t - tpre[lo]) * tile;
-      n = p.seg_base[lo] + p.seg_count[lo];
+      row0 = (uint64_t)lo * p.seg_stride + (t - tpre[lo]) * tile;
+      n = (uint64_t)lo * p.seg_stride + p.seg_count[lo];
       row = lane_base<R>(row0, 0, lane);
     } else {
       row = lane_base<R>(row0, threadIdx.x >> 5, lane);
@@ -1038,7 +1038,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
       const uint32_t b = sbid[e];
       const uint64_t g = gpos[b] + (e - lstart[b]);
       if (g >= sp.seg_cap) continue;
-      const uint64_t idx = sp.seg_base[b] + g;
+      const uint64_t idx = (uint64_t)b * sp.seg_stride + g;
       sp.out_key[idx] = skey[e];
 #pragma unroll
       for (int c = 0; c < NV; ++c)

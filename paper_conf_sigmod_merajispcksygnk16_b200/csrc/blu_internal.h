@@ -47,6 +47,7 @@ struct blu_gby_plan_s {
   int32_t sms;
   uint32_t parts;         // path b: buckets of the partitioned two-pass mode (1 = one pass)
   uint32_t part_shift;    // log2(cap) - log2(parts)
+  mutable std::atomic<uint64_t> part_chunk{0};  // rows per partitioned chunk (decided at first execute)
   mutable std::atomic<uint32_t> retries_last{0};
 };
 

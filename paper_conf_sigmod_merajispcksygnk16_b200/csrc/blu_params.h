@@ -93,8 +93,9 @@ struct AggParams {
   uint32_t soff[kMaxFields];     // per field: byte offset of its SoA array
   uint32_t colmask[kMaxFields];  // per kernel value column: bit j = field j reads it
   uint32_t cntmask;              // fields that count the constant 1
-  // partitioned pass 2 (segments mode): rows of segment b are [seg_base[b], seg_base[b] + seg_count[b])
-  const uint64_t* seg_base;
+  // partitioned pass 2 (segments mode, seg_stride > 0): rows of segment b are
+  // [b * seg_stride, b * seg_stride + seg_count[b])
+  uint64_t seg_stride;
   const uint64_t* seg_count;
   uint32_t n_segs;
   uint64_t* tile_ctr;            // segments mode: dynamic warp-tile counter (zeroed per launch)
@@ -125,7 +126,7 @@ struct FinalParams {
 struct ScatterParams {
   uint32_t B;
   uint32_t shift;            // bucket = (fmix64(key) & cap_mask) >> shift
-  const uint64_t* seg_base;  // B: first row of each bucket in the partition buffers
+  uint64_t seg_stride;       // bucket b starts at row b * seg_stride of the partition buffers
   uint64_t* cursor;          // B: rows appended so far (zeroed per chunk)
   uint64_t seg_cap;          // rows per bucket
   uint64_t* out_key;         // packed keys (u64)

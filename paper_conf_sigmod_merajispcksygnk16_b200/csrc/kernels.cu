@@ -107,7 +107,7 @@ __global__ void __launch_bounds__(512, 2) k_agg_dense_smem(AggParams p, FinalPar
 }
 
 template <int NV, int R, bool FRONT, bool DIRECT, int MODE>
-__global__ void __launch_bounds__(512) k_agg_global(AggParams p, RecSrc rs) {
+__global__ void __launch_bounds__(512, 2) k_agg_global(AggParams p, RecSrc rs) {
   global_body<GenericSpec, NV, R, FRONT, DIRECT, MODE>(p, rs);
 }
 
@@ -403,13 +403,14 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
       // 2 CTAs x 512 threads per SM: <= 64 registers (one resident wave, see plan.cpp)
       if (launch_jit(body, decl, p, args, st, grid, block, smem, name, 2)) return 0;
     } else {
-      const int front = p.front_slots > 0, direct = path == BLU_PATH_DIRECT_GLOBAL, mode = p.seg_base ? 2 : 0;
+      const int front = p.front_slots > 0, direct = path == BLU_PATH_DIRECT_GLOBAL, mode = p.seg_stride ? 2 : 0;
       snprintf(name, sizeof name, "blu_jit_global_%d_%d_%d_%d_%d", nv, r, front, direct, mode);
       snprintf(decl, sizeof decl, "%s(blu::AggParams p, blu::RecSrc rs)", name);
       snprintf(body, sizeof body, "blu::global_body<blu::JitSpec, %d, %d, %s, %s, %d>(p, rs);", nv, r,
                front ? "true" : "false", direct ? "true" : "false", mode);
       void* args[] = {&pc, &rc};
-      if (launch_jit(body, decl, p, args, st, grid, block, smem, name)) return 0;
+      // <= 64 registers: 2 CTAs of 512 (front) or 4 of 256 threads per SM stay resident
+      if (launch_jit(body, decl, p, args, st, grid, block, smem, name, 2)) return 0;
     }
   }
   if (path == BLU_PATH_DENSE_SMEM) {
@@ -431,7 +432,7 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
       k = k_agg_global<NV, R, false, false, 0>;
     } else {
       if (records) k = k_agg_global<NV, R, false, false, 1>;
-      else if (p.seg_base) k = k_agg_global<NV, R, false, false, 2>;
+      else if (p.seg_stride) k = k_agg_global<NV, R, false, false, 2>;
       else if (direct) k = front ? k_agg_global<NV, R, true, true, 0> : k_agg_global<NV, R, false, true, 0>;
       else k = front ? k_agg_global<NV, R, true, false, 0> : k_agg_global<NV, R, false, false, 0>;
     }

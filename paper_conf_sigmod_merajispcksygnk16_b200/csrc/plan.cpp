@@ -161,7 +161,7 @@ void fill_smem_layout(AggParams& p, uint32_t S, bool with_keys) {
     p.soff[j] = o;
     o += (S * (uint32_t)L.f[j].ssize + 15) / 16 * 16;
   }
-  p.seg_base = nullptr;
+  p.seg_stride = 0;
   p.seg_count = nullptr;
   p.n_segs = 0;
   p.gate = nullptr;

@@ -11,7 +11,11 @@ torch.cuda.synchronize()
 plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
 print(json.dumps(plan.info()))
 bg.blu_gby_set_timing(True)
+flush = torch.empty(512 * 2**20, dtype=torch.uint8, device="cuda") if os.environ.get("FLUSH") else None
 for i in range(int(os.environ.get('ITERS', '4'))):
+    if flush is not None:
+        flush.zero_()
+        torch.cuda.synchronize()
     t0 = time.perf_counter()
     r = bg.blu_gby_execute(plan, kc, vc)
     t1 = time.perf_counter()
