@@ -112,7 +112,7 @@ __global__ void __launch_bounds__(512, 2) k_agg_global(AggParams p, RecSrc rs) {
 }
 
 template <int NV, int R>
-__global__ void __launch_bounds__(512) k_scatter(AggParams p, ScatterParams sp) {
+__global__ void __launch_bounds__(512, 2) k_scatter(AggParams p, ScatterParams sp) {
   scatter_body<GenericSpec, NV, R>(p, sp);
 }
 
@@ -128,7 +128,7 @@ static int launch_scatter_nv(const AggParams& p, const ScatterParams& sp, cudaSt
     AggParams pc = p;
     ScatterParams sc = sp;
     void* args[] = {&pc, &sc};
-    if (launch_jit(body, decl, p, args, st, grid, 512, (uint32_t)smem, name)) return 0;
+    if (launch_jit(body, decl, p, args, st, grid, 512, (uint32_t)smem, name, 2)) return 0;
   }
   auto k = k_scatter<NV, R>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
