@@ -202,6 +202,18 @@ blu_status_t blu_gby_merge_records(blu_gby_plan_t plan, const void* records, uin
                                    void* stream, int32_t partial_out, blu_gby_result_t* out);
 uint32_t blu_gby_record_bytes(blu_gby_plan_t plan);
 
+/* ---- group-count estimate --------------------------------------------
+ * KMV ("K-minimum values") estimate of the number of distinct key tuples in n_rows DEVICE key
+ * columns — the estimate the paper computes on CPU threads right after hashing and feeds to the GPU
+ * runtime ("use a simple hash function and KMV[2] algorithm to estimate the number of
+ * groups"). est = (k-1) * 2^64 / (k-th smallest distinct 64-bit key hash); if fewer than k
+ * distinct hashes exist the count is exact (*exact = 1). Relative standard error ~ 1/sqrt(k-2).
+ * k in [16, 2048]. Depends only on the set of keys (not on row order or launch shape). Synchronises
+ * `stream`. Errors: BLU_E_INVALID, BLU_E_UNSUPPORTED, BLU_E_KEY_RANGE (a code outside its
+ * dictionary), BLU_E_OOM. */
+blu_status_t blu_gby_estimate_groups(const blu_key_desc_t* keys, int32_t n_keys, const void* const* key_cols,
+                                     uint64_t n_rows, uint32_t k, void* stream, double* est, int32_t* exact);
+
 /* ---- S4 table initialisation (Table 1) -------------------------------------
  * The slot template ("hash table mask"): key all-ones ("M/4 Fs"), SUM 0, MAX the type minimum,
  * MIN the type maximum, COUNT 0, padding 0. slot_template copies slot_bytes bytes into `out`

@@ -86,6 +86,7 @@ def _load():
         "blu_gby_partition": ([vp, P(ResultC), i32, vp, vp, P(u64)], i32),
         "blu_gby_merge_records": ([vp, vp, u64, vp, i32, P(ResultC)], i32),
         "blu_gby_record_bytes": ([vp], u32),
+        "blu_gby_estimate_groups": ([P(KeyDesc), i32, P(vp), u64, u32, vp, P(ctypes.c_double), P(i32)], i32),
         "blu_gby_slot_template": ([vp, vp, u32, P(u32)], i32),
         "blu_gby_init_table": ([vp, vp, u64, vp], i32),
         "blu_gby_set_timing": ([i32], None),
@@ -199,6 +200,13 @@ def blu_gby_plan(keys: Sequence[Tuple[int, int]], vals: Sequence[int], aggs: Seq
 def plan_for(schema, est_groups: int, n_rows: int) -> Plan:
     """Plan from any object with .keys / .vals / .aggs (e.g. blugen.Schema)."""
     return blu_gby_plan(schema.keys, schema.vals, schema.aggs, est_groups, n_rows)
+
+
+def plan_estimated(schema, key_cols, n_rows: Optional[int] = None, k: int = 2048, stream=None) -> Plan:
+    """The paper's pipeline: KMV-estimate the group count on the device, then plan."""
+    est, _ = blu_gby_estimate_groups(schema.keys, key_cols, k=k, n_rows=n_rows, stream=stream)
+    n = int(len(key_cols[0]) if n_rows is None else n_rows)
+    return blu_gby_plan(schema.keys, schema.vals, schema.aggs, max(1, int(round(est))), n)
 
 
 # ---------------------------------------------------------------------------------------------
@@ -402,6 +410,17 @@ def blu_gby_finalize_dense_state(plan: Plan, state_arrays, stream=None) -> Resul
     rc = ResultC()
     _check(lib.blu_gby_finalize_dense_state(plan.handle, _ptrs(state_arrays), s, ctypes.byref(rc)))
     return Result(rc, _key_dtypes(plan), _out_dtypes(plan, False), s, _device_of(state_arrays))
+
+
+def blu_gby_estimate_groups(keys: Sequence[Tuple[int, int]], key_cols, k: int = 2048, n_rows: Optional[int] = None,
+                            stream=None) -> Tuple[float, bool]:
+    """KMV estimate of the number of distinct key tuples: (estimate, exact)."""
+    kd = (KeyDesc * max(1, len(keys)))(*[KeyDesc(int(d), int(s)) for d, s in keys])
+    n = int(len(key_cols[0]) if n_rows is None else n_rows)
+    est, exact = ctypes.c_double(), ctypes.c_int32()
+    _check(lib.blu_gby_estimate_groups(kd, len(keys), _ptrs(key_cols), n, int(k), _stream_handle(stream),
+                                       ctypes.byref(est), ctypes.byref(exact)))
+    return est.value, bool(exact.value)
 
 
 def blu_gby_init_table(plan: Plan, dev_table, n_slots: int, stream=None):

@@ -365,3 +365,64 @@ def test_partitioned_with_regrow(bg, oracles, monkeypatch):
     res = bg.blu_gby_execute(plan, kc, vc)
     gk, ga = gpu_sorted(res, w.schema)
     assert_parity(gk, ga, o, w.schema)
+
+
+def _kmv_reference(keys_packed, k):
+    """Independent numpy statement of the KMV estimate (same definition, no shared code):
+    h = fmix64(packed ^ salt); est = (k-1) * 2^64 / (k-th smallest distinct h), exact if < k."""
+    M = (1 << 64) - 1
+    h = (keys_packed.astype(np.uint64) ^ np.uint64(0x6b6d765f73616c74))
+    with np.errstate(over="ignore"):
+        h ^= h >> np.uint64(33)
+        h *= np.uint64(0xff51afd7ed558ccd)
+        h ^= h >> np.uint64(33)
+        h *= np.uint64(0xc4ceb9fe1a85ec53)
+        h ^= h >> np.uint64(33)
+    u = np.unique(h)
+    u = u[u != np.uint64(M)]
+    if u.size < k:
+        return float(u.size), True
+    return (k - 1) * 18446744073709551616.0 / float(int(u[k - 1])), False
+
+
+@pytest.mark.parametrize("G,n,k", [(700, 200_000, 2048), (50_000, 3_000_000, 2048), (1_000_000, 4_000_000, 1024)])
+def test_kmv_estimate(bg, G, n, k):
+    """NEXT-3: on-GPU KMV estimate equals the numpy statement of the same definition,
+    is exact below k distinct keys, and lands within 5 standard errors of the true count."""
+    w = blugen.workload("C3", n_rows=n, n_groups=G)
+    kc, _ = blugen.device_columns(w)
+    est, exact = bg.blu_gby_estimate_groups(w.schema.keys, kc, k=k)
+    host = kc[0].cpu().numpy()
+    ref, ref_exact = _kmv_reference(host, k)
+    true = len(np.unique(host))
+    assert exact == ref_exact and est == ref
+    if exact:
+        assert est == true
+    else:
+        assert abs(est - true) <= 5 * true / np.sqrt(k - 2)
+    # order invariance: the same key set in a different row order gives the same estimate
+    perm = torch.randperm(n, device="cuda")
+    est2, _ = bg.blu_gby_estimate_groups(w.schema.keys, [kc[0][perm].contiguous()], k=k)
+    assert est2 == est
+
+
+def test_kmv_dense_composite_keys(bg):
+    w = blugen.workload("C4", n_rows=2_000_000)
+    kc, _ = blugen.device_columns(w)
+    est, exact = bg.blu_gby_estimate_groups(w.schema.keys, kc, k=2048)
+    packed = kc[0].long() + 100 * kc[1].long() + 5000 * kc[2].long()
+    ref, ref_exact = _kmv_reference(packed.cpu().numpy(), 2048)
+    assert est == ref and exact == ref_exact
+    true = int(torch.unique(packed).numel())
+    assert abs(est - true) <= 5 * true / np.sqrt(2046)
+
+
+def test_plan_from_device_estimate(bg, oracles):
+    """Estimate -> plan -> execute, the paper's runtime order."""
+    w, o = oracles("C5")
+    kc, vc = blugen.device_columns(w)
+    plan = bg.plan_estimated(w.schema, kc)
+    assert abs(plan.info()["est_groups"] - w.expected_groups) <= 0.15 * w.expected_groups
+    res = bg.blu_gby_execute(plan, kc, vc)
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
