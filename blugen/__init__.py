@@ -243,7 +243,20 @@ def _c5(n_rows=4_000_000_000, n_groups=50_000_000) -> Workload:
                     "1 sparse i64 key, 50M groups; COUNT, SUM, AVG; sharded over GPUs")
 
 
-WORKLOADS = {"C1": _c1, "C2": _c2, "C3": _c3, "C4": _c4, "C5": _c5}
+def _k3(n_rows=100_000_000, n_groups=50_000_000) -> Workload:
+    """Kernel-3 study: many aggregates (8 state fields) and a low
+    rows/groups ratio (2 rows per group) — where the paper prefers one row lock over per-field atomics."""
+    seed = 0x5EED0013
+    keys = [Col(I64, SPARSE_KEY, 0, n_groups=n_groups)]
+    vals = [Col(I32, UNIFORM, 1, 1, 101), Col(I64, UNIFORM, 2, 0, 10**7), Col(F64, DYADIC, 3),
+            Col(I64, UNIFORM, 4, -(10**9), 10**9)]
+    sch = Schema([(I64, 0)], [I32, I64, F64, I64],
+                 [(COUNT, -1), (SUM, 0), (MIN, 0), (MAX, 0), (SUM, 1), (AVG, 2), (MIN, 3), (MAX, 3)])
+    return Workload("K3", n_rows, seed, keys, vals, sch, n_groups, n_groups,
+                    "kernel-3 study: sparse i64 key, 2 rows/group, 8 aggregates")
+
+
+WORKLOADS = {"C1": _c1, "C2": _c2, "C3": _c3, "C4": _c4, "C5": _c5, "K3": _k3}
 
 
 def workload(name: str, n_rows: Optional[int] = None, n_groups: Optional[int] = None) -> Workload:

@@ -136,6 +136,7 @@ typedef struct {
     int32_t state_dtypes[32];/* blu_dtype_t of each state field                                   */
     uint32_t grid, block;    /* aggregation launch shape                                          */
     uint32_t retries_last;
+    int32_t row_lock;        /* (b): kernel 3 — one row lock per slot, then every aggregate */
 } blu_gby_plan_desc_t;
 blu_status_t blu_gby_plan_describe(blu_gby_plan_t plan, blu_gby_plan_desc_t* out);
 

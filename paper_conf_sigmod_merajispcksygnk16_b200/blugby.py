@@ -56,7 +56,7 @@ class PlanDescC(ctypes.Structure):
                 ("slot_bytes", ctypes.c_uint32), ("smem_bytes", ctypes.c_uint32), ("hot_front", ctypes.c_int32),
                 ("front_slots", ctypes.c_uint32), ("partitions", ctypes.c_uint32), ("n_states", ctypes.c_int32),
                 ("state_dtypes", ctypes.c_int32 * 32), ("grid", ctypes.c_uint32), ("block", ctypes.c_uint32),
-                ("retries_last", ctypes.c_uint32)]
+                ("retries_last", ctypes.c_uint32), ("row_lock", ctypes.c_int32)]
 
 
 class TimingC(ctypes.Structure):

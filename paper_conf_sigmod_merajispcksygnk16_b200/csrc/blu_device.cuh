@@ -613,6 +613,77 @@ __device__ __forceinline__ void dense_body(const AggParams& p, const FinalParams
 // ------------------------------------------------------------------------------------------------
 // S5b: path (b) global hash table / path (b') direct-mapped, optional shared-memory hot-key front
 // ------------------------------------------------------------------------------------------------
+// ---- kernel 3: one row lock per slot, then every aggregate with plain L2 accesses -------
+__device__ __forceinline__ void row_lock_acquire(uint32_t* l) {
+  for (;;) {
+    uint32_t old;
+    asm volatile("atom.acquire.gpu.global.cas.b32 %0, [%1], 0, 1;" : "=r"(old) : "l"(l) : "memory");
+    if (old == 0) return;
+    __nanosleep(32);
+  }
+}
+__device__ __forceinline__ void row_lock_release(uint32_t* l) {
+  asm volatile("st.release.gpu.global.b32 [%0], 0;" ::"l"(l) : "memory");
+}
+
+// field update under the row lock (the stored encodings of g_upd: 4-byte i32 MIN/MAX, ordered f64)
+template <int K>
+__device__ __forceinline__ void locked_upd(uint8_t* a, uint64_t raw) {
+  const uint64_t x = enc<K, true>(raw);
+  if constexpr (K == FK_COUNT || K == FK_SUMI) {
+    __stcg((unsigned long long*)a, __ldcg((const unsigned long long*)a) + x);
+  } else if constexpr (K == FK_SUMF) {
+    const double o = __longlong_as_double((long long)__ldcg((const unsigned long long*)a));
+    __stcg((unsigned long long*)a, (unsigned long long)__double_as_longlong(o + __longlong_as_double((long long)x)));
+  } else if constexpr (K == FK_MINI32 || K == FK_MAXI32) {
+    const int o = __ldcg((const int*)a), v = (int)x;
+    if (K == FK_MINI32 ? v < o : v > o) __stcg((int*)a, v);
+  } else if constexpr (K == FK_MINI64 || K == FK_MINF64) {
+    const long long o = (long long)__ldcg((const unsigned long long*)a);
+    if ((long long)x < o) __stcg((unsigned long long*)a, x);
+  } else {
+    const long long o = (long long)__ldcg((const unsigned long long*)a);
+    if ((long long)x > o) __stcg((unsigned long long*)a, x);
+  }
+}
+
+// Kernel 3: for each row in `mask`, lock its slot, apply every aggregate, unlock ("each thread
+// locks the entire row of the hash table after it finds out that its key matches ... goes through all
+// the aggregation functions and applies them one by one. Finally, the thread releases the lock").
+template <class SP, int NV, int R>
+__device__ __forceinline__ void global_apply_rows_locked(const AggParams& p, const uint64_t (&slot)[R], uint32_t mask,
+                                                         const uint64_t (&v)[NV][R]) {
+  const Layout& L = p.lay;
+  uint8_t* tb = (uint8_t*)p.table;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    if (!(mask >> r & 1)) continue;
+    uint8_t* s = tb + slot[r] * L.slot_bytes;
+    uint32_t* lk = (uint32_t*)(s + L.lock_off);
+    row_lock_acquire(lk);
+    if constexpr (SP::kStatic) {
+      sfor<0, SP::NF>([&](auto jc) {
+        constexpr int j = decltype(jc)::v;
+        constexpr int c = SP::COL[j], KK = c < 0 ? FK_COUNT : SP::KIND[j], goff = SP::GOFF[j];
+        locked_upd<KK>(s + goff, c < 0 ? 1ull : v[c < 0 ? 0 : c][r]);
+      });
+    } else {
+      for (int j = 0; j < L.n_fields; ++j) {
+        const int c = L.f[j].col;
+        uint64_t x = 1ull;
+#pragma unroll
+        for (int cc = 0; cc < NV; ++cc)
+          if (cc == c) x = v[cc][r];
+        dispatch_kind(c < 0 ? (int)FK_COUNT : L.f[j].kind, [&](auto kc) {
+          constexpr int K = decltype(kc)::v;
+          locked_upd<K>(s + L.f[j].goff, x);
+        });
+      }
+    }
+    row_lock_release(lk);
+  }
+}
+
 // ---- JIT front path with warp-level pre-aggregation (skewed keys) -----------------------------
 template <int K>
 __device__ __forceinline__ uint64_t combine_vals(uint64_t a, uint64_t b) {
@@ -918,7 +989,8 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
       }
       __syncwarp();  // reconverge before the field reductions so each RED instruction is warp-wide
     }
-    global_apply_rows<SP, NV, R, DIRECT>(p, slot, miss, v);
+    if (!DIRECT && L.lock_off) global_apply_rows_locked<SP, NV, R>(p, slot, miss, v);  // kernel 3
+    else global_apply_rows<SP, NV, R, DIRECT>(p, slot, miss, v);
     t = t_next;
   }
   if (FRONT) {

@@ -66,6 +66,7 @@ struct Layout {
   uint32_t slot_bytes;           // global AoS slot (key + fields, padded)
   int32_t n_group[4];            // fields per StateGroup
   uint32_t smem_entry_bytes;     // per entry of a shared-memory table (no key)
+  int32_t lock_off;              // kernel 3: byte offset of the slot's row lock, 0 = none
 };
 
 // ---------------------------------------------------------------------------------------------

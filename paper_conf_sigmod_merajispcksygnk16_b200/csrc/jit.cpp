@@ -129,6 +129,7 @@ std::string spec_source(const char* name, const Layout& L) {
   s += "  static constexpr int SIDX[24] = " + arr(si, L.n_fields, 24) + ";\n";
   s += "  static constexpr unsigned long long SLOT = " + std::to_string(L.slot_bytes) + "ULL;\n";
   s += "  static constexpr unsigned long long DOMAIN = " + std::to_string((unsigned long long)L.domain) + "ULL;\n";
+  s += "  static constexpr int LOCKOFF = " + std::to_string(L.lock_off) + ";\n";
   const char* dd = getenv("BLU_GBY_DEDUPE");
   s += std::string("  static constexpr int DEDUPE = ") + (dd && dd[0] == '1' ? "1" : "0") + ";\n";
   s += "};\n}  // namespace blu\n";

@@ -54,6 +54,7 @@ constexpr uint64_t kMinCap = 1024;
 constexpr uint64_t kFrontRatio = 1000;          // rows/groups above which the front pays off
 constexpr uint32_t kFrontBudget = 110 * 1024;
 constexpr uint64_t kDirectMin = 1ull << 20;
+constexpr uint64_t kRowLockRatio = 16;          // kernel 3 when rows/groups <= this
 constexpr uint32_t kPartBudgetMB = 48;          // L2 slice per bucket (126 MB L2)
 
 static int32_t field_gsize(int kind) { return (kind == FK_MINI32 || kind == FK_MAXI32) ? 4 : 8; }
@@ -96,6 +97,15 @@ static void finish_layout(Layout& L) {
   if (sb < raw) sb = (raw + 63) / 64 * 64;
   L.slot_bytes = sb;
   L.smem_entry_bytes = smem_entry_bytes(L);
+  if (L.lock_off) {  // kernel 3: a 4-byte row lock after the fields (re-padded slot)
+    uint32_t lo = (off + 3) / 4 * 4;
+    L.lock_off = (int32_t)lo;
+    uint32_t raw2 = (lo + 4 + 7) / 8 * 8;
+    uint32_t sb2 = 16;
+    while (sb2 < raw2 && sb2 < 128) sb2 <<= 1;
+    if (sb2 < raw2) sb2 = (raw2 + 63) / 64 * 64;
+    L.slot_bytes = sb2;
+  }
 }
 
 static int add_field(Layout& L, int kind, int col, int is_count) {
@@ -307,6 +317,24 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   }
   P->cap = path == BLU_PATH_HASH_GLOBAL ? cap_est : D;
 
+  // Kernel 3: "if both 1) the number of aggregation functions is large [more than 5] 2) number
+  // of rows/number groups is small, this kernel would have very good performance" — lock the slot
+  // once and apply every aggregate, instead of one atomic per aggregate. Hash path only (AoS slots).
+  // On B200 every aggregate of this library has a native fire-and-forget 64-bit L2 reduction, and the
+  // lock costs two round trips per row: measured slower even in the paper's regime (K3: 14.3 vs 11.0
+  // ms; C4 hot keys: 53 vs 3 ms per 1e8 rows), so the rule is kept but off unless requested
+  // (BLU_GBY_ROW_LOCK=1, or =rule to apply the paper's rule).
+  {
+    const bool rule = path == BLU_PATH_HASH_GLOBAL && L.n_fields > 5 && n_rows <= kRowLockRatio * P->est_groups;
+    bool lock = false;
+    if (const char* rl = env("BLU_GBY_ROW_LOCK"))
+      lock = path == BLU_PATH_HASH_GLOBAL && (rl[0] == '1' || (rl[0] == 'r' && rule));
+    if (lock) {
+      L.lock_off = 1;  // placeholder: finish_layout assigns the real offset
+      finish_layout(L);
+    }
+  }
+
   // Partitioned two-pass mode for path (b) when the table exceeds an L2-sized budget: rows are
   // first scattered into B buckets by the top bits of their slot, then aggregated bucket by bucket
   // so each bucket's slice of the table stays L2-resident (126 MB L2).
@@ -384,6 +412,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   // merge layout: rows are (keys, one column per state field); COUNT becomes SUM of counts.
   Layout& M = P->merge_lay;
   M = L;
+  M.lock_off = 0;
   M.n_vals = L.n_fields;
   for (int j = 0; j < L.n_fields; ++j) {
     int k = L.f[j].kind;
@@ -424,6 +453,7 @@ blu_status_t blu_gby_plan_describe(blu_gby_plan_t P, blu_gby_plan_desc_t* o) {
   o->grid = P->grid;
   o->block = P->block;
   o->retries_last = P->retries_last.load();
+  o->row_lock = P->lay.lock_off ? 1 : 0;
   return BLU_OK;
 }
 

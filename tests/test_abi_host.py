@@ -152,3 +152,17 @@ def test_forced_path_env(bg, monkeypatch):
 def test_record_bytes(bg):
     p = bg.plan_for(blugen.workload("C3").schema, 10**7, 10**9)
     assert p.record_bytes == 8 * (1 + 3)
+
+
+def test_planner_kernel3_rule(bg, monkeypatch):
+    """more than 5 aggregation functions and a low rows/groups ratio -> kernel 3 (row lock).
+    Off by default on B200 (native 64-bit REDs measured faster); BLU_GBY_ROW_LOCK=rule applies it."""
+    k3 = bg.plan_for(blugen.workload("K3").schema, 50_000_000, 100_000_000).info()
+    assert k3["path"] == bg.BLU_PATH_HASH_GLOBAL and k3["row_lock"] == 0 and k3["n_states"] == 8
+    monkeypatch.setenv("BLU_GBY_ROW_LOCK", "rule")
+    k3 = bg.plan_for(blugen.workload("K3").schema, 50_000_000, 100_000_000).info()
+    assert k3["row_lock"] == 1
+    c3 = bg.plan_for(blugen.workload("C3").schema, 10**7, 10**9).info()
+    assert c3["row_lock"] == 0  # 3 fields
+    hi = bg.plan_for(blugen.workload("K3").schema, 1000, 100_000_000).info()
+    assert hi["row_lock"] == 0  # 1e5 rows per group: contention, keep per-field atomics

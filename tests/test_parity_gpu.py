@@ -32,6 +32,7 @@ SCALED = {
     "C3": dict(n_rows=2_000_003, n_groups=60_000),
     "C4": dict(n_rows=3_000_017),
     "C5": dict(n_rows=2_500_001, n_groups=150_000),
+    "K3": dict(n_rows=2_000_003, n_groups=1_000_000),
 }
 
 
@@ -423,6 +424,23 @@ def test_plan_from_device_estimate(bg, oracles):
     kc, vc = blugen.device_columns(w)
     plan = bg.plan_estimated(w.schema, kc)
     assert abs(plan.info()["est_groups"] - w.expected_groups) <= 0.15 * w.expected_groups
+    res = bg.blu_gby_execute(plan, kc, vc)
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
+@pytest.mark.parametrize("name,lock", [("K3", "rule"), ("K3", "0"), ("C3", "1"), ("C4", "1")])
+def test_kernel3_row_lock(bg, oracles, monkeypatch, name, lock):
+    """NEXT-1: kernel 3 locks the slot once and applies every aggregate. Chosen automatically
+    for > 5 aggregates at a low rows/groups ratio (K3); forced on C3/C4 (hash path) for parity."""
+    w, o = oracles(name)
+    kc, vc = blugen.device_columns(w)
+    if lock is not None:
+        monkeypatch.setenv("BLU_GBY_ROW_LOCK", lock)
+    if name == "C4":
+        monkeypatch.setenv("BLU_GBY_FORCE_PATH", "b")
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    assert plan.info()["row_lock"] == (0 if lock == "0" else 1)
     res = bg.blu_gby_execute(plan, kc, vc)
     gk, ga = gpu_sorted(res, w.schema)
     assert_parity(gk, ga, o, w.schema)
