@@ -45,7 +45,7 @@ extern "C" {
 typedef enum {
     BLU_OK = 0,
     BLU_E_INVALID = 1,      /* bad argument or schema                                          */
-    BLU_E_UNSUPPORTED = 2,  /* valid SQL, not supported: K > 1 sparse keys, dense domain >= 2^62 */
+    BLU_E_UNSUPPORTED = 2,  /* valid SQL, not supported: key tuple wider than 128 bits, > 2 sparse */
     BLU_E_KEY_RANGE = 3,    /* a key code outside [0, dict_size) or a negative sparse code      */
     BLU_E_OOM = 4,          /* device or host allocation failed                                */
     BLU_E_CUDA = 5          /* other CUDA runtime error                                         */
@@ -56,8 +56,12 @@ typedef enum { BLU_I32 = 0, BLU_I64 = 1, BLU_F64 = 2 } blu_dtype_t;
 typedef enum { BLU_COUNT = 0, BLU_SUM = 1, BLU_MIN = 2, BLU_MAX = 3, BLU_AVG = 4 } blu_aggop_t;
 
 /* One grouping column: dictionary codes in [0, dict_size) (P:109 LCOG loads "grouping keys";
- * DB2 BLU columns are dictionary encoded). dict_size == 0 means a sparse non-negative code, allowed
- * only when it is the single key column (dtype I32 or I64). Keys must be I32 or I64. */
+ * DB2 BLU columns are dictionary encoded). dict_size == 0 means a sparse non-negative code.
+ * Keys must be I32 or I64. The key tuple is packed into one 64-bit word when it is a single sparse
+ * column or dense columns with prod(dict_size) < 2^62; otherwise into TWO words ("wide keys",
+ * P:153 "If the key size is larger than 64 bit ..."): each sparse column (at most two) takes a
+ * whole word, dense columns fill the words greedily in column order with a per-word product < 2^62.
+ * Wide keys always plan path (b) with a 16-byte key CAS (no hot front, no partitioning). */
 typedef struct {
     blu_dtype_t dtype;
     uint64_t dict_size;
@@ -188,10 +192,12 @@ blu_status_t blu_gby_execute_dense_state(blu_gby_plan_t plan, const void* const*
 blu_status_t blu_gby_finalize_dense_state(blu_gby_plan_t plan, void* const* state_arrays, void* stream,
                                           blu_gby_result_t* out);
 
-/* Hash path exchange (path b): records are rows of (1 + n_states) 64-bit words:
- *   word 0 = packed key (the code for a sparse key; mixed radix sum code_j * prod_{i<j} d_i for a
- *            dense composite key), words 1.. = state fields as 64-bit (i32 states sign-extended,
- *            f64 states as their bits).
+/* Hash path exchange (path b): records are rows of (W + n_states) 64-bit words, W = 1 (or 2 for
+ * wide keys, see blu_key_desc_t):
+ *   words 0..W-1 = packed key (the code for a sparse key; mixed radix sum code_j * prod_{i<j} d_i
+ *            for a dense composite key; per word for wide keys), words W.. = state fields as 64-bit
+ *            (i32 states sign-extended, f64 states as their bits). Wide-key owners use
+ *            mulhi(fmix64(w0 ^ fmix64(w1 ^ 0x9E3779B97F4A7C15)), n_parts).
  * blu_gby_partition writes the groups of `partial` into send_buf (DEVICE, capacity
  * n_groups x record bytes) bucketed by owner rank = mulhi(fmix64(packed), n_parts) — bits
  * independent of the slot bits — in rank order, and sets send_counts[p] (HOST) to the number of

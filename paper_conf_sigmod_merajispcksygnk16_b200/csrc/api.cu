@@ -621,7 +621,7 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
   // fused init + compaction needs exactly one aggregation launch
   const bool single = n <= (((uint64_t)P->grid * (1ull << 30)) & ~3ull);
   Feeder feed = [&](AggParams& base, uint32_t* launches, Work& w, const FinalParams* fin) -> cudaError_t {
-    base.jit_ok = 1;
+    base.jit_ok = L.key_words == 2 ? 0 : 1;
     if (P->path == BLU_PATH_HASH_GLOBAL && P->parts > 1 && n >= 4096 * (uint64_t)P->parts)
       return partitioned_feed(P, base, keys, vals, n, st, launches, w);
     return agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, launches, fin);
@@ -705,7 +705,7 @@ blu_status_t blu_gby_execute_host(blu_gby_plan_t P, const void* const* hkeys, co
   float h2d_ms = 0.f;
   Feeder feed = [&](AggParams& base, uint32_t* launches, Work&, const FinalParams*) -> cudaError_t {
     if (!n) return cudaSuccess;
-    base.jit_ok = 1;
+    base.jit_ok = L.key_words == 2 ? 0 : 1;
     cudaEventRecord(t0, st);
     cudaStreamWaitEvent(cs, t0, 0);  // staging buffers are allocated on st
     uint64_t nchunks = (n + chunk - 1) / chunk;
@@ -792,7 +792,7 @@ blu_status_t blu_gby_merge_records(blu_gby_plan_t P, const void* records, uint64
   uint64_t cap = 1024;
   while ((double)cap * 0.7 < (double)est) cap <<= 1;
   uint32_t grid = (uint32_t)P->sms * 8, block = 256;
-  RecSrc rs{(const uint64_t*)records, (uint32_t)(1 + M.n_vals)};
+  RecSrc rs{(const uint64_t*)records, (uint32_t)((M.key_words == 2 ? 2 : 1) + M.n_vals)};
   Feeder feed = [&](AggParams& base, uint32_t* launches, Work&, const FinalParams*) -> cudaError_t {
     if (!n) return cudaSuccess;
     return agg_batch(P, BLU_PATH_HASH_GLOBAL, base, nullptr, nullptr, n, &rs, st, grid, block, 0, launches);
@@ -825,7 +825,7 @@ blu_status_t blu_gby_execute_dense_state(blu_gby_plan_t P, const void* const* ke
   base.front_slots = P->hot_front ? P->front_slots : 0;
   base.flags = (uint32_t*)small;
   fill_smem_layout(base, P->path == BLU_PATH_DENSE_SMEM ? (uint32_t)L.domain : base.front_slots, base.front_slots > 0);
-  base.jit_ok = 1;
+  base.jit_ok = L.key_words == 2 ? 0 : 1;
   CK(agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, nullptr), "aggregate");
   uint64_t* hs = pinned_scratch();
   uint64_t hb[2] = {0, 0};

@@ -67,6 +67,11 @@ struct Layout {
   int32_t n_group[4];            // fields per StateGroup
   uint32_t smem_entry_bytes;     // per entry of a shared-memory table (no key)
   int32_t lock_off;              // kernel 3: byte offset of the slot's row lock, 0 = none
+  // wide keys (> 64 bits; NEXT-2): key_words = 2 packs the key columns into two 64-bit words
+  // (mixed radix within a word; a sparse code occupies a whole word); kword[k] = word of column k and
+  // stride[k] its stride within that word. The slot key is then 16 bytes, claimed with a 16-byte CAS.
+  int32_t key_words;
+  int32_t kword[kMaxKeys];
 };
 
 // ---------------------------------------------------------------------------------------------

@@ -148,6 +148,118 @@ int launch_scatter(const AggParams& p, const ScatterParams& sp, void* stream, ui
   return launch_scatter_nv<16, 1>(p, sp, st, grid);
 }
 
+
+__device__ __forceinline__ uint64_t hash128(uint64_t w0, uint64_t w1) { return fmix64(w0 ^ fmix64(w1 ^ 0x9E3779B97F4A7C15ull)); }
+
+// ------------------------------------------------------------------------------------------------
+// Wide keys (> 64 bits; "If the key size is larger than 64 bit, we can not use CUDA atomic
+// operations any more so we try to acquire a lock ... Murmur hashing"). On sm_100a a 16-byte CAS is
+// native (ATOMG.E.CAS.128), so the 128-bit packed key is claimed exactly like the 64-bit one: read
+// both words, compare, CAS EMPTY -> key. Hash: Murmur3 finalizer over both words. Path (b) only.
+// MODE 0: columns; 1: records [w0, w1, states...].
+// ------------------------------------------------------------------------------------------------
+__device__ __forceinline__ void cas128(unsigned long long* a, unsigned long long cl, unsigned long long ch,
+                                       unsigned long long nl, unsigned long long nh, unsigned long long& ol,
+                                       unsigned long long& oh) {
+  asm volatile("{\n\t.reg .b128 d, c, n;\n\tmov.b128 c, {%2, %3};\n\tmov.b128 n, {%4, %5};\n\t"
+               "atom.global.cas.b128 d, [%6], c, n;\n\tmov.b128 {%0, %1}, d;\n\t}"
+               : "=l"(ol), "=l"(oh)
+               : "l"(cl), "l"(ch), "l"(nl), "l"(nh), "l"(a)
+               : "memory");
+}
+
+__device__ __forceinline__ bool hash_locate128(uint8_t* table, uint64_t mask, uint32_t sb, uint64_t k0, uint64_t k1,
+                                               uint32_t max_probe, uint64_t& out) {
+  uint64_t idx = hash128(k0, k1) & mask;
+  for (uint32_t q = 0; q < max_probe; ++q) {
+    unsigned long long* kp = (unsigned long long*)(table + idx * sb);
+    const ulonglong2 cur = __ldcg((const ulonglong2*)kp);
+    if (cur.x == k0 && cur.y == k1) { out = idx; return true; }
+    if (cur.x == kEmpty && cur.y == kEmpty) {
+      unsigned long long ol, oh;
+      cas128(kp, kEmpty, kEmpty, k0, k1, ol, oh);
+      if ((ol == kEmpty && oh == kEmpty) || (ol == k0 && oh == k1)) { out = idx; return true; }
+    }
+    idx = (idx + 1) & mask;
+  }
+  return false;
+}
+
+template <int NV, int R, int MODE>
+__global__ void __launch_bounds__(256) k_agg_wide(AggParams p, RecSrc rs) {
+  const Layout& L = p.lay;
+  const uint64_t pol = evict_first_policy();
+  const uint64_t n = p.n_rows;
+  const uint64_t tile = (uint64_t)blockDim.x * R;
+  const uint64_t ntiles = (n + tile - 1) / tile;
+  uint8_t* tb = (uint8_t*)p.table;
+  uint32_t flag_seen = 0;
+  for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    if (flag_seen) break;
+    flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);
+    const uint64_t row = lane_base<R>(t * tile, threadIdx.x >> 5, threadIdx.x & 31);
+    uint64_t w0[R], w1[R], v[NV][R];
+    uint32_t valid = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      w0[r] = w1[r] = 0;
+#pragma unroll
+      for (int c = 0; c < NV; ++c) v[c][r] = 0;
+      if (row_of<R>(row, r) < n) valid |= 1u << r;
+    }
+    if (MODE == 1) {
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const uint64_t rr = row_of<R>(row, r);
+        if (rr >= n) continue;
+        const unsigned long long* rec = (const unsigned long long*)rs.rec + rr * rs.words;
+        w0[r] = __ldg(rec);
+        w1[r] = __ldg(rec + 1);
+#pragma unroll
+        for (int c = 0; c < NV; ++c)
+          if (c < L.n_vals) {
+            const uint64_t x = __ldg(rec + 2 + c);
+            v[c][r] = L.val_dtype[c] == BLU_I32 ? (uint64_t)(int64_t)(int32_t)(uint32_t)x : x;
+          }
+      }
+    } else {
+      uint32_t bad = 0;
+      for (int k = 0; k < L.n_keys; ++k) {
+        uint64_t c[R];
+        load_rows<R>(p.key[k], L.key_dtype[k], row, n, p.vec_ok, pol, c);
+        const uint64_t d = L.dict[k], st = L.stride[k];
+        const int wd = L.kword[k];
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (d ? c[r] >= d : (int64_t)c[r] < 0) bad |= 1u << r;
+          const uint64_t x = d ? c[r] * st : c[r];
+          if (wd) w1[r] += x;
+          else w0[r] += x;
+        }
+      }
+      bad &= valid;
+      if (bad) atomicOr(p.flags, FLAG_KEY_RANGE);
+      valid &= ~bad;
+      load_vals<GenericSpec, NV, R>(p, row, n, pol, v);
+    }
+    uint64_t slot[R];
+    uint32_t ok = valid;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      slot[r] = 0;
+      if (!(valid >> r & 1)) continue;
+      uint64_t sl;
+      if (hash_locate128(tb, p.cap_mask, L.slot_bytes, w0[r], w1[r], p.max_probe, sl)) {
+        slot[r] = sl;
+      } else {
+        ok &= ~(1u << r);
+        atomicOr(p.flags, FLAG_OVERFLOW);
+      }
+    }
+    __syncwarp();
+    global_apply_rows<GenericSpec, NV, R, false>(p, slot, ok, v);
+  }
+}
 // ------------------------------------------------------------------------------------------------
 // S8: compaction (path (c))
 // ------------------------------------------------------------------------------------------------
@@ -249,10 +361,19 @@ __global__ void __launch_bounds__(kCT) k_compact_emit(CompactParams p) {
     before += __popc(bal & ((1u << lane) - 1u));
     if (occ) {
       uint64_t pos = out_pos + before;
-      uint64_t key = p.source == 0 ? __ldg((const unsigned long long*)((const uint8_t*)p.table + e * L.slot_bytes)) : e;
-      for (int k = 0; k < L.n_keys; ++k) {
-        uint64_t code = L.sparse ? key : (key / L.stride[k]) % L.dict[k];
-        store_as(p.out_keys[k], pos, L.key_dtype[k], code);
+      const unsigned long long* kp = (const unsigned long long*)((const uint8_t*)p.table + e * L.slot_bytes);
+      uint64_t key = p.source == 0 ? __ldg(kp) : e;
+      if (L.key_words == 2) {  // wide keys: per-word mixed radix (a sparse code is its whole word)
+        const uint64_t w[2] = {key, __ldg(kp + 1)};
+        for (int k = 0; k < L.n_keys; ++k) {
+          const uint64_t x = w[L.kword[k]];
+          store_as(p.out_keys[k], pos, L.key_dtype[k], L.dict[k] ? (x / L.stride[k]) % L.dict[k] : x);
+        }
+      } else {
+        for (int k = 0; k < L.n_keys; ++k) {
+          uint64_t code = L.sparse ? key : (key / L.stride[k]) % L.dict[k];
+          store_as(p.out_keys[k], pos, L.key_dtype[k], code);
+        }
       }
       if (p.partial) {
         for (int j = 0; j < L.n_fields; ++j) {
@@ -299,6 +420,17 @@ struct PartParams {
   uint32_t words;
 };
 
+__device__ __forceinline__ void pack_row_wide(const PartParams& p, uint64_t i, uint64_t& w0, uint64_t& w1) {
+  const Layout& L = p.lay;
+  w0 = w1 = 0;
+  for (int k = 0; k < L.n_keys; ++k) {
+    uint64_t c = L.key_dtype[k] == BLU_I32 ? (uint64_t)(int64_t)((const int32_t*)p.key[k])[i] : ((const uint64_t*)p.key[k])[i];
+    uint64_t x = L.dict[k] ? c * L.stride[k] : c;
+    if (L.kword[k]) w1 += x;
+    else w0 += x;
+  }
+}
+
 __device__ __forceinline__ uint64_t pack_row(const PartParams& p, uint64_t i) {
   const Layout& L = p.lay;
   if (L.sparse) {
@@ -316,21 +448,39 @@ __device__ __forceinline__ uint32_t owner_of(uint64_t key, int32_t P) { return (
 
 __global__ void __launch_bounds__(256) k_partition_hist(PartParams p) {
   uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.n; i += stride)
-    atomicAdd((unsigned long long*)&p.counts[owner_of(pack_row(p, i), p.n_parts)], 1ull);
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.n; i += stride) {
+    uint32_t o;
+    if (p.lay.key_words == 2) {
+      uint64_t w0, w1;
+      pack_row_wide(p, i, w0, w1);
+      o = (uint32_t)__umul64hi(hash128(w0, w1), (uint64_t)p.n_parts);
+    } else {
+      o = owner_of(pack_row(p, i), p.n_parts);
+    }
+    atomicAdd((unsigned long long*)&p.counts[o], 1ull);
+  }
 }
 
 __global__ void __launch_bounds__(256) k_partition_scatter(PartParams p) {
   uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.n; i += stride) {
-    uint64_t key = pack_row(p, i);
-    uint32_t o = owner_of(key, p.n_parts);
+    const int kw = p.lay.key_words == 2 ? 2 : 1;
+    uint64_t key = 0, key1 = 0;
+    uint32_t o;
+    if (kw == 2) {
+      pack_row_wide(p, i, key, key1);
+      o = (uint32_t)__umul64hi(hash128(key, key1), (uint64_t)p.n_parts);
+    } else {
+      key = pack_row(p, i);
+      o = owner_of(key, p.n_parts);
+    }
     uint64_t pos = p.offsets[o] + atomicAdd((unsigned long long*)&p.counts[o], 1ull);
     uint64_t* rec = p.out + pos * p.words;
     rec[0] = key;
+    if (kw == 2) rec[1] = key1;
     for (int j = 0; j < p.lay.n_vals; ++j) {
       uint64_t w = p.lay.val_dtype[j] == BLU_I32 ? (uint64_t)(int64_t)((const int32_t*)p.st[j])[i] : ((const uint64_t*)p.st[j])[i];
-      rec[1 + j] = w;
+      rec[kw + j] = w;
     }
   }
 }
@@ -386,7 +536,7 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
                          void* stream, uint32_t grid, uint32_t block, uint32_t smem, const FinalParams* fin) {
   cudaStream_t st = (cudaStream_t)stream;
   cudaError_t e = cudaSuccess;
-  if (!records && p.jit_ok) {
+  if (!records && p.jit_ok && p.lay.key_words != 2) {
     const int nv = p.lay.n_vals < 1 ? 1 : p.lay.n_vals;
     int r = rows_per_thread(p.lay.n_vals);
     char body[256], decl[160], name[64];
@@ -427,6 +577,17 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
     void (*k)(AggParams, RecSrc);
     bool front = p.front_slots > 0;
     bool direct = path == BLU_PATH_DIRECT_GLOBAL;
+    if (p.lay.key_words == 2) {  // wide keys: 16-byte key CAS (hash path only)
+      if constexpr (NV <= 16) {
+        k = records ? k_agg_wide<NV, R, 1> : k_agg_wide<NV, R, 0>;
+        note_kernel("k_agg_wide (generic)");
+        k<<<grid, block < 256 ? block : 256, 0, st>>>(p, rs);
+        count_launch(1);
+        return (int)cudaGetLastError();
+      } else {
+        return (int)cudaErrorInvalidValue;
+      }
+    }
     if constexpr (NV > 16) {  // merges of wide states: no front, no records
       if (records || front || direct) return (int)cudaErrorInvalidValue;
       k = k_agg_global<NV, R, false, false, 0>;
@@ -486,7 +647,7 @@ int launch_partition(const Layout& lay, const void* const* key_cols, const void*
   p.counts = d_counts;
   p.offsets = d_offsets;
   p.out = (uint64_t*)send_buf;
-  p.words = 1 + lay.n_vals;
+  p.words = (lay.key_words == 2 ? 2 : 1) + lay.n_vals;
   int grid = grid_for(n, 256, 148 * 8);
   k_partition_hist<<<grid, 256, 0, st>>>(p);
   count_launch(1);

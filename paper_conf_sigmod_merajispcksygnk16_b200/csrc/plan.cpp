@@ -78,7 +78,7 @@ uint32_t smem_entry_bytes(const Layout& lay) {
 
 // Assign AoS offsets (natural alignment, in field order after the 8-byte key) and dense groups.
 static void finish_layout(Layout& L) {
-  uint32_t off = 8;
+  uint32_t off = 8 * (L.key_words == 2 ? 2 : 1);
   int32_t gcount[4] = {0, 0, 0, 0};
   for (int j = 0; j < L.n_fields; ++j) {
     Field& f = L.f[j];
@@ -146,6 +146,7 @@ void build_slot_template(const Layout& L, uint8_t* out) {
   memset(out, 0, L.slot_bytes);
   uint64_t key = kEmpty;
   memcpy(out, &key, 8);
+  if (L.key_words == 2) memcpy(out + 8, &key, 8);
   for (int j = 0; j < L.n_fields; ++j) {
     const Field& f = L.f[j];
     uint8_t* p = out + f.goff;
@@ -227,10 +228,54 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
       return fail(BLU_E_INVALID, "agg %d: val_col %d out of range", a, s->aggs[a].val_col);
   }
   bool sparse = false;
+  int n_sparse = 0;
   for (int k = 0; k < s->n_keys; ++k)
-    if (s->keys[k].dict_size == 0) sparse = true;
-  if (sparse && s->n_keys > 1)
-    return fail(BLU_E_UNSUPPORTED, "a sparse key (dict_size 0) must be the only key column (wide keys: NEXT-2)");
+    if (s->keys[k].dict_size == 0) {
+      sparse = true;
+      ++n_sparse;
+    }
+  for (int k = 0; k < s->n_keys; ++k)
+    if (s->keys[k].dtype == BLU_I32 && s->keys[k].dict_size > (1ull << 31))
+      return fail(BLU_E_INVALID, "key %d: dict_size %llu exceeds the i32 code range", k,
+                  (unsigned long long)s->keys[k].dict_size);
+  // one 64-bit word: a single sparse key, or dense keys with D < 2^62; otherwise try two words
+  bool wide = false;
+  {
+    uint64_t Dt = 1;
+    bool over = false;
+    for (int k = 0; k < s->n_keys && !sparse; ++k) {
+      const uint64_t d = s->keys[k].dict_size;
+      if (Dt > ((1ull << 62) / d)) over = true;
+      else Dt *= d;
+    }
+    wide = (sparse && s->n_keys > 1) || over;
+  }
+  int kword[kMaxKeys] = {0};
+  uint64_t kstride[kMaxKeys] = {0};
+  if (wide) {  // greedy two-word packing: each sparse column takes a word; dense columns fill up
+    if (n_sparse > 2) return fail(BLU_E_UNSUPPORTED, "more than two sparse key columns (> 128-bit keys)");
+    uint64_t prod[2] = {1, 1};
+    bool full[2] = {false, false};
+    int w = 0;
+    for (int k = 0; k < s->n_keys; ++k)
+      if (s->keys[k].dict_size == 0) {
+        kword[k] = w;
+        kstride[k] = 1;
+        full[w] = true;
+        ++w;
+      }
+    for (int k = 0; k < s->n_keys; ++k) {
+      const uint64_t d = s->keys[k].dict_size;
+      if (!d) continue;
+      int t = -1;
+      for (int c = 0; c < 2 && t < 0; ++c)
+        if (!full[c] && prod[c] <= ((1ull << 62) / d)) t = c;
+      if (t < 0) return fail(BLU_E_UNSUPPORTED, "key tuple does not fit in 128 bits");
+      kword[k] = t;
+      kstride[k] = prod[t];
+      prod[t] *= d;
+    }
+  }
 
   auto* P = new blu_gby_plan_s();
   P->keys.assign(s->keys, s->keys + s->n_keys);
@@ -245,23 +290,19 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   L.sparse = sparse ? 1 : 0;
   L.count_field = -1;
   uint64_t D = 1;
+  L.key_words = wide ? 2 : 1;
   for (int k = 0; k < s->n_keys; ++k) {
     L.key_dtype[k] = s->keys[k].dtype;
     L.dict[k] = s->keys[k].dict_size;
-    L.stride[k] = D;
-    if (!sparse) {
-      uint64_t d = s->keys[k].dict_size;
-      if (s->keys[k].dtype == BLU_I32 && d > (1ull << 31)) {
-        delete P;
-        return fail(BLU_E_INVALID, "key %d: dict_size %llu exceeds the i32 code range", k, (unsigned long long)d);
-      }
-      if (D > ((1ull << 62) / d)) {
-        delete P;
-        return fail(BLU_E_UNSUPPORTED, "dense key domain >= 2^62 (wide keys: NEXT-2)");
-      }
-      D *= d;
+    if (wide) {
+      L.kword[k] = kword[k];
+      L.stride[k] = kstride[k];
+      continue;
     }
+    L.stride[k] = D;
+    if (!sparse) D *= s->keys[k].dict_size;
   }
+  if (wide) sparse = true;  // no dense domain: hash path only
   L.domain = sparse ? 0 : D;
   L.n_vals = s->n_vals;
   for (int c = 0; c < s->n_vals; ++c) L.val_dtype[c] = s->vals[c];
@@ -294,6 +335,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   // ---- moderator: pick the path ---------------------------------------------
   uint64_t cap_est = std::max<uint64_t>(kMinCap, next_pow2((uint64_t)((double)P->est_groups / kMaxLoad + 0.999999)));
   uint32_t entry_with_count = L.smem_entry_bytes + (L.count_field < 0 ? 4u : 0u);
+  L.sparse = sparse ? 1 : 0;
   int path;
   if (!sparse && D * (uint64_t)entry_with_count <= kSmemDenseMax) path = BLU_PATH_DENSE_SMEM;
   else if (!sparse && D <= std::max<uint64_t>(2 * cap_est, kDirectMin)) path = BLU_PATH_DIRECT_GLOBAL;
@@ -310,6 +352,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     }
     path = want;
   }
+  if (L.key_words == 2) path = BLU_PATH_HASH_GLOBAL;  // wide keys: 16-byte key CAS, hash path only
   P->path = path;
   if (path != BLU_PATH_HASH_GLOBAL && L.count_field < 0) {  // dense occupancy = COUNT > 0
     add_field(L, FK_COUNT, -1, 1);
@@ -340,7 +383,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   // so each bucket's slice of the table stays L2-resident (126 MB L2).
   P->parts = 1;
   P->part_shift = 0;
-  if (path == BLU_PATH_HASH_GLOBAL) {
+  if (path == BLU_PATH_HASH_GLOBAL && L.key_words == 1) {
     uint64_t budget = (uint64_t)kPartBudgetMB << 20;
     if (const char* pm = env("BLU_GBY_PART_MB")) budget = (uint64_t)atoi(pm) << 20;
     uint64_t tbytes = P->cap * (uint64_t)L.slot_bytes;
@@ -366,7 +409,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   // hot-key front (path b / b')
   P->hot_front = 0;
   P->front_slots = 0;
-  if (path != BLU_PATH_DENSE_SMEM) {
+  if (path != BLU_PATH_DENSE_SMEM && L.key_words == 1) {
     bool on = n_rows >= kFrontRatio * P->est_groups;
     if (const char* hf = env("BLU_GBY_HOT_FRONT")) on = hf[0] == '1';
     if (on) {
@@ -469,7 +512,9 @@ blu_status_t blu_gby_dense_state_shape(blu_gby_plan_t P, int32_t* n_isum, int32_
   return BLU_OK;
 }
 
-uint32_t blu_gby_record_bytes(blu_gby_plan_t P) { return P ? 8u * (1u + (uint32_t)P->lay.n_fields) : 0u; }
+uint32_t blu_gby_record_bytes(blu_gby_plan_t P) {
+  return P ? 8u * ((P->lay.key_words == 2 ? 2u : 1u) + (uint32_t)P->lay.n_fields) : 0u;
+}
 
 blu_status_t blu_gby_slot_template(blu_gby_plan_t P, void* out, uint32_t cap, uint32_t* slot_bytes) {
   if (!P) return fail(BLU_E_INVALID, "NULL plan");

@@ -127,11 +127,14 @@ def test_schema_validation(bg):
     with pytest.raises(bg.BluError) as e:
         bg.blu_gby_plan([(F64, 4)], [I64], [(SUM, 0)], 1, 1)
     assert e.value.status == bg.BLU_E_INVALID
-    with pytest.raises(bg.BluError) as e:  # sparse key with another key column: NEXT-2
-        bg.blu_gby_plan([(I64, 0), (I32, 4)], [I64], [(SUM, 0)], 1, 1)
+    with pytest.raises(bg.BluError) as e:  # three sparse key columns: wider than 128 bits
+        bg.blu_gby_plan([(I64, 0), (I64, 0), (I32, 0)], [I64], [(SUM, 0)], 1, 1)
     assert e.value.status == bg.BLU_E_UNSUPPORTED
-    with pytest.raises(bg.BluError) as e:  # dense domain >= 2^62
-        bg.blu_gby_plan([(I64, 2**40), (I64, 2**30)], [I64], [(SUM, 0)], 1, 1)
+    with pytest.raises(bg.BluError) as e:  # dense tuple of 2^120 codes does not fit two 2^62 words
+        bg.blu_gby_plan([(I64, 2**40), (I64, 2**40), (I64, 2**40)], [I64], [(SUM, 0)], 1, 1)
+    assert e.value.status == bg.BLU_E_UNSUPPORTED
+    with pytest.raises(bg.BluError) as e:  # sparse + sparse + any dense column: no room
+        bg.blu_gby_plan([(I64, 0), (I64, 0), (I32, 4)], [I64], [(SUM, 0)], 1, 1)
     assert e.value.status == bg.BLU_E_UNSUPPORTED
     with pytest.raises(bg.BluError) as e:
         bg.blu_gby_plan([(I32, 4)], [I64], [(7, 0)], 1, 1)
@@ -166,3 +169,19 @@ def test_planner_kernel3_rule(bg, monkeypatch):
     assert c3["row_lock"] == 0  # 3 fields
     hi = bg.plan_for(blugen.workload("K3").schema, 1000, 100_000_000).info()
     assert hi["row_lock"] == 0  # 1e5 rows per group: contention, keep per-field atomics
+
+
+@pytest.mark.parametrize("keys, n_fields", [
+    ([(I64, 0), (I32, 4)], 1),                 # sparse + dense
+    ([(I64, 2**40), (I64, 2**30)], 1),         # dense domain >= 2^62
+    ([(I64, 0), (I64, 0)], 1),                 # two sparse columns
+])
+def test_wide_key_plans(bg, keys, n_fields):
+    """Key tuples wider than one 64-bit word plan path (b) with a two-word key."""
+    p = bg.blu_gby_plan(keys, [I64], [(SUM, 0)], 1000, 10**6)
+    d = p.info()
+    assert d["path"] == bg.BLU_PATH_HASH_GLOBAL
+    assert d["hot_front"] == 0 and d["partitions"] == 1
+    assert d["n_states"] == n_fields
+    assert p.record_bytes == 8 * (2 + n_fields)
+    assert d["slot_bytes"] >= 16 + 8

@@ -444,3 +444,88 @@ def test_kernel3_row_lock(bg, oracles, monkeypatch, name, lock):
     res = bg.blu_gby_execute(plan, kc, vc)
     gk, ga = gpu_sorted(res, w.schema)
     assert_parity(gk, ga, o, w.schema)
+
+
+# ---- NEXT-2: wide keys (> 64-bit packed key) --------------------------------------------
+WIDE = {
+    # two sparse i64 columns: 128-bit key, heavy duplication
+    "ss": lambda rng, n: ([(I64, 0), (I64, 0)],
+                          [rng.integers(0, 2**62, 997)[rng.integers(0, 997, n)],
+                           rng.integers(0, 2**40, 31)[rng.integers(0, 31, n)]]),
+    # sparse + two dense columns (dense ones share word 1)
+    "sdd": lambda rng, n: ([(I64, 0), (I32, 7), (I64, 1000)],
+                           [rng.integers(0, 2**50, 5000)[rng.integers(0, 5000, n)],
+                            rng.integers(0, 7, n).astype(np.int32), rng.integers(0, 1000, n)]),
+    # dense tuple with domain 2^70: spills into the second word
+    "dd": lambda rng, n: ([(I64, 2**40), (I64, 2**30)],
+                          [rng.integers(0, 2**40, 3000)[rng.integers(0, 3000, n)],
+                           rng.integers(2**30 - 5, 2**30, n)]),
+}
+
+
+@pytest.mark.parametrize("n", [0, 1, 33, 65_537, 1_000_003])
+@pytest.mark.parametrize("kind", sorted(WIDE))
+def test_wide_keys_parity(bg, kind, n):
+    rng = np.random.default_rng(sorted(WIDE).index(kind) * 1000 + n)
+    keys, kc = WIDE[kind](rng, n)
+    kc = [k.astype(np.int32 if d == I32 else np.int64) for k, (d, _) in zip(kc, keys)]
+    sch = blugen.Schema(keys, [I32, I64, F64], ALL(3))
+    vc = [rng.integers(-(2**31), 2**31, n).astype(np.int32), rng.integers(-(2**40), 2**40, n),
+          rng.integers(-(2**20), 2**20, n) / 64.0]
+    o = oracle.groupby_arrays(sch, kc, vc)
+    plan = bg.plan_for(sch, max(1, o.keys.shape[0] // 2), n)  # under-estimate: exercises regrow
+    assert plan.info()["path"] == bg.BLU_PATH_HASH_GLOBAL
+    dk, dv = _mk(kc, vc)
+    res = bg.blu_gby_execute(plan, dk, dv, n_rows=n)
+    gk, ga = gpu_sorted(res, sch)
+    assert_parity(gk, ga, o, sch)
+
+
+def test_wide_keys_partition_and_merge(bg):
+    """Partial -> partition records (2 key words) -> merge_records, and partial merge, for wide keys."""
+    rng = np.random.default_rng(5)
+    n = 400_001
+    keys, kc = WIDE["sdd"](rng, n)
+    kc = [k.astype(np.int32 if d == I32 else np.int64) for k, (d, _) in zip(kc, keys)]
+    sch = blugen.Schema(keys, [I64, F64], [(COUNT, -1), (SUM, 0), (MIN, 1), (MAX, 0), (AVG, 1)])
+    vc = [rng.integers(-(2**40), 2**40, n), rng.integers(-(2**20), 2**20, n) / 64.0]
+    o = oracle.groupby_arrays(sch, kc, vc)
+    plan = bg.plan_for(sch, o.keys.shape[0], n)
+    dk, dv = _mk(kc, vc)
+    P = 3
+    cuts = np.linspace(0, n, P + 1).astype(int)
+    parts = [bg.blu_gby_execute_partial(plan, [k[cuts[r]:cuts[r + 1]] for k in dk],
+                                        [v[cuts[r]:cuts[r + 1]] for v in dv]) for r in range(P)]
+    gk, ga = gpu_sorted(bg.blu_gby_merge(plan, parts), sch)
+    assert_parity(gk, ga, o, sch)
+    rb = plan.record_bytes
+    inbox = [[] for _ in range(P)]
+    for part in parts:
+        buf = torch.empty(max(1, part.n_groups) * rb // 8, dtype=torch.int64, device="cuda")
+        counts = bg.blu_gby_partition(plan, part, P, buf)
+        off = 0
+        for dst in range(P):
+            inbox[dst].append(buf[off * rb // 8:(off + counts[dst]) * rb // 8])
+            off += counts[dst]
+    keys_, aggs = [], []
+    for dst in range(P):
+        recs = torch.cat(inbox[dst])
+        k, a = gpu_sorted(bg.blu_gby_merge_records(plan, recs, recs.numel() * 8 // rb), sch)
+        keys_.append(k)
+        aggs.append(a)
+    allk = np.concatenate(keys_)
+    order = np.lexsort(allk.T[::-1])
+    assert_parity(allk[order], [np.concatenate([a[i] for a in aggs])[order] for i in range(len(sch.aggs))], o, sch)
+
+
+def test_wide_keys_host_columns(bg):
+    rng = np.random.default_rng(9)
+    n = 300_007
+    keys, kc = WIDE["ss"](rng, n)
+    sch = blugen.Schema(keys, [I64], [(COUNT, -1), (SUM, 0), (MAX, 0)])
+    vc = [rng.integers(-(2**40), 2**40, n)]
+    o = oracle.groupby_arrays(sch, kc, vc)
+    plan = bg.plan_for(sch, o.keys.shape[0], n)
+    res = bg.blu_gby_execute_host(plan, kc, vc)
+    gk, ga = host_sorted(res, sch)
+    assert_parity(gk, ga, o, sch)
