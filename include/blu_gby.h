@@ -243,6 +243,21 @@ void blu_gby_set_timing(int32_t enable);
 blu_status_t blu_gby_last_timing(blu_gby_timing_t* out);
 uint64_t blu_gby_launch_count(void);
 
+/* Diagnostics: compile (NVRTC, no GPU needed, nothing launched) the plan-specialised kernels that
+ * execute would JIT for this plan, with the NVRTC the library loads. Returns BLU_OK if every program
+ * compiled; BLU_E_UNSUPPORTED if one failed (its log goes to `log`, HOST, log_cap bytes, may be
+ * NULL) or the plan has no JIT kernels (wide keys, BLU_GBY_JIT=0) — execute then runs the generic
+ * precompiled kernels. *n_programs (may be NULL) = programs compiled. */
+blu_status_t blu_gby_jit_probe(blu_gby_plan_t plan, char* log, uint32_t log_cap, int32_t* n_programs);
+
+/* Measurement helper (SURVEY.md §8(d) roofline denominator (i)): reads n_cols DEVICE columns of
+ * bytes[i] bytes each (16-byte aligned) once, with the same 128-bit evict-first streaming loads the
+ * aggregation kernels use, and XOR-folds them into *dev_out (DEVICE u64) so nothing is elided. The
+ * caller times it; bytes / time is the read-only ceiling for the input stream. Grid = 2 CTAs/SM x
+ * 512 threads, like path (a). */
+blu_status_t blu_gby_read_roofline(const void* const* cols, const uint64_t* bytes, int32_t n_cols, void* stream,
+                                   uint64_t* dev_out);
+
 /* Make `device` the current CUDA device of the calling thread for this library (one process per
  * GPU: pass the local rank). */
 blu_status_t blu_gby_bind_device(int32_t device);

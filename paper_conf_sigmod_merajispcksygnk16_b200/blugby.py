@@ -92,6 +92,8 @@ def _load():
         "blu_gby_set_timing": ([i32], None),
         "blu_gby_last_timing": ([P(TimingC)], i32),
         "blu_gby_launch_count": ([], u64),
+        "blu_gby_read_roofline": ([P(vp), P(u64), i32, vp, vp], i32),
+        "blu_gby_jit_probe": ([vp, ctypes.c_char_p, u32, P(i32)], i32),
         "blu_gby_bind_device": ([i32], i32),
         "blu_gby_result_free": ([P(ResultC), vp], None),
         "blu_gby_plan_destroy": ([vp], None),
@@ -441,6 +443,22 @@ def blu_gby_last_timing() -> dict:
 
 def blu_gby_launch_count() -> int:
     return int(lib.blu_gby_launch_count())
+
+
+def blu_gby_jit_probe(plan: Plan) -> Tuple[int, int, str]:
+    """Compile (no GPU needed) the plan-specialised kernels execute would JIT: (status, programs, log)."""
+    buf = ctypes.create_string_buffer(1 << 16)
+    n = ctypes.c_int32()
+    st = int(lib.blu_gby_jit_probe(plan.handle, buf, len(buf), ctypes.byref(n)))
+    return st, n.value, buf.value.decode(errors="replace")
+
+
+def blu_gby_read_roofline(cols, out, stream=None):
+    """Measurement helper: stream every byte of `cols` (device tensors) once with the aggregation
+    kernels' load instructions; XOR-fold into `out` (device int64 tensor of 1 element)."""
+    n = len(cols)
+    by = (ctypes.c_uint64 * n)(*[c.numel() * c.element_size() for c in cols])
+    _check(lib.blu_gby_read_roofline(_ptrs(cols), by, n, _stream_handle(stream), ctypes.c_void_p(out.data_ptr())))
 
 
 def blu_gby_bind_device(device: int):

@@ -229,6 +229,12 @@ static cudaError_t agg_batch(const blu_gby_plan_s* P, int path, AggParams p, con
       }
     }
     p.vec_ok = vec ? 1 : 0;
+    if (vec) {
+      bool v32 = true;
+      for (int k = 0; k < L.n_keys; ++k) v32 = v32 && ((uintptr_t)p.key[k] & 31) == 0;
+      for (int c = 0; c < L.n_vals; ++c) v32 = v32 && ((uintptr_t)p.val[c] & 31) == 0;
+      if (v32) p.vec_ok |= 2;
+    }
     p.n_rows = m;
     RecSrc r{nullptr, 0};
     if (rs) r = RecSrc{rs->rec + r0 * rs->words, rs->words};
@@ -261,13 +267,6 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     // path (a) with a small domain: init (S4) and compaction (S8) fused into the aggregation kernel
     const bool fuse = fuse_req && path == BLU_PATH_DENSE_SMEM && D <= 65536 && !partial && !host_out &&
                       !getenv("BLU_GBY_NO_FUSE");
-    if (dense) {
-      for (int g = 0; g < 4; ++g) CK(w.alloc(&dense_g[g], (size_t)lay.n_group[g] * D * 8), "dense state alloc");
-      if (!fuse) CK(launch_init_dense(lay, dense_g, D, st), "init dense");
-    } else {
-      CK(w.alloc(&table, (size_t)cap * lay.slot_bytes), "hash table alloc");
-      CK(launch_init_slots(lay, table, cap, st), "init slots");
-    }
     const uint64_t n_entries = dense ? D : cap;
     const uint64_t nb = (n_entries + 4095) / 4096;
     void* small = nullptr;
@@ -276,7 +275,14 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     uint64_t* d_ngroups = (uint64_t*)((uint8_t*)small + 8);
     uint64_t* d_bcounts = (uint64_t*)((uint8_t*)small + 64);
     uint64_t* d_boffs = d_bcounts + std::max<uint64_t>(nb, 1);
-    CK(cudaMemsetAsync(small, 0, 64, st), "memset flags");
+    if (dense) {
+      for (int g = 0; g < 4; ++g) CK(w.alloc(&dense_g[g], (size_t)lay.n_group[g] * D * 8), "dense state alloc");
+      if (!fuse) CK(launch_init_dense(lay, dense_g, D, st, (uint64_t*)small, 8), "init dense");  // + flags
+      else CK(cudaMemsetAsync(small, 0, 64, st), "memset flags");
+    } else {
+      CK(w.alloc(&table, (size_t)cap * lay.slot_bytes), "hash table alloc");
+      CK(launch_init_slots(lay, table, cap, st, (uint64_t*)small, 8), "init slots");  // + flags
+    }
     if (t_timing) cudaEventRecord(t_ev.e[1], st);
 
     AggParams base{};
@@ -646,6 +652,52 @@ blu_status_t blu_gby_last_timing(blu_gby_timing_t* out) {
 }
 
 uint64_t blu_gby_launch_count(void) { return launches_total(); }
+
+blu_status_t blu_gby_jit_probe(blu_gby_plan_t P, char* log, uint32_t log_cap, int32_t* n_programs) {
+  if (!P) return fail(BLU_E_INVALID, "NULL plan");
+  if (log && log_cap) log[0] = 0;
+  if (n_programs) *n_programs = 0;
+  if (!jit_enabled() || P->lay.key_words == 2) return fail(BLU_E_UNSUPPORTED, "no JIT kernels for this plan");
+  JitProbe pr;
+  jit_probe_begin(&pr);
+  AggParams p{};
+  p.lay = P->lay;
+  p.jit_ok = 1;
+  p.n_rows = 1;
+  p.front_slots = P->hot_front ? P->front_slots : 0;
+  fill_smem_layout(p, P->path == BLU_PATH_DENSE_SMEM ? (uint32_t)P->lay.domain : p.front_slots, p.front_slots > 0);
+  int rc = launch_aggregate_impl(P, P->path, p, RecSrc{nullptr, 0}, false, nullptr, P->grid, P->block, P->smem_bytes);
+  if (P->path == BLU_PATH_HASH_GLOBAL && P->parts > 1) {  // partitioned mode: scatter + segment pass
+    ScatterParams sp{};
+    sp.B = P->parts;
+    if (!rc) rc = launch_scatter(p, sp, nullptr, P->grid);
+    AggParams p2 = p;
+    p2.seg_stride = 1;
+    if (!rc) rc = launch_aggregate_impl(P, P->path, p2, RecSrc{nullptr, 0}, false, nullptr, P->grid, P->block, P->smem_bytes);
+  }
+  jit_probe_end();
+  if (n_programs) *n_programs = pr.programs;
+  if (log && log_cap) {
+    strncpy(log, pr.log.c_str(), log_cap - 1);
+    log[log_cap - 1] = 0;
+  }
+  if (rc || pr.failed || !pr.programs)
+    return fail(BLU_E_UNSUPPORTED, "JIT probe: %d of %d programs failed", pr.failed, pr.programs);
+  return BLU_OK;
+}
+
+blu_status_t blu_gby_read_roofline(const void* const* cols, const uint64_t* bytes, int32_t n_cols, void* stream,
+                                   uint64_t* dev_out) {
+  if (n_cols < 1 || n_cols > kMaxKeys + kMaxVals || !cols || !bytes || !dev_out)
+    return fail(BLU_E_INVALID, "bad read_roofline arguments");
+  for (int j = 0; j < n_cols; ++j)
+    if (!cols[j] || ((uintptr_t)cols[j] & 15) || (bytes[j] & 15)) return fail(BLU_E_INVALID, "column %d: not 16-byte aligned", j);
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  CK(launch_read_roofline(cols, bytes, n_cols, stream, dev_out, sms), "read roofline");
+  return BLU_OK;
+}
 
 blu_status_t blu_gby_execute(blu_gby_plan_t P, const void* const* key_cols, const void* const* val_cols, uint64_t n_rows,
                              void* stream, blu_gby_result_t* out) {

@@ -49,6 +49,29 @@ __device__ __forceinline__ int4 ld_stream_v4(const void* p, uint64_t pol) {
       : "l"(p), "l"(pol));
   return r;
 }
+// 256-bit streaming load (LDG.E.256 on sm_100a): one instruction per 32 contiguous bytes per lane.
+// Needs PTX ISA 8.8 (CUDA >= 12.9); the JIT passes BLU_LDG256 from the NVRTC version it loaded.
+#ifndef BLU_LDG256
+#if defined(__CUDACC_VER_MAJOR__) && (__CUDACC_VER_MAJOR__ > 12 || (__CUDACC_VER_MAJOR__ == 12 && __CUDACC_VER_MINOR__ >= 9))
+#define BLU_LDG256 1
+#else
+#define BLU_LDG256 0
+#endif
+#endif
+__device__ __forceinline__ void ld_stream_v4u64(const void* p, uint64_t pol, uint64_t& a, uint64_t& b, uint64_t& c,
+                                                uint64_t& d) {
+#if BLU_LDG256
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+      : "=l"(a), "=l"(b), "=l"(c), "=l"(d)
+      : "l"(p), "l"(pol));
+#else
+  const int4 x = ld_stream_v4(p, pol), y = ld_stream_v4((const uint8_t*)p + 16, pol);
+  a = (uint64_t)(uint32_t)x.x | ((uint64_t)(uint32_t)x.y << 32);
+  b = (uint64_t)(uint32_t)x.z | ((uint64_t)(uint32_t)x.w << 32);
+  c = (uint64_t)(uint32_t)y.x | ((uint64_t)(uint32_t)y.y << 32);
+  d = (uint64_t)(uint32_t)y.z | ((uint64_t)(uint32_t)y.w << 32);
+#endif
+}
 __device__ __forceinline__ int32_t ld_stream_s32(const void* p, uint64_t pol) {
   int32_t r;
   asm("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
@@ -82,8 +105,9 @@ __device__ __forceinline__ int2 ld_stream_v2(const void* p, uint64_t pol) {
 }
 
 // Load this lane's R rows of one column as 64-bit patterns (i32 sign-extended). Rows >= n read 0.
+// vec: bit 0 = every column 16-byte aligned, bit 1 = 32-byte aligned (256-bit loads allowed).
 template <int R, bool PAIR = true>
-__device__ __forceinline__ void load_rows(const void* base, int dt, uint64_t lb, uint64_t n, bool vec,
+__device__ __forceinline__ void load_rows(const void* base, int dt, uint64_t lb, uint64_t n, uint32_t vec,
                                           uint64_t pol, uint64_t (&out)[R]) {
   if (!PAIR && R >= 4) {  // quad mapping: rows lb..lb+R-1 (path (a): 16-byte loads, 4 i32 rows each)
     if (dt == BLU_I32) {
@@ -103,7 +127,10 @@ __device__ __forceinline__ void load_rows(const void* base, int dt, uint64_t lb,
       }
     } else {
       const uint64_t* p = (const uint64_t*)base + lb;
-      if (vec && lb + R <= n) {
+      if ((vec & 2) && R % 4 == 0 && lb + R <= n) {  // 32 contiguous bytes per lane: whole sectors
+#pragma unroll
+        for (int r = 0; r < R; r += 4) ld_stream_v4u64(p + r, pol, out[r], out[(r + 1) % R], out[(r + 2) % R], out[(r + 3) % R]);
+      } else if (vec && lb + R <= n) {
 #pragma unroll
         for (int r = 0; r < R; r += 2) {
           int4 v = ld_stream_v4(p + r, pol);
@@ -544,7 +571,7 @@ __device__ __forceinline__ void dense_finalize_block(const AggParams& p, const F
 
 // FUSE (small inputs, where launch latency dominates): S4 init and S8 compaction run inside this
 // kernel. Kept out of the large-input instantiation, whose register budget it would squeeze.
-template <class SP, int NV, int R, bool FUSE = false>
+template <class SP, int NV, int R, bool FUSE = false, bool PAIRMAP = false>
 __device__ __forceinline__ void dense_body(const AggParams& p, const FinalParams& fp) {
   extern __shared__ __align__(16) uint8_t sm[];
   const Layout& L = p.lay;
@@ -567,11 +594,11 @@ __device__ __forceinline__ void dense_body(const AggParams& p, const FinalParams
   for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
     if (flag_seen) break;
     flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);  // warp-uniform, seen next tile
-    const uint64_t row = lane_base<R, false>(t * tile, threadIdx.x >> 5, threadIdx.x & 31);
+    const uint64_t row = lane_base<R, PAIRMAP>(t * tile, threadIdx.x >> 5, threadIdx.x & 31);
     uint64_t key[R];
-    const uint32_t valid = pack_keys<SP, R, false>(p, row, n, pol, key);
+    const uint32_t valid = pack_keys<SP, R, PAIRMAP>(p, row, n, pol, key);
     uint64_t v[NV][R];
-    load_vals<SP, NV, R, false>(p, row, n, pol, v);
+    load_vals<SP, NV, R, PAIRMAP>(p, row, n, pol, v);
     uint32_t e[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) e[r] = (uint32_t)key[r];

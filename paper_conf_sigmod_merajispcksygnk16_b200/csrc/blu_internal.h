@@ -68,9 +68,13 @@ int launch_aggregate_impl(const blu_gby_plan_s* P, int path, const AggParams& p,
 uint64_t launches_total();
 int launch_scatter(const AggParams& p, const ScatterParams& s, void* stream, uint32_t grid);
 blu_status_t fail(blu_status_t s, const char* fmt, ...);
-int launch_init_slots(const Layout& lay, void* table, uint64_t n_slots, void* stream);
-int launch_init_dense(const Layout& lay, void* const dense[4], uint64_t D, void* stream);
+int launch_init_slots(const Layout& lay, void* table, uint64_t n_slots, void* stream, uint64_t* zero = nullptr,
+                      uint32_t n_zero = 0);
+int launch_init_dense(const Layout& lay, void* const dense[4], uint64_t D, void* stream, uint64_t* zero = nullptr,
+                      uint32_t n_zero = 0);
 int launch_compact(const CompactParams& p, void* stream, uint32_t* launches);
+int launch_read_roofline(const void* const* cols, const uint64_t* bytes, int n_cols, void* stream, uint64_t* out,
+                         int sms);
 int launch_partition(const Layout& lay, const void* const* key_cols, const void* const* state_cols,
                      uint64_t n, int32_t n_parts, void* send_buf, uint64_t* d_counts, uint64_t* d_offsets,
                      void* stream);
@@ -79,6 +83,13 @@ void count_launch(uint64_t n);
 
 // NVRTC specialisation (jit.cpp)
 bool jit_enabled();
+struct JitProbe {  // compile-only mode of the JIT (blu_gby_jit_probe)
+  int programs = 0, failed = 0;
+  std::string log;
+};
+void jit_probe_begin(JitProbe* pr);
+void jit_probe_end();
+bool jit_probe_active();
 const void* jit_kernel(const std::string& spec_src, const std::string& entry_src, const char* entry);
 std::string jit_spec(const char* name, const Layout& L);
 

@@ -85,7 +85,7 @@ struct AggParams {
   const void* key[kMaxKeys];
   const void* val[kMaxVals];
   uint64_t n_rows;
-  int32_t vec_ok;        // all column pointers 16-byte aligned
+  int32_t vec_ok;        // bit 0: all column pointers 16-byte aligned; bit 1: 32-byte aligned
   // targets
   void* table;           // path b: AoS slots (cap x slot_bytes)
   uint64_t cap_mask;     // cap - 1 (power of two)

@@ -47,10 +47,12 @@ Nvrtc* nvrtc() {
   static Nvrtc n;
   static std::once_flag once;
   std::call_once(once, [] {
-    const char* names[] = {"libnvrtc.so.12", "libnvrtc.so", "/usr/local/cuda/lib64/libnvrtc.so.12"};
+    // The toolkit's NVRTC first (same release as the nvcc that built the AOT kernels; the copy torch
+    // bundles can be older and reject sm_100a-only PTX such as 256-bit loads), then the soname.
+    const char* names[] = {"/usr/local/cuda/lib64/libnvrtc.so.12", "libnvrtc.so.12", "libnvrtc.so"};
     void* h = nullptr;
     for (const char* nm : names)
-      if ((h = dlopen(nm, RTLD_NOW | RTLD_GLOBAL))) break;
+      if ((h = dlopen(nm, RTLD_NOW | RTLD_LOCAL))) break;
     if (!h) return;
     n.create = (decltype(n.create))dlsym(h, "nvrtcCreateProgram");
     n.compile = (decltype(n.compile))dlsym(h, "nvrtcCompileProgram");
@@ -173,9 +175,12 @@ bool compile(const std::string& src, std::vector<char>& cubin, std::string& log)
     log = "nvrtcCreateProgram failed";
     return false;
   }
+  int major = 0, minor = 0;
+  if (n->version) n->version(&major, &minor);
+  const bool ldg256 = major > 12 || (major == 12 && minor >= 9);  // 256-bit LDG needs PTX ISA 8.8
   const char* opts[] = {"--gpu-architecture=sm_100a", "--std=c++17", "-lineinfo", "--device-as-default-execution-space", "--diag-suppress=128,177",
-                        "-DNDEBUG"};
-  int rc = n->compile(prog, 6, opts);
+                        "-DNDEBUG", ldg256 ? "-DBLU_LDG256=1" : "-DBLU_LDG256=0"};
+  int rc = n->compile(prog, 7, opts);
   size_t ls = 0;
   n->log_size(prog, &ls);
   log.assign(ls, '\0');
@@ -201,8 +206,35 @@ bool jit_enabled() {
 
 // Returns a kernel handle (usable with cudaLaunchKernel / cudaFuncSetAttribute) for `entry` in the
 // program made of `spec_src` + `entry_src`, or nullptr (caller falls back to the generic kernels).
+thread_local JitProbe* t_probe = nullptr;
+void jit_probe_begin(JitProbe* pr) { t_probe = pr; }
+void jit_probe_end() { t_probe = nullptr; }
+bool jit_probe_active() { return t_probe != nullptr; }
+
+// Compile-only probe (blu_gby_jit_probe): NVRTC compile of the program, no module load, no launch.
+static void probe_compile(const std::string& body) {
+  JitProbe& pr = *t_probe;
+  ++pr.programs;
+  if (!nvrtc()->ok) {
+    ++pr.failed;
+    pr.log += "NVRTC not found\n";
+    return;
+  }
+  std::string src = std::string(kPreamble) + kSrc_blu_params_h + "\n" + kSrc_blu_device_cuh + "\n" + body;
+  std::vector<char> cubin;
+  std::string log;
+  if (!compile(src, cubin, log) || cubin.empty()) {
+    ++pr.failed;
+    pr.log += log.empty() ? std::string("compile failed\n") : log;
+  }
+}
+
 const void* jit_kernel(const std::string& spec_src, const std::string& entry_src, const char* entry) {
   if (!jit_enabled()) return nullptr;
+  if (t_probe) {
+    probe_compile(spec_src + entry_src);
+    return nullptr;
+  }
   int dev = 0;
   cudaGetDevice(&dev);
   const std::string body = spec_src + entry_src;

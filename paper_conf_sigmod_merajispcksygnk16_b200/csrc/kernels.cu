@@ -19,6 +19,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
 #include <atomic>
 
 #include "blu_internal.h"
@@ -59,6 +60,7 @@ static bool launch_jit(const char* body, const char* entry_decl, const AggParams
   src += body;
   src += " }\n";
   const void* k = jit_kernel(spec, src, entry);
+  if (jit_probe_active()) return true;  // compile-only probe: nothing is launched
   if (!k) return false;
   if (smem > 48 * 1024 && cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
     cudaGetLastError();
@@ -82,9 +84,11 @@ struct SlotTemplate {
   uint32_t words;  // slot_bytes / 8
 };
 
-__global__ void __launch_bounds__(256) k_init_slots(SlotTemplate t, uint64_t* table, uint64_t n_words2) {
-  // n_words2 = number of 16-byte chunks; slot_bytes is a multiple of 16
+__global__ void __launch_bounds__(256) k_init_slots(SlotTemplate t, uint64_t* table, uint64_t n_words2, uint64_t* zero,
+                                                   uint32_t n_zero) {
+  // n_words2 = number of 16-byte chunks; slot_bytes is a multiple of 16; zero: optional u64 block set to 0
   uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  if (zero && blockIdx.x == 0 && threadIdx.x < n_zero) zero[threadIdx.x] = 0;
   uint32_t pairs = t.words / 2;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_words2; i += stride) {
     uint32_t w = (uint32_t)(i % pairs) * 2;
@@ -341,13 +345,15 @@ __global__ void __launch_bounds__(1024) k_compact_scan(uint64_t* counts, uint64_
   if (threadIdx.x == 0) *total = carry;
 }
 
+// SINGLE: one CTA covers all n_entries (<= kCB) and publishes n_groups itself (no count/scan launches).
+template <bool SINGLE>
 __global__ void __launch_bounds__(kCT) k_compact_emit(CompactParams p) {
   __shared__ uint32_t ws[kCT / 32];
   const uint64_t base = (uint64_t)blockIdx.x * kCB;
-  uint64_t out_pos = p.block_offsets[blockIdx.x];
+  uint64_t out_pos = SINGLE ? 0 : p.block_offsets[blockIdx.x];
   const Layout& L = p.lay;
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  for (int i = 0; i < kCRounds; ++i) {
+  for (int i = 0; i < kCRounds && base + (uint64_t)i * kCT < p.n_entries; ++i) {
     uint64_t e = base + (uint64_t)i * kCT + threadIdx.x;
     bool occ = e < p.n_entries && occupied(p, e);
     unsigned bal = __ballot_sync(0xffffffffu, occ);
@@ -403,6 +409,7 @@ __global__ void __launch_bounds__(kCT) k_compact_emit(CompactParams p) {
     __syncthreads();
     out_pos += tot;
   }
+  if (SINGLE && threadIdx.x == 0) *p.n_groups = out_pos;
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -486,6 +493,54 @@ __global__ void __launch_bounds__(256) k_partition_scatter(PartParams p) {
 }
 
 // ------------------------------------------------------------------------------------------------
+// read-only roofline (measurement helper): stream every column once, XOR-fold, one RED per CTA
+// ------------------------------------------------------------------------------------------------
+struct ReadCols {
+  const int4* c[kMaxKeys + kMaxVals];
+  uint64_t n16[kMaxKeys + kMaxVals];  // 16-byte chunks per column
+  int n;
+  unsigned long long* out;
+};
+
+__global__ void __launch_bounds__(512, 2) k_read_roofline(ReadCols rc) {
+  const uint64_t pol = evict_first_policy();
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  uint64_t acc = 0;
+  for (int j = 0; j < rc.n; ++j) {
+    const int4* p = rc.c[j];
+    const uint64_t n = rc.n16[j];
+    uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    for (; i + 3 * stride < n; i += 4 * stride) {  // 4 independent loads in flight per thread
+      const int4 a = ld_stream_v4(p + i, pol), b = ld_stream_v4(p + i + stride, pol);
+      const int4 c = ld_stream_v4(p + i + 2 * stride, pol), d = ld_stream_v4(p + i + 3 * stride, pol);
+      acc ^= (uint64_t)(uint32_t)(a.x ^ b.x ^ c.x ^ d.x) | (uint64_t)(uint32_t)(a.y ^ b.y ^ c.y ^ d.y) << 32;
+      acc ^= (uint64_t)(uint32_t)(a.z ^ b.z ^ c.z ^ d.z) | (uint64_t)(uint32_t)(a.w ^ b.w ^ c.w ^ d.w) << 32;
+    }
+    for (; i < n; i += stride) {
+      const int4 a = ld_stream_v4(p + i, pol);
+      acc ^= (uint64_t)(uint32_t)a.x | (uint64_t)(uint32_t)a.y << 32;
+      acc ^= (uint64_t)(uint32_t)a.z | (uint64_t)(uint32_t)a.w << 32;
+    }
+  }
+  for (int o = 16; o; o >>= 1) acc ^= __shfl_xor_sync(0xffffffffu, acc, o);
+  if ((threadIdx.x & 31) == 0) atomicXor(rc.out, (unsigned long long)acc);
+}
+
+int launch_read_roofline(const void* const* cols, const uint64_t* bytes, int n_cols, void* stream, uint64_t* out,
+                         int sms) {
+  ReadCols rc{};
+  rc.n = n_cols;
+  rc.out = (unsigned long long*)out;
+  for (int j = 0; j < n_cols; ++j) {
+    rc.c[j] = (const int4*)cols[j];
+    rc.n16[j] = bytes[j] / 16;
+  }
+  k_read_roofline<<<2 * sms, 512, 0, (cudaStream_t)stream>>>(rc);
+  count_launch(1);
+  return (int)cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------
 // launchers
 // ------------------------------------------------------------------------------------------------
 static int grid_for(uint64_t n, int threads, int max_blocks) {
@@ -494,15 +549,17 @@ static int grid_for(uint64_t n, int threads, int max_blocks) {
   return (int)(b ? b : 1);
 }
 
-int launch_init_slots(const Layout& lay, void* table, uint64_t n_slots, void* stream) {
-  if (!n_slots) return 0;
+int launch_init_slots(const Layout& lay, void* table, uint64_t n_slots, void* stream, uint64_t* zero, uint32_t n_zero) {
+  if (!n_slots && !zero) return 0;
   SlotTemplate t{};
   uint8_t buf[256];
   build_slot_template(lay, buf);
   memcpy(t.w, buf, lay.slot_bytes);
   t.words = lay.slot_bytes / 8;
   uint64_t chunks = n_slots * (lay.slot_bytes / 16);
-  k_init_slots<<<grid_for(chunks, 256, 148 * 16), 256, 0, (cudaStream_t)stream>>>(t, (uint64_t*)table, chunks);
+  if (!chunks && !zero) return 0;
+  k_init_slots<<<grid_for(std::max<uint64_t>(chunks, 1), 256, 148 * 16), 256, 0, (cudaStream_t)stream>>>(
+      t, (uint64_t*)table, chunks, zero, zero ? n_zero : 0);
   count_launch(1);
   return (int)cudaGetLastError();
 }
@@ -517,16 +574,39 @@ static uint64_t identity_host(int k) {
   }
 }
 
-int launch_init_dense(const Layout& lay, void* const dense[4], uint64_t D, void* stream) {
-  // Dense state groups: ISUM/FSUM -> 0; MIN -> INT64_MAX (covers widened i32 and ordered f64);
-  // MAX -> INT64_MIN. Each group is one contiguous array.
+struct DenseInit {
+  uint64_t* a[4];
+  uint64_t n[4];
+  uint64_t* zero;  // optional block of n_zero u64 words set to 0 (the execute's flag/counter block)
+  uint32_t n_zero;
+};
+
+__global__ void __launch_bounds__(256) k_init_dense_all(DenseInit d) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x, t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (d.zero && t < d.n_zero) d.zero[t] = 0;
+#pragma unroll
   for (int g = 0; g < 4; ++g) {
-    uint64_t n = (uint64_t)lay.n_group[g] * D;
-    if (!n) continue;
-    uint64_t v = g == SG_MIN ? (uint64_t)INT64_MAX : g == SG_MAX ? (uint64_t)INT64_MIN : 0ull;
-    k_fill_u64<<<grid_for(n, 256, 148 * 16), 256, 0, (cudaStream_t)stream>>>((uint64_t*)dense[g], n, v);
-    count_launch(1);
+    const uint64_t v = g == SG_MIN ? (uint64_t)INT64_MAX : g == SG_MAX ? (uint64_t)INT64_MIN : 0ull;
+    for (uint64_t i = t; i < d.n[g]; i += stride) d.a[g][i] = v;
   }
+}
+
+int launch_init_dense(const Layout& lay, void* const dense[4], uint64_t D, void* stream, uint64_t* zero,
+                      uint32_t n_zero) {
+  // Dense state groups: ISUM/FSUM -> 0; MIN -> INT64_MAX (covers widened i32 and ordered f64);
+  // MAX -> INT64_MIN. Each group is one contiguous array; one launch initialises all of them.
+  DenseInit d{};
+  uint64_t tot = n_zero;
+  for (int g = 0; g < 4; ++g) {
+    d.a[g] = (uint64_t*)dense[g];
+    d.n[g] = (uint64_t)lay.n_group[g] * D;
+    tot = std::max<uint64_t>(tot, d.n[g]);
+  }
+  d.zero = zero;
+  d.n_zero = zero ? n_zero : 0;
+  if (!tot) return 0;
+  k_init_dense_all<<<grid_for(tot, 256, 148 * 16), 256, 0, (cudaStream_t)stream>>>(d);
+  count_launch(1);
   (void)identity_host;
   return (int)cudaGetLastError();
 }
@@ -547,7 +627,9 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
       const int fuse = fin && fin->enabled;
       snprintf(name, sizeof name, "blu_jit_dense_%d_%d%s", nv, r, fuse ? "_fused" : "");
       snprintf(decl, sizeof decl, "%s(blu::AggParams p, blu::FinalParams fp)", name);
-      snprintf(body, sizeof body, "blu::dense_body<blu::JitSpec, %d, %d, %s>(p, fp);", nv, r, fuse ? "true" : "false");
+      const int pairmap = r == 4 && jit_env("BLU_GBY_DENSE_PAIR", 0);
+      snprintf(body, sizeof body, "blu::dense_body<blu::JitSpec, %d, %d, %s, %s>(p, fp);", nv, r, fuse ? "true" : "false",
+               pairmap ? "true" : "false");
       FinalParams fpc = fin ? *fin : FinalParams{};
       void* args[] = {&pc, &fpc};
       // 2 CTAs x 512 threads per SM: <= 64 registers (one resident wave, see plan.cpp)
@@ -624,9 +706,15 @@ int launch_compact(const CompactParams& p, void* stream, uint32_t* launches) {
     cudaMemsetAsync(p.n_groups, 0, 8, st);
     return (int)cudaGetLastError();
   }
+  if (nb == 1) {  // small table / dense domain: one CTA, one launch
+    k_compact_emit<true><<<1, kCT, 0, st>>>(p);
+    count_launch(1);
+    if (launches) *launches += 1;
+    return (int)cudaGetLastError();
+  }
   k_compact_count<<<(unsigned)nb, kCT, 0, st>>>(p);
   k_compact_scan<<<1, 1024, 0, st>>>(p.block_counts, p.block_offsets, nb, p.n_groups);
-  k_compact_emit<<<(unsigned)nb, kCT, 0, st>>>(p);
+  k_compact_emit<false><<<(unsigned)nb, kCT, 0, st>>>(p);
   count_launch(3);
   if (launches) *launches += 3;
   return (int)cudaGetLastError();

@@ -185,3 +185,21 @@ def test_wide_key_plans(bg, keys, n_fields):
     assert d["n_states"] == n_fields
     assert p.record_bytes == 8 * (2 + n_fields)
     assert d["slot_bytes"] >= 16 + 8
+
+
+@pytest.mark.parametrize("name", ["C1", "C2", "C3", "C4", "C5", "K3"])
+def test_jit_probe_compiles_plan_kernels(bg, name):
+    """The NVRTC programs execute would JIT for each config compile with the NVRTC the library loads
+    (no GPU needed); a failure here would silently fall back to the generic kernels on the GPU."""
+    import blugen
+    w = blugen.workload(name)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    st, n, log = bg.blu_gby_jit_probe(plan)
+    assert st == bg.BLU_OK, log
+    assert n >= (3 if plan.info()["partitions"] > 1 else 1)
+
+
+def test_jit_probe_wide_keys_unsupported(bg):
+    plan = bg.blu_gby_plan([(I64, 0), (I64, 0)], [I64], [(SUM, 0)], 100, 1000)
+    st, n, _ = bg.blu_gby_jit_probe(plan)
+    assert st == bg.BLU_E_UNSUPPORTED and n == 0
