@@ -628,6 +628,25 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
   const bool single = n <= (((uint64_t)P->grid * (1ull << 30)) & ~3ull);
   Feeder feed = [&](AggParams& base, uint32_t* launches, Work& w, const FinalParams* fin) -> cudaError_t {
     base.jit_ok = L.key_words == 2 ? 0 : 1;
+    // hot-key front seeded with the heavy hitters of a row sample (needs a COUNT field to tell
+    // seeded keys that received rows from those that did not)
+    static const bool no_seed = getenv("BLU_GBY_NO_SEED") != nullptr;
+    if (base.front_slots > 0 && L.count_field >= 0 && !no_seed && n >= (1u << 16)) {
+      void* ws = nullptr;
+      cudaError_t e = w.alloc(&ws, front_seed_bytes(base.front_slots));
+      if (e) return e;
+      AggParams pk = base;
+      uint32_t vec = 1;
+      for (int k = 0; k < L.n_keys; ++k) {
+        pk.key[k] = keys[k];
+        if (((uintptr_t)keys[k] & 15) != 0) vec = 0;
+      }
+      pk.vec_ok = (int32_t)vec;
+      const uint64_t* front = nullptr;
+      int rc = launch_front_seed(pk, n, base.front_slots, ws, st, (int)P->sms, &front);
+      if (rc) return (cudaError_t)rc;
+      base.front_seed = front;
+    }
     if (P->path == BLU_PATH_HASH_GLOBAL && P->parts > 1 && n >= 4096 * (uint64_t)P->parts)
       return partitioned_feed(P, base, keys, vals, n, st, launches, w);
     return agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, launches, fin);

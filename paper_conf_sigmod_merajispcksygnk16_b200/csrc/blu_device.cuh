@@ -30,6 +30,11 @@ __device__ __forceinline__ uint64_t fmix64(uint64_t h) {  // Murmur3 finalizer (
   return h;
 }
 
+// home slot of a key in the shared-memory front (bits independent of the table's slot bits)
+__device__ __forceinline__ uint32_t front_home(uint64_t key, uint32_t S) {
+  return (uint32_t)(fmix64(key ^ 0x5bd1e995ull) >> 40) & (S - 1);
+}
+
 // Order-preserving map of IEEE-754 f64 bits onto int64 (an involution).
 __device__ __forceinline__ int64_t ord_f64(uint64_t bits) {
   int64_t b = (int64_t)bits;
@@ -845,7 +850,9 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
     __syncthreads();
   }
   if (FRONT) {
-    for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) ((uint64_t*)(sm + p.key_off))[e] = kEmpty;
+    const uint64_t* seed = p.front_seed;
+    for (uint32_t e = threadIdx.x; e < S; e += blockDim.x)
+      ((uint64_t*)(sm + p.key_off))[e] = seed ? __ldg((const unsigned long long*)seed + e) : kEmpty;
     for (int j = 0; j < L.n_fields; ++j)
       for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) smem_init_entry(sm + p.soff[j], L.f[j].kind, e, S);
     __syncthreads();
@@ -936,23 +943,34 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
     if (FRONT && !deduped) {
       // hot-key front: small open-addressing table per CTA in shared memory
       uint64_t* fk = (uint64_t*)(sm + p.key_off);
+      const bool seeded = p.front_seed != nullptr;
       uint32_t fe[R];
       uint32_t hit = 0;
 #pragma unroll
       for (int r = 0; r < R; ++r) {
         fe[r] = 0;
         if (!(valid >> r & 1)) continue;
-        uint32_t s = (uint32_t)(fmix64(key[r] ^ 0x5bd1e995ull) >> 40) & (S - 1);
+        uint32_t s = front_home(key[r], S);
+        if (seeded) {  // read-only front (load <= 1/2): stop at the key or the first empty slot
 #pragma unroll 1
-        for (int q = 0; q < 8; ++q) {
-          uint64_t cur = *(volatile uint64_t*)(fk + s);
-          if (cur == key[r]) { hit |= 1u << r; break; }
-          if (cur == kEmpty) {
-            unsigned long long old = atomicCAS((unsigned long long*)(fk + s), (unsigned long long)kEmpty,
-                                               (unsigned long long)key[r]);
-            if (old == kEmpty || old == key[r]) { hit |= 1u << r; break; }
+          for (int q = 0; q < 8; ++q) {
+            const uint64_t cur = fk[s];
+            if (cur == key[r]) { hit |= 1u << r; break; }
+            if (cur == kEmpty) break;
+            s = (s + 1) & (S - 1);
           }
-          s = (s + 1) & (S - 1);
+        } else {
+#pragma unroll 1
+          for (int q = 0; q < 8; ++q) {
+            uint64_t cur = *(volatile uint64_t*)(fk + s);
+            if (cur == key[r]) { hit |= 1u << r; break; }
+            if (cur == kEmpty) {
+              unsigned long long old = atomicCAS((unsigned long long*)(fk + s), (unsigned long long)kEmpty,
+                                                 (unsigned long long)key[r]);
+              if (old == kEmpty || old == key[r]) { hit |= 1u << r; break; }
+            }
+            s = (s + 1) & (S - 1);
+          }
         }
         fe[r] = s;
       }
@@ -1024,9 +1042,11 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
     // merge the front into the global table
     __syncthreads();
     const uint64_t* fk = (const uint64_t*)(sm + p.key_off);
+    const int cf = L.count_field;
     for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) {
       const uint64_t key = fk[e];
       if (key == kEmpty) continue;
+      if (p.front_seed && s_read<FK_COUNT>(sm + p.soff[cf], e, S) == 0) continue;  // seeded, no rows here
       uint64_t s = key;
       if (!DIRECT) {
         uint64_t idx = fmix64(key) & p.cap_mask;

@@ -41,6 +41,7 @@ struct blu_gby_plan_s {
   uint64_t n_rows;
   uint64_t cap;           // hash slots (path b) or D (paths a, b')
   int32_t hot_front;
+  int32_t front_wide;  // 1: one 1024-thread CTA per SM with a double-size front
   uint32_t front_slots;   // entries of the shared-memory front
   uint32_t smem_bytes;    // dynamic shared memory of the aggregation kernel
   uint32_t grid, block;
@@ -73,6 +74,9 @@ int launch_init_slots(const Layout& lay, void* table, uint64_t n_slots, void* st
 int launch_init_dense(const Layout& lay, void* const dense[4], uint64_t D, void* stream, uint64_t* zero = nullptr,
                       uint32_t n_zero = 0);
 int launch_compact(const CompactParams& p, void* stream, uint32_t* launches);
+size_t front_seed_bytes(uint32_t S);
+int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, void* ws, void* stream, int sms,
+                      const uint64_t** front_out);
 int launch_read_roofline(const void* const* cols, const uint64_t* bytes, int n_cols, void* stream, uint64_t* out,
                          int sms);
 int launch_partition(const Layout& lay, const void* const* key_cols, const void* const* state_cols,

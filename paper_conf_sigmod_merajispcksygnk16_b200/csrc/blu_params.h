@@ -113,6 +113,10 @@ struct AggParams {
   // compacts it into the result (FinalParams::enabled); sync[0] = init done, sync[1] = CTAs done
   uint32_t fuse_init;
   uint32_t* sync;
+  // seeded hot-key front (heavy hitters from a sample, [20] via P:38): S keys laid out as the
+  // front's open-addressing image; CTAs copy it and only look keys up (no inserts). NULL = the
+  // front is filled first-come with CAS inserts.
+  const uint64_t* front_seed;
 };
 
 // Path (a) in-kernel compaction (S8 fused into S5a/S7 for small dense domains).

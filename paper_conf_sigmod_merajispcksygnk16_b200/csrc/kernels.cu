@@ -53,8 +53,10 @@ static bool launch_jit(const char* body, const char* entry_decl, const AggParams
                        uint32_t grid, uint32_t block, uint32_t smem, const char* entry, int min_blocks = 1) {
   if (!p.jit_ok || !jit_enabled()) return false;
   const std::string spec = jit_spec("JitSpec", p.lay);
-  std::string src = "extern \"C\" __global__ void __launch_bounds__(512, " +
-                    std::to_string(jit_env("BLU_GBY_JIT_MINB", min_blocks)) + ") ";
+  // 1024-thread CTAs (one per SM, wide hot-key front) keep the same 64-register budget
+  const int maxt = block > 512 ? 1024 : 512, minb = block > 512 ? 1 : jit_env("BLU_GBY_JIT_MINB", min_blocks);
+  std::string src = "extern \"C\" __global__ void __launch_bounds__(" + std::to_string(maxt) + ", " +
+                    std::to_string(minb) + ") ";
   src += entry_decl;
   src += " { ";
   src += body;
@@ -493,6 +495,131 @@ __global__ void __launch_bounds__(256) k_partition_scatter(PartParams p) {
 }
 
 // ------------------------------------------------------------------------------------------------
+// Seeded hot-key front: heavy hitters of a row sample (the heavy-hitter aggregation of [20],
+// P:38 / P:316). 1) count the packed keys of ~2^20 sampled rows in a global sample table;
+// 2) histogram their counts; 3) pick the count threshold that keeps <= K keys; 4) lay those keys
+// out as the front's open-addressing image (load <= 1/2) that every CTA copies into shared memory.
+// ------------------------------------------------------------------------------------------------
+static int grid_for(uint64_t n, int threads, int max_blocks);
+
+struct HHParams {
+  uint64_t* skey;       // sample table keys (cap_s, kEmpty = free)
+  uint32_t* scnt;       // sample table counts
+  uint64_t cap_s;       // power of two
+  uint32_t* hist;       // kHHBins counts-of-counts
+  uint32_t* ctl;        // [0] threshold, [1] keys placed
+  uint64_t* front;      // S-slot front image
+  uint32_t S, K;
+  uint64_t blocks, block_rows, block_stride;  // sample = `blocks` runs of block_rows rows
+};
+constexpr uint32_t kHHBins = 4096;
+
+__global__ void __launch_bounds__(512) k_hh_count(AggParams p, HHParams h) {
+  constexpr int R = 4;
+  const uint64_t pol = evict_first_policy();
+  const uint64_t tiles_per_block = (h.block_rows + 512 * R - 1) / (512 * R);
+  for (uint64_t w = blockIdx.x; w < h.blocks * tiles_per_block; w += gridDim.x) {
+    const uint64_t b = w / tiles_per_block, t = w % tiles_per_block;
+    const uint64_t r0 = b * h.block_stride + t * 512 * R;
+    const uint64_t n = std::min<uint64_t>(p.n_rows, b * h.block_stride + h.block_rows);
+    const uint64_t row = lane_base<R>(r0, threadIdx.x >> 5, threadIdx.x & 31);
+    uint64_t key[R];
+    const uint32_t valid = pack_keys<GenericSpec, R>(p, row, n, pol, key);
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!(valid >> r & 1)) continue;
+      uint64_t s = fmix64(key[r] ^ 0x68686868ull) & (h.cap_s - 1);
+      for (int q = 0; q < 64; ++q) {
+        uint64_t cur = __ldcg((const unsigned long long*)h.skey + s);
+        if (cur == kEmpty) {
+          cur = atomicCAS((unsigned long long*)h.skey + s, (unsigned long long)kEmpty, (unsigned long long)key[r]);
+          if (cur == kEmpty) cur = key[r];
+        }
+        if (cur == key[r]) {
+          atomicAdd(h.scnt + s, 1u);
+          break;
+        }
+        s = (s + 1) & (h.cap_s - 1);
+      }
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_hh_hist(HHParams h) {
+  __shared__ uint32_t sh[kHHBins];
+  for (uint32_t i = threadIdx.x; i < kHHBins; i += blockDim.x) sh[i] = 0;
+  __syncthreads();
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < h.cap_s; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = h.scnt[i];
+    if (c) atomicAdd(&sh[std::min<uint32_t>(c, kHHBins - 1)], 1u);
+  }
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < kHHBins; i += blockDim.x)
+    if (sh[i]) atomicAdd(&h.hist[i], sh[i]);
+}
+
+// smallest threshold t >= 2 with #(keys with count >= t) <= K (one warp, bins scanned from the top)
+__global__ void k_hh_pick(HHParams h) {
+  if (threadIdx.x != 0) return;
+  uint64_t acc = 0;
+  uint32_t t = kHHBins;
+  for (int b = kHHBins - 1; b >= 2; --b) {
+    if (acc + h.hist[b] > h.K) break;
+    acc += h.hist[b];
+    t = b;
+  }
+  if (t == kHHBins) t = kHHBins - 1;  // even the top bin overflows K: take its keys first come
+  h.ctl[0] = t;
+}
+
+__global__ void __launch_bounds__(256) k_hh_build(HHParams h) {
+  const uint32_t t = h.ctl[0];
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < h.cap_s; i += (uint64_t)gridDim.x * blockDim.x) {
+    if (h.scnt[i] < t) continue;
+    if (atomicAdd(&h.ctl[1], 1u) >= h.K) continue;
+    const uint64_t key = h.skey[i];
+    uint32_t s = front_home(key, h.S);
+    for (uint32_t q = 0; q < h.S; ++q) {  // load <= 1/2: always finds a free slot
+      if (atomicCAS((unsigned long long*)h.front + s, (unsigned long long)kEmpty, (unsigned long long)key) == kEmpty) break;
+      s = (s + 1) & (h.S - 1);
+    }
+  }
+}
+
+size_t front_seed_bytes(uint32_t S) { return (size_t)S * 8 + ((size_t)1 << 18) * 12 + kHHBins * 4 + 64; }
+
+int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, void* ws, void* stream, int sms,
+                      const uint64_t** front_out) {
+  cudaStream_t st = (cudaStream_t)stream;
+  HHParams h{};
+  h.S = S;
+  h.K = S / 2;
+  h.cap_s = (uint64_t)1 << 18;
+  uint8_t* w = (uint8_t*)ws;
+  h.front = (uint64_t*)w;
+  h.skey = (uint64_t*)(w + (size_t)S * 8);
+  h.scnt = (uint32_t*)(h.skey + h.cap_s);
+  h.hist = h.scnt + h.cap_s;
+  h.ctl = h.hist + kHHBins;
+  // sample: up to 256 evenly spaced runs of 4096 rows (2^20 rows; all rows if fewer)
+  h.block_rows = 4096;
+  h.blocks = std::min<uint64_t>(256, (n + h.block_rows - 1) / h.block_rows);
+  h.block_stride = h.blocks > 1 ? (n - h.block_rows) / (h.blocks - 1) / 4 * 4 : 0;
+  if (h.blocks <= 1) h.block_rows = n;
+  k_fill_u64<<<grid_for((uint64_t)S + h.cap_s, 256, sms * 8), 256, 0, st>>>(h.front, (uint64_t)S + h.cap_s, kEmpty);
+  cudaMemsetAsync(h.scnt, 0, h.cap_s * 4 + kHHBins * 4 + 64, st);
+  AggParams p = base;
+  p.n_rows = n;
+  k_hh_count<<<sms * 2, 512, 0, st>>>(p, h);
+  k_hh_hist<<<sms, 256, 0, st>>>(h);
+  k_hh_pick<<<1, 32, 0, st>>>(h);
+  k_hh_build<<<sms, 256, 0, st>>>(h);
+  count_launch(5);
+  *front_out = h.front;
+  return (int)cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------------
 // read-only roofline (measurement helper): stream every column once, XOR-fold, one RED per CTA
 // ------------------------------------------------------------------------------------------------
 struct ReadCols {
@@ -682,7 +809,7 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
     if (smem > 48 * 1024) e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e) return (int)e;
     if (!p.gate || p.gate_run_if == 0) note_kernel("k_agg_global (generic)");
-    k<<<grid, block, smem, st>>>(p, rs);
+    k<<<grid, block > 512 ? 512 : block, smem, st>>>(p, rs);  // generic kernels: <= 512 threads
   }
   count_launch(1);
   return (int)cudaGetLastError();

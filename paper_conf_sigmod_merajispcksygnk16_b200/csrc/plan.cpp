@@ -53,6 +53,7 @@ constexpr double kMaxLoadPart = 0.5;            // partitioned mode (buckets are
 constexpr uint64_t kMinCap = 1024;
 constexpr uint64_t kFrontRatio = 1000;          // rows/groups above which the front pays off
 constexpr uint32_t kFrontBudget = 110 * 1024;
+constexpr uint32_t kFrontBudgetWide = 220 * 1024;  // one CTA per SM
 constexpr uint64_t kDirectMin = 1ull << 20;
 constexpr uint64_t kRowLockRatio = 16;          // kernel 3 when rows/groups <= this
 constexpr uint32_t kPartBudgetMB = 48;          // L2 slice per bucket (126 MB L2)
@@ -415,12 +416,20 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     if (on) {
       uint32_t per = 8 + L.smem_entry_bytes;
       uint32_t budget = kFrontBudget;
-      uint32_t S = 4096;
+      uint32_t S = 8192;
       if (const char* fs = env("BLU_GBY_FRONT_SLOTS")) S = (uint32_t)atoi(fs);
-      while (S > 64 && S * per > budget) S >>= 1;  // power of two, >= 64: 4-way buckets
-      if (S * per <= 200 * 1024) {
+      uint32_t S1 = S, S2 = S;
+      while (S1 > 64 && S1 * per > budget) S1 >>= 1;  // power of two, >= 64
+      while (S2 > 64 && S2 * per > kFrontBudgetWide) S2 >>= 1;
+      // a front twice as large in one 1024-thread CTA per SM holds twice the heavy hitters (the
+      // seeded front keeps S/2 keys); same threads and registers per SM as 2 x 512
+      bool wide = S2 > S1;
+      if (const char* fw = env("BLU_GBY_FRONT_WIDE")) wide = wide && fw[0] == '1';
+      S = wide ? S2 : S1;
+      if (S * per <= 200 * 1024 || wide) {
         P->hot_front = 1;
         P->front_slots = S;
+        P->front_wide = wide ? 1 : 0;
       }
     }
   }
@@ -436,7 +445,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     uint32_t b = P->front_slots * 8;
     for (int j = 0; j < L.n_fields; ++j) b += (P->front_slots * L.f[j].ssize + 15) / 16 * 16;
     P->smem_bytes = b;
-    P->block = 512;
+    P->block = P->front_wide ? 1024 : 512;
   } else {
     P->smem_bytes = 0;
     P->block = 256;

@@ -66,6 +66,11 @@ def main():
         "shared_atom_bank_conflicts": num("l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_atom.sum"),
         "global_red_inst": num("smsp__inst_executed_op_global_red.sum"),
         "inst_executed": num("smsp__inst_executed.sum"),
+        "lsu_data_pipe_pct": num("l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed"),
+        "shared_wavefronts": num("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum"),
+        "shared_ld_wavefronts": num("l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum"),
+        "shared_atom_wavefronts": num("l1tex__data_pipe_lsu_wavefronts_mem_shared_op_atom.sum"),
+        "global_ld_sectors": num("l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum"),
         "top_stalls_pct": {k: round(100 * v / tot, 1) for k, v in top},
         "sm_clock_hz": num("gpc__cycles_elapsed.avg.per_second"),
         "note": a.note,
