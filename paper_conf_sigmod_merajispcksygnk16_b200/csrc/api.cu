@@ -206,6 +206,10 @@ static OutSpec make_outspec(const blu_gby_plan_s* P, const Layout& lay, bool par
 using Feeder = std::function<cudaError_t(AggParams& base, uint32_t* launches, Work& w, const FinalParams* fin)>;
 
 static bool ptr_aligned(const void* p) { return ((uintptr_t)p & 15) == 0; }
+static uint32_t prefetch_enabled() {  // scatter prefetch distance in tiles (BLU_GBY_PREFETCH, default 1)
+  static const uint32_t d = getenv("BLU_GBY_PREFETCH") ? (uint32_t)atoi(getenv("BLU_GBY_PREFETCH")) : 1u;
+  return d;
+}
 
 // Launch the aggregation for rows [0, n) of one batch, chunked so per-CTA 32-bit shared counters
 // cannot overflow.
@@ -550,6 +554,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       vec = vec && ptr_aligned(p1.val[c]);
     }
     p1.vec_ok = vec;
+    p1.prefetch = prefetch_enabled();
     p1.n_rows = m;
     ScatterParams sp{};
     sp.B = B;

@@ -188,6 +188,23 @@ __device__ __forceinline__ void load_rows(const void* base, int dt, uint64_t lb,
   }
 }
 
+// L2 prefetch of the column bytes of rows [r0, r1) (one prefetch per 128-byte line, spread over the
+// CTA): issued one tile ahead so HBM reads stay in flight while the CTA works on the current tile.
+template <class SP>
+__device__ __forceinline__ void prefetch_rows_l2(const AggParams& p, uint64_t r0, uint64_t r1) {
+  if (r0 >= r1) return;
+  const int nk = p.lay.n_keys, nv = p.lay.n_vals;
+  for (int c = 0; c < nk + nv; ++c) {
+    const bool is_key = c < nk;
+    const int dt = is_key ? p.lay.key_dtype[c] : p.lay.val_dtype[c - nk];
+    const uint32_t w = dt == BLU_I32 ? 4 : 8;
+    const uint8_t* base = (const uint8_t*)(is_key ? p.key[c] : p.val[c - nk]);
+    const uintptr_t a0 = ((uintptr_t)(base + r0 * w)) & ~(uintptr_t)127, a1 = (uintptr_t)(base + r1 * w);
+    for (uintptr_t a = a0 + (uintptr_t)threadIdx.x * 128; a < a1; a += (uintptr_t)blockDim.x * 128)
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(a));
+  }
+}
+
 // Identity (the mask value of P:151) of a field in its encoded 64-bit form.
 __device__ __forceinline__ uint64_t identity64(int k) {
   switch (k) {
@@ -1125,6 +1142,10 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
     const uint32_t valid = pack_keys<SP, R>(p, row, n, pol, key);
     uint64_t v[NV][R];
     load_vals<SP, NV, R>(p, row, n, pol, v);
+    if (p.prefetch) {  // a later tile of this CTA: in flight during the sort and the writes below
+      const uint64_t nt = t + (uint64_t)gridDim.x * p.prefetch;
+      prefetch_rows_l2<SP>(p, nt * TILE, nt * TILE + TILE < n ? nt * TILE + TILE : n);
+    }
     uint32_t bb[R], pos[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) {

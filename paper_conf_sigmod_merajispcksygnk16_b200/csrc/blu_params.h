@@ -117,6 +117,7 @@ struct AggParams {
   // front's open-addressing image; CTAs copy it and only look keys up (no inserts). NULL = the
   // front is filled first-come with CAS inserts.
   const uint64_t* front_seed;
+  uint32_t prefetch;             // scatter: L2-prefetch the column bytes of the tile this many tiles ahead (0 = off)
 };
 
 // Path (a) in-kernel compaction (S8 fused into S5a/S7 for small dense domains).
