@@ -22,11 +22,11 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libblugen.so")
 
 # dtype / op numbering — identical to include/blu_gby.h (by convention; no shared code).
-I32, I64, F64 = 0, 1, 2
+I32, I64, F64, I128 = 0, 1, 2, 3  # I128 columns: int64 arrays of shape (n, 2) = (lo, hi) words
 COUNT, SUM, MIN, MAX, AVG = 0, 1, 2, 3, 4
-DTYPE_NAMES = {I32: "i32", I64: "i64", F64: "f64"}
+DTYPE_NAMES = {I32: "i32", I64: "i64", F64: "f64", I128: "i128"}
 OP_NAMES = {COUNT: "COUNT", SUM: "SUM", MIN: "MIN", MAX: "MAX", AVG: "AVG"}
-NP_DTYPE = {I32: np.int32, I64: np.int64, F64: np.float64}
+NP_DTYPE = {I32: np.int32, I64: np.int64, F64: np.float64, I128: np.int64}
 
 # generator kinds (blu_gen_kind_t)
 UNIFORM, DYADIC, SPARSE_KEY, ZIPF_DIGIT, CYCLIC_DIGIT, LINEAR, REAL, UNIFORM_DIGIT = range(8)
@@ -79,7 +79,7 @@ class Schema:
             return F64
         vd = self.vals[col]
         if op == SUM:
-            return F64 if vd == F64 else I64
+            return vd if vd in (F64, I128) else I64
         return vd  # MIN / MAX keep the input dtype
 
 

@@ -15,7 +15,7 @@ from typing import List, Optional, Sequence
 import numpy as np
 
 import blugen
-from blugen import COUNT, SUM, MIN, MAX, AVG, I32, I64, F64
+from blugen import COUNT, SUM, MIN, MAX, AVG, I32, I64, F64, I128
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "liboracle.so")
@@ -91,7 +91,7 @@ def _fetch(h, s: blugen.Schema) -> OracleResult:
     aggs, sumabs = [], []
     for a, (op, col) in enumerate(s.aggs):
         od = s.agg_out_dtype(a)
-        aggs.append(np.zeros(G, np.float64 if od == F64 else np.int64))
+        aggs.append(np.zeros((G, 2) if od == I128 else G, np.float64 if od == F64 else np.int64))
         f64_in = op in (SUM, AVG) and s.vals[col] == F64
         sumabs.append(np.zeros(G, np.float64) if f64_in else None)
     agg_ptrs = (ctypes.c_void_p * max(1, len(aggs)))(*[x.ctypes.data for x in aggs])

@@ -23,7 +23,10 @@
  *   A12 AVG is f64: (double)(int64)sum / (double)count, IEEE round-to-nearest;
  *   A13 f64 SUM accumulates in long double (x86 80-bit) plus sum |v| for the tolerance check;
  *   A14 MIN/MAX use < and > (inputs hold no NaN, no -0.0);
- *   A15 all columns NOT NULL, COUNT means COUNT(*).
+ *   A15 all columns NOT NULL, COUNT means COUNT(*);
+ *   A18 128-bit integer payloads ("128bit Integer or Decimal data type", NEXT-2): SUM wraps
+ *       mod 2^128 (accumulated in unsigned __int128), MIN/MAX compare as signed __int128, AVG is
+ *       (double)(__int128)sum / (double)count (GCC's correctly rounded __int128 -> double).
  *
  * Parity pins for this file live in tests/test_oracle_pins.py (brute force, closed forms,
  * invariants, special cases).
@@ -40,7 +43,7 @@
 
 namespace {
 
-enum { O_I32 = 0, O_I64 = 1, O_F64 = 2 };
+enum { O_I32 = 0, O_I64 = 1, O_F64 = 2, O_I128 = 3 };
 enum { O_COUNT = 0, O_SUM = 1, O_MIN = 2, O_MAX = 3, O_AVG = 4 };
 
 struct Schema {
@@ -59,6 +62,8 @@ struct AggState {
     long double fabs_sum = 0.0L;
     int64_t imm = 0;          // integer MIN or MAX
     double fmm = 0.0;         // f64 MIN or MAX
+    unsigned __int128 qsum = 0;  // 128-bit SUM / AVG numerator, wraps mod 2^128
+    __int128 qmm = 0;            // 128-bit MIN or MAX
 };
 
 struct Group {
@@ -75,10 +80,11 @@ struct Result {
 struct Val {
     int64_t i;
     double d;
+    __int128 q;  // 128-bit payloads only
 };
 
 Val widen(int dtype, uint64_t bits) {
-    Val v{0, 0.0};
+    Val v{0, 0.0, 0};
     if (dtype == O_I32) v.i = (int64_t)(int32_t)(uint32_t)bits;
     else if (dtype == O_I64) v.i = (int64_t)bits;
     else memcpy(&v.d, &bits, sizeof(double));
@@ -88,6 +94,14 @@ Val widen(int dtype, uint64_t bits) {
 uint64_t read_bits(int dtype, const void* col, uint64_t i) {
     if (dtype == O_I32) return (uint64_t)(uint32_t)((const int32_t*)col)[i];
     return ((const uint64_t*)col)[i];
+}
+
+// A 128-bit payload: 16 bytes per row, low 64-bit word first (two's complement).
+Val read_i128(const void* col, uint64_t i) {
+    const uint64_t lo = ((const uint64_t*)col)[2 * i], hi = ((const uint64_t*)col)[2 * i + 1];
+    Val v{0, 0.0, 0};
+    v.q = (__int128)(((unsigned __int128)hi << 64) | lo);
+    return v;
 }
 
 // The per-row step: find or insert the group, then apply every aggregate.
@@ -110,6 +124,12 @@ void add_row(Result& r, const std::vector<int64_t>& key, const std::vector<Val>&
         int dt = s.val_dtypes[c];
         const Val& v = vals[c];
         AggState& st = g.a[a];
+        if (dt == O_I128) {
+            if (op == O_SUM || op == O_AVG) st.qsum += (unsigned __int128)v.q;
+            else if (op == O_MIN) { if (first || v.q < st.qmm) st.qmm = v.q; }
+            else if (op == O_MAX) { if (first || v.q > st.qmm) st.qmm = v.q; }
+            continue;
+        }
         if (op == O_SUM || op == O_AVG) {
             if (dt == O_F64) {
                 st.fsum += (long double)v.d;
@@ -187,7 +207,9 @@ void* oracle_groupby_arrays(const oracle_schema_t* sc, const void* const* keys, 
         for (int k = 0; k < sc->n_keys; ++k) key[k] = widen(sc->key_dtypes[k], read_bits(sc->key_dtypes[k], keys[k], i)).i;
         if (!in_slice(key, slice_p, slice_P)) continue;
         if (filter_keys && !filter.count(key)) continue;
-        for (int c = 0; c < sc->n_vals; ++c) v[c] = widen(sc->val_dtypes[c], read_bits(sc->val_dtypes[c], vals[c], i));
+        for (int c = 0; c < sc->n_vals; ++c)
+            v[c] = sc->val_dtypes[c] == O_I128 ? read_i128(vals[c], i)
+                                               : widen(sc->val_dtypes[c], read_bits(sc->val_dtypes[c], vals[c], i));
         add_row(*r, key, v);
     }
     return r;
@@ -229,7 +251,8 @@ uint64_t oracle_n_groups(void* h) { return ((Result*)h)->groups.size(); }
  *   keys_out:   n_groups x n_keys int64 (row-major)
  *   count_out:  n_groups int64
  *   agg_out[a]: n_groups elements: COUNT -> int64; SUM(int) -> int64; SUM(f64) -> double;
- *               MIN/MAX -> int64 (integer inputs, widened) or double; AVG -> double
+ *               MIN/MAX -> int64 (integer inputs, widened) or double; AVG -> double;
+ *               SUM/MIN/MAX of a 128-bit column -> 2 x uint64 per group (low word first)
  *   sumabs_out[a] (optional, may be NULL or hold NULLs): sum |v| per group for f64 SUM/AVG. */
 void oracle_fetch(void* h, int64_t* keys_out, int64_t* count_out, void* const* agg_out, double* const* sumabs_out) {
     Result* r = (Result*)h;
@@ -244,6 +267,16 @@ void oracle_fetch(void* h, int64_t* keys_out, int64_t* count_out, void* const* a
             int op = s.agg_ops[a];
             int dt = op == O_COUNT ? O_I64 : s.val_dtypes[s.agg_cols[a]];
             const AggState& st = G.a[a];
+            if (dt == O_I128 && op != O_COUNT) {
+                if (op == O_AVG) {
+                    ((double*)agg_out[a])[g] = (double)(__int128)st.qsum / (double)G.count;
+                } else {
+                    const unsigned __int128 x = op == O_SUM ? st.qsum : (unsigned __int128)st.qmm;
+                    ((uint64_t*)agg_out[a])[2 * g] = (uint64_t)x;
+                    ((uint64_t*)agg_out[a])[2 * g + 1] = (uint64_t)(x >> 64);
+                }
+                continue;
+            }
             if (op == O_COUNT) {
                 ((int64_t*)agg_out[a])[g] = G.count;
             } else if (op == O_SUM) {

@@ -304,3 +304,63 @@ def test_filter_is_subset_and_generated_equals_arrays():
     assert np.array_equal(sub.keys, pick)
     for x, y in zip(sub.aggs, full_a.aggs):
         assert np.array_equal(x, y[idx])
+
+
+# ---- 128-bit payloads (NEXT-2, reading A18) ------------------------------------------------------
+def i128_cols(ints):
+    """Python ints -> (n, 2) int64 (low word, high word), two's complement mod 2^128."""
+    out = np.zeros((len(ints), 2), np.int64)
+    for i, x in enumerate(ints):
+        u = x % (1 << 128)
+        out[i, 0] = np.int64(np.uint64(u & ((1 << 64) - 1)).view(np.int64))
+        out[i, 1] = np.int64(np.uint64(u >> 64).view(np.int64))
+    return out
+
+
+def i128_value(row):
+    u = (int(np.uint64(row[1]).view(np.uint64)) << 64) | int(np.int64(row[0]).view(np.uint64))
+    return u - (1 << 128) if u >> 127 else u
+
+
+def test_i128_brute_force():
+    """SUM (mod 2^128), MIN, MAX, AVG, COUNT over 128-bit payloads vs Python integers."""
+    rng = np.random.default_rng(128)
+    n = 3000
+    keys = rng.integers(0, 9, n)
+    vals = [int(x) for x in rng.integers(-(2**62), 2**62, n)]
+    vals = [v * (1 << 64) + int(rng.integers(0, 2**62)) if i % 3 else v for i, v in enumerate(vals)]  # full range
+    sch = blugen.Schema([(I64, 9)], [blugen.I128], [(COUNT, -1), (SUM, 0), (MIN, 0), (MAX, 0), (AVG, 0)])
+    o = oracle.groupby_arrays(sch, [keys.astype(np.int64)], [i128_cols(vals)])
+    assert list(o.keys[:, 0]) == sorted(set(keys.tolist()))
+    for gi, k in enumerate(o.keys[:, 0]):
+        g = [v for kk, v in zip(keys, vals) if kk == k]
+        s = sum(g) % (1 << 128)
+        s = s - (1 << 128) if s >> 127 else s
+        assert o.aggs[0][gi] == len(g)
+        assert i128_value(o.aggs[1][gi]) == s
+        assert i128_value(o.aggs[2][gi]) == min(g)
+        assert i128_value(o.aggs[3][gi]) == max(g)
+        assert o.aggs[4][gi] == float(s) / len(g)  # (double)sum correctly rounded, then IEEE division
+
+
+def test_i128_sum_wraps_mod_2_128():
+    """Closed form: 4 rows of 2^126 sum to 2^128 = 0; 5 rows of 2^126 to 2^126 (mod 2^128)."""
+    sch = blugen.Schema([(I64, 2)], [blugen.I128], [(SUM, 0)])
+    keys = np.array([0, 0, 0, 0, 1, 1, 1, 1, 1], np.int64)
+    o = oracle.groupby_arrays(sch, [keys], [i128_cols([1 << 126] * 9)])
+    assert i128_value(o.aggs[0][0]) == 0 and i128_value(o.aggs[0][1]) == 1 << 126
+
+
+def test_i128_in_int64_range_equals_i64_column():
+    """Special case: 128-bit payloads that fit 64 bits give the i64 results (sums far from wrapping)."""
+    rng = np.random.default_rng(7)
+    n = 5000
+    keys = rng.integers(0, 13, n).astype(np.int64)
+    v = rng.integers(-(2**40), 2**40, n)
+    s64 = blugen.Schema([(I64, 13)], [I64], [(SUM, 0), (MIN, 0), (MAX, 0), (AVG, 0)])
+    s128 = blugen.Schema([(I64, 13)], [blugen.I128], [(SUM, 0), (MIN, 0), (MAX, 0), (AVG, 0)])
+    a = oracle.groupby_arrays(s64, [keys], [v])
+    b = oracle.groupby_arrays(s128, [keys], [i128_cols([int(x) for x in v])])
+    for j in range(3):
+        assert np.array_equal(b.aggs[j][:, 0], a.aggs[j]) and np.array_equal(b.aggs[j][:, 1], a.aggs[j] >> 63)
+    assert np.array_equal(b.aggs[3], a.aggs[3])
