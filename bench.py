@@ -38,10 +38,10 @@ def load_peaks():
     return PEAKS_FALLBACK["hbm_gbs"], "fallback (B200_PROFILING.md)"
 
 
-def load_traffic(config):
-    """Per-launch DRAM traffic (read + write bytes) of the aggregation kernel from the committed
-    ncu --set full summary (profiles/), or None."""
-    p = os.path.join(ROOT, "profiles", f"ncu_{config}_summary.json")
+def load_traffic(config, phase=None):
+    """Per-launch DRAM traffic (read + write bytes) of the aggregation kernel (or of one phase of the
+    partitioned path) from the committed ncu --set full summary (profiles/), or None."""
+    p = os.path.join(ROOT, "profiles", f"ncu_{config}_{phase + '_' if phase else ''}summary.json")
     if os.path.exists(p):
         d = json.load(open(p))
         return d.get("dram_bytes_per_launch"), d.get("rows_per_launch")
@@ -234,6 +234,7 @@ def main():
     del r
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     agg_ms = []
+    part_t = []
     agg_kernel = ""
     sampler = ClockSampler(local if not args.no_clocks else -1)
     if world > 1:
@@ -250,6 +251,7 @@ def main():
         t = bg.blu_gby_last_timing()
         agg_ms.append(t["aggregate_ms"] / max(1, t["aggregate_launches"]))
         agg_kernel = t["kernel"]
+        part_t.append((t["scatter_ms"], t["pass2_ms"], t["part_chunks"]))
         del r
     torch.cuda.synchronize()
     launches = bg.blu_gby_launch_count() - c0
@@ -271,10 +273,39 @@ def main():
     # dominant kernel: the aggregation kernel (S5), timed with CUDA events on its launch stream
     agg_avg_ms = statistics.mean(agg_ms)
     rows_per_launch = n  # one aggregate launch per execute (rows < grid * 2^30)
-    achieved = rows_per_launch * bpr / (agg_avg_ms / 1000.0) / 1e9
+    alg_bytes = rows_per_launch * bpr
     traffic, traffic_rows = load_traffic(args.config)
-    if traffic is not None and traffic_rows:
-        traffic = traffic * rows_per_launch / traffic_rows
+    phases = None
+    chunks = max(c for _, _, c in part_t) if part_t else 0
+    if chunks:
+        # partitioned path (b): two kernels per chunk — the scatter (reads the input columns, writes
+        # the bucket records) and pass 2 (reads the records); the longer one is the dominant kernel
+        rec_bytes = 8 + sum(v.element_size() for v in vc)
+        sc_ms = statistics.mean(a for a, _, _ in part_t) / chunks
+        p2_ms = statistics.mean(b for _, b, _ in part_t) / chunks
+        rows_per_launch = n / chunks
+        sc_alg, p2_alg = rows_per_launch * (bpr + rec_bytes), rows_per_launch * rec_bytes
+        tr_sc, tr_rows_sc = load_traffic(args.config, "scatter")
+        tr_p2, tr_rows_p2 = load_traffic(args.config, "pass2")
+        phases = {
+            "scatter": {"avg_launch_ms": sc_ms, "algorithmic_bytes_per_launch": sc_alg,
+                        "achieved_gbs": sc_alg / (sc_ms / 1e3) / 1e9,
+                        "traffic": tr_sc * rows_per_launch / tr_rows_sc if tr_sc and tr_rows_sc else None},
+            "pass2": {"avg_launch_ms": p2_ms, "algorithmic_bytes_per_launch": p2_alg,
+                      "achieved_gbs": p2_alg / (p2_ms / 1e3) / 1e9,
+                      "traffic": tr_p2 * rows_per_launch / tr_rows_p2 if tr_p2 and tr_rows_p2 else None},
+            "launches_per_step": chunks,
+        }
+        dom = "pass2" if p2_ms >= sc_ms else "scatter"
+        agg_avg_ms = phases[dom]["avg_launch_ms"]
+        alg_bytes = phases[dom]["algorithmic_bytes_per_launch"]
+        traffic = phases[dom]["traffic"]
+        agg_kernel = f"{dom}: " + (agg_kernel if dom == "pass2" else "blu_jit_scatter")
+        achieved = alg_bytes / (agg_avg_ms / 1000.0) / 1e9
+    else:
+        achieved = alg_bytes / (agg_avg_ms / 1000.0) / 1e9
+        if traffic is not None and traffic_rows:
+            traffic = traffic * rows_per_launch / traffic_rows
     # SURVEY §8(d) denominator (i): the same input columns streamed read-only by our own kernel with the
     # aggregation kernels' load instructions (L2 flushed before each launch, like the steps)
     rr_out = torch.zeros(1, dtype=torch.int64, device=dev)
@@ -291,7 +322,7 @@ def main():
     read_gbs = n * bpr / (statistics.median(rr_ms) / 1000.0) / 1e9
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": traffic, "kernel": agg_kernel,
-                "algorithmic_bytes_per_launch": rows_per_launch * bpr, "avg_launch_ms": agg_avg_ms,
+                "algorithmic_bytes_per_launch": alg_bytes, "avg_launch_ms": agg_avg_ms, "phases": phases,
                 "peak_source": peak_src, "share_of_step": agg_avg_ms / (tot_ms / args.steps),
                 "read_only_ceiling_gbs": read_gbs, "frac_of_read_only_ceiling": achieved / read_gbs,
                 "spec_peak_gbs": 8000.0, "frac_of_spec": achieved / 8000.0}

@@ -141,6 +141,9 @@ typedef struct {
     uint32_t grid, block;    /* aggregation launch shape                                          */
     uint32_t retries_last;
     int32_t row_lock;        /* (b): kernel 3 — one row lock per slot, then every aggregate */
+    int32_t part_smem;       /* (b) partitioned: 1 = pass 2 aggregates each bucket in a per-CTA
+                                shared-memory table and merges it once per piece       */
+    uint32_t bucket_entries; /* part_smem: entries of that table                                   */
 } blu_gby_plan_desc_t;
 blu_status_t blu_gby_plan_describe(blu_gby_plan_t plan, blu_gby_plan_desc_t* out);
 
@@ -238,6 +241,10 @@ typedef struct {
     float init_ms, aggregate_ms, compact_ms, h2d_ms, total_ms;
     uint32_t aggregate_launches, retries;
     char kernel[64];     /* name of the last aggregation kernel launched (JIT entry or generic) */
+    /* partitioned path (b): the two passes of aggregate_ms, summed over chunks/retries */
+    float scatter_ms, pass2_ms;
+    uint32_t part_chunks;
+    uint32_t part_fallbacks; /* chunks in which a bucket overflowed and the one-pass fallback ran */
 } blu_gby_timing_t;
 void blu_gby_set_timing(int32_t enable);
 blu_status_t blu_gby_last_timing(blu_gby_timing_t* out);

@@ -56,13 +56,16 @@ class PlanDescC(ctypes.Structure):
                 ("slot_bytes", ctypes.c_uint32), ("smem_bytes", ctypes.c_uint32), ("hot_front", ctypes.c_int32),
                 ("front_slots", ctypes.c_uint32), ("partitions", ctypes.c_uint32), ("n_states", ctypes.c_int32),
                 ("state_dtypes", ctypes.c_int32 * 32), ("grid", ctypes.c_uint32), ("block", ctypes.c_uint32),
-                ("retries_last", ctypes.c_uint32), ("row_lock", ctypes.c_int32)]
+                ("retries_last", ctypes.c_uint32), ("row_lock", ctypes.c_int32), ("part_smem", ctypes.c_int32),
+                ("bucket_entries", ctypes.c_uint32)]
 
 
 class TimingC(ctypes.Structure):
     _fields_ = [("init_ms", ctypes.c_float), ("aggregate_ms", ctypes.c_float), ("compact_ms", ctypes.c_float),
                 ("h2d_ms", ctypes.c_float), ("total_ms", ctypes.c_float),
-                ("aggregate_launches", ctypes.c_uint32), ("retries", ctypes.c_uint32), ("kernel", ctypes.c_char * 64)]
+                ("aggregate_launches", ctypes.c_uint32), ("retries", ctypes.c_uint32), ("kernel", ctypes.c_char * 64),
+                ("scatter_ms", ctypes.c_float), ("pass2_ms", ctypes.c_float), ("part_chunks", ctypes.c_uint32),
+                ("part_fallbacks", ctypes.c_uint32)]
 
 
 def _load():

@@ -36,6 +36,30 @@ struct Events {
 };
 static thread_local Events t_ev;
 
+// Partitioned path (b): three events per chunk (before the scatter, between the passes, after pass 2),
+// read by run_core after its synchronisation.
+struct PartEvents {
+  std::vector<cudaEvent_t> ev;
+  size_t used = 0;
+  uint32_t* gates = nullptr;  // pinned: per chunk, 1 if a bucket overflowed (fallback ran)
+  uint32_t* gate_slot(size_t chunk) {
+    if (!gates && cudaMallocHost((void**)&gates, 4 * 256) != cudaSuccess) {
+      cudaGetLastError();
+      gates = nullptr;
+    }
+    return gates && chunk < 256 ? gates + chunk : nullptr;
+  }
+  cudaEvent_t next() {
+    if (used == ev.size()) {
+      cudaEvent_t e;
+      cudaEventCreate(&e);
+      ev.push_back(e);
+    }
+    return ev[used++];
+  }
+};
+static thread_local PartEvents t_pev;
+
 static uint64_t* pinned_scratch() {
   static thread_local uint64_t* p = nullptr;
   if (!p) {
@@ -405,6 +429,16 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       tm.aggregate_ms += b;
       tm.compact_ms += c;
       tm.aggregate_launches += launches;
+      for (size_t i = 0; i + 3 <= t_pev.used; i += 3) {
+        float x = 0, y = 0;
+        cudaEventElapsedTime(&x, t_pev.ev[i], t_pev.ev[i + 1]);
+        cudaEventElapsedTime(&y, t_pev.ev[i + 1], t_pev.ev[i + 2]);
+        tm.scatter_ms += x;
+        tm.pass2_ms += y;
+        tm.part_chunks += 1;
+        if (t_pev.gates && i / 3 < 256) tm.part_fallbacks += t_pev.gates[i / 3];
+      }
+      t_pev.used = 0;
     }
     if (flags & FLAG_KEY_RANGE) {
       free_owner();
@@ -517,13 +551,18 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       cudaGetLastError();
     }
     free_b += cache_idle_bytes();  // idle workspace blocks are reusable
-    uint64_t budget_rows = (uint64_t)((double)free_b * 0.6 / (double)row_bytes / 1.03);
+    uint64_t budget_rows = (uint64_t)((double)free_b * 0.6 / (double)row_bytes / 1.1);
     M = std::max<uint64_t>(budget_rows, 1ull << 22);
     P->part_chunk.store(M);
   }
   M = std::min<uint64_t>(n, M);
   if (const char* cr = getenv("BLU_GBY_PART_CHUNK")) M = std::min<uint64_t>(n, std::max<uint64_t>(1024, strtoull(cr, 0, 10)));
-  uint64_t seg_cap = ((uint64_t)((double)((M + B - 1) / B) * 1.03) + 4096 + 63) & ~63ull;
+  // bucket capacity: the mean plus slack for the spread of the number of GROUPS per bucket (keys
+  // hash uniformly: relative sd 1/sqrt(est/B); 6 sd) and of rows per group; heavier skew overflows a
+  // bucket and takes the gated one-pass fallback
+  const double gpb = std::max(1.0, (double)P->est_groups / (double)B);
+  const double slack = 1.03 + std::min(1.0, 6.0 / std::sqrt(gpb));
+  uint64_t seg_cap = ((uint64_t)((double)((M + B - 1) / B) * slack) + 4096 + 63) & ~63ull;
   uint64_t rows_alloc = seg_cap * B;
   void* kbuf = nullptr;
   void* vbuf[kMaxVals] = {};
@@ -533,9 +572,9 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   if (e == cudaSuccess) e = w.alloc(&meta, (size_t)B * 16 + 64);
   if (e != cudaSuccess) return e;
   const double h1 = now();
-  uint64_t* d_cursor = (uint64_t*)meta;
+  uint64_t* d_cursor = (uint64_t*)meta;  // B cursors, gate, tile counter
   uint32_t* d_gate = (uint32_t*)(d_cursor + B);
-  uint32_t scatter_grid = (uint32_t)P->sms * 2;
+  const uint32_t sgrid = scatter_grid((uint32_t)P->sms, B);
   Layout L2 = L;  // pass 2 reads the packed u64 key as a single sparse key column
   L2.n_keys = 1;
   L2.sparse = 1;
@@ -554,6 +593,12 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       vec = vec && ptr_aligned(p1.val[c]);
     }
     p1.vec_ok = vec;
+    if (vec) {  // 256-bit loads when every column is 32-byte aligned
+      bool v32 = true;
+      for (int k = 0; k < L.n_keys; ++k) v32 = v32 && ((uintptr_t)p1.key[k] & 31) == 0;
+      for (int c = 0; c < L.n_vals; ++c) v32 = v32 && ((uintptr_t)p1.val[c] & 31) == 0;
+      if (v32) p1.vec_ok |= 2;
+    }
     p1.prefetch = prefetch_enabled();
     p1.n_rows = m;
     ScatterParams sp{};
@@ -575,12 +620,20 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       for (auto& x : ev) cudaEventCreate(&x);
       cudaEventRecord(ev[0], st);
     }
-    int le = launch_scatter(p1, sp, st, scatter_grid);
+    cudaEvent_t tev[3] = {nullptr, nullptr, nullptr};
+    if (t_timing) {
+      for (auto& x : tev) x = t_pev.next();
+      cudaEventRecord(tev[0], st);
+    }
+    int le = 0;
+    le = launch_scatter(p1, sp, st, sgrid);
     if (le) return (cudaError_t)le;
     if (dbg) cudaEventRecord(ev[1], st);
+    if (t_timing) cudaEventRecord(tev[1], st);
     // pass 2 (runs if no bucket overflowed)
     AggParams p2 = base;
     p2.lay = L2;
+    if (P->part_smem) fill_smem_layout(p2, P->bucket_S, true);
     p2.key[0] = kbuf;
     for (int c = 0; c < L.n_vals; ++c) p2.val[c] = vbuf[c];
     p2.vec_ok = 1;
@@ -592,8 +645,25 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     p2.gate = d_gate;
     p2.gate_run_if = 0;
     p2.front_slots = 0;
-    le = launch_aggregate_impl(P, BLU_PATH_HASH_GLOBAL, p2, RecSrc{nullptr, 0}, false, st, P->grid, P->block, 0);
+    if (P->part_smem) {
+      // bucket-local shared-memory tables: pieces of ~1/div of the mean bucket, whole 4096-row tiles
+      const uint64_t div = getenv("BLU_GBY_PIECE_DIV") ? std::max(1, atoi(getenv("BLU_GBY_PIECE_DIV"))) : 2;
+      const uint64_t mean = (m + B - 1) / B;
+      uint64_t piece = ((mean + div - 1) / div + 4095) / 4096 * 4096;
+      piece = std::min<uint64_t>(std::max<uint64_t>(piece, 4096), 1ull << 30);
+      p2.piece_rows = piece;
+      p2.aux_off = bucket_table_bytes(L2, P->bucket_S);
+      p2.tile_ctr = (uint64_t*)(d_cursor + B + 1);
+      p2.vec_ok = 3;  // segments start at multiples of 64 rows of 8-byte-aligned buffers
+      le = launch_bucket(p2, st, (uint32_t)P->sms, P->bucket_smem);
+    } else {
+      le = launch_aggregate_impl(P, BLU_PATH_HASH_GLOBAL, p2, RecSrc{nullptr, 0}, false, st, P->grid, P->block, 0);
+    }
     if (le) return (cudaError_t)le;
+    if (t_timing) {
+      cudaEventRecord(tev[2], st);
+      if (uint32_t* g = t_pev.gate_slot(t_pev.used / 3 - 1)) cudaMemcpyAsync(g, d_gate, 4, cudaMemcpyDeviceToHost, st);
+    }
     // fallback one-pass over the chunk's rows (runs only if a bucket overflowed)
     AggParams p3 = p1;
     p3.jit_ok = 0;  // gated fallback, normally a no-op: keep the precompiled kernel
@@ -696,8 +766,16 @@ blu_status_t blu_gby_jit_probe(blu_gby_plan_t P, char* log, uint32_t log_cap, in
     sp.B = P->parts;
     if (!rc) rc = launch_scatter(p, sp, nullptr, P->grid);
     AggParams p2 = p;
-    p2.seg_stride = 1;
-    if (!rc) rc = launch_aggregate_impl(P, P->path, p2, RecSrc{nullptr, 0}, false, nullptr, P->grid, P->block, P->smem_bytes);
+    p2.lay.n_keys = 1;
+    p2.lay.sparse = 1;
+    p2.lay.key_dtype[0] = BLU_I64;
+    if (P->part_smem) {
+      fill_smem_layout(p2, P->bucket_S, true);
+      if (!rc) rc = launch_bucket(p2, nullptr, (uint32_t)P->sms, P->bucket_smem);
+    } else {
+      p2.seg_stride = 1;
+      if (!rc) rc = launch_aggregate_impl(P, P->path, p2, RecSrc{nullptr, 0}, false, nullptr, P->grid, P->block, P->smem_bytes);
+    }
   }
   jit_probe_end();
   if (n_programs) *n_programs = pr.programs;

@@ -1086,16 +1086,197 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
 }
 
 // ------------------------------------------------------------------------------------------------
+// Partitioned path (b), pass 2 with bucket-local shared-memory tables. After the scatter, the rows
+// of bucket b hold exactly the groups whose slot lies in slice b of the global table, and no other
+// bucket holds any of them. So a CTA can aggregate a piece of one bucket in an open-addressing table
+// of its own shared memory (the paper's shared-memory kernel, applied per bucket instead
+// of per query) and merge it into the global table once per piece ("merged"): one CAS + one
+// RED per field per GROUP and piece instead of per ROW. Rows whose key finds no room within
+// kBucketProbe slots (a bucket with more groups than the table holds) take the global path.
+// Work items = (bucket, piece) handed out in bucket order by one global counter. p.S = table
+// entries (any multiple of 16), p.lay = the records' layout (packed u64 key, value columns).
+// ------------------------------------------------------------------------------------------------
+constexpr uint32_t kBucketProbe = 32;
+
+// The table is 4-way bucketed: entries [4h, 4h + 4) form bucket h; a key's home bucket comes from the
+// high half of a second hash (independent of the slot bits that chose the partition). One probe step
+// reads the bucket's four keys with two 16-byte loads, so at the table's load (<= 0.7) almost every
+// row resolves in the first step (linear probing by single entries needed ~14 convergent steps per
+// warp tile at load 0.6: the longest of 128 probe sequences).
+__device__ __forceinline__ uint32_t bucket_home(uint64_t key, uint32_t nbk) {
+  return (uint32_t)(((fmix64(key ^ 0x2545F4914F6CDD1Dull) >> 32) * (uint64_t)nbk) >> 32);
+}
+
+__device__ __forceinline__ void lds_v2_volatile(const uint64_t* p, uint64_t& a, uint64_t& b) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(p);
+  asm volatile("ld.volatile.shared.v2.u64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "r"(s));
+}
+
+// Merge entry e of the shared table into the global table, then reset it to the mask.
+__device__ __forceinline__ void bucket_flush_entry(const AggParams& p, uint8_t* sm, uint32_t e) {
+  const Layout& L = p.lay;
+  const uint32_t S = p.S;
+  uint64_t* fk = (uint64_t*)(sm + p.key_off);
+  const uint64_t key = fk[e];
+  if (key == kEmpty) return;
+  uint8_t* tb = (uint8_t*)p.table;
+  const uint64_t idx = fmix64(key) & p.cap_mask;
+  uint64_t s;
+  const bool ok = hash_locate(tb, p.cap_mask, L.slot_bytes, key, __ldcg((const unsigned long long*)(tb + idx * L.slot_bytes)),
+                              idx, p.max_probe, s);
+  if (!ok) atomicOr(p.flags, FLAG_OVERFLOW);
+  for (int j = 0; j < L.n_fields; ++j) {
+    uint8_t* b = sm + p.soff[j];
+    const int kind = L.f[j].kind;
+    if (ok)
+      dispatch_kind(kind, [&](auto kc) {
+        constexpr int K = decltype(kc)::v;
+        g_upd<K, false>(tb + s * L.slot_bytes + L.f[j].goff, s_read<K>(b, e, S));
+      });
+    smem_init_entry(b, kind, e, S);
+  }
+  fk[e] = kEmpty;
+}
+
+template <class SP, int NV, int R>
+__device__ __forceinline__ void bucket_body(const AggParams& p) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  if (p.gate && ((*(volatile const uint32_t*)p.gate != 0) != (p.gate_run_if != 0))) return;
+  const Layout& L = p.lay;
+  const uint32_t S = p.S;
+  const uint32_t nb = p.n_segs;
+  uint32_t* ppre = (uint32_t*)(sm + p.aux_off);  // nb + 1 piece prefix, then 2 scalars
+  volatile uint32_t* s_item = ppre + nb + 1;
+  uint64_t* fk = (uint64_t*)(sm + p.key_off);
+  const uint64_t piece = p.piece_rows;
+  // piece prefix over the buckets (warp 0) and the table mask (all threads)
+  if (threadIdx.x < 32) {
+    uint32_t carry = 0;
+    for (uint32_t b0 = 0; b0 < nb; b0 += 32) {
+      const uint32_t b = b0 + threadIdx.x;
+      const uint32_t x = b < nb ? (uint32_t)((p.seg_count[b] + piece - 1) / piece) : 0u;
+      uint32_t inc = x;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if ((int)threadIdx.x >= o) inc += y;
+      }
+      if (b < nb) ppre[b] = carry + inc - x;
+      carry += __shfl_sync(0xffffffffu, inc, 31);
+    }
+    if (threadIdx.x == 0) ppre[nb] = carry;
+  }
+  for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) fk[e] = kEmpty;
+  for (int j = 0; j < L.n_fields; ++j)
+    for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) smem_init_entry(sm + p.soff[j], L.f[j].kind, e, S);
+  const uint64_t pol = evict_first_policy();
+  const uint64_t tile = (uint64_t)blockDim.x * R;
+  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint8_t* tb = (uint8_t*)p.table;
+  for (;;) {
+    __syncthreads();  // prefix ready / previous piece flushed and the table reset
+    if (threadIdx.x == 0) {
+      s_item[0] = (uint32_t)atomicAdd((unsigned long long*)p.tile_ctr, 1ull);
+      s_item[1] = *(volatile uint32_t*)p.flags;
+    }
+    __syncthreads();
+    const uint32_t item = s_item[0];
+    if (item >= ppre[nb] || (s_item[1] & FLAG_OVERFLOW)) break;
+    uint32_t lo = 0, hi = nb - 1;  // bucket of the item: largest b with ppre[b] <= item
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi + 1) >> 1;
+      if (ppre[mid] <= item) lo = mid; else hi = mid - 1;
+    }
+    const uint64_t seg0 = (uint64_t)lo * p.seg_stride;
+    const uint64_t r0 = seg0 + (uint64_t)(item - ppre[lo]) * piece;
+    const uint64_t cnt = p.seg_count[lo];
+    const uint64_t r1 = seg0 + ((uint64_t)(item - ppre[lo]) * piece + piece < cnt ? (uint64_t)(item - ppre[lo]) * piece + piece : cnt);
+    for (uint64_t row0 = r0; row0 < r1; row0 += tile) {
+      const uint64_t row = lane_base<R>(row0, warp, lane);
+      uint64_t key[R];
+      uint64_t v[NV][R];
+      const uint32_t valid = pack_keys<SP, R>(p, row, r1, pol, key);
+      load_vals<SP, NV, R>(p, row, r1, pol, v);
+      // convergent probe of the shared table: every pending row inspects one 4-entry bucket per step
+      const uint32_t nbk = S >> 2;
+      uint32_t e[R], h[R];
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        h[r] = bucket_home(key[r], nbk);
+        e[r] = 0;
+      }
+      uint32_t pending = valid, hit = 0;
+      for (uint32_t it = 0; it < kBucketProbe; ++it) {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (!(pending >> r & 1)) continue;
+          const uint64_t* q = fk + 4 * h[r];
+          uint64_t k0, k1, k2, k3;
+          lds_v2_volatile(q, k0, k1);
+          lds_v2_volatile(q + 2, k2, k3);
+          const uint64_t kk = key[r];
+          int m = k0 == kk ? 0 : k1 == kk ? 1 : k2 == kk ? 2 : k3 == kk ? 3 : -1;
+          if (m < 0) {
+            const int z = k0 == kEmpty ? 0 : k1 == kEmpty ? 1 : k2 == kEmpty ? 2 : k3 == kEmpty ? 3 : -1;
+            if (z >= 0) {  // claim the first empty entry; on a lost race re-read this bucket next step
+              const unsigned long long old = atomicCAS((unsigned long long*)(q + z), (unsigned long long)kEmpty,
+                                                       (unsigned long long)kk);
+              if (old == kEmpty || old == kk) m = z;
+            } else {
+              h[r] = h[r] + 1 == nbk ? 0u : h[r] + 1;
+            }
+          }
+          if (m >= 0) {
+            e[r] = 4 * h[r] + (uint32_t)m;
+            pending &= ~(1u << r);
+            hit |= 1u << r;
+          }
+        }
+        if (!__any_sync(0xffffffffu, pending)) break;
+      }
+      __syncwarp();
+      smem_apply_rows<SP, NV, R>(p, sm, e, hit, v);
+      if (__any_sync(0xffffffffu, pending)) {  // no room in the shared table: global table (S5b)
+        uint64_t slot[R];
+        uint32_t miss = pending;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          slot[r] = 0;
+          if (!(miss >> r & 1)) continue;
+          const uint64_t idx = fmix64(key[r]) & p.cap_mask;
+          if (!hash_locate(tb, p.cap_mask, L.slot_bytes, key[r], __ldcg((const unsigned long long*)(tb + idx * L.slot_bytes)),
+                           idx, p.max_probe, slot[r])) {
+            miss &= ~(1u << r);
+            atomicOr(p.flags, FLAG_OVERFLOW);
+          }
+        }
+        __syncwarp();
+        global_apply_rows<SP, NV, R, false>(p, slot, miss, v);
+      }
+    }
+    __syncthreads();  // every row of the piece applied
+    for (uint32_t x = threadIdx.x; x < S; x += blockDim.x) bucket_flush_entry(p, sm, x);
+  }
+}
+
+// ------------------------------------------------------------------------------------------------
 // Partitioned path (b), pass 1: radix scatter of rows into B buckets by the top bits of their slot.
 // Per tile: shared-memory counting sort by bucket, one global cursor reservation per (tile,
 // bucket), then coalesced writes of each bucket's contiguous segment (packed u64 key + values).
 // ------------------------------------------------------------------------------------------------
-__device__ __forceinline__ void block_excl_scan_512(uint32_t* a, uint32_t* out, uint32_t B, uint32_t* warp_tot,
-                                                    uint32_t* total) {
-  // exclusive scan of a[0..B) (B <= 2 * blockDim.x, blockDim.x == 512) into out
-  const unsigned t = threadIdx.x, lane = t & 31, w = t >> 5;
-  uint32_t x0 = 2 * t < B ? a[2 * t] : 0, x1 = 2 * t + 1 < B ? a[2 * t + 1] : 0;
-  uint32_t sum = x0 + x1, inc = sum;
+__device__ __forceinline__ void block_excl_scan(uint32_t* a, uint32_t* out, uint32_t B, uint32_t* warp_tot,
+                                                uint32_t* total) {
+  // exclusive scan of a[0..B) into out (B <= 4 * blockDim.x; blockDim.x a multiple of 32, <= 1024):
+  // thread t owns the C consecutive elements [C*t, C*t + C)
+  const unsigned t = threadIdx.x, lane = t & 31, w = t >> 5, nw = blockDim.x >> 5;
+  const uint32_t C = (B + blockDim.x - 1) / blockDim.x;
+  uint32_t x[4], sum = 0;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t k = C * t + i;
+    x[i] = (i < (int)C && k < B) ? a[k] : 0u;
+    sum += x[i];
+  }
+  uint32_t inc = sum;
   for (int o = 1; o < 32; o <<= 1) {
     uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
     if ((int)lane >= o) inc += y;
@@ -1103,18 +1284,22 @@ __device__ __forceinline__ void block_excl_scan_512(uint32_t* a, uint32_t* out, 
   if (lane == 31) warp_tot[w] = inc;
   __syncthreads();
   if (w == 0) {
-    uint32_t v = lane < blockDim.x / 32 ? warp_tot[lane] : 0, vi = v;
+    uint32_t v = lane < nw ? warp_tot[lane] : 0, vi = v;
     for (int o = 1; o < 32; o <<= 1) {
       uint32_t y = __shfl_up_sync(0xffffffffu, vi, o);
       if ((int)lane >= o) vi += y;
     }
-    if (lane < blockDim.x / 32) warp_tot[lane] = vi - v;
+    if (lane < nw) warp_tot[lane] = vi - v;
     if (lane == 31) *total = vi;
   }
   __syncthreads();
   uint32_t excl = warp_tot[w] + inc - sum;
-  if (2 * t < B) out[2 * t] = excl;
-  if (2 * t + 1 < B) out[2 * t + 1] = excl + x0;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const uint32_t k = C * t + i;
+    if (i < (int)C && k < B) out[k] = excl;
+    excl += x[i];
+  }
 }
 
 template <class SP, int NV, int R>
@@ -1153,7 +1338,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
       pos[r] = (valid >> r & 1) ? atomicAdd(&hist[bb[r]], 1u) : 0u;
     }
     __syncthreads();
-    block_excl_scan_512(hist, lstart, B, wtot, total);
+    block_excl_scan(hist, lstart, B, wtot, total);
     for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
       uint32_t h = hist[b];
       if (h) {

@@ -48,6 +48,9 @@ struct blu_gby_plan_s {
   int32_t sms;
   uint32_t parts;         // path b: buckets of the partitioned two-pass mode (1 = one pass)
   uint32_t part_shift;    // log2(cap) - log2(parts)
+  int32_t part_smem;      // partitioned pass 2: 1 = bucket-local shared-memory tables, 0 = L2-resident slices
+  uint32_t bucket_S;      // part_smem: entries of the per-CTA bucket table
+  uint32_t bucket_smem;   // part_smem: dynamic shared memory of the bucket kernel
   mutable std::atomic<uint64_t> part_chunk{0};  // rows per partitioned chunk (decided at first execute)
   mutable std::atomic<uint32_t> retries_last{0};
 };
@@ -68,6 +71,13 @@ int launch_aggregate_impl(const blu_gby_plan_s* P, int path, const AggParams& p,
                           const FinalParams* fin = nullptr);
 uint64_t launches_total();
 int launch_scatter(const AggParams& p, const ScatterParams& s, void* stream, uint32_t grid);
+uint32_t scatter_block(uint32_t B);
+uint32_t scatter_grid(uint32_t sms, uint32_t B);
+size_t scatter_smem(int nv, uint32_t B);
+int launch_bucket(const AggParams& p, void* stream, uint32_t grid, uint32_t smem);
+// bucket table sizing: bytes of an S-entry table (keys + SoA fields) and the kernel's total smem
+uint32_t bucket_table_bytes(const Layout& L, uint32_t S);
+uint32_t bucket_smem_bytes(const Layout& L, uint32_t S, uint32_t B);
 blu_status_t fail(blu_status_t s, const char* fmt, ...);
 int launch_init_slots(const Layout& lay, void* table, uint64_t n_slots, void* stream, uint64_t* zero = nullptr,
                       uint32_t n_zero = 0);

@@ -118,6 +118,11 @@ struct AggParams {
   // front is filled first-come with CAS inserts.
   const uint64_t* front_seed;
   uint32_t prefetch;             // scatter: L2-prefetch the column bytes of the tile this many tiles ahead (0 = off)
+  // partitioned pass 2 with bucket-local shared-memory tables (bucket_body): a bucket's rows are
+  // cut into pieces of piece_rows rows (a multiple of the CTA tile); aux_off = byte offset of the
+  // per-bucket piece prefix (n_segs + 1 u32) behind the S-entry table in dynamic shared memory.
+  uint64_t piece_rows;
+  uint32_t aux_off;
 };
 
 // Path (a) in-kernel compaction (S8 fused into S5a/S7 for small dense domains).

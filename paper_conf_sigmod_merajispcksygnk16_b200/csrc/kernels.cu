@@ -122,11 +122,28 @@ __global__ void __launch_bounds__(512, 2) k_scatter(AggParams p, ScatterParams s
   scatter_body<GenericSpec, NV, R>(p, sp);
 }
 
+// wide fan-out (B > 512): one 1024-thread CTA per SM, a tile twice as long (more rows per bucket
+// per cursor reservation)
+template <int NV, int R>
+__global__ void __launch_bounds__(1024, 1) k_scatter_wide(AggParams p, ScatterParams sp) {
+  scatter_body<GenericSpec, NV, R>(p, sp);
+}
+
+uint32_t scatter_block(uint32_t B) { return B > 512 ? 1024u : 512u; }
+uint32_t scatter_grid(uint32_t sms, uint32_t B) { return B > 512 ? sms : 2 * sms; }  // resident CTAs
+
+size_t scatter_smem(int nv, uint32_t B) {
+  const int R = rows_per_thread(nv);
+  const size_t NV = nv <= 1 ? 1 : nv <= 2 ? 2 : nv <= 4 ? 4 : nv <= 8 ? 8 : 16;
+  const size_t TILE = (size_t)scatter_block(B) * R;
+  return TILE * 8 * (1 + NV) + (size_t)B * 16 + 36 * 4 + 16 + TILE * 2;
+}
+
 template <int NV, int R>
 static int launch_scatter_nv(const AggParams& p, const ScatterParams& sp, cudaStream_t st, uint32_t grid) {
-  const uint32_t TILE = 512 * R;
-  size_t smem = (size_t)TILE * 8 * (1 + NV) + (size_t)sp.B * 16 + 36 * 4 + 16 + (size_t)TILE * 2;
-  if (p.jit_ok) {
+  const uint32_t block = scatter_block(sp.B);
+  const size_t smem = scatter_smem(p.lay.n_vals, sp.B);
+  if (p.jit_ok && jit_env("BLU_GBY_JIT_SCATTER", 1)) {
     char body[160], decl[160], name[64];
     snprintf(name, sizeof name, "blu_jit_scatter_%d_%d", NV, R);
     snprintf(decl, sizeof decl, "%s(blu::AggParams p, blu::ScatterParams sp)", name);
@@ -134,12 +151,12 @@ static int launch_scatter_nv(const AggParams& p, const ScatterParams& sp, cudaSt
     AggParams pc = p;
     ScatterParams sc = sp;
     void* args[] = {&pc, &sc};
-    if (launch_jit(body, decl, p, args, st, grid, 512, (uint32_t)smem, name, 2)) return 0;
+    if (launch_jit(body, decl, p, args, st, grid, block, (uint32_t)smem, name, 2)) return 0;
   }
-  auto k = k_scatter<NV, R>;
+  auto k = block > 512 ? k_scatter_wide<NV, R> : k_scatter<NV, R>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e) return (int)e;
-  k<<<grid, 512, smem, st>>>(p, sp);
+  k<<<grid, block, smem, st>>>(p, sp);
   count_launch(1);
   return (int)cudaGetLastError();
 }
@@ -154,6 +171,43 @@ int launch_scatter(const AggParams& p, const ScatterParams& sp, void* stream, ui
   return launch_scatter_nv<16, 1>(p, sp, st, grid);
 }
 
+// ------------------------------------------------------------------------------------------------
+// Partitioned pass 2 with bucket-local shared-memory tables (bucket_body): one 1024-thread CTA per SM
+// ------------------------------------------------------------------------------------------------
+template <int NV, int R>
+__global__ void __launch_bounds__(1024, 1) k_agg_bucket(AggParams p) {
+  bucket_body<GenericSpec, NV, R>(p);
+}
+
+template <int NV, int R>
+static int launch_bucket_nv(const AggParams& p, cudaStream_t st, uint32_t grid, uint32_t smem) {
+  if (p.jit_ok) {
+    char body[160], decl[160], name[64];
+    snprintf(name, sizeof name, "blu_jit_bucket_%d_%d", NV, R);
+    snprintf(decl, sizeof decl, "%s(blu::AggParams p)", name);
+    snprintf(body, sizeof body, "blu::bucket_body<blu::JitSpec, %d, %d>(p);", NV, R);
+    AggParams pc = p;
+    void* args[] = {&pc};
+    if (launch_jit(body, decl, p, args, st, grid, 1024, smem, name, 1)) return 0;
+  }
+  auto k = k_agg_bucket<NV, R>;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e) return (int)e;
+  if (!p.gate || p.gate_run_if == 0) note_kernel("k_agg_bucket (generic)");
+  k<<<grid, 1024, smem, st>>>(p);
+  count_launch(1);
+  return (int)cudaGetLastError();
+}
+
+int launch_bucket(const AggParams& p, void* stream, uint32_t grid, uint32_t smem) {
+  cudaStream_t st = (cudaStream_t)stream;
+  int nv = p.lay.n_vals;
+  if (nv <= 1) return launch_bucket_nv<1, 4>(p, st, grid, smem);
+  if (nv <= 2) return launch_bucket_nv<2, 4>(p, st, grid, smem);
+  if (nv <= 4) return launch_bucket_nv<4, 4>(p, st, grid, smem);
+  if (nv <= 8) return launch_bucket_nv<8, 2>(p, st, grid, smem);
+  return launch_bucket_nv<16, 1>(p, st, grid, smem);
+}
 
 __device__ __forceinline__ uint64_t hash128(uint64_t w0, uint64_t w1) { return fmix64(w0 ^ fmix64(w1 ^ 0x9E3779B97F4A7C15ull)); }
 

@@ -57,6 +57,9 @@ constexpr uint32_t kFrontBudgetWide = 220 * 1024;  // one CTA per SM
 constexpr uint64_t kDirectMin = 1ull << 20;
 constexpr uint64_t kRowLockRatio = 16;          // kernel 3 when rows/groups <= this
 constexpr uint32_t kPartBudgetMB = 48;          // L2 slice per bucket (126 MB L2)
+constexpr uint32_t kSmemMax = 232448;           // dynamic shared memory per CTA (227 KB opt-in)
+constexpr uint32_t kMaxBuckets = 4096;          // one-pass scatter fan-out
+constexpr double kBucketLoad = 0.7;             // mean groups per bucket / bucket table entries
 
 static int32_t field_gsize(int kind) { return (kind == FK_MINI32 || kind == FK_MAXI32) ? 4 : 8; }
 static int32_t field_ssize(int kind) {
@@ -161,6 +164,16 @@ void build_slot_template(const Layout& L, uint8_t* out) {
       default: memcpy(p, &v64, 8); break;  // COUNT, SUM: 0
     }
   }
+}
+
+uint32_t bucket_table_bytes(const Layout& L, uint32_t S) {
+  uint32_t o = S * 8;
+  for (int j = 0; j < L.n_fields; ++j) o += (S * (uint32_t)L.f[j].ssize + 15) / 16 * 16;
+  return o;
+}
+
+uint32_t bucket_smem_bytes(const Layout& L, uint32_t S, uint32_t B) {
+  return bucket_table_bytes(L, S) + ((B + 1 + 2) * 4 + 15) / 16 * 16;
 }
 
 void fill_smem_layout(AggParams& p, uint32_t S, bool with_keys) {
@@ -380,24 +393,53 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   }
 
   // Partitioned two-pass mode for path (b) when the table exceeds an L2-sized budget: rows are
-  // first scattered into B buckets by the top bits of their slot, then aggregated bucket by bucket
-  // so each bucket's slice of the table stays L2-resident (126 MB L2).
+  // first scattered into B buckets by the top bits of their slot, then aggregated bucket by bucket.
+  // Pass 2 either applies every row to the bucket's L2-resident slice of the global table (default;
+  // 126 MB L2) or builds each bucket's groups in a shared-memory table per CTA
+  // and merges them into the global table once per piece (part_smem, BLU_GBY_PART_SMEM=1).
   P->parts = 1;
   P->part_shift = 0;
+  P->part_smem = 0;
+  P->bucket_S = 0;
+  P->bucket_smem = 0;
   if (path == BLU_PATH_HASH_GLOBAL && L.key_words == 1) {
     uint64_t budget = (uint64_t)kPartBudgetMB << 20;
     if (const char* pm = env("BLU_GBY_PART_MB")) budget = (uint64_t)atoi(pm) << 20;
     uint64_t tbytes = P->cap * (uint64_t)L.slot_bytes;
+    // shared-memory bucket tables are opt-in: measured on C3 (10^9 rows, 10^7 groups) they need
+    // >= 2048 buckets, whose scatter costs 32 ms against 10 ms for the 32-bucket L2 mode
+    bool smem_mode = false;
+    if (const char* ps = env("BLU_GBY_PART_SMEM")) smem_mode = !L.lock_off && ps[0] == '1';
     uint64_t B = 1;
-    while (budget && B < 1024 && tbytes / B > budget && B < P->cap / 1024) B <<= 1;
-    if (const char* pp = env("BLU_GBY_PARTS")) B = std::max(1, atoi(pp));
-    if (B > 1 && !env("BLU_GBY_PARTS")) {
-      // partitioned tables live in L2 one bucket at a time: trade HBM footprint for short probes
-      uint64_t cap2 = std::max<uint64_t>(kMinCap, next_pow2((uint64_t)((double)P->est_groups / kMaxLoadPart + 0.999999)));
-      if (cap2 > P->cap) {
-        P->cap = cap2;
-        tbytes = P->cap * (uint64_t)L.slot_bytes;
-        while (budget && B < 1024 && tbytes / B > budget && B < P->cap / 1024) B <<= 1;
+    const char* forced = env("BLU_GBY_PARTS");
+    if (smem_mode && ((budget && tbytes > budget) || (forced && atoi(forced) > 1))) {
+      // smallest B whose buckets hold <= kBucketLoad * S groups on average, within the scatter's
+      // shared memory and <= kMaxBuckets; the records' layout has the same fields as L
+      auto S_of = [&](uint32_t b) {
+        uint32_t S = 16;
+        while (bucket_smem_bytes(L, S + 16, b) <= kSmemMax) S += 16;
+        return S;
+      };
+      B = 2;
+      while (B < kMaxBuckets && (double)P->est_groups > kBucketLoad * S_of((uint32_t)B) * (double)B &&
+             scatter_smem(L.n_vals, (uint32_t)B * 2) <= kSmemMax && B * 2 <= P->cap / 1024)
+        B <<= 1;
+      if (forced) B = std::max(2, std::min((int)kMaxBuckets, atoi(forced)));
+      while (B > 2 && scatter_smem(L.n_vals, (uint32_t)B) > kSmemMax) B >>= 1;
+      P->part_smem = 1;
+      P->bucket_S = S_of((uint32_t)B);
+      P->bucket_smem = bucket_smem_bytes(L, P->bucket_S, (uint32_t)B);
+    } else {
+      while (budget && B < 1024 && tbytes / B > budget && B < P->cap / 1024) B <<= 1;
+      if (const char* pp = env("BLU_GBY_PARTS")) B = std::max(1, atoi(pp));
+      if (B > 1 && !env("BLU_GBY_PARTS")) {
+        // partitioned tables live in L2 one bucket at a time: trade HBM footprint for short probes
+        uint64_t cap2 = std::max<uint64_t>(kMinCap, next_pow2((uint64_t)((double)P->est_groups / kMaxLoadPart + 0.999999)));
+        if (cap2 > P->cap) {
+          P->cap = cap2;
+          tbytes = P->cap * (uint64_t)L.slot_bytes;
+          while (budget && B < 1024 && tbytes / B > budget && B < P->cap / 1024) B <<= 1;
+        }
       }
     }
     P->parts = (uint32_t)B;
@@ -506,6 +548,8 @@ blu_status_t blu_gby_plan_describe(blu_gby_plan_t P, blu_gby_plan_desc_t* o) {
   o->block = P->block;
   o->retries_last = P->retries_last.load();
   o->row_lock = P->lay.lock_off ? 1 : 0;
+  o->part_smem = P->part_smem;
+  o->bucket_entries = P->bucket_S;
   return BLU_OK;
 }
 

@@ -79,6 +79,7 @@ def test_planner_paths_for_the_five_configs(bg):
     assert c1["capacity"] == 16 and c2["capacity"] == 1024
     # C3: 537 MB at load 0.6 exceeds the L2 budget -> partitioned mode, sized at load <= 0.5
     assert c3["path"] == bg.BLU_PATH_HASH_GLOBAL and c3["capacity"] == 2**25 and c3["slot_bytes"] == 32
+    assert c3["part_smem"] == 0
     assert c3["partitions"] >= 16 and c3["capacity"] * 32 // c3["partitions"] <= 48 * 2**20
     assert c3["hot_front"] == 0
     assert c4["path"] == bg.BLU_PATH_DIRECT_GLOBAL and c4["capacity"] == 100_000 and c4["hot_front"] == 1
@@ -86,18 +87,36 @@ def test_planner_paths_for_the_five_configs(bg):
     assert c1["partitions"] == c2["partitions"] == c4["partitions"] == 1
 
 
+def test_planner_partitioned_smem_mode(bg, monkeypatch):
+    """BLU_GBY_PART_SMEM=1: pass 2 in per-CTA shared-memory bucket tables; buckets hold <= 0.7 x the
+    table's entries on average (C3: 10^7 / 2048 = 4883 of 8000); the global table keeps load <= 0.7;
+    the one-pass scatter fans out to at most 4096 buckets (C5)."""
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
+    c3 = _plan(bg, blugen.workload("C3")).info()
+    assert c3["part_smem"] == 1 and c3["capacity"] == 2**24
+    assert c3["partitions"] == 2048 and c3["bucket_entries"] >= 7900
+    assert 10**7 / c3["partitions"] <= 0.7 * c3["bucket_entries"]
+    c5 = _plan(bg, blugen.workload("C5")).info()
+    assert c5["part_smem"] == 1 and c5["partitions"] == 4096
+
+
 @pytest.mark.parametrize("est,cap", [(1, 1024), (700, 1024), (716, 1024), (717, 2048), (10_000_000, 2**24),
                                      (50_000_000, 2**27)])
 def test_capacity_rounding(bg, monkeypatch, est, cap):
     """cap = next_pow2(ceil(max(est,1)/0.7)), >= 1024 (P:151 "slightly larger", reading A5);
-    one-pass mode (the partitioned mode sizes its L2-resident buckets at load <= 0.5)."""
+    one-pass mode and the shared-memory partitioned mode (the L2-slice partitioned mode sizes its
+    buckets at load <= 0.5)."""
     monkeypatch.setenv("BLU_GBY_PART_MB", "0")
     p = bg.blu_gby_plan([(I64, 0)], [I64], [(SUM, 0)], est, 10**10)
     assert p.info()["capacity"] == cap and p.info()["partitions"] == 1
     monkeypatch.delenv("BLU_GBY_PART_MB")
     p2 = bg.blu_gby_plan([(I64, 0)], [I64], [(SUM, 0)], est, 10**10)
-    if p2.info()["partitions"] > 1:
+    if p2.info()["partitions"] > 1:  # L2-resident slices: load <= 0.5
         assert p2.info()["capacity"] >= 2 * est
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
+    p3 = bg.blu_gby_plan([(I64, 0)], [I64], [(SUM, 0)], est, 10**10)
+    if p3.info()["partitions"] > 1:  # shared-memory bucket tables: the global table keeps load <= 0.7
+        assert p3.info()["part_smem"] == 1 and p3.info()["capacity"] == cap
 
 
 def test_est_clamped_to_rows(bg):
@@ -196,7 +215,8 @@ def test_jit_probe_compiles_plan_kernels(bg, name):
     plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
     st, n, log = bg.blu_gby_jit_probe(plan)
     assert st == bg.BLU_OK, log
-    assert n >= (3 if plan.info()["partitions"] > 1 else 1)
+    info = plan.info()
+    assert n >= (1 if info["partitions"] == 1 else 3)
 
 
 def test_jit_probe_wide_keys_unsupported(bg):

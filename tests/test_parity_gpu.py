@@ -328,22 +328,60 @@ def test_launch_count_and_timing(bg):
         del os.environ["BLU_GBY_NO_FUSE"]
 
 
-@pytest.mark.parametrize("parts,chunk", [("8", None), ("16", "300000"), ("64", "1000003")])
-def test_partitioned_two_pass(bg, oracles, monkeypatch, parts, chunk):
+@pytest.mark.parametrize("smem", ["1", "0"])
+@pytest.mark.parametrize("parts,chunk,div", [("8", None, None), ("16", "300000", None), ("64", "1000003", None),
+                                             ("2", None, None), ("256", None, "7"), ("128", "700001", "64")])
+def test_partitioned_two_pass(bg, oracles, monkeypatch, parts, chunk, div, smem):
     """Path (b) partitioned mode: scatter into buckets by slot bits, then bucket-by-bucket
-    aggregation; several chunks; identical to the oracle."""
+    aggregation — in per-CTA shared-memory bucket tables merged once per piece (smem=1; with 2
+    buckets most groups find no room and take the global path inside the same kernel; div cuts
+    buckets into many pieces, so one bucket is merged from several CTAs) or directly into the
+    bucket's L2-resident table slice (smem=0); several chunks; identical to the oracle."""
     w, o = oracles("C3")
     kc, vc = blugen.device_columns(w)
     monkeypatch.setenv("BLU_GBY_PARTS", parts)
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", smem)
     if chunk:
         monkeypatch.setenv("BLU_GBY_PART_CHUNK", chunk)
+    if div:
+        monkeypatch.setenv("BLU_GBY_PIECE_DIV", div)
     plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    info = plan.info()
+    assert info["partitions"] == int(parts) and info["part_smem"] == int(smem), info
+    bg.blu_gby_set_timing(True)
     res = bg.blu_gby_execute(plan, kc, vc)
+    t = bg.blu_gby_last_timing()
+    bg.blu_gby_set_timing(False)
+    assert t["part_chunks"] >= 1 and t["scatter_ms"] > 0 and t["pass2_ms"] > 0, t
+    assert t["part_fallbacks"] == 0, t  # pass 2 ran (no bucket overflowed)
     gk, ga = gpu_sorted(res, w.schema)
     assert_parity(gk, ga, o, w.schema)
 
 
-def test_partitioned_skew_falls_back(bg, monkeypatch):
+@pytest.mark.parametrize("parts", [None, "4096"])
+def test_partitioned_wide_fanout(bg, monkeypatch, parts):
+    """Shared-memory bucket tables as planned for 2M groups (several hundred buckets, the 1024-thread
+    wide scatter) and with a forced 4096-way scatter, at 20M rows, against the oracle."""
+    w = blugen.workload("C3", n_rows=20_000_003, n_groups=2_000_000)
+    o = oracle.groupby_generated(w)
+    kc, vc = blugen.device_columns(w)
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
+    if parts:
+        monkeypatch.setenv("BLU_GBY_PARTS", parts)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    info = plan.info()
+    assert info["part_smem"] == 1 and info["partitions"] >= 256, info
+    bg.blu_gby_set_timing(True)
+    res = bg.blu_gby_execute(plan, kc, vc)
+    t = bg.blu_gby_last_timing()
+    bg.blu_gby_set_timing(False)
+    assert t["part_chunks"] == 1 and t["part_fallbacks"] == 0, t
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
+@pytest.mark.parametrize("smem", ["1", "0"])
+def test_partitioned_skew_falls_back(bg, monkeypatch, smem):
     """A bucket overflow (every row in one bucket) takes the device-side fallback: still exact."""
     n = 600_000
     rng = np.random.default_rng(3)
@@ -352,17 +390,24 @@ def test_partitioned_skew_falls_back(bg, monkeypatch):
     v = [rng.integers(-(2**40), 2**40, n), rng.integers(-(2**20), 2**20, n) / 64.0]
     o = oracle.groupby_arrays(sch, [k], v)
     monkeypatch.setenv("BLU_GBY_PARTS", "16")
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", smem)
     dk, dv = _mk([k], v)
     plan = bg.plan_for(sch, 5000, n)
+    bg.blu_gby_set_timing(True)
     res = bg.blu_gby_execute(plan, dk, dv)
+    t = bg.blu_gby_last_timing()
+    bg.blu_gby_set_timing(False)
+    assert t["part_fallbacks"] == t["part_chunks"] == 1, t
     gk, ga = gpu_sorted(res, sch)
     assert_parity(gk, ga, o, sch)
 
 
-def test_partitioned_with_regrow(bg, oracles, monkeypatch):
+@pytest.mark.parametrize("smem", ["1", "0"])
+def test_partitioned_with_regrow(bg, oracles, monkeypatch, smem):
     w, o = oracles("C5")
     kc, vc = blugen.device_columns(w)
     monkeypatch.setenv("BLU_GBY_PARTS", "4")
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", smem)
     plan = bg.plan_for(w.schema, 1000, w.n_rows)  # under-estimate: partitioned + regrow
     res = bg.blu_gby_execute(plan, kc, vc)
     gk, ga = gpu_sorted(res, w.schema)
