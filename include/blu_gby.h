@@ -51,7 +51,14 @@ typedef enum {
     BLU_E_CUDA = 5          /* other CUDA runtime error                                         */
 } blu_status_t;
 
-typedef enum { BLU_I32 = 0, BLU_I64 = 1, BLU_F64 = 2 } blu_dtype_t;
+/* Column dtypes. BLU_I128 (value columns only): a 128-bit two's-complement integer stored as 16
+ * bytes per row, low 64-bit word first — the paper's "128bit Integer or Decimal data type" whose
+ * aggregates it applies with atomicCAS (a DECIMAL(31) column is its scaled 128-bit integer).
+ * SUM(i128) wraps mod 2^128 and, like MIN/MAX(i128), returns an i128 column; AVG(i128) returns
+ * f64 = (double)SUM / (double)COUNT, both conversions round-to-nearest-even. Plans with an i128
+ * column use path (b) in one pass (no hot front, no partitioning, no per-plan JIT); the multi-GPU
+ * record helpers (blu_gby_partition, blu_gby_merge_records) return BLU_E_UNSUPPORTED for them. */
+typedef enum { BLU_I32 = 0, BLU_I64 = 1, BLU_F64 = 2, BLU_I128 = 3 } blu_dtype_t;
 
 typedef enum { BLU_COUNT = 0, BLU_SUM = 1, BLU_MIN = 2, BLU_MAX = 3, BLU_AVG = 4 } blu_aggop_t;
 
@@ -77,7 +84,7 @@ typedef struct {
 typedef struct {
     int32_t n_keys;               /* 1..8; composite keys are concatenated (CCAT)           */
     const blu_key_desc_t* keys;
-    int32_t n_vals;               /* 0..16 value (payload) columns, dtype I32, I64 or F64           */
+    int32_t n_vals;               /* 0..16 value (payload) columns, dtype I32, I64, F64 or I128     */
     const blu_dtype_t* vals;
     int32_t n_aggs;               /* 1..16                                                         */
     const blu_agg_desc_t* aggs;

@@ -16,7 +16,7 @@ LIB_PATH = os.path.join(_HERE, "libblugby.so")
 
 # enums (include/blu_gby.h)
 BLU_OK, BLU_E_INVALID, BLU_E_UNSUPPORTED, BLU_E_KEY_RANGE, BLU_E_OOM, BLU_E_CUDA = range(6)
-BLU_I32, BLU_I64, BLU_F64 = 0, 1, 2
+BLU_I32, BLU_I64, BLU_F64, BLU_I128 = 0, 1, 2, 3  # I128: int64 tensors of shape (n, 2) = (lo, hi)
 BLU_COUNT, BLU_SUM, BLU_MIN, BLU_MAX, BLU_AVG = range(5)
 BLU_PATH_DENSE_SMEM, BLU_PATH_HASH_GLOBAL, BLU_PATH_DIRECT_GLOBAL = range(3)
 PATH_NAMES = {0: "a:dense_smem", 1: "b:hash_global", 2: "b':direct_global"}
@@ -224,7 +224,7 @@ def _torch_dtype(dt):
     global _TORCH_DT
     import torch
     if _TORCH_DT is None:
-        _TORCH_DT = {BLU_I32: torch.int32, BLU_I64: torch.int64, BLU_F64: torch.float64}
+        _TORCH_DT = {BLU_I32: torch.int32, BLU_I64: torch.int64, BLU_F64: torch.float64, BLU_I128: torch.int64}
     return _TORCH_DT[dt]
 
 
@@ -253,9 +253,10 @@ class _DevArray:
     """__cuda_array_interface__ provider that keeps the result's owner alive while a tensor views it."""
 
     def __init__(self, owner: _Owner, ptr: int, n: int, dt: int):
-        typestr = {BLU_I32: "<i4", BLU_I64: "<i8", BLU_F64: "<f8"}[dt]
+        typestr = {BLU_I32: "<i4", BLU_I64: "<i8", BLU_F64: "<f8", BLU_I128: "<i8"}[dt]
         self._owner = owner
-        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr if n else 0, False),
+        shape = (n, 2) if dt == BLU_I128 else (n,)
+        self.__cuda_array_interface__ = {"shape": shape, "typestr": typestr, "data": (ptr if n else 0, False),
                                          "version": 3, "strides": None}
 
 
@@ -281,14 +282,16 @@ class Result:
     def _wrap(self, ptr, n, dt, device):
         if self.is_host:
             import numpy as np
-            npdt = {BLU_I32: np.int32, BLU_I64: np.int64, BLU_F64: np.float64}[dt]
+            npdt = {BLU_I32: np.int32, BLU_I64: np.int64, BLU_F64: np.float64, BLU_I128: np.int64}[dt]
+            w = 2 if dt == BLU_I128 else 1
             if n == 0:
-                return np.zeros(0, npdt)
-            buf = (ctypes.c_char * (n * np.dtype(npdt).itemsize)).from_address(ptr)
-            return np.frombuffer(buf, npdt).copy()  # host results are small; copy and free below
+                return np.zeros((0, 2) if w == 2 else 0, npdt)
+            buf = (ctypes.c_char * (n * w * np.dtype(npdt).itemsize)).from_address(ptr)
+            a = np.frombuffer(buf, npdt).copy()  # host results are small; copy and free below
+            return a.reshape(n, 2) if w == 2 else a
         import torch
         if n == 0:
-            return torch.zeros(0, dtype=_torch_dtype(dt), device=device or "cuda")
+            return torch.zeros((0, 2) if dt == BLU_I128 else 0, dtype=_torch_dtype(dt), device=device or "cuda")
         return torch.as_tensor(_DevArray(self._owner, ptr, n, dt), device=device or "cuda")
 
     @property
@@ -310,7 +313,7 @@ def _out_dtypes(plan: Plan, partial: bool) -> List[int]:
         elif op == BLU_AVG:
             out.append(BLU_F64)
         elif op == BLU_SUM:
-            out.append(BLU_F64 if plan.vals[col] == BLU_F64 else BLU_I64)
+            out.append(plan.vals[col] if plan.vals[col] in (BLU_F64, BLU_I128) else BLU_I64)
         else:
             out.append(plan.vals[col])
     return out

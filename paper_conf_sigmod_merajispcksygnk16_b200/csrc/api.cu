@@ -110,7 +110,7 @@ struct Owner {
   std::vector<void*> host;
 };
 
-static size_t dtype_bytes(int dt) { return dt == BLU_I32 ? 4 : 8; }
+static size_t dtype_bytes(int dt) { return dt == BLU_I32 ? 4 : dt == BLU_I128 ? 16 : 8; }
 
 // Workspace cache (per process, per device): the hash table, dense state and partition buffers of
 // an execute come from blocks that are cudaMalloc'd once and reused by later executes — the B200
@@ -211,7 +211,9 @@ static OutSpec make_outspec(const blu_gby_plan_s* P, const Layout& lay, bool par
     o.n_out = lay.n_fields;
     for (int j = 0; j < lay.n_fields; ++j) {
       int k = lay.f[j].kind;
-      o.out_dtype[j] = (k == FK_MINI32 || k == FK_MAXI32) ? BLU_I32 : (k == FK_SUMF || k == FK_MINF64 || k == FK_MAXF64) ? BLU_F64 : BLU_I64;
+      o.out_dtype[j] = (k == FK_MINI32 || k == FK_MAXI32) ? BLU_I32
+                       : (k == FK_SUMF || k == FK_MINF64 || k == FK_MAXF64) ? BLU_F64
+                       : (k == FK_SUMQ || k == FK_MINQ || k == FK_MAXQ) ? BLU_I128 : BLU_I64;
     }
   } else {
     o.n_out = (int)P->amap.size();
@@ -751,7 +753,7 @@ blu_status_t blu_gby_jit_probe(blu_gby_plan_t P, char* log, uint32_t log_cap, in
   if (!P) return fail(BLU_E_INVALID, "NULL plan");
   if (log && log_cap) log[0] = 0;
   if (n_programs) *n_programs = 0;
-  if (!jit_enabled() || P->lay.key_words == 2) return fail(BLU_E_UNSUPPORTED, "no JIT kernels for this plan");
+  if (!jit_enabled() || P->lay.key_words == 2 || P->lay.has_q) return fail(BLU_E_UNSUPPORTED, "no JIT kernels for this plan");
   JitProbe pr;
   jit_probe_begin(&pr);
   AggParams p{};
@@ -940,6 +942,7 @@ blu_status_t blu_gby_merge_partial(blu_gby_plan_t P, const blu_gby_result_t* par
 blu_status_t blu_gby_merge_records(blu_gby_plan_t P, const void* records, uint64_t n, void* stream, int32_t partial_out,
                                    blu_gby_result_t* out) {
   if (!P || !out || (n && !records)) return fail(BLU_E_INVALID, "bad merge_records arguments");
+  if (P->lay.has_q) return fail(BLU_E_UNSUPPORTED, "merge_records: 128-bit payloads have no record format");
   cudaStream_t st = (cudaStream_t)stream;
   const Layout& M = P->merge_lay;
   uint64_t est = std::max<uint64_t>(1, std::min<uint64_t>(n, std::max<uint64_t>(P->est_groups, 1)));
@@ -1012,6 +1015,7 @@ blu_status_t blu_gby_finalize_dense_state(blu_gby_plan_t P, void* const* state_a
 blu_status_t blu_gby_partition(blu_gby_plan_t P, const blu_gby_result_t* partial, int32_t n_parts, void* stream, void* send_buf,
                                uint64_t* send_counts) {
   if (!P || !partial || !send_counts || n_parts < 1 || n_parts > 1024) return fail(BLU_E_INVALID, "bad partition arguments");
+  if (P->lay.has_q) return fail(BLU_E_UNSUPPORTED, "partition: 128-bit payloads have no record format");
   if (!partial->is_partial || partial->is_host) return fail(BLU_E_INVALID, "partition needs a device partial result");
   if (partial->n_groups && !send_buf) return fail(BLU_E_INVALID, "NULL send_buf");
   cudaStream_t st = (cudaStream_t)stream;

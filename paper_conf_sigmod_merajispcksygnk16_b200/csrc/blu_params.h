@@ -10,7 +10,7 @@
 
 // dtype / op numbering of include/blu_gby.h (repeated so this header stands alone under NVRTC)
 #ifndef BLU_GBY_H
-enum { BLU_I32 = 0, BLU_I64 = 1, BLU_F64 = 2 };
+enum { BLU_I32 = 0, BLU_I64 = 1, BLU_F64 = 2, BLU_I128 = 3 };
 #endif
 
 namespace blu {
@@ -33,6 +33,10 @@ enum FieldKind : int32_t {
   FK_MAXI64 = 6,  // MAX over i64 (init INT64_MIN, Table 1)
   FK_MINF64 = 7,  // MIN over f64 through the order-preserving int64 map (init +INT64_MAX)
   FK_MAXF64 = 8,  // MAX over f64 (init INT64_MIN)
+  // 128-bit integer payloads ("128bit Integer or Decimal"): 16-byte fields, low word first
+  FK_SUMQ = 9,    // sum mod 2^128: atomic add of the low word, carry into a RED on the high word
+  FK_MINQ = 10,   // MIN over i128 (init INT128_MAX): 16-byte CAS loop
+  FK_MAXQ = 11,   // MAX over i128 (init INT128_MIN)
 };
 
 // Where the dense state of a field lives in the 4 allreduce groups (blu_gby.h execute_dense_state).
@@ -72,6 +76,7 @@ struct Layout {
   // stride[k] its stride within that word. The slot key is then 16 bytes, claimed with a 16-byte CAS.
   int32_t key_words;
   int32_t kword[kMaxKeys];
+  int32_t has_q;  // 1: some value column is i128 / some field is 128-bit (generic k_agg_q kernel)
 };
 
 // ---------------------------------------------------------------------------------------------

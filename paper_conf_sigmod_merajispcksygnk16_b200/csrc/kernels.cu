@@ -321,6 +321,141 @@ __global__ void __launch_bounds__(256) k_agg_wide(AggParams p, RecSrc rs) {
   }
 }
 // ------------------------------------------------------------------------------------------------
+// 128-bit integer payloads ("the 128bit Integer or Decimal data type" aggregated with
+// atomicCAS). Path (b), one pass, generic kernel. SUM mod 2^128: the low word is added atomically
+// and the carry it produced is added with the high word — addition mod 2^128 is associative and each
+// low-word wrap is seen by exactly one adder, so the high word ends at sum(hi) + #wraps. MIN/MAX: a
+// 16-byte CAS loop (atom.global.cas.b128); a value that looks no better than the field is confirmed
+// with a CAS that writes back what it read, so a torn 16-byte read can never skip an update.
+// ------------------------------------------------------------------------------------------------
+__device__ __forceinline__ bool lt128(uint64_t al, uint64_t ah, uint64_t bl, uint64_t bh) {
+  return (int64_t)ah < (int64_t)bh || (ah == bh && al < bl);
+}
+
+__device__ __forceinline__ void q_add(uint8_t* a, uint64_t lo, uint64_t hi) {
+  const unsigned long long old = atomicAdd((unsigned long long*)a, (unsigned long long)lo);
+  const uint64_t h = hi + (old + lo < old ? 1ull : 0ull);
+  if (h) atomicAdd((unsigned long long*)(a + 8), (unsigned long long)h);
+}
+
+template <bool MIN>
+__device__ __forceinline__ void q_minmax(uint8_t* a, uint64_t lo, uint64_t hi) {
+  unsigned long long* w = (unsigned long long*)a;
+  const ulonglong2 c0 = __ldcg((const ulonglong2*)a);
+  unsigned long long cl = c0.x, ch = c0.y;
+  for (;;) {
+    const bool better = MIN ? lt128(lo, hi, cl, ch) : lt128(cl, ch, lo, hi);
+    unsigned long long ol, oh;
+    if (better) cas128(w, cl, ch, lo, hi, ol, oh);
+    else cas128(w, cl, ch, cl, ch, ol, oh);  // confirm the value compared against
+    if (ol == cl && oh == ch) return;
+    cl = ol;
+    ch = oh;
+  }
+}
+
+__device__ __forceinline__ void ld_q(const void* base, uint64_t row, uint64_t pol, uint64_t& lo, uint64_t& hi) {
+  const uint8_t* q = (const uint8_t*)base + row * 16;
+  if (((uintptr_t)base & 15) == 0) {
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;" : "=l"(lo), "=l"(hi) : "l"(q), "l"(pol));
+  } else {
+    lo = ld_stream_u64(q, pol);
+    hi = ld_stream_u64(q + 8, pol);
+  }
+}
+
+template <int NV>
+__global__ void __launch_bounds__(256) k_agg_q(AggParams p) {
+  constexpr int R = 2;
+  const Layout& L = p.lay;
+  const uint64_t pol = evict_first_policy();
+  const uint64_t n = p.n_rows, tile = (uint64_t)blockDim.x * R;
+  uint8_t* tb = (uint8_t*)p.table;
+  for (uint64_t t = blockIdx.x; t * tile < n; t += gridDim.x) {
+    if (*(volatile uint32_t*)p.flags & FLAG_OVERFLOW) break;
+    const uint64_t row = lane_base<R>(t * tile, threadIdx.x >> 5, threadIdx.x & 31);
+    uint64_t key[R];
+    const uint32_t valid = pack_keys<GenericSpec, R>(p, row, n, pol, key);
+    uint64_t vlo[NV][R], vhi[NV][R];
+#pragma unroll
+    for (int c = 0; c < NV; ++c) {
+#pragma unroll
+      for (int r = 0; r < R; ++r) vlo[c][r] = vhi[c][r] = 0;
+      if (c >= L.n_vals) continue;
+      if (L.val_dtype[c] == BLU_I128) {
+#pragma unroll
+        for (int r = 0; r < R; ++r)
+          if (row_of<R>(row, r) < n) ld_q(p.val[c], row_of<R>(row, r), pol, vlo[c][r], vhi[c][r]);
+      } else {
+        load_rows<R>(p.val[c], L.val_dtype[c], row, n, p.vec_ok, pol, vlo[c]);
+      }
+    }
+    uint64_t slot[R];
+    uint32_t ok = valid;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      slot[r] = 0;
+      if (!(valid >> r & 1)) continue;
+      const uint64_t idx = fmix64(key[r]) & p.cap_mask;
+      if (!hash_locate(tb, p.cap_mask, L.slot_bytes, key[r], __ldcg((const unsigned long long*)(tb + idx * L.slot_bytes)),
+                       idx, p.max_probe, slot[r])) {
+        ok &= ~(1u << r);
+        atomicOr(p.flags, FLAG_OVERFLOW);
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (!(ok >> r & 1)) continue;
+      uint8_t* sl = tb + slot[r] * L.slot_bytes;
+      for (uint32_t m = p.cntmask; m; m &= m - 1) g_upd<FK_COUNT, true>(sl + L.f[__ffs(m) - 1].goff, 1ull);
+#pragma unroll
+      for (int c = 0; c < NV; ++c) {
+        if (c >= L.n_vals) break;
+        for (uint32_t m = p.colmask[c]; m; m &= m - 1) {
+          const Field& f = L.f[__ffs(m) - 1];
+          uint8_t* a = sl + f.goff;
+          if (f.kind == FK_SUMQ) {
+            // a 64-bit column summed into a 128-bit field (merges of COUNT never land here)
+            q_add(a, vlo[c][r], L.val_dtype[c] == BLU_I128 ? vhi[c][r] : (uint64_t)((int64_t)vlo[c][r] >> 63));
+          } else if (f.kind == FK_MINQ) {
+            q_minmax<true>(a, vlo[c][r], vhi[c][r]);
+          } else if (f.kind == FK_MAXQ) {
+            q_minmax<false>(a, vlo[c][r], vhi[c][r]);
+          } else {
+            dispatch_kind(f.kind, [&](auto kc) {
+              constexpr int K = decltype(kc)::v;
+              g_upd<K, true>(a, vlo[c][r]);
+            });
+          }
+        }
+      }
+    }
+  }
+}
+
+// Correctly rounded (round-to-nearest-even) conversion of a two's-complement 128-bit integer to f64:
+// the top 64 significant bits are converted with the sticky OR of the rest folded into bit 0 (below
+// the 11 bits __ull2double_rn drops), then scaled by an exact power of two.
+__device__ __forceinline__ double i128_to_f64(uint64_t lo, uint64_t hi) {
+  const bool neg = (int64_t)hi < 0;
+  if (neg) {
+    lo = ~lo + 1ull;
+    hi = ~hi + (lo == 0 ? 1ull : 0ull);
+  }
+  double r;
+  if (hi == 0) {
+    r = __ull2double_rn(lo);
+  } else {
+    const int z = __clzll((long long)hi);  // 0..63
+    const uint64_t top = z ? (hi << z) | (lo >> (64 - z)) : hi;
+    const uint64_t rest = z ? lo << z : lo;
+    r = __ull2double_rn(top | (rest != 0 ? 1ull : 0ull));
+    r *= __longlong_as_double((long long)(1023 + 64 - z) << 52);  // 2^(64 - z), exact
+  }
+  return neg ? -r : r;
+}
+
+// ------------------------------------------------------------------------------------------------
 // S8: compaction (path (c))
 // ------------------------------------------------------------------------------------------------
 constexpr int kCT = 256;        // threads
@@ -348,6 +483,17 @@ __device__ __forceinline__ uint64_t read_field(const CompactParams& p, int j, ui
 __device__ __forceinline__ void store_as(void* out, uint64_t pos, int dtype, uint64_t bits) {
   if (dtype == BLU_I32) ((int32_t*)out)[pos] = (int32_t)(uint32_t)bits;
   else ((uint64_t*)out)[pos] = bits;
+}
+
+// high word of a 16-byte field (hash table only)
+__device__ __forceinline__ uint64_t read_field_hi(const CompactParams& p, int j, uint64_t e) {
+  const uint8_t* a = (const uint8_t*)p.table + e * p.lay.slot_bytes + p.lay.f[j].goff + 8;
+  return __ldg((const unsigned long long*)a);
+}
+
+__device__ __forceinline__ void store_q(void* out, uint64_t pos, uint64_t lo, uint64_t hi) {
+  ((uint64_t*)out)[2 * pos] = lo;
+  ((uint64_t*)out)[2 * pos + 1] = hi;
 }
 
 __global__ void __launch_bounds__(kCT) k_compact_count(CompactParams p) {
@@ -441,6 +587,10 @@ __global__ void __launch_bounds__(kCT) k_compact_emit(CompactParams p) {
         for (int j = 0; j < L.n_fields; ++j) {
           uint64_t x = read_field(p, j, e);
           int k = L.f[j].kind;
+          if (L.f[j].gsize == 16) {
+            store_q(p.out_vals[j], pos, x, read_field_hi(p, j, e));
+            continue;
+          }
           if (k == FK_MINF64 || k == FK_MAXF64) x = unord_f64((int64_t)x);
           int dt = (k == FK_MINI32 || k == FK_MAXI32) ? BLU_I32 : BLU_I64;
           store_as(p.out_vals[j], pos, dt, x);
@@ -452,9 +602,13 @@ __global__ void __launch_bounds__(kCT) k_compact_emit(CompactParams p) {
           int k = L.f[j].kind;
           if (p.out_kind[o] == 1) {  // AVG = (double)SUM / (double)COUNT (reading A12)
             uint64_t cnt = read_field(p, p.out_field2[o], e);
-            double s = k == FK_SUMF ? __longlong_as_double((long long)x) : (double)(long long)x;
+            double s = k == FK_SUMF ? __longlong_as_double((long long)x)
+                       : k == FK_SUMQ ? i128_to_f64(x, read_field_hi(p, j, e)) : (double)(long long)x;
             double a = s / (double)(long long)cnt;
             x = (uint64_t)__double_as_longlong(a);
+          } else if (L.f[j].gsize == 16) {
+            store_q(p.out_vals[o], pos, x, read_field_hi(p, j, e));
+            continue;
           } else if (k == FK_MINF64 || k == FK_MAXF64) {
             x = unord_f64((int64_t)x);
           }
@@ -797,6 +951,13 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
                          void* stream, uint32_t grid, uint32_t block, uint32_t smem, const FinalParams* fin) {
   cudaStream_t st = (cudaStream_t)stream;
   cudaError_t e = cudaSuccess;
+  if (p.lay.has_q) {  // 128-bit payloads: path (b), columns, generic kernel
+    if (records || path != BLU_PATH_HASH_GLOBAL || p.lay.key_words == 2) return (int)cudaErrorInvalidValue;
+    note_kernel("k_agg_q (generic)");
+    k_agg_q<NV><<<grid, 256, 0, st>>>(p);
+    count_launch(1);
+    return (int)cudaGetLastError();
+  }
   if (!records && p.jit_ok && p.lay.key_words != 2) {
     const int nv = p.lay.n_vals < 1 ? 1 : p.lay.n_vals;
     int r = rows_per_thread(p.lay.n_vals);

@@ -61,15 +61,18 @@ constexpr uint32_t kSmemMax = 232448;           // dynamic shared memory per CTA
 constexpr uint32_t kMaxBuckets = 4096;          // one-pass scatter fan-out
 constexpr double kBucketLoad = 0.7;             // mean groups per bucket / bucket table entries
 
-static int32_t field_gsize(int kind) { return (kind == FK_MINI32 || kind == FK_MAXI32) ? 4 : 8; }
+static bool field_q(int kind) { return kind == FK_SUMQ || kind == FK_MINQ || kind == FK_MAXQ; }
+static int32_t field_gsize(int kind) {
+  return field_q(kind) ? 16 : (kind == FK_MINI32 || kind == FK_MAXI32) ? 4 : 8;
+}
 static int32_t field_ssize(int kind) {
-  return (kind == FK_COUNT || kind == FK_MINI32 || kind == FK_MAXI32) ? 4 : 8;
+  return field_q(kind) ? 16 : (kind == FK_COUNT || kind == FK_MINI32 || kind == FK_MAXI32) ? 4 : 8;
 }
 static int32_t field_group(int kind) {
   switch (kind) {
-    case FK_COUNT: case FK_SUMI: return SG_ISUM;
+    case FK_COUNT: case FK_SUMI: case FK_SUMQ: return SG_ISUM;
     case FK_SUMF: return SG_FSUM;
-    case FK_MINI32: case FK_MINI64: case FK_MINF64: return SG_MIN;
+    case FK_MINI32: case FK_MINI64: case FK_MINF64: case FK_MINQ: return SG_MIN;
     default: return SG_MAX;
   }
 }
@@ -95,6 +98,9 @@ static void finish_layout(Layout& L) {
     f.sidx = gcount[f.sgroup]++;
   }
   for (int g = 0; g < 4; ++g) L.n_group[g] = gcount[g];
+  L.has_q = 0;
+  for (int j = 0; j < L.n_fields; ++j) L.has_q |= field_q(L.f[j].kind) ? 1 : 0;
+  for (int c = 0; c < L.n_vals; ++c) L.has_q |= L.val_dtype[c] == BLU_I128 ? 1 : 0;
   uint32_t raw = (off + 7) / 8 * 8;
   uint32_t sb = 16;
   while (sb < raw && sb < 128) sb <<= 1;
@@ -161,6 +167,17 @@ void build_slot_template(const Layout& L, uint8_t* out) {
       case FK_MAXI32: v32 = INT32_MIN; memcpy(p, &v32, 4); break;
       case FK_MINI64: case FK_MINF64: v64 = INT64_MAX; memcpy(p, &v64, 8); break;
       case FK_MAXI64: case FK_MAXF64: v64 = INT64_MIN; memcpy(p, &v64, 8); break;
+      case FK_MINQ: {  // INT128_MAX: low word all ones, high word INT64_MAX
+        const uint64_t w[2] = {~0ull, (uint64_t)INT64_MAX};
+        memcpy(p, w, 16);
+        break;
+      }
+      case FK_MAXQ: {  // INT128_MIN
+        const uint64_t w[2] = {0ull, (uint64_t)INT64_MIN};
+        memcpy(p, w, 16);
+        break;
+      }
+      case FK_SUMQ: memset(p, 0, 16); break;
       default: memcpy(p, &v64, 8); break;  // COUNT, SUM: 0
     }
   }
@@ -233,7 +250,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     if (s->keys[k].dtype != BLU_I32 && s->keys[k].dtype != BLU_I64)
       return fail(BLU_E_INVALID, "key %d: dtype must be BLU_I32 or BLU_I64", k);
   for (int c = 0; c < s->n_vals; ++c)
-    if (s->vals[c] != BLU_I32 && s->vals[c] != BLU_I64 && s->vals[c] != BLU_F64)
+    if (s->vals[c] != BLU_I32 && s->vals[c] != BLU_I64 && s->vals[c] != BLU_F64 && s->vals[c] != BLU_I128)
       return fail(BLU_E_INVALID, "value %d: bad dtype %d", c, (int)s->vals[c]);
   for (int a = 0; a < s->n_aggs; ++a) {
     int op = s->aggs[a].op;
@@ -291,6 +308,11 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     }
   }
 
+  {
+    bool q = false;
+    for (int c = 0; c < s->n_vals; ++c) q = q || s->vals[c] == BLU_I128;
+    if (q && wide) return fail(BLU_E_UNSUPPORTED, "128-bit payloads with a key tuple wider than 64 bits");
+  }
   auto* P = new blu_gby_plan_s();
   P->keys.assign(s->keys, s->keys + s->n_keys);
   P->vals.assign(s->vals, s->vals + s->n_vals);
@@ -333,14 +355,16 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
       m.field = add_field(L, FK_COUNT, -1, 1);
       m.out_dtype = BLU_I64;
     } else if (op == BLU_SUM || op == BLU_AVG) {
-      m.field = add_field(L, dt == BLU_F64 ? FK_SUMF : FK_SUMI, col, 0);
+      m.field = add_field(L, dt == BLU_F64 ? FK_SUMF : dt == BLU_I128 ? FK_SUMQ : FK_SUMI, col, 0);
       if (op == BLU_AVG) m.field2 = add_field(L, FK_COUNT, -1, 1);
-      m.out_dtype = op == BLU_AVG ? BLU_F64 : (dt == BLU_F64 ? BLU_F64 : BLU_I64);
+      m.out_dtype = op == BLU_AVG ? BLU_F64 : (dt == BLU_F64 || dt == BLU_I128 ? dt : BLU_I64);
     } else if (op == BLU_MIN) {
-      m.field = add_field(L, dt == BLU_I32 ? FK_MINI32 : dt == BLU_I64 ? FK_MINI64 : FK_MINF64, col, 0);
+      m.field = add_field(L, dt == BLU_I32 ? FK_MINI32 : dt == BLU_I64 ? FK_MINI64 : dt == BLU_I128 ? FK_MINQ : FK_MINF64,
+                          col, 0);
       m.out_dtype = dt;
     } else {
-      m.field = add_field(L, dt == BLU_I32 ? FK_MAXI32 : dt == BLU_I64 ? FK_MAXI64 : FK_MAXF64, col, 0);
+      m.field = add_field(L, dt == BLU_I32 ? FK_MAXI32 : dt == BLU_I64 ? FK_MAXI64 : dt == BLU_I128 ? FK_MAXQ : FK_MAXF64,
+                          col, 0);
       m.out_dtype = dt;
     }
   }
@@ -367,6 +391,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     path = want;
   }
   if (L.key_words == 2) path = BLU_PATH_HASH_GLOBAL;  // wide keys: 16-byte key CAS, hash path only
+  if (L.has_q) path = BLU_PATH_HASH_GLOBAL;            // 128-bit payloads: 16-byte global fields only
   P->path = path;
   if (path != BLU_PATH_HASH_GLOBAL && L.count_field < 0) {  // dense occupancy = COUNT > 0
     add_field(L, FK_COUNT, -1, 1);
@@ -385,7 +410,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     const bool rule = path == BLU_PATH_HASH_GLOBAL && L.n_fields > 5 && n_rows <= kRowLockRatio * P->est_groups;
     bool lock = false;
     if (const char* rl = env("BLU_GBY_ROW_LOCK"))
-      lock = path == BLU_PATH_HASH_GLOBAL && (rl[0] == '1' || (rl[0] == 'r' && rule));
+      lock = path == BLU_PATH_HASH_GLOBAL && !L.has_q && (rl[0] == '1' || (rl[0] == 'r' && rule));
     if (lock) {
       L.lock_off = 1;  // placeholder: finish_layout assigns the real offset
       finish_layout(L);
@@ -402,7 +427,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   P->part_smem = 0;
   P->bucket_S = 0;
   P->bucket_smem = 0;
-  if (path == BLU_PATH_HASH_GLOBAL && L.key_words == 1) {
+  if (path == BLU_PATH_HASH_GLOBAL && L.key_words == 1 && !L.has_q) {
     uint64_t budget = (uint64_t)kPartBudgetMB << 20;
     if (const char* pm = env("BLU_GBY_PART_MB")) budget = (uint64_t)atoi(pm) << 20;
     uint64_t tbytes = P->cap * (uint64_t)L.slot_bytes;
@@ -452,7 +477,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   // hot-key front (path b / b')
   P->hot_front = 0;
   P->front_slots = 0;
-  if (path != BLU_PATH_DENSE_SMEM && L.key_words == 1) {
+  if (path != BLU_PATH_DENSE_SMEM && L.key_words == 1 && !L.has_q) {
     bool on = n_rows >= kFrontRatio * P->est_groups;
     if (const char* hf = env("BLU_GBY_HOT_FRONT")) on = hf[0] == '1';
     if (on) {
@@ -511,7 +536,8 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   for (int j = 0; j < L.n_fields; ++j) {
     int k = L.f[j].kind;
     M.val_dtype[j] = (k == FK_MINI32 || k == FK_MAXI32) ? BLU_I32
-                     : (k == FK_SUMF || k == FK_MINF64 || k == FK_MAXF64) ? BLU_F64 : BLU_I64;
+                     : (k == FK_SUMF || k == FK_MINF64 || k == FK_MAXF64) ? BLU_F64
+                     : field_q(k) ? BLU_I128 : BLU_I64;
     M.f[j].col = j;
     if (k == FK_COUNT) M.f[j].kind = FK_SUMI;  // is_count stays 1
   }

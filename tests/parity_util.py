@@ -3,14 +3,18 @@ import numpy as np
 
 import blugen
 import oracle
-from blugen import AVG, F64, MAX, MIN, SUM
+from blugen import AVG, F64, I128, MAX, MIN, SUM
+
+
+def _empty_aggs(schema):
+    return [np.zeros((0, 2) if schema.agg_out_dtype(a) == I128 else 0) for a in range(len(schema.aggs))]
 
 
 def gpu_sorted(res, schema):
     """(keys (G,K) int64 lexsorted, [agg arrays in the same order]) from a finalized Result."""
     K = len(schema.keys)
     if res.n_groups == 0:
-        return np.zeros((0, K), np.int64), [np.zeros(0) for _ in schema.aggs]
+        return np.zeros((0, K), np.int64), _empty_aggs(schema)
     keys = np.stack([k.cpu().numpy().astype(np.int64) for k in res.keys], axis=1)
     order = np.lexsort(keys.T[::-1])
     aggs = [a.cpu().numpy()[order] for a in res.aggs]
@@ -20,7 +24,7 @@ def gpu_sorted(res, schema):
 def host_sorted(res, schema):
     K = len(schema.keys)
     if res.n_groups == 0:
-        return np.zeros((0, K), np.int64), [np.zeros(0) for _ in schema.aggs]
+        return np.zeros((0, K), np.int64), _empty_aggs(schema)
     keys = np.stack([k.astype(np.int64) for k in res.keys], axis=1)
     order = np.lexsort(keys.T[::-1])
     return keys[order], [a[order] for a in res.aggs]

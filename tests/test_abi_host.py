@@ -223,3 +223,25 @@ def test_jit_probe_wide_keys_unsupported(bg):
     plan = bg.blu_gby_plan([(I64, 0), (I64, 0)], [I64], [(SUM, 0)], 100, 1000)
     st, n, _ = bg.blu_gby_jit_probe(plan)
     assert st == bg.BLU_E_UNSUPPORTED and n == 0
+
+
+def test_i128_plan_and_mask(bg):
+    """128-bit payloads: path (b) in one pass (no front, no partitions, no kernel 3); the
+    states are 16-byte fields at 16-byte offsets whose mask values are SUM 0, MIN INT128_MAX,
+    MAX INT128_MIN (the Table 1 rule for a 128-bit type: "for MAX ... the minimum value")."""
+    I128 = blugen.I128
+    p = bg.blu_gby_plan([(I64, 0)], [I128, I64], [(COUNT, -1), (SUM, 0), (MIN, 0), (MAX, 0), (AVG, 0)], 10**7, 10**9)
+    info = p.info()
+    assert info["path"] == bg.BLU_PATH_HASH_GLOBAL and info["partitions"] == 1 and info["hot_front"] == 0
+    assert sorted(info["state_dtypes"]) == [I64, I128, I128, I128]  # COUNT, SUM, MIN, MAX
+    t = p.slot_template()
+    assert struct.unpack_from("<q", t, 0)[0] == -1  # EMPTY key
+    words = [struct.unpack_from("<QQ", t, o) for o in range(16, len(t) - 15, 16)]
+    assert (0, 0) in words
+    assert ((1 << 64) - 1, (1 << 63) - 1) in words   # INT128_MAX (MIN's identity)
+    assert (0, 1 << 63) in words                     # INT128_MIN (MAX's identity)
+    st, n, _ = bg.blu_gby_jit_probe(p)
+    assert st == bg.BLU_E_UNSUPPORTED and n == 0     # generic k_agg_q only
+    with pytest.raises(bg.BluError) as e:            # 128-bit payloads with two-word keys
+        bg.blu_gby_plan([(I64, 0), (I64, 0)], [I128], [(SUM, 0)], 100, 1000)
+    assert e.value.status == bg.BLU_E_UNSUPPORTED

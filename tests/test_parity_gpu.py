@@ -575,3 +575,90 @@ def test_wide_keys_host_columns(bg):
     res = bg.blu_gby_execute_host(plan, kc, vc)
     gk, ga = host_sorted(res, sch)
     assert_parity(gk, ga, o, sch)
+
+
+# ---- 128-bit integer payloads (NEXT-2; "128bit Integer or Decimal"; reading A18) ------
+I128 = blugen.I128
+
+
+def _i128(rng, n, kind):
+    """(n, 2) int64 = (lo, hi) words of 128-bit values: the full range, the int64 range (sign
+    extended) or values near +-2^126 so that group sums wrap mod 2^128."""
+    lo = rng.integers(-(2**63), 2**63, n, dtype=np.int64)
+    if kind == "full":
+        hi = rng.integers(-(2**63), 2**63, n, dtype=np.int64)
+    elif kind == "small":
+        hi = lo >> 63
+    else:
+        hi = rng.choice(np.array([2**62, 2**62 - 1, -(2**62), -(2**62) - 1], np.int64), n)
+    return np.ascontiguousarray(np.stack([lo, hi], axis=1))
+
+
+def _i128_case(rng, n, kind):
+    G = max(1, n // 40)
+    codes = rng.integers(0, 2**62, G, dtype=np.int64)
+    k = codes[rng.integers(0, G, n)] if n else np.zeros(0, np.int64)
+    v64 = rng.integers(-(2**62), 2**62, n, dtype=np.int64)
+    sch = blugen.Schema([(I64, 0)], [I128, I64],
+                        [(COUNT, -1), (SUM, 0), (MIN, 0), (MAX, 0), (AVG, 0), (SUM, 1), (MAX, 1)])
+    return sch, [k], [_i128(rng, n, kind), v64], G
+
+
+@pytest.mark.parametrize("kind", ["full", "small", "wrap"])
+@pytest.mark.parametrize("n", [0, 1, 33, 4097, 300_001])
+def test_i128_payload_parity(bg, n, kind):
+    """SUM mod 2^128, MIN/MAX (signed), AVG = RN(RN(sum)/count) of a 128-bit column beside an int64
+    column, bit-exact against the oracle's __int128 arithmetic (path (b), one pass, k_agg_q)."""
+    rng = np.random.default_rng(1000 + n)
+    sch, kc, vc, G = _i128_case(rng, n, kind)
+    o = oracle.groupby_arrays(sch, kc, vc)
+    plan = bg.plan_for(sch, G, max(n, 1))
+    info = plan.info()
+    assert info["path"] == bg.BLU_PATH_HASH_GLOBAL and info["partitions"] == 1 and info["hot_front"] == 0
+    dk, dv = _mk(kc, vc)
+    bg.blu_gby_set_timing(True)
+    res = bg.blu_gby_execute(plan, dk, dv, n_rows=n)
+    t = bg.blu_gby_last_timing()
+    bg.blu_gby_set_timing(False)
+    if n:
+        assert t["kernel"].startswith("k_agg_q"), t["kernel"]
+    gk, ga = gpu_sorted(res, sch)
+    if n:
+        assert ga[1].shape == (res.n_groups, 2)
+    assert_parity(gk, ga, o, sch)
+
+
+def test_i128_regrow_partial_merge_and_host(bg):
+    """Under-estimated groups (regrow), 3 partial shards merged on the device (128-bit states),
+    and host columns through blu_gby_execute_host — all equal to the oracle."""
+    rng = np.random.default_rng(77)
+    n = 200_003
+    sch, kc, vc, G = _i128_case(rng, n, "full")
+    o = oracle.groupby_arrays(sch, kc, vc)
+    dk, dv = _mk(kc, vc)
+    plan = bg.plan_for(sch, 1, n)
+    gk, ga = gpu_sorted(bg.blu_gby_execute(plan, dk, dv), sch)
+    assert_parity(gk, ga, o, sch)
+    assert plan.info()["retries_last"] >= 1
+    plan = bg.plan_for(sch, G, n)
+    cuts = [0, 70_001, 140_000, n]
+    parts = [bg.blu_gby_execute_partial(plan, [k[a:b] for k in dk], [v[a:b] for v in dv], n_rows=b - a)
+             for a, b in zip(cuts[:-1], cuts[1:])]
+    assert parts[0].states[1].shape[1] == 2  # the 128-bit SUM state travels as (lo, hi)
+    gk, ga = gpu_sorted(bg.blu_gby_merge(plan, parts), sch)
+    assert_parity(gk, ga, o, sch)
+    hk, ha = host_sorted(bg.blu_gby_execute_host(plan, [torch.from_numpy(k) for k in kc],
+                                                 [torch.from_numpy(v) for v in vc]), sch)
+    assert_parity(hk, ha, o, sch)
+
+
+def test_i128_record_helpers_unsupported(bg):
+    rng = np.random.default_rng(5)
+    sch, kc, vc, G = _i128_case(rng, 1000, "small")
+    plan = bg.plan_for(sch, G, 1000)
+    dk, dv = _mk(kc, vc)
+    part = bg.blu_gby_execute_partial(plan, dk, dv)
+    buf = torch.empty(1 << 20, dtype=torch.uint8, device="cuda")
+    with pytest.raises(bg.BluError) as e:
+        bg.blu_gby_partition(plan, part, 2, buf)
+    assert e.value.status == bg.BLU_E_UNSUPPORTED
