@@ -24,8 +24,8 @@ $(PKG)/libblugby.so: $(BLUGBY_SRCS) $(BLUGBY_HDRS)
 blugen/libblugen.so: blugen/csrc/gen.cu include/blu_gen.h
 	$(NVCC) $(NVFLAGS) -shared -o $@ blugen/csrc/gen.cu
 
-oracle/liboracle.so: oracle/blu_oracle.cpp include/blu_gen.h
-	$(CXX) -O2 -std=c++17 -fPIC -shared -Wall -Iinclude -o $@ oracle/blu_oracle.cpp
+oracle/liboracle.so: oracle/blu_oracle.cpp oracle/sort_oracle.cpp include/blu_gen.h
+	$(CXX) -O2 -std=c++17 -fPIC -shared -Wall -Iinclude -o $@ oracle/blu_oracle.cpp oracle/sort_oracle.cpp
 
 clean:
 	rm -f $(PKG)/libblugby.so blugen/libblugen.so oracle/liboracle.so

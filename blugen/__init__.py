@@ -293,3 +293,25 @@ def host_specs(w: Workload):
         vs[i], k = host_spec(c, w.seed)
         keep.append(k)
     return ks, vs, keep
+
+
+# ---- sort offload workload (§3) ---------------------------------
+SORT_SEED = 0x5EED0050
+
+
+def sort_rows(n: int, W: int = 16, seed: int = SORT_SEED, cards=(1823, 502)) -> np.ndarray:
+    """(n, W) uint8 binary-sortable keys (W a multiple of 4) shaped like an ORDER BY over TPC-DS
+    store_sales: 4-byte word 0 a sold-date code (1823 distinct), word 1 a store code (502
+    distinct), the remaining words uniform random bytes (item / ticket). Each word is stored most
+    significant byte first, so lexicographic byte order is numeric order per word. Seeded numpy
+    generator; no sort arithmetic here."""
+    assert W % 4 == 0 and W >= 4
+    rng = np.random.default_rng(seed)
+    words = []
+    for w in range(W // 4):
+        if w < len(cards) and cards[w]:
+            words.append(rng.integers(0, cards[w], n, dtype=np.uint32))
+        else:
+            words.append(rng.integers(0, 2**32, n, dtype=np.uint32))
+    be = np.stack(words, axis=1).astype(">u4")
+    return np.ascontiguousarray(be.view(np.uint8).reshape(n, W))

@@ -56,6 +56,15 @@ def lib():
         L.oracle_fetch.restype = None
         L.oracle_free.argtypes = [vp]
         L.oracle_free.restype = None
+        u64 = ctypes.c_uint64
+        L.oracle_partial_keys.argtypes = [vp, u64, ctypes.c_uint32, ctypes.c_uint32, vp]
+        L.oracle_partial_keys.restype = None
+        L.oracle_sort_pairs.argtypes = [vp, vp, u64, vp, vp]
+        L.oracle_sort_pairs.restype = None
+        L.oracle_dup_ranges.argtypes = [vp, u64, vp, vp]
+        L.oracle_dup_ranges.restype = u64
+        L.oracle_sort_rows.argtypes = [vp, u64, ctypes.c_uint32, vp]
+        L.oracle_sort_rows.restype = None
         _lib = L
     return _lib
 
@@ -143,3 +152,40 @@ def concat(results: Sequence[OracleResult]) -> OracleResult:
         else:
             sumabs.append(np.concatenate([r.sumabs[a] for r in results])[order])
     return OracleResult(keys[order], np.concatenate([r.count for r in results])[order], aggs, sumabs)
+
+
+# ---- sort offload (§3; oracle/sort_oracle.cpp) -----------------------------------
+def partial_keys(rows: np.ndarray, word: int) -> np.ndarray:
+    """4-byte binary-sortable partial keys of word `word` of (n, W) uint8 rows."""
+    rows = np.ascontiguousarray(rows, np.uint8)
+    n, W = rows.shape
+    out = np.zeros(n, np.uint32)
+    lib().oracle_partial_keys(rows.ctypes.data, n, W, word, out.ctypes.data)
+    return out
+
+
+def sort_pairs(keys: np.ndarray, payload: np.ndarray):
+    """Stable sort of the partial key buffer by its 4-byte key."""
+    k = np.ascontiguousarray(keys, np.uint32)
+    p = np.ascontiguousarray(payload, np.uint32)
+    ko, po = np.zeros_like(k), np.zeros_like(p)
+    lib().oracle_sort_pairs(k.ctypes.data, p.ctypes.data, len(k), ko.ctypes.data, po.ctypes.data)
+    return ko, po
+
+
+def dup_ranges(sorted_keys: np.ndarray):
+    """(starts, lens) of the duplicate ranges of a sorted buffer."""
+    k = np.ascontiguousarray(sorted_keys, np.uint32)
+    m = max(1, len(k) // 2)
+    st, ln = np.zeros(m, np.uint64), np.zeros(m, np.uint64)
+    r = lib().oracle_dup_ranges(k.ctypes.data, len(k), st.ctypes.data, ln.ctypes.data)
+    return st[:r].astype(np.int64), ln[:r].astype(np.int64)
+
+
+def sort_rows(rows: np.ndarray) -> np.ndarray:
+    """The completed sort: stable lexicographic order of (n, W) uint8 rows, as row indices."""
+    rows = np.ascontiguousarray(rows, np.uint8)
+    n, W = rows.shape
+    out = np.zeros(n, np.uint32)
+    lib().oracle_sort_rows(rows.ctypes.data, n, W, out.ctypes.data)
+    return out

@@ -364,3 +364,98 @@ def test_i128_in_int64_range_equals_i64_column():
     for j in range(3):
         assert np.array_equal(b.aggs[j][:, 0], a.aggs[j]) and np.array_equal(b.aggs[j][:, 1], a.aggs[j] >> 63)
     assert np.array_equal(b.aggs[3], a.aggs[3])
+
+
+# ---- sort offload oracle (§3; oracle/sort_oracle.cpp) -----------------------------
+def _rows(rng, n, W, alphabet=4):
+    """Small-alphabet byte rows: many shared prefixes, so duplicate ranges occur at every word."""
+    return rng.integers(0, alphabet, (n, W), dtype=np.uint8)
+
+
+def test_partial_key_is_big_endian_and_order_isomorphic():
+    """P:78 "partial binary sortable representation": the u32 of bytes [4w, 4w+4) read most
+    significant first; comparing two partial keys = comparing those 4 bytes lexicographically."""
+    rng = np.random.default_rng(11)
+    rows = rng.integers(0, 256, (300, 12), dtype=np.uint8)
+    for w in range(3):
+        k = oracle.partial_keys(rows, w)
+        for i in range(300):
+            assert int(k[i]) == int.from_bytes(bytes(rows[i, 4 * w:4 * w + 4]), "big")
+        for i in range(0, 299):
+            a, b = bytes(rows[i, 4 * w:4 * w + 4]), bytes(rows[i + 1, 4 * w:4 * w + 4])
+            assert (k[i] < k[i + 1]) == (a < b) and (k[i] == k[i + 1]) == (a == b)
+
+
+@pytest.mark.parametrize("n,card", [(0, 3), (1, 3), (500, 3), (2000, 50), (2000, 2**32)])
+def test_sort_pairs_is_stable_sort_by_key(n, card):
+    """The sorted partial key buffer equals Python's (stable) sorted() by key, and numpy's
+    stable argsort; payload order within equal keys is buffer order."""
+    rng = np.random.default_rng(n + 5)
+    keys = rng.integers(0, card, n, dtype=np.uint64).astype(np.uint32)
+    pay = rng.permutation(n).astype(np.uint32)
+    ko, po = oracle.sort_pairs(keys, pay)
+    order = sorted(range(n), key=lambda i: int(keys[i]))
+    assert [int(x) for x in po] == [int(pay[i]) for i in order]
+    assert np.array_equal(ko, keys[order] if n else keys)
+    assert np.array_equal(po, pay[np.argsort(keys, kind="stable")])
+
+
+def test_dup_ranges_brute_force():
+    """Duplicate ranges = maximal runs of >= 2 equal keys, by itertools.groupby."""
+    import itertools
+    rng = np.random.default_rng(3)
+    for n, card in [(0, 2), (1, 2), (7, 1), (400, 5), (400, 1000)]:
+        keys = np.sort(rng.integers(0, card, n)).astype(np.uint32)
+        st, ln = oracle.dup_ranges(keys)
+        exp, pos = [], 0
+        for _, g in itertools.groupby(keys.tolist()):
+            c = len(list(g))
+            if c >= 2:
+                exp.append((pos, c))
+            pos += c
+        assert list(zip(st.tolist(), ln.tolist())) == exp
+        assert int(ln.sum()) == sum(c for _, c in exp)
+
+
+@pytest.mark.parametrize("W", [4, 8, 12, 16])
+def test_sort_rows_brute_force(W):
+    """The completed sort = Python's stable sorted() of row indices by the key bytes."""
+    rng = np.random.default_rng(W)
+    for n in (0, 1, 2, 37, 700):
+        rows = _rows(rng, n, W)
+        perm = oracle.sort_rows(rows)
+        exp = sorted(range(n), key=lambda i: bytes(rows[i]))
+        assert [int(x) for x in perm] == exp
+
+
+def test_sort_rows_special_cases_and_invariants():
+    rng = np.random.default_rng(9)
+    n, W = 1000, 8
+    same = np.tile(rng.integers(0, 256, (1, W), dtype=np.uint8), (n, 1))
+    assert np.array_equal(oracle.sort_rows(same), np.arange(n))           # all equal: row order
+    distinct = np.stack([np.frombuffer(int(x).to_bytes(W, "big"), np.uint8) for x in range(n)])
+    assert np.array_equal(oracle.sort_rows(distinct), np.arange(n))       # already sorted
+    assert np.array_equal(oracle.sort_rows(distinct[::-1].copy()), np.arange(n)[::-1])  # reversed
+    rows = _rows(rng, 5000, 12)
+    perm = oracle.sort_rows(rows)
+    assert np.array_equal(np.sort(perm), np.arange(5000))                 # a permutation
+    s = rows[perm]
+    for i in range(4999):                                                  # non-decreasing, stable
+        a, b = bytes(s[i]), bytes(s[i + 1])
+        assert a < b or (a == b and perm[i] < perm[i + 1])
+    # the job queue of P:84-86 written out step by step reaches the same order: sort by word 0,
+    # then every duplicate range by the next word, until no range is left
+    order = np.arange(5000)
+    ranges = [(0, 5000)]
+    for w in range(3):
+        nxt = []
+        for a, b in ranges:
+            seg = order[a:b]
+            k = oracle.partial_keys(rows[seg], w)
+            _, po = oracle.sort_pairs(k, np.arange(b - a, dtype=np.uint32))
+            order[a:b] = seg[po.astype(np.int64)]
+            ks = k[po.astype(np.int64)]
+            st, ln = oracle.dup_ranges(ks)
+            nxt += [(a + int(x), a + int(x) + int(y)) for x, y in zip(st, ln)]
+        ranges = nxt
+    assert np.array_equal(order, perm)
