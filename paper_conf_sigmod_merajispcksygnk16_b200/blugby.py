@@ -68,6 +68,11 @@ class TimingC(ctypes.Structure):
                 ("part_fallbacks", ctypes.c_uint32)]
 
 
+class SortStatsC(ctypes.Structure):
+    _fields_ = [("levels", ctypes.c_uint32), ("ranges", ctypes.c_uint64 * 256), ("active", ctypes.c_uint64 * 256),
+                ("ms", ctypes.c_float * 256)]
+
+
 def _load():
     if not os.path.exists(LIB_PATH):
         raise ImportError(f"libblugby.so not built ({LIB_PATH}); run `make` or __graft_entry__.build()")
@@ -93,6 +98,10 @@ def _load():
         "blu_gby_slot_template": ([vp, vp, u32, P(u32)], i32),
         "blu_gby_init_table": ([vp, vp, u64, vp], i32),
         "blu_gby_set_timing": ([i32], None),
+        "blu_sort_partial_keys": ([vp, u64, ctypes.c_uint32, ctypes.c_uint32, vp, vp], i32),
+        "blu_sort_pairs": ([vp, vp, u64, vp, vp, vp], i32),
+        "blu_sort_dup_ranges": ([vp, u64, vp, vp, u64, P(u64), vp], i32),
+        "blu_sort_rows": ([vp, u64, ctypes.c_uint32, vp, vp, P(SortStatsC)], i32),
         "blu_gby_last_timing": ([P(TimingC)], i32),
         "blu_gby_launch_count": ([], u64),
         "blu_gby_read_roofline": ([P(vp), P(u64), i32, vp, vp], i32),
@@ -469,3 +478,47 @@ def blu_gby_read_roofline(cols, out, stream=None):
 
 def blu_gby_bind_device(device: int):
     _check(lib.blu_gby_bind_device(int(device)))
+
+
+# ---- sort offload (include/blu_sort.h; §3) ----------------------------------------
+# u32 partial keys / payloads / permutations travel as torch.int32 tensors holding the same bits.
+def blu_sort_partial_keys(rows, word: int, stream=None):
+    """big-endian 4-byte partial keys of word `word` of (n, W) uint8 device rows."""
+    import torch
+    n, W = rows.shape
+    out = torch.empty(n, dtype=torch.int32, device=rows.device)
+    _check(lib.blu_sort_partial_keys(_ptr(rows), n, W, word, _ptr(out), _stream_handle(stream)))
+    return out
+
+
+def blu_sort_pairs(keys, payload, stream=None):
+    """stable sort of the partial key buffer by its unsigned 4-byte key."""
+    import torch
+    ko, po = torch.empty_like(keys), torch.empty_like(payload)
+    _check(lib.blu_sort_pairs(_ptr(keys), _ptr(payload), keys.numel(), _ptr(ko), _ptr(po), _stream_handle(stream)))
+    return ko, po
+
+
+def blu_sort_dup_ranges(sorted_keys, stream=None):
+    """(starts, lens) int64 device tensors of the duplicate ranges of a sorted buffer."""
+    import torch
+    n = sorted_keys.numel()
+    cap = max(1, n // 2)
+    st = torch.empty(cap, dtype=torch.int64, device=sorted_keys.device)
+    ln = torch.empty(cap, dtype=torch.int64, device=sorted_keys.device)
+    r = ctypes.c_uint64()
+    _check(lib.blu_sort_dup_ranges(_ptr(sorted_keys), n, _ptr(st), _ptr(ln), cap, ctypes.byref(r), _stream_handle(stream)))
+    return st[: r.value], ln[: r.value]
+
+
+def blu_sort_rows(rows, stream=None):
+    """(perm, stats): perm[p] = row at position p of the stable lexicographic order of the
+    (n, W) uint8 device rows; stats = levels, ranges / active rows / ms per level."""
+    import torch
+    n, W = rows.shape
+    perm = torch.empty(n, dtype=torch.int32, device=rows.device)
+    st = SortStatsC()
+    _check(lib.blu_sort_rows(_ptr(rows), n, W, _ptr(perm), _stream_handle(stream), ctypes.byref(st)))
+    L = st.levels
+    stats = {"levels": L, "ranges": list(st.ranges[:L]), "active": list(st.active[:L]), "ms": list(st.ms[:L])}
+    return perm, stats

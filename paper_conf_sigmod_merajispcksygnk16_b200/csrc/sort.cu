@@ -1,0 +1,550 @@
+// sort.cu — libblugby's sort offload (§3; include/blu_sort.h).
+//
+//   k_rs_upsweep / k_rs_scan / k_rs_downsweep   one pass of a stable LSD radix sort (8-bit digit):
+//       every CTA owns one contiguous range of tiles; the upsweep counts its digits, one CTA scans
+//       the digit-major count matrix into output offsets, the downsweep ranks each tile's keys with
+//       warp matching (__match_any_sync: lanes with equal digits, the lowest one bumps a per-warp
+//       counter) and scatters them after all earlier CTAs' and tiles' keys of the same digit —
+//       stable, no global atomics. Used for the partial key buffer (u32 keys, "Duane sort"
+//       [18]) and for the batched duplicate-range jobs (u64 keys = range id << 32 | partial key).
+//   k_partial_keys        P:78 4-byte big-endian partial key of one word of every row
+//   k_dup_mark / k_dup_count / k_dup_emit   P:84 duplicate ranges: run boundaries, block counts,
+//       one-CTA scan, compaction into (start, len) or into the next level's active set
+//   k_level_keys / k_level_scatter           one batched level of the job queue
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "blu_internal.h"
+#include "blu_sort.h"
+
+namespace blu {
+
+namespace {
+
+constexpr int kRT = 256;  // threads per radix CTA (= number of digits: thread d owns digit d)
+
+template <typename KT>
+struct RadixCfg {
+  static constexpr int ITEMS = sizeof(KT) == 4 ? 16 : 8;  // keys per thread per tile
+  static constexpr int WARP_CHUNK = 32 * ITEMS;           // contiguous keys per warp
+  static constexpr int TILE = kRT * ITEMS;
+};
+
+__device__ __forceinline__ void tile_span(uint64_t ntiles, uint64_t& t0, uint64_t& t1) {
+  t0 = ntiles * blockIdx.x / gridDim.x;
+  t1 = ntiles * (blockIdx.x + 1) / gridDim.x;
+}
+
+template <typename KT>
+__device__ __forceinline__ uint32_t digit_of(KT k, uint32_t shift) {
+  return (uint32_t)(k >> shift) & 255u;
+}
+
+template <typename KT>
+__global__ void __launch_bounds__(kRT) k_rs_upsweep(const KT* __restrict__ keys, uint64_t n, uint32_t shift,
+                                                    uint32_t* __restrict__ counts) {
+  using C = RadixCfg<KT>;
+  __shared__ uint32_t h[256];
+  h[threadIdx.x] = 0;
+  __syncthreads();
+  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t t0, t1;
+  tile_span((n + C::TILE - 1) / C::TILE, t0, t1);
+  for (uint64_t t = t0; t < t1; ++t) {
+    const uint64_t b = t * C::TILE + (uint64_t)warp * C::WARP_CHUNK + lane;
+#pragma unroll
+    for (int i = 0; i < C::ITEMS; ++i) {
+      const uint64_t e = b + (uint64_t)i * 32;
+      const bool valid = e < n;
+      const uint32_t d = valid ? digit_of(keys[e], shift) : 256u + lane;
+      const uint32_t peers = __match_any_sync(0xffffffffu, d);
+      if (valid && lane == (unsigned)(__ffs(peers) - 1)) atomicAdd(&h[d], (uint32_t)__popc(peers));
+    }
+  }
+  __syncthreads();
+  counts[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x] = h[threadIdx.x];
+}
+
+// Exclusive scan, in place, of a[0..L) (one CTA of 1024 threads, contiguous chunk per thread).
+__global__ void __launch_bounds__(1024) k_rs_scan(uint32_t* a, uint64_t L) {
+  __shared__ uint32_t ws[32];
+  const uint64_t per = (L + blockDim.x - 1) / blockDim.x;
+  const uint64_t b = per * threadIdx.x, e = b + per < L ? b + per : L;
+  uint32_t s = 0;
+  for (uint64_t i = b; i < e; ++i) s += a[i];
+  const unsigned lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t inc = s;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+    if ((int)lane >= o) inc += y;
+  }
+  if (lane == 31) ws[w] = inc;
+  __syncthreads();
+  if (w == 0) {
+    const uint32_t v = ws[lane];
+    uint32_t vi = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, vi, o);
+      if ((int)lane >= o) vi += y;
+    }
+    ws[lane] = vi - v;
+  }
+  __syncthreads();
+  uint32_t run = ws[w] + inc - s;
+  for (uint64_t i = b; i < e; ++i) {
+    const uint32_t x = a[i];
+    a[i] = run;
+    run += x;
+  }
+}
+
+template <typename KT>
+__global__ void __launch_bounds__(kRT) k_rs_downsweep(const KT* __restrict__ kin, const uint32_t* __restrict__ vin,
+                                                      KT* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
+                                                      uint32_t shift, const uint32_t* __restrict__ offsets) {
+  using C = RadixCfg<KT>;
+  __shared__ uint32_t base[256];
+  __shared__ uint32_t ttot[256];
+  __shared__ uint32_t wcnt[kRT / 32][256];
+  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t lt_mask = (1u << lane) - 1u;
+  base[threadIdx.x] = offsets[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x];
+  uint64_t t0, t1;
+  tile_span((n + C::TILE - 1) / C::TILE, t0, t1);
+  for (uint64_t t = t0; t < t1; ++t) {
+#pragma unroll
+    for (int w = 0; w < kRT / 32; ++w) wcnt[w][threadIdx.x] = 0;
+    __syncthreads();
+    // warp-striped tile: warp w owns keys [w * WARP_CHUNK, +WARP_CHUNK); item i of lane l is key
+    // i * 32 + l of that chunk, so (warp, i, lane) order is input order (stability)
+    const uint64_t b = t * C::TILE + (uint64_t)warp * C::WARP_CHUNK + lane;
+    KT k[C::ITEMS];
+    uint32_t v[C::ITEMS], rank[C::ITEMS];
+#pragma unroll
+    for (int i = 0; i < C::ITEMS; ++i) {
+      const uint64_t e = b + (uint64_t)i * 32;
+      k[i] = e < n ? kin[e] : (KT)0;
+      v[i] = e < n ? vin[e] : 0u;
+    }
+#pragma unroll
+    for (int i = 0; i < C::ITEMS; ++i) {
+      const bool valid = b + (uint64_t)i * 32 < n;
+      const uint32_t d = valid ? digit_of(k[i], shift) : 256u + lane;
+      const uint32_t peers = __match_any_sync(0xffffffffu, d);
+      const int leader = __ffs(peers) - 1;
+      uint32_t c = 0;
+      if (valid && (int)lane == leader) {
+        c = wcnt[warp][d];
+        wcnt[warp][d] = c + (uint32_t)__popc(peers);
+      }
+      c = __shfl_sync(0xffffffffu, c, leader);
+      rank[i] = c + (uint32_t)__popc(peers & lt_mask);
+      __syncwarp();
+    }
+    __syncthreads();
+    {  // per digit: exclusive prefix over the warps, tile total
+      uint32_t run = 0;
+#pragma unroll
+      for (int w = 0; w < kRT / 32; ++w) {
+        const uint32_t x = wcnt[w][threadIdx.x];
+        wcnt[w][threadIdx.x] = run;
+        run += x;
+      }
+      ttot[threadIdx.x] = run;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int i = 0; i < C::ITEMS; ++i) {
+      if (b + (uint64_t)i * 32 >= n) continue;
+      const uint32_t d = digit_of(k[i], shift);
+      const uint32_t pos = base[d] + wcnt[warp][d] + rank[i];
+      kout[pos] = k[i];
+      vout[pos] = v[i];
+    }
+    __syncthreads();
+    base[threadIdx.x] += ttot[threadIdx.x];
+  }
+}
+
+// big-endian 4-byte partial key of word `word` (bytes past W read as 0); payload = row index.
+template <typename KT>
+__global__ void k_partial_keys(const uint8_t* __restrict__ rows, uint64_t n, uint32_t W, uint32_t word,
+                               KT* __restrict__ keys, uint32_t* __restrict__ payload) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t p = 4 * word;
+    uint32_t k;
+    if (p + 4 <= W && (W & 3) == 0 && ((uintptr_t)rows & 3) == 0) {
+      k = __byte_perm(__ldg((const unsigned int*)(rows + i * W + p)), 0, 0x0123);  // bswap
+    } else {
+      k = 0;
+      for (uint32_t q = 0; q < 4; ++q) k = (k << 8) | (p + q < W ? rows[i * W + p + q] : 0u);
+    }
+    keys[i] = (KT)k;
+    if (payload) payload[i] = (uint32_t)i;
+  }
+}
+
+// ---- duplicate ranges: marks -> block counts -> scan -> emit ---------------------------------------
+constexpr int kDT = 256, kDR = 16;  // threads, elements per thread (4096 per block)
+constexpr uint64_t kDB = (uint64_t)kDT * kDR;
+
+template <typename KT>
+__device__ __forceinline__ void dup_flags(const KT* k, uint64_t m, uint64_t j, bool& act, bool& start, bool& end) {
+  const bool sp = j > 0 && k[j] == k[j - 1];
+  const bool sn = j + 1 < m && k[j] == k[j + 1];
+  act = sp || sn;
+  start = act && !sp;
+  end = act && !sn;
+}
+
+// per block: number of active elements (in a duplicate range) and of range starts
+template <typename KT>
+__global__ void __launch_bounds__(kDT) k_dup_count(const KT* __restrict__ k, uint64_t m, uint32_t* __restrict__ cnt_act,
+                                                   uint32_t* __restrict__ cnt_start) {
+  uint32_t a = 0, s = 0;
+  for (int r = 0; r < kDR; ++r) {
+    const uint64_t j = (uint64_t)blockIdx.x * kDB + (uint64_t)r * kDT + threadIdx.x;
+    if (j >= m) break;
+    bool act, st, en;
+    dup_flags(k, m, j, act, st, en);
+    a += act;
+    s += st;
+  }
+  __shared__ uint32_t wa[kDT / 32], wsum[kDT / 32];
+  for (int o = 16; o; o >>= 1) {
+    a += __shfl_xor_sync(0xffffffffu, a, o);
+    s += __shfl_xor_sync(0xffffffffu, s, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    wa[threadIdx.x >> 5] = a;
+    wsum[threadIdx.x >> 5] = s;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t ta = 0, ts = 0;
+    for (int w = 0; w < kDT / 32; ++w) {
+      ta += wa[w];
+      ts += wsum[w];
+    }
+    cnt_act[blockIdx.x] = ta;
+    cnt_start[blockIdx.x] = ts;
+  }
+}
+
+// Emit, in order, per active element j: its position act_pos (the caller's position list, or j
+// itself if NULL) into next_pos and its range id (0-based, in order) into next_seg; per range its
+// start and its end (exclusive; k_range_lens turns it into a length) into r_start / r_len (if
+// non-NULL, ids < cap).
+template <typename KT>
+__global__ void __launch_bounds__(kDT) k_dup_emit(const KT* __restrict__ k, uint64_t m, const uint32_t* __restrict__ off_act,
+                                                  const uint32_t* __restrict__ off_start, const uint32_t* __restrict__ act_pos,
+                                                  uint32_t* __restrict__ next_pos, uint32_t* __restrict__ next_seg,
+                                                  uint64_t* __restrict__ r_start, uint64_t* __restrict__ r_len, uint64_t cap) {
+  __shared__ uint32_t wa[kDT / 32], wsum[kDT / 32];
+  uint32_t base_a = off_act[blockIdx.x], base_s = off_start[blockIdx.x];
+  const unsigned lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  for (int r = 0; r < kDR; ++r) {
+    const uint64_t j = (uint64_t)blockIdx.x * kDB + (uint64_t)r * kDT + threadIdx.x;
+    bool act = false, st = false, en = false;
+    if (j < m) dup_flags(k, m, j, act, st, en);
+    const uint32_t ba = __ballot_sync(0xffffffffu, act), bs = __ballot_sync(0xffffffffu, st);
+    if (lane == 0) {
+      wa[w] = __popc(ba);
+      wsum[w] = __popc(bs);
+    }
+    __syncthreads();
+    uint32_t pa = 0, ps = 0, ta = 0, ts = 0;
+    for (unsigned q = 0; q < kDT / 32; ++q) {
+      if (q < w) {
+        pa += wa[q];
+        ps += wsum[q];
+      }
+      ta += wa[q];
+      ts += wsum[q];
+    }
+    pa += __popc(ba & ((1u << lane) - 1u));
+    ps += __popc(bs & ((1u << lane) - 1u));
+    const uint32_t ia = base_a + pa;                      // index among active elements
+    const uint32_t seg = base_s + ps + (st ? 1u : 0u) - 1u;  // range id (inclusive count - 1)
+    if (act) {
+      if (next_pos) next_pos[ia] = act_pos ? act_pos[j] : (uint32_t)j;
+      if (next_seg) next_seg[ia] = seg;
+    }
+    if (r_start && seg < cap) {
+      if (st) r_start[seg] = j;
+      if (en) r_len[seg] = j + 1;
+    }
+    __syncthreads();
+    base_a += ta;
+    base_s += ts;
+  }
+}
+
+__global__ void k_range_lens(const uint64_t* __restrict__ r_start, uint64_t* __restrict__ r_len, uint64_t cnt) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += (uint64_t)gridDim.x * blockDim.x)
+    r_len[i] -= r_start[i];
+}
+
+// One batched level: key = (range id << 32) | partial key `word` of the row at buffer position
+// pos[j]; payload = that row id.
+__global__ void k_level_keys(const uint8_t* __restrict__ rows, uint32_t W, uint32_t word, const uint32_t* __restrict__ pos,
+                             const uint32_t* __restrict__ seg, const uint32_t* __restrict__ perm, uint64_t m,
+                             uint64_t* __restrict__ keys, uint32_t* __restrict__ payload) {
+  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < m; j += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t row = perm[pos[j]];
+    const uint32_t p = 4 * word;
+    uint32_t k = 0;
+    if ((W & 3) == 0 && p + 4 <= W && ((uintptr_t)rows & 3) == 0) {
+      k = __byte_perm(__ldg((const unsigned int*)(rows + (uint64_t)row * W + p)), 0, 0x0123);
+    } else {
+      for (uint32_t q = 0; q < 4; ++q) k = (k << 8) | (p + q < W ? rows[(uint64_t)row * W + p + q] : 0u);
+    }
+    keys[j] = ((uint64_t)seg[j] << 32) | k;
+    payload[j] = row;
+  }
+}
+
+// Sorted level results back into the positions its ranges occupy (same ranges, same order).
+__global__ void k_level_scatter(const uint32_t* __restrict__ pos, const uint32_t* __restrict__ rows_sorted, uint64_t m,
+                                uint32_t* __restrict__ perm) {
+  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < m; j += (uint64_t)gridDim.x * blockDim.x)
+    perm[pos[j]] = rows_sorted[j];
+}
+
+int sms_now() {
+  int dev = 0, s = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&s, cudaDevAttrMultiProcessorCount, dev);
+  return s;
+}
+
+uint32_t elem_grid(uint64_t n) {
+  const uint64_t g = (n + 255) / 256;
+  return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(g, (uint64_t)sms_now() * 16));
+}
+
+struct DevBuf {  // stream-ordered scratch
+  void* p = nullptr;
+  cudaStream_t st;
+  explicit DevBuf(cudaStream_t s) : st(s) {}
+  cudaError_t alloc(size_t b) { return cudaMallocAsync(&p, std::max<size_t>(b, 16), st); }
+  ~DevBuf() {
+    if (p) cudaFreeAsync(p, st);
+  }
+};
+
+// Stable LSD radix sort of the low `bits` key bits: (kin, vin) -> (kout, vout); kt/vt scratch (n).
+template <typename KT>
+cudaError_t radix_sort(const KT* kin, const uint32_t* vin, KT* kout, uint32_t* vout, KT* kt, uint32_t* vt, uint64_t n,
+                       uint32_t bits, uint32_t* counts, uint32_t grid, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  const int passes = std::max(1, (int)((bits + 7) / 8));
+  const KT* sk = kin;
+  const uint32_t* sv = vin;
+  for (int p = 0; p < passes; ++p) {
+    const bool to_out = ((passes - 1 - p) % 2) == 0;
+    KT* dk = to_out ? kout : kt;
+    uint32_t* dv = to_out ? vout : vt;
+    k_rs_upsweep<KT><<<grid, kRT, 0, st>>>(sk, n, 8u * p, counts);
+    k_rs_scan<<<1, 1024, 0, st>>>(counts, (uint64_t)256 * grid);
+    k_rs_downsweep<KT><<<grid, kRT, 0, st>>>(sk, sv, dk, dv, n, 8u * p, counts);
+    count_launch(3);
+    sk = dk;
+    sv = dv;
+  }
+  return cudaGetLastError();
+}
+
+uint32_t radix_grid() { return (uint32_t)sms_now() * 8; }  // 8 x 256 threads per SM
+
+blu_status_t cuda_err(cudaError_t e, const char* what) {
+  cudaGetLastError();
+  if (e == cudaErrorMemoryAllocation) return fail(BLU_E_OOM, "%s: %s", what, cudaGetErrorString(e));
+  return fail(BLU_E_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+#define SCK(x, what)                                 \
+  do {                                               \
+    cudaError_t e_ = (x);                            \
+    if (e_ != cudaSuccess) return cuda_err(e_, what); \
+  } while (0)
+
+// Duplicate ranges of sorted keys k[0..m): counts, host scan result (#active, #ranges), emit.
+template <typename KT>
+blu_status_t dup_pass(const KT* k, uint64_t m, const uint32_t* act_pos, uint32_t* next_pos, uint32_t* next_seg,
+                      uint64_t* r_start, uint64_t* r_len, uint64_t cap, uint64_t* n_act, uint64_t* n_rng,
+                      cudaStream_t st) {
+  *n_act = *n_rng = 0;
+  if (m == 0) return BLU_OK;
+  const uint64_t nb = (m + kDB - 1) / kDB;
+  DevBuf w(st);
+  SCK(w.alloc(nb * 8 + 16), "dup workspace");
+  uint32_t* ca = (uint32_t*)w.p;
+  uint32_t* cs = ca + nb;
+  uint32_t* tot = cs + nb;  // 2 totals
+  k_dup_count<KT><<<(unsigned)nb, kDT, 0, st>>>(k, m, ca, cs);
+  // totals: sum of the last offsets + counts after the scans
+  SCK(cudaMemcpyAsync(tot, ca + nb - 1, 4, cudaMemcpyDeviceToDevice, st), "dup totals");
+  SCK(cudaMemcpyAsync(tot + 1, cs + nb - 1, 4, cudaMemcpyDeviceToDevice, st), "dup totals");
+  k_rs_scan<<<1, 1024, 0, st>>>(ca, nb);
+  k_rs_scan<<<1, 1024, 0, st>>>(cs, nb);
+  k_dup_emit<KT><<<(unsigned)nb, kDT, 0, st>>>(k, m, ca, cs, act_pos, next_pos, next_seg, r_start, r_len, cap);
+  count_launch(4);
+  uint32_t h[4];
+  SCK(cudaMemcpyAsync(h, ca + nb - 1, 4, cudaMemcpyDeviceToHost, st), "dup D2H");
+  SCK(cudaMemcpyAsync(h + 1, cs + nb - 1, 4, cudaMemcpyDeviceToHost, st), "dup D2H");
+  SCK(cudaMemcpyAsync(h + 2, tot, 8, cudaMemcpyDeviceToHost, st), "dup D2H");
+  SCK(cudaStreamSynchronize(st), "dup sync");
+  *n_act = (uint64_t)h[0] + h[2];
+  *n_rng = (uint64_t)h[1] + h[3];
+  if (r_start && *n_rng) {
+    const uint64_t c = std::min(cap, *n_rng);
+    k_range_lens<<<elem_grid(c), 256, 0, st>>>(r_start, r_len, c);
+    count_launch(1);
+    SCK(cudaGetLastError(), "range lens");
+  }
+  return BLU_OK;
+}
+
+}  // namespace
+}  // namespace blu
+
+using namespace blu;
+
+extern "C" {
+
+blu_status_t blu_sort_partial_keys(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t word, uint32_t* keys_out,
+                                   void* stream) {
+  if (n && (!rows || !keys_out)) return fail(BLU_E_INVALID, "NULL pointer");
+  if (W < 4 || W > 1024 || (W & 3) || 4 * word >= W) return fail(BLU_E_INVALID, "bad W %u / word %u", W, word);
+  if (!n) return BLU_OK;
+  cudaStream_t st = (cudaStream_t)stream;
+  k_partial_keys<uint32_t><<<elem_grid(n), 256, 0, st>>>(rows, n, W, word, keys_out, nullptr);
+  count_launch(1);
+  SCK(cudaGetLastError(), "partial keys");
+  return BLU_OK;
+}
+
+blu_status_t blu_sort_pairs(const uint32_t* keys_in, const uint32_t* payload_in, uint64_t n, uint32_t* keys_out,
+                            uint32_t* payload_out, void* stream) {
+  if (n && (!keys_in || !payload_in || !keys_out || !payload_out)) return fail(BLU_E_INVALID, "NULL pointer");
+  if (n >= (1ull << 32)) return fail(BLU_E_INVALID, "n >= 2^32");
+  if (n && ((const void*)keys_out == (const void*)keys_in || (const void*)payload_out == (const void*)payload_in))
+    return fail(BLU_E_INVALID, "outputs alias inputs");
+  if (!n) return BLU_OK;
+  cudaStream_t st = (cudaStream_t)stream;
+  const uint32_t grid = radix_grid();
+  DevBuf w(st);
+  SCK(w.alloc((size_t)n * 8 + (size_t)256 * grid * 4), "sort workspace");
+  uint32_t* kt = (uint32_t*)w.p;
+  uint32_t* vt = kt + n;
+  uint32_t* counts = vt + n;
+  SCK(radix_sort<uint32_t>(keys_in, payload_in, keys_out, payload_out, kt, vt, n, 32, counts, grid, st), "radix sort");
+  return BLU_OK;
+}
+
+blu_status_t blu_sort_dup_ranges(const uint32_t* sorted_keys, uint64_t n, uint64_t* starts, uint64_t* lens, uint64_t cap,
+                                 uint64_t* n_ranges, void* stream) {
+  if (!n_ranges || (n && !sorted_keys) || (cap && (!starts || !lens))) return fail(BLU_E_INVALID, "NULL pointer");
+  if (n >= (1ull << 32)) return fail(BLU_E_INVALID, "n >= 2^32");
+  uint64_t na = 0;
+  return dup_pass<uint32_t>(sorted_keys, n, nullptr, nullptr, nullptr, cap ? starts : nullptr, cap ? lens : nullptr, cap, &na,
+                            n_ranges, (cudaStream_t)stream);
+}
+
+blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t* perm_out, void* stream,
+                           blu_sort_stats_t* stats) {
+  if (n && (!rows || !perm_out)) return fail(BLU_E_INVALID, "NULL pointer");
+  if (W < 4 || W > 1024 || (W & 3)) return fail(BLU_E_INVALID, "W must be a multiple of 4 in [4, 1024] (got %u)", W);
+  if (n >= (1ull << 32)) return fail(BLU_E_INVALID, "n >= 2^32");
+  if (stats) memset(stats, 0, sizeof *stats);
+  if (!n) return BLU_OK;
+  cudaStream_t st = (cudaStream_t)stream;
+  const uint32_t grid = radix_grid();
+  cudaEvent_t e0 = nullptr, e1 = nullptr;
+  if (stats) {
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+  }
+  auto level_time = [&](uint32_t l) {
+    if (!stats || l >= 256) return;
+    cudaEventRecord(e1, st);
+    cudaEventSynchronize(e1);
+    cudaEventElapsedTime(&stats->ms[l], e0, e1);
+  };
+  // workspace: level-0 keys/payload scratch (u32) + level keys (u64 x2) + payload x2 + pos/seg x2
+  DevBuf w(st);
+  const size_t need = (size_t)n * (4 + 4 + 8 + 8 + 8 + 4 + 4 + 4 + 4 * 4) + (size_t)256 * grid * 4 + 256;
+  SCK(w.alloc(need), "sort workspace");
+  uint8_t* q = (uint8_t*)w.p;
+  auto take = [&](size_t b) {
+    uint8_t* r = q;
+    q += (b + 15) & ~(size_t)15;
+    return r;
+  };
+  uint32_t* k32a = (uint32_t*)take(n * 4);
+  uint32_t* k32b = (uint32_t*)take(n * 4);
+  uint64_t* k64a = (uint64_t*)take(n * 8);
+  uint64_t* k64b = (uint64_t*)take(n * 8);
+  uint64_t* k64c = (uint64_t*)take(n * 8);  // radix scratch (never an input of the same sort)
+  uint32_t* pa = (uint32_t*)take(n * 4);
+  uint32_t* pb = (uint32_t*)take(n * 4);
+  uint32_t* pc = (uint32_t*)take(n * 4);
+  uint32_t* pos0 = (uint32_t*)take(n * 4);
+  uint32_t* seg0 = (uint32_t*)take(n * 4);
+  uint32_t* pos1 = (uint32_t*)take(n * 4);
+  uint32_t* seg1 = (uint32_t*)take(n * 4);
+  uint32_t* counts = (uint32_t*)take((size_t)256 * grid * 4);
+  if (stats) cudaEventRecord(e0, st);
+  // level 0: the whole buffer is one job ("Initially there is only one job")
+  k_partial_keys<uint32_t><<<elem_grid(n), 256, 0, st>>>(rows, n, W, 0, k32a, pa);
+  count_launch(1);
+  SCK(radix_sort<uint32_t>(k32a, pa, k32b, perm_out, (uint32_t*)k64c, pc, n, 32, counts, grid, st), "level 0 sort");
+  uint64_t m = 0, nr = 0;
+  blu_status_t s = dup_pass<uint32_t>(k32b, n, nullptr, pos0, seg0, nullptr, nullptr, 0, &m, &nr, st);
+  if (s != BLU_OK) return s;
+  uint32_t level = 1;
+  if (stats) {
+    stats->ranges[0] = nr;
+    stats->active[0] = m;
+    level_time(0);
+  }
+  // level l: every duplicate range left is a job sorted by its next 4 bytes; all of them in
+  // one batched sort keyed by (range id, partial key)
+  for (uint32_t word = 1; m > 0 && 4 * word < W; ++word, ++level) {
+    if (stats) cudaEventRecord(e0, st);
+    uint32_t bits_seg = 0;
+    while (bits_seg < 32 && (1ull << bits_seg) < nr) ++bits_seg;
+    k_level_keys<<<elem_grid(m), 256, 0, st>>>(rows, W, word, pos0, seg0, perm_out, m, k64a, pa);
+    count_launch(1);
+    SCK(radix_sort<uint64_t>(k64a, pa, k64b, pb, k64c, pc, m, 32 + bits_seg, counts, grid, st), "level sort");
+    k_level_scatter<<<elem_grid(m), 256, 0, st>>>(pos0, pb, m, perm_out);
+    count_launch(1);
+    uint64_t m2 = 0, nr2 = 0;
+    s = dup_pass<uint64_t>(k64b, m, pos0, pos1, seg1, nullptr, nullptr, 0, &m2, &nr2, st);
+    if (s != BLU_OK) return s;
+    std::swap(pos0, pos1);
+    std::swap(seg0, seg1);
+    m = m2;
+    nr = nr2;
+    if (stats && level < 256) {
+      stats->ranges[level] = nr;
+      stats->active[level] = m;
+      level_time(level);
+    }
+  }
+  if (stats) {
+    stats->levels = level;
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+  }
+  SCK(cudaGetLastError(), "sort rows");
+  return BLU_OK;
+}
+
+}  // extern "C"

@@ -29,6 +29,22 @@ def test_library_exports_every_header_symbol(bg):
     assert not missing, missing
 
 
+def test_library_exports_sort_header_symbols(bg):
+    """include/blu_sort.h (NEXT-4 sort offload, P:76-88): every declared entry point is exported;
+    argument checks run without a GPU."""
+    hdr = open(os.path.join(ROOT, "include", "blu_sort.h")).read()
+    names = set(re.findall(r"\b(blu_sort_[a-z_0-9]+)\s*\(", hdr))
+    assert names == {"blu_sort_partial_keys", "blu_sort_pairs", "blu_sort_dup_ranges", "blu_sort_rows"}
+    lib = ctypes.CDLL(bg.LIB_PATH)
+    assert all(hasattr(lib, n) for n in names)
+    st = bg.lib.blu_sort_rows(None, 10, 6, None, None, None)       # W not a multiple of 4
+    assert st == bg.BLU_E_INVALID
+    st = bg.lib.blu_sort_rows(None, 0, 16, None, None, None)       # empty input: nothing to do
+    assert st == bg.BLU_OK
+    st = bg.lib.blu_sort_pairs(None, None, 5, None, None, None)    # NULL buffers
+    assert st == bg.BLU_E_INVALID
+
+
 def test_generator_library_exports():
     hdr = open(os.path.join(ROOT, "include", "blu_gen.h")).read()
     names = set(re.findall(r"^(?:int|void)\s+(blu_gen_[a-z_0-9]+)\s*\(", hdr, re.M))
