@@ -169,6 +169,140 @@ def run_reference(args):
 
 
 # ----------------------------------------------------------------------------------------------
+# S1: the sort offload (§3) — a second workload, not the
+# BASELINE metric: 10^8 rows of 16-byte binary-sortable keys shaped like an ORDER BY over
+# store_sales (sold date, store, item/ticket), sorted into a stable permutation.
+# ----------------------------------------------------------------------------------------------
+SORT_METRIC = "sort offload rows/s (partial-key radix sort + duplicate-range jobs, P:76-88)"
+SORT_N, SORT_W = 100_000_000, 16
+
+
+def sort_cpu(rows_np, n):
+    import oracle
+    t0 = time.perf_counter()
+    oracle.sort_rows(rows_np[:n])
+    return n / (time.perf_counter() - t0)
+
+
+def run_sort_reference(args):
+    if int(os.environ.get("RANK", "0")) != 0:
+        return 0
+    import blugen
+    n = int(os.environ.get("BLU_BENCH_SORT_REF_ROWS", "2000000"))
+    rows = blugen.sort_rows(n, SORT_W)
+    for _ in range(args.warmup):
+        sort_cpu(rows, n // 4)
+    rates = [sort_cpu(rows, n) for _ in range(args.steps)]
+    value = statistics.mean(rates)
+    line = {"impl": "reference", "metric": SORT_METRIC, "value": value, "unit": "rows/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * n / value, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": f"S1: {SORT_W}-byte keys, rows per step {n} of {SORT_N}"},
+            "cpu_baseline": {"value": value, "unit": "rows/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{n} rows of S1, std::stable_sort + memcmp oracle, single thread"},
+            "e2e": {"value": value, "unit": "rows/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_sort(args):
+    import torch
+    import torch.distributed as dist
+
+    import blugen
+    from paper_conf_sigmod_merajispcksygnk16_b200 import blugby as bg
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream(dev)
+    n = args.rows or SORT_N
+    rows_np = blugen.sort_rows(n, SORT_W, seed=blugen.SORT_SEED + rank)  # every rank its own rows (weak)
+    rows = torch.from_numpy(rows_np).to(dev)
+    flush = torch.empty(512 * 2**20, dtype=torch.uint8, device=dev)
+    for _ in range(args.warmup):
+        flush.zero_()
+        perm, stats = bg.blu_sort_rows(rows, stream=stream)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    sampler = ClockSampler(local if not args.no_clocks else -1)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler.start()
+    time.sleep(1.0)  # nvidia-smi (NVML) start-up stalls the driver for ~0.5 s: let it finish first
+    c0 = bg.blu_gby_launch_count()
+    ds_ms, ds_bytes, ds_launch = [], [], []
+    for i in range(args.steps):
+        flush.zero_()
+        ev[i][0].record(stream)
+        perm, stats = bg.blu_sort_rows(rows, stream=stream)
+        ev[i][1].record(stream)
+        ds_ms.append(stats["downsweep_ms"])
+        ds_bytes.append(stats["downsweep_bytes"])
+        ds_launch.append(stats["downsweep_launches"])
+    torch.cuda.synchronize()
+    launches = bg.blu_gby_launch_count() - c0
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop()
+    tot_ms = sum(a.elapsed_time(b) for a, b in ev)
+    if world > 1:
+        t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        tot_ms = float(t.item())
+    value = n * world * args.steps / (tot_ms / 1000.0)
+    peak, peak_src = load_peaks()
+    per_launch_ms = sum(ds_ms) / max(1, sum(ds_launch))
+    per_launch_bytes = sum(ds_bytes) / max(1, sum(ds_launch))
+    achieved = per_launch_bytes / (per_launch_ms / 1000.0) / 1e9
+    tr = load_traffic("S1")
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": tr[0] if tr[0] else None, "kernel": "k_rs_downsweep (radix pass: read + scatter of key, payload)",
+                "algorithmic_bytes_per_launch": per_launch_bytes, "avg_launch_ms": per_launch_ms,
+                "launches_per_step": sum(ds_launch) / args.steps,
+                "share_of_step": sum(ds_ms) / tot_ms, "peak_source": peak_src,
+                "levels": stats["levels"], "active_rows_per_level": stats["active"], "ms_per_level": stats["ms"]}
+    e2e = None
+    if not args.no_e2e and world == 1:
+        hrows = rows.cpu().pin_memory()
+        hperm = torch.empty(n, dtype=torch.int32).pin_memory()
+        e_steps = min(3, args.steps)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(e_steps):
+            d = hrows.to(dev, non_blocking=True)
+            p, _ = bg.blu_sort_rows(d, stream=stream)
+            hperm.copy_(p, non_blocking=True)
+            torch.cuda.synchronize()
+        dt = (time.perf_counter() - t0) / e_steps
+        e2e = {"value": n / dt, "unit": "rows/s", "h2d_bytes_per_step": n * SORT_W, "d2h_bytes_per_step": n * 4,
+               "ms_per_step": dt * 1000, "note": "pinned host rows -> device, blu_sort_rows, permutation -> host"}
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        m = 2_000_000
+        cpu = {"value": sort_cpu(rows_np, m), "unit": "rows/s", "cores": 1, "kind": "oracle",
+               "sample": f"first {m} rows of S1, std::stable_sort + memcmp oracle, single thread"}
+    if rank == 0:
+        line = {"metric": SORT_METRIC, "value": value, "unit": "rows/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": tot_ms / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+                "config": {"workload": f"S1: sort offload, {n} rows x {SORT_W}-byte keys (date 1823, store 502, "
+                                       f"8 random bytes), stable permutation", "rows_per_gpu": n,
+                           "parallelism": f"replicas x{world}",
+                           "l2": "flushed between steps (512 MB memset, outside step events); inputs > L2"},
+                "input_gbs": value * SORT_W / 1e9, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                "gpu_launches": launches, "clocks": clocks}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+# ----------------------------------------------------------------------------------------------
 # GPU leg
 # ----------------------------------------------------------------------------------------------
 def main():
@@ -176,7 +310,8 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5"])
+    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5", "S1"],
+                    help="C1-C5: GROUP BY configs (BASELINE.json); S1: the sort offload (NEXT-4, P:76-88)")
     ap.add_argument("--impl", default="blugby", choices=["blugby", "reference"])
     ap.add_argument("--rows", type=int, default=None, help="override rows per rank (testing only)")
     ap.add_argument("--no-e2e", action="store_true")
@@ -185,7 +320,9 @@ def main():
     args = ap.parse_args()
     args.warmup = max(3, args.warmup)
     if args.impl == "reference":
-        return run_reference(args)
+        return run_sort_reference(args) if args.config == "S1" else run_reference(args)
+    if args.config == "S1":
+        return run_sort(args)
 
     import torch
     import torch.distributed as dist
@@ -241,7 +378,7 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     sampler.start()
-    time.sleep(0.15)
+    time.sleep(1.0)  # nvidia-smi (NVML) start-up stalls the driver for ~0.5 s: let it finish first
     c0 = bg.blu_gby_launch_count()
     for i in range(args.steps):
         flush.zero_()

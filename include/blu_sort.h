@@ -49,6 +49,11 @@ typedef struct {
     uint64_t ranges[256];   /* ranges[l] = duplicate ranges left after level l                        */
     uint64_t active[256];   /* active[l] = rows inside those ranges (the next level's job size)      */
     float ms[256];          /* device time of level l (sort + range detection), CUDA events          */
+    /* the dominant kernel, the radix downsweep (read + scatter of keys and payloads), timed per
+       launch with CUDA events on `stream`: summed time, launches, algorithmic bytes moved          */
+    float downsweep_ms;
+    uint32_t downsweep_launches;
+    uint64_t downsweep_bytes;
 } blu_sort_stats_t;
 
 /* P:76-86, the whole job queue: perm_out[p] (DEVICE, n u32) = the row at position p of the stable

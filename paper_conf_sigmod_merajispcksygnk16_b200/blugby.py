@@ -70,7 +70,8 @@ class TimingC(ctypes.Structure):
 
 class SortStatsC(ctypes.Structure):
     _fields_ = [("levels", ctypes.c_uint32), ("ranges", ctypes.c_uint64 * 256), ("active", ctypes.c_uint64 * 256),
-                ("ms", ctypes.c_float * 256)]
+                ("ms", ctypes.c_float * 256), ("downsweep_ms", ctypes.c_float), ("downsweep_launches", ctypes.c_uint32),
+                ("downsweep_bytes", ctypes.c_uint64)]
 
 
 def _load():
@@ -520,5 +521,7 @@ def blu_sort_rows(rows, stream=None):
     st = SortStatsC()
     _check(lib.blu_sort_rows(_ptr(rows), n, W, _ptr(perm), _stream_handle(stream), ctypes.byref(st)))
     L = st.levels
-    stats = {"levels": L, "ranges": list(st.ranges[:L]), "active": list(st.active[:L]), "ms": list(st.ms[:L])}
+    stats = {"levels": L, "ranges": list(st.ranges[:L]), "active": list(st.active[:L]), "ms": list(st.ms[:L]),
+             "downsweep_ms": st.downsweep_ms, "downsweep_launches": st.downsweep_launches,
+             "downsweep_bytes": st.downsweep_bytes}
     return perm, stats

@@ -127,7 +127,7 @@ struct CacheBlock {
 static std::mutex g_cache_mu;
 static std::vector<CacheBlock> g_cache;
 
-static cudaError_t cache_get(void** out, size_t bytes) {
+cudaError_t cache_get(void** out, size_t bytes) {
   int dev = 0;
   cudaGetDevice(&dev);
   bytes = (bytes + (2u << 20) - 1) & ~(size_t)((2u << 20) - 1);
@@ -173,7 +173,7 @@ static size_t cache_idle_bytes() {
   return t;
 }
 
-static void cache_put(void* p) {
+void cache_put(void* p) {
   std::lock_guard<std::mutex> lk(g_cache_mu);
   for (auto& b : g_cache)
     if (b.p == p) b.busy = false;

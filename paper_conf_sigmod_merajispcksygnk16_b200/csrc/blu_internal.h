@@ -95,6 +95,11 @@ int launch_partition(const Layout& lay, const void* const* key_cols, const void*
 
 void count_launch(uint64_t n);
 
+// Workspace block cache (api.cu): cudaMalloc'd blocks reused across calls; a block may be put back
+// only after the stream that used it has been synchronised.
+cudaError_t cache_get(void** out, size_t bytes);
+void cache_put(void* p);
+
 // NVRTC specialisation (jit.cpp)
 bool jit_enabled();
 struct JitProbe {  // compile-only mode of the JIT (blu_gby_jit_probe)

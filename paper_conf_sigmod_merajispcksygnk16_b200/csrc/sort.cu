@@ -15,6 +15,7 @@
 #include <stdint.h>
 #include <stdio.h>
 #include <string.h>
+#include <time.h>
 
 #include <algorithm>
 #include <vector>
@@ -30,7 +31,7 @@ constexpr int kRT = 256;  // threads per radix CTA (= number of digits: thread d
 
 template <typename KT>
 struct RadixCfg {
-  static constexpr int ITEMS = sizeof(KT) == 4 ? 16 : 8;  // keys per thread per tile
+  static constexpr int ITEMS = 8;                          // keys per thread per tile
   static constexpr int WARP_CHUNK = 32 * ITEMS;           // contiguous keys per warp
   static constexpr int TILE = kRT * ITEMS;
 };
@@ -103,17 +104,65 @@ __global__ void __launch_bounds__(1024) k_rs_scan(uint32_t* a, uint64_t L) {
   }
 }
 
+// Exclusive scan of each digit's row of the count matrix (CTA d scans counts[d][0..G), coalesced,
+// 256 at a time); the row total goes to digit_tot[d]. The downsweep adds the digit bases itself.
+__global__ void __launch_bounds__(kRT) k_rs_scan_rows(uint32_t* __restrict__ counts, uint32_t G,
+                                                      uint32_t* __restrict__ digit_tot) {
+  __shared__ uint32_t ws[kRT / 32];
+  uint32_t* row = counts + (uint64_t)blockIdx.x * G;
+  const unsigned lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint32_t carry = 0;
+  for (uint32_t c0 = 0; c0 < G; c0 += kRT) {
+    const uint32_t c = c0 + threadIdx.x;
+    const uint32_t x = c < G ? row[c] : 0u;
+    uint32_t inc = x;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+      if ((int)lane >= o) inc += y;
+    }
+    if (lane == 31) ws[w] = inc;
+    __syncthreads();
+    uint32_t before = 0, tot = 0;
+    for (unsigned q = 0; q < kRT / 32; ++q) {
+      if (q < w) before += ws[q];
+      tot += ws[q];
+    }
+    if (c < G) row[c] = carry + before + inc - x;
+    carry += tot;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) digit_tot[blockIdx.x] = carry;
+}
+
 template <typename KT>
-__global__ void __launch_bounds__(kRT) k_rs_downsweep(const KT* __restrict__ kin, const uint32_t* __restrict__ vin,
+__global__ void __launch_bounds__(kRT, 4) k_rs_downsweep(const KT* __restrict__ kin, const uint32_t* __restrict__ vin,
                                                       KT* __restrict__ kout, uint32_t* __restrict__ vout, uint64_t n,
-                                                      uint32_t shift, const uint32_t* __restrict__ offsets) {
+                                                      uint32_t shift, const uint32_t* __restrict__ offsets,
+                                                      const uint32_t* __restrict__ digit_tot) {
   using C = RadixCfg<KT>;
   __shared__ uint32_t base[256];
   __shared__ uint32_t ttot[256];
+  __shared__ uint32_t tstart[256];
+  __shared__ uint32_t wsum[kRT / 32];
   __shared__ uint32_t wcnt[kRT / 32][256];
+  __shared__ KT sk[C::TILE];
+  __shared__ uint32_t sv[C::TILE];
   const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint32_t lt_mask = (1u << lane) - 1u;
-  base[threadIdx.x] = offsets[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x];
+  {  // digit bases: exclusive scan of the 256 digit totals (thread d owns digit d)
+    const uint32_t x = digit_tot[threadIdx.x];
+    uint32_t inc = x;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+      if ((int)lane >= o) inc += y;
+    }
+    if (lane == 31) ttot[warp] = inc;
+    __syncthreads();
+    uint32_t before = 0;
+    for (unsigned q = 0; q < warp; ++q) before += ttot[q];
+    base[threadIdx.x] = before + inc - x + offsets[(uint64_t)threadIdx.x * gridDim.x + blockIdx.x];
+    __syncthreads();
+  }
   uint64_t t0, t1;
   tile_span((n + C::TILE - 1) / C::TILE, t0, t1);
   for (uint64_t t = t0; t < t1; ++t) {
@@ -147,6 +196,7 @@ __global__ void __launch_bounds__(kRT) k_rs_downsweep(const KT* __restrict__ kin
       __syncwarp();
     }
     __syncthreads();
+    uint32_t tot_d;
     {  // per digit: exclusive prefix over the warps, tile total
       uint32_t run = 0;
 #pragma unroll
@@ -155,19 +205,64 @@ __global__ void __launch_bounds__(kRT) k_rs_downsweep(const KT* __restrict__ kin
         wcnt[w][threadIdx.x] = run;
         run += x;
       }
-      ttot[threadIdx.x] = run;
+      tot_d = run;
+    }
+    {  // tile-local start of each digit: exclusive scan of the tile totals over the 256 digits
+      uint32_t inc = tot_d;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if ((int)lane >= o) inc += y;
+      }
+      if (lane == 31) wsum[warp] = inc;
+      __syncthreads();
+      uint32_t before = 0;
+      for (unsigned q = 0; q < warp; ++q) before += wsum[q];
+      tstart[threadIdx.x] = before + inc - tot_d;
+      ttot[threadIdx.x] = tot_d;
     }
     __syncthreads();
+    // stage the tile in digit order in shared memory ...
 #pragma unroll
     for (int i = 0; i < C::ITEMS; ++i) {
       if (b + (uint64_t)i * 32 >= n) continue;
       const uint32_t d = digit_of(k[i], shift);
-      const uint32_t pos = base[d] + wcnt[warp][d] + rank[i];
-      kout[pos] = k[i];
-      vout[pos] = v[i];
+      const uint32_t lp = tstart[d] + wcnt[warp][d] + rank[i];
+      sk[lp] = k[i];
+      sv[lp] = v[i];
+    }
+    __syncthreads();
+    // ... then write it out: consecutive threads write consecutive addresses of each digit's run
+    const uint64_t tile0 = t * C::TILE;
+    const uint32_t cnt = (uint32_t)(n - tile0 < (uint64_t)C::TILE ? n - tile0 : (uint64_t)C::TILE);
+    for (uint32_t e = threadIdx.x; e < cnt; e += kRT) {
+      const KT key = sk[e];
+      const uint32_t d = digit_of(key, shift);
+      const uint32_t pos = base[d] + (e - tstart[d]);
+      kout[pos] = key;
+      vout[pos] = sv[e];
     }
     __syncthreads();
     base[threadIdx.x] += ttot[threadIdx.x];
+  }
+}
+
+// OR and AND of all keys: a digit whose 8 bits agree in both is the same for every key, and its
+// LSD pass is the identity permutation (skipped).
+template <typename KT>
+__global__ void k_key_bits(const KT* __restrict__ keys, uint64_t n, unsigned long long* __restrict__ or_and) {
+  unsigned long long o = 0, a = ~0ull;
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const unsigned long long k = (unsigned long long)keys[i];
+    o |= k;
+    a &= k;
+  }
+  for (int s = 16; s; s >>= 1) {
+    o |= __shfl_xor_sync(0xffffffffu, o, s);
+    a &= __shfl_xor_sync(0xffffffffu, a, s);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicOr(or_and, o);
+    atomicAnd(or_and + 1, a);
   }
 }
 
@@ -328,6 +423,14 @@ uint32_t elem_grid(uint64_t n) {
   return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(g, (uint64_t)sms_now() * 16));
 }
 
+struct CachedBuf {  // workspace from the block cache (callers synchronise before it is released)
+  void* p = nullptr;
+  cudaError_t alloc(size_t b) { return cache_get(&p, std::max<size_t>(b, 16)); }
+  ~CachedBuf() {
+    if (p) cache_put(p);
+  }
+};
+
 struct DevBuf {  // stream-ordered scratch
   void* p = nullptr;
   cudaStream_t st;
@@ -338,21 +441,64 @@ struct DevBuf {  // stream-ordered scratch
   }
 };
 
+// Per-launch CUDA events around the downsweeps (blu_sort_stats_t), read after the caller syncs.
+struct RsTiming {
+  std::vector<cudaEvent_t> ev;
+  size_t used = 0;
+  uint64_t bytes = 0;
+  cudaEvent_t next() {
+    if (used == ev.size()) {
+      cudaEvent_t e;
+      cudaEventCreate(&e);
+      ev.push_back(e);
+    }
+    return ev[used++];
+  }
+  ~RsTiming() {
+    for (auto e : ev) cudaEventDestroy(e);
+  }
+};
+
 // Stable LSD radix sort of the low `bits` key bits: (kin, vin) -> (kout, vout); kt/vt scratch (n).
 template <typename KT>
 cudaError_t radix_sort(const KT* kin, const uint32_t* vin, KT* kout, uint32_t* vout, KT* kt, uint32_t* vt, uint64_t n,
-                       uint32_t bits, uint32_t* counts, uint32_t grid, cudaStream_t st) {
+                       uint32_t bits, uint32_t* counts, uint32_t grid, cudaStream_t st, RsTiming* tm = nullptr) {
   if (n == 0) return cudaSuccess;
-  const int passes = std::max(1, (int)((bits + 7) / 8));
+  // digits that vary (one small reduction + one synchronisation)
+  int digits[8], passes = 0;
+  {
+    unsigned long long* oa = (unsigned long long*)(counts + (size_t)256 * (grid + 1));
+    const unsigned long long init[2] = {0ull, ~0ull};
+    cudaError_t e = cudaMemcpyAsync(oa, init, 16, cudaMemcpyHostToDevice, st);
+    if (e) return e;
+    k_key_bits<KT><<<elem_grid(n), 256, 0, st>>>(kin, n, oa);
+    count_launch(1);
+    unsigned long long h[2];
+    if ((e = cudaMemcpyAsync(h, oa, 16, cudaMemcpyDeviceToHost, st)) || (e = cudaStreamSynchronize(st))) return e;
+    const int nd = std::max(1, (int)((bits + 7) / 8));
+    for (int p = 0; p < nd; ++p)
+      if ((((h[0] ^ h[1]) >> (8 * p)) & 255ull) != 0) digits[passes++] = p;
+  }
+  if (passes == 0) {  // every key equal: the stable order is the input order
+    cudaError_t e = cudaMemcpyAsync(kout, kin, n * sizeof(KT), cudaMemcpyDeviceToDevice, st);
+    if (!e) e = cudaMemcpyAsync(vout, vin, n * 4, cudaMemcpyDeviceToDevice, st);
+    return e;
+  }
   const KT* sk = kin;
   const uint32_t* sv = vin;
   for (int p = 0; p < passes; ++p) {
     const bool to_out = ((passes - 1 - p) % 2) == 0;
     KT* dk = to_out ? kout : kt;
     uint32_t* dv = to_out ? vout : vt;
-    k_rs_upsweep<KT><<<grid, kRT, 0, st>>>(sk, n, 8u * p, counts);
-    k_rs_scan<<<1, 1024, 0, st>>>(counts, (uint64_t)256 * grid);
-    k_rs_downsweep<KT><<<grid, kRT, 0, st>>>(sk, sv, dk, dv, n, 8u * p, counts);
+    const uint32_t shift = 8u * (uint32_t)digits[p];
+    k_rs_upsweep<KT><<<grid, kRT, 0, st>>>(sk, n, shift, counts);
+    k_rs_scan_rows<<<256, kRT, 0, st>>>(counts, grid, counts + (size_t)256 * grid);
+    if (tm) cudaEventRecord(tm->next(), st);
+    k_rs_downsweep<KT><<<grid, kRT, 0, st>>>(sk, sv, dk, dv, n, shift, counts, counts + (size_t)256 * grid);
+    if (tm) {
+      cudaEventRecord(tm->next(), st);
+      tm->bytes += 2ull * n * (sizeof(KT) + 4);
+    }
     count_launch(3);
     sk = dk;
     sv = dv;
@@ -440,7 +586,7 @@ blu_status_t blu_sort_pairs(const uint32_t* keys_in, const uint32_t* payload_in,
   cudaStream_t st = (cudaStream_t)stream;
   const uint32_t grid = radix_grid();
   DevBuf w(st);
-  SCK(w.alloc((size_t)n * 8 + (size_t)256 * grid * 4), "sort workspace");
+  SCK(w.alloc((size_t)n * 8 + (size_t)256 * (grid + 1) * 4 + 64), "sort workspace");
   uint32_t* kt = (uint32_t*)w.p;
   uint32_t* vt = kt + n;
   uint32_t* counts = vt + n;
@@ -477,10 +623,19 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
     cudaEventSynchronize(e1);
     cudaEventElapsedTime(&stats->ms[l], e0, e1);
   };
-  // workspace: level-0 keys/payload scratch (u32) + level keys (u64 x2) + payload x2 + pos/seg x2
-  DevBuf w(st);
-  const size_t need = (size_t)n * (4 + 4 + 8 + 8 + 8 + 4 + 4 + 4 + 4 * 4) + (size_t)256 * grid * 4 + 256;
+  // workspace: level-0 keys/payload scratch (u32) + level keys (u64 x3) + payload x3 + pos/seg x2;
+  // from the block cache (every level ends with a synchronisation, so it is idle on return)
+  static const bool dbg = getenv("BLU_SORT_DEBUG") != nullptr;
+  auto hnow = [] {
+    timespec ts;
+    clock_gettime(CLOCK_MONOTONIC, &ts);
+    return ts.tv_sec * 1e3 + ts.tv_nsec * 1e-6;
+  };
+  const double h0 = hnow();
+  CachedBuf w;
+  const size_t need = (size_t)n * (4 + 4 + 8 + 8 + 8 + 4 + 4 + 4 + 4 * 4) + (size_t)256 * (grid + 1) * 4 + 256;
   SCK(w.alloc(need), "sort workspace");
+  if (dbg) fprintf(stderr, "[blu_sort] workspace %.3f ms\n", hnow() - h0);
   uint8_t* q = (uint8_t*)w.p;
   auto take = [&](size_t b) {
     uint8_t* r = q;
@@ -499,12 +654,14 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
   uint32_t* seg0 = (uint32_t*)take(n * 4);
   uint32_t* pos1 = (uint32_t*)take(n * 4);
   uint32_t* seg1 = (uint32_t*)take(n * 4);
-  uint32_t* counts = (uint32_t*)take((size_t)256 * grid * 4);
+  uint32_t* counts = (uint32_t*)take((size_t)256 * (grid + 1) * 4 + 64);
   if (stats) cudaEventRecord(e0, st);
   // level 0: the whole buffer is one job ("Initially there is only one job")
   k_partial_keys<uint32_t><<<elem_grid(n), 256, 0, st>>>(rows, n, W, 0, k32a, pa);
   count_launch(1);
-  SCK(radix_sort<uint32_t>(k32a, pa, k32b, perm_out, (uint32_t*)k64c, pc, n, 32, counts, grid, st), "level 0 sort");
+  RsTiming rtm;
+  RsTiming* tm = stats ? &rtm : nullptr;
+  SCK(radix_sort<uint32_t>(k32a, pa, k32b, perm_out, (uint32_t*)k64c, pc, n, 32, counts, grid, st, tm), "level 0 sort");
   uint64_t m = 0, nr = 0;
   blu_status_t s = dup_pass<uint32_t>(k32b, n, nullptr, pos0, seg0, nullptr, nullptr, 0, &m, &nr, st);
   if (s != BLU_OK) return s;
@@ -522,7 +679,7 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
     while (bits_seg < 32 && (1ull << bits_seg) < nr) ++bits_seg;
     k_level_keys<<<elem_grid(m), 256, 0, st>>>(rows, W, word, pos0, seg0, perm_out, m, k64a, pa);
     count_launch(1);
-    SCK(radix_sort<uint64_t>(k64a, pa, k64b, pb, k64c, pc, m, 32 + bits_seg, counts, grid, st), "level sort");
+    SCK(radix_sort<uint64_t>(k64a, pa, k64b, pb, k64c, pc, m, 32 + bits_seg, counts, grid, st, tm), "level sort");
     k_level_scatter<<<elem_grid(m), 256, 0, st>>>(pos0, pb, m, perm_out);
     count_launch(1);
     uint64_t m2 = 0, nr2 = 0;
@@ -532,6 +689,7 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
     std::swap(seg0, seg1);
     m = m2;
     nr = nr2;
+    if (dbg) fprintf(stderr, "[blu_sort] level %u done at %.3f ms (m=%llu)\n", level, hnow() - h0, (unsigned long long)m);
     if (stats && level < 256) {
       stats->ranges[level] = nr;
       stats->active[level] = m;
@@ -542,6 +700,14 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
     stats->levels = level;
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
+    cudaStreamSynchronize(st);
+    for (size_t i = 0; i + 1 < rtm.used; i += 2) {
+      float x = 0;
+      cudaEventElapsedTime(&x, rtm.ev[i], rtm.ev[i + 1]);
+      stats->downsweep_ms += x;
+      stats->downsweep_launches += 1;
+    }
+    stats->downsweep_bytes = rtm.bytes;
   }
   SCK(cudaGetLastError(), "sort rows");
   return BLU_OK;
