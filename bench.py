@@ -259,9 +259,12 @@ def run_sort(args):
     per_launch_ms = sum(ds_ms) / max(1, sum(ds_launch))
     per_launch_bytes = sum(ds_bytes) / max(1, sum(ds_launch))
     achieved = per_launch_bytes / (per_launch_ms / 1000.0) / 1e9
-    tr = load_traffic("S1")
+    traffic = None
+    sp = os.path.join(ROOT, "profiles", "ncu_S1_summary.json")
+    if os.path.exists(sp):  # DRAM bytes / algorithmic bytes of the captured downsweep, per average launch
+        traffic = json.load(open(sp)).get("traffic_over_algorithmic", 0) * per_launch_bytes or None
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": tr[0] if tr[0] else None, "kernel": "k_rs_downsweep (radix pass: read + scatter of key, payload)",
+                "traffic": traffic, "kernel": "k_rs_downsweep (radix pass: read + scatter of key, payload)",
                 "algorithmic_bytes_per_launch": per_launch_bytes, "avg_launch_ms": per_launch_ms,
                 "launches_per_step": sum(ds_launch) / args.steps,
                 "share_of_step": sum(ds_ms) / tot_ms, "peak_source": peak_src,

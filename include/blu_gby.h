@@ -219,6 +219,23 @@ blu_status_t blu_gby_merge_records(blu_gby_plan_t plan, const void* records, uin
                                    void* stream, int32_t partial_out, blu_gby_result_t* out);
 uint32_t blu_gby_record_bytes(blu_gby_plan_t plan);
 
+/* Rows mode of the hash-path exchange (chosen when est_groups >= rows per rank,
+ * i.e. partial states would not be smaller than the rows): raw ROWS are bucketed by owner and the
+ * owner aggregates them. Row records are (W + n_vals) 64-bit words: the packed key as above, then
+ * every value column as 64 bits (i32 sign-extended, f64 bits). blu_gby_partition_rows writes the
+ * n_rows rows of key_cols / val_cols (DEVICE, the execute layout) into send_buf (DEVICE, capacity
+ * n_rows x row record bytes) by owner, sets send_counts[p] (HOST), and synchronises `stream`.
+ * Errors: BLU_E_KEY_RANGE (a key outside its dictionary / negative sparse code; nothing usable is
+ * written), BLU_E_UNSUPPORTED for 128-bit payloads. blu_gby_execute_records runs S4-S8 over
+ * n_records such records (DEVICE) with a hash table sized from the plan's estimate: the rows this
+ * rank owns, aggregated into a finalized (or partial) result. */
+blu_status_t blu_gby_partition_rows(blu_gby_plan_t plan, const void* const* key_cols, const void* const* val_cols,
+                                    uint64_t n_rows, int32_t n_parts, void* stream, void* send_buf,
+                                    uint64_t* send_counts);
+blu_status_t blu_gby_execute_records(blu_gby_plan_t plan, const void* records, uint64_t n_records, void* stream,
+                                     int32_t partial_out, blu_gby_result_t* out);
+uint32_t blu_gby_row_record_bytes(blu_gby_plan_t plan);
+
 /* ---- group-count estimate --------------------------------------------
  * KMV ("K-minimum values") estimate of the number of distinct key tuples in n_rows DEVICE key
  * columns — the estimate the paper computes on CPU threads right after hashing and feeds to the GPU

@@ -95,6 +95,9 @@ def _load():
         "blu_gby_partition": ([vp, P(ResultC), i32, vp, vp, P(u64)], i32),
         "blu_gby_merge_records": ([vp, vp, u64, vp, i32, P(ResultC)], i32),
         "blu_gby_record_bytes": ([vp], u32),
+        "blu_gby_row_record_bytes": ([vp], u32),
+        "blu_gby_partition_rows": ([vp, P(vp), P(vp), u64, i32, vp, vp, P(u64)], i32),
+        "blu_gby_execute_records": ([vp, vp, u64, vp, i32, P(ResultC)], i32),
         "blu_gby_estimate_groups": ([P(KeyDesc), i32, P(vp), u64, u32, vp, P(ctypes.c_double), P(i32)], i32),
         "blu_gby_slot_template": ([vp, vp, u32, P(u32)], i32),
         "blu_gby_init_table": ([vp, vp, u64, vp], i32),
@@ -198,6 +201,10 @@ class Plan:
     @property
     def record_bytes(self) -> int:
         return int(lib.blu_gby_record_bytes(self.handle))
+
+    @property
+    def row_record_bytes(self) -> int:
+        return int(lib.blu_gby_row_record_bytes(self.handle))
 
 
 def blu_gby_plan(keys: Sequence[Tuple[int, int]], vals: Sequence[int], aggs: Sequence[Tuple[int, int]],
@@ -403,6 +410,26 @@ def blu_gby_partition(plan: Plan, partial: Result, n_parts: int, send_buf, strea
     counts = (ctypes.c_uint64 * n_parts)()
     _check(lib.blu_gby_partition(plan.handle, ctypes.byref(partial.c), n_parts, s, _ptr(send_buf), counts))
     return [int(c) for c in counts]
+
+
+def blu_gby_partition_rows(plan: Plan, key_cols, val_cols, n_parts: int, send_buf, n_rows: Optional[int] = None,
+                           stream=None) -> List[int]:
+    """Rows mode of the exchange: raw rows bucketed by owner rank into send_buf (row records)."""
+    n = int(len(key_cols[0]) if n_rows is None else n_rows)
+    s = _stream_handle(stream)
+    counts = (ctypes.c_uint64 * n_parts)()
+    _check(lib.blu_gby_partition_rows(plan.handle, _ptrs(key_cols), _ptrs(val_cols), n, n_parts, s, _ptr(send_buf),
+                                      counts))
+    return [int(c) for c in counts]
+
+
+def blu_gby_execute_records(plan: Plan, records, n_records: int, stream=None, partial_out: bool = False) -> Result:
+    """S4-S8 over row records (the rows this rank owns after a rows-mode exchange)."""
+    s = _stream_handle(stream)
+    rc = ResultC()
+    _check(lib.blu_gby_execute_records(plan.handle, _ptr(records), int(n_records), s, int(partial_out),
+                                       ctypes.byref(rc)))
+    return Result(rc, _key_dtypes(plan), _out_dtypes(plan, partial_out), s, getattr(records, "device", None))
 
 
 def dense_state_arrays(plan: Plan, device="cuda"):

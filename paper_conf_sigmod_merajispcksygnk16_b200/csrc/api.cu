@@ -1012,6 +1012,52 @@ blu_status_t blu_gby_finalize_dense_state(blu_gby_plan_t P, void* const* state_a
   return run_core(P, L, P->path, false, L.domain, L.domain, feed, false, st, out, false, nullptr);
 }
 
+blu_status_t blu_gby_execute_records(blu_gby_plan_t P, const void* records, uint64_t n, void* stream, int32_t partial_out,
+                                     blu_gby_result_t* out) {
+  if (!P || !out || (n && !records)) return fail(BLU_E_INVALID, "bad execute_records arguments");
+  if (P->lay.has_q) return fail(BLU_E_UNSUPPORTED, "execute_records: 128-bit payloads have no record format");
+  cudaStream_t st = (cudaStream_t)stream;
+  const Layout& L = P->lay;
+  uint64_t est = std::max<uint64_t>(1, std::min<uint64_t>(n, std::max<uint64_t>(P->est_groups, 1)));
+  uint64_t cap = 1024;
+  while ((double)cap * 0.7 < (double)est) cap <<= 1;
+  uint32_t grid = (uint32_t)P->sms * 8, block = 256;
+  RecSrc rs{(const uint64_t*)records, (uint32_t)((L.key_words == 2 ? 2 : 1) + L.n_vals)};
+  Feeder feed = [&](AggParams& base, uint32_t* launches, Work&, const FinalParams*) -> cudaError_t {
+    if (!n) return cudaSuccess;
+    return agg_batch(P, BLU_PATH_HASH_GLOBAL, base, nullptr, nullptr, n, &rs, st, grid, block, 0, launches);
+  };
+  return run_core(P, L, BLU_PATH_HASH_GLOBAL, false, cap, n, feed, partial_out != 0, st, out, false, nullptr);
+}
+
+blu_status_t blu_gby_partition_rows(blu_gby_plan_t P, const void* const* key_cols, const void* const* val_cols,
+                                    uint64_t n, int32_t n_parts, void* stream, void* send_buf, uint64_t* send_counts) {
+  if (!P || !send_counts || n_parts < 1 || n_parts > 1024) return fail(BLU_E_INVALID, "bad partition_rows arguments");
+  if (P->lay.has_q) return fail(BLU_E_UNSUPPORTED, "partition_rows: 128-bit payloads have no record format");
+  if (n && (!send_buf || !nonnull_cols(key_cols, P->lay.n_keys) || !nonnull_cols(val_cols, P->lay.n_vals)))
+    return fail(BLU_E_INVALID, "NULL column or send_buf");
+  cudaStream_t st = (cudaStream_t)stream;
+  setup_pool();
+  if (!n) {
+    for (int i = 0; i < n_parts; ++i) send_counts[i] = 0;
+    return BLU_OK;
+  }
+  Work w(st);
+  void* tmp = nullptr;
+  CK(w.alloc(&tmp, 16 * (size_t)n_parts + 16), "partition workspace");
+  CK(cudaMemsetAsync(tmp, 0, 16 * (size_t)n_parts + 16, st), "memset");
+  uint64_t* d_counts = (uint64_t*)tmp;
+  uint64_t* d_offs = d_counts + n_parts;
+  uint32_t* d_flags = (uint32_t*)(d_offs + n_parts);
+  CK(launch_partition(P->lay, key_cols, val_cols, n, n_parts, send_buf, d_counts, d_offs, st, d_flags), "partition rows");
+  uint32_t flags = 0;
+  CK(cudaMemcpyAsync(send_counts, d_counts, 8 * (size_t)n_parts, cudaMemcpyDeviceToHost, st), "counts D2H");
+  CK(cudaMemcpyAsync(&flags, d_flags, 4, cudaMemcpyDeviceToHost, st), "flags D2H");
+  CK(cudaStreamSynchronize(st), "sync");
+  if (flags & FLAG_KEY_RANGE) return fail(BLU_E_KEY_RANGE, "a key code is outside its dictionary (or negative)");
+  return BLU_OK;
+}
+
 blu_status_t blu_gby_partition(blu_gby_plan_t P, const blu_gby_result_t* partial, int32_t n_parts, void* stream, void* send_buf,
                                uint64_t* send_counts) {
   if (!P || !partial || !send_counts || n_parts < 1 || n_parts > 1024) return fail(BLU_E_INVALID, "bad partition arguments");

@@ -91,7 +91,7 @@ int launch_read_roofline(const void* const* cols, const uint64_t* bytes, int n_c
                          int sms);
 int launch_partition(const Layout& lay, const void* const* key_cols, const void* const* state_cols,
                      uint64_t n, int32_t n_parts, void* send_buf, uint64_t* d_counts, uint64_t* d_offsets,
-                     void* stream);
+                     void* stream, uint32_t* d_flags = nullptr);
 
 void count_launch(uint64_t n);
 

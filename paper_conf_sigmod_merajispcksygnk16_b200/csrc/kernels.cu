@@ -635,7 +635,18 @@ struct PartParams {
   uint64_t* offsets;  // n_parts
   uint64_t* out;
   uint32_t words;
+  uint32_t* flags;    // rows mode: FLAG_KEY_RANGE if a key code is outside its dictionary (else NULL)
 };
+
+// rows mode: a key code outside [0, dict) (or a negative sparse code) would pack into another key
+__device__ __forceinline__ bool row_keys_bad(const PartParams& p, uint64_t i) {
+  const Layout& L = p.lay;
+  for (int k = 0; k < L.n_keys; ++k) {
+    const int64_t c = L.key_dtype[k] == BLU_I32 ? (int64_t)((const int32_t*)p.key[k])[i] : ((const int64_t*)p.key[k])[i];
+    if (c < 0 || (L.dict[k] && (uint64_t)c >= L.dict[k])) return true;
+  }
+  return false;
+}
 
 __device__ __forceinline__ void pack_row_wide(const PartParams& p, uint64_t i, uint64_t& w0, uint64_t& w1) {
   const Layout& L = p.lay;
@@ -666,6 +677,10 @@ __device__ __forceinline__ uint32_t owner_of(uint64_t key, int32_t P) { return (
 __global__ void __launch_bounds__(256) k_partition_hist(PartParams p) {
   uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.n; i += stride) {
+    if (p.flags && row_keys_bad(p, i)) {
+      atomicOr(p.flags, FLAG_KEY_RANGE);
+      continue;
+    }
     uint32_t o;
     if (p.lay.key_words == 2) {
       uint64_t w0, w1;
@@ -681,6 +696,7 @@ __global__ void __launch_bounds__(256) k_partition_hist(PartParams p) {
 __global__ void __launch_bounds__(256) k_partition_scatter(PartParams p) {
   uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.n; i += stride) {
+    if (p.flags && row_keys_bad(p, i)) continue;
     const int kw = p.lay.key_words == 2 ? 2 : 1;
     uint64_t key = 0, key1 = 0;
     uint32_t o;
@@ -1063,7 +1079,8 @@ int launch_compact(const CompactParams& p, void* stream, uint32_t* launches) {
 }
 
 int launch_partition(const Layout& lay, const void* const* key_cols, const void* const* state_cols, uint64_t n,
-                     int32_t n_parts, void* send_buf, uint64_t* d_counts, uint64_t* d_offsets, void* stream) {
+                     int32_t n_parts, void* send_buf, uint64_t* d_counts, uint64_t* d_offsets, void* stream,
+                     uint32_t* d_flags) {
   // two-phase: histogram -> (host) offsets -> scatter. The caller passes d_counts zeroed; this
   // launcher runs the histogram, copies counts to the host, scans, uploads offsets, re-zeroes the
   // cursors and scatters.
@@ -1078,6 +1095,7 @@ int launch_partition(const Layout& lay, const void* const* key_cols, const void*
   p.offsets = d_offsets;
   p.out = (uint64_t*)send_buf;
   p.words = (lay.key_words == 2 ? 2 : 1) + lay.n_vals;
+  p.flags = d_flags;
   int grid = grid_for(n, 256, 148 * 8);
   k_partition_hist<<<grid, 256, 0, st>>>(p);
   count_launch(1);

@@ -595,6 +595,10 @@ uint32_t blu_gby_record_bytes(blu_gby_plan_t P) {
   return P ? 8u * ((P->lay.key_words == 2 ? 2u : 1u) + (uint32_t)P->lay.n_fields) : 0u;
 }
 
+uint32_t blu_gby_row_record_bytes(blu_gby_plan_t P) {
+  return P ? 8u * ((P->lay.key_words == 2 ? 2u : 1u) + (uint32_t)P->lay.n_vals) : 0u;
+}
+
 blu_status_t blu_gby_slot_template(blu_gby_plan_t P, void* out, uint32_t cap, uint32_t* slot_bytes) {
   if (!P) return fail(BLU_E_INVALID, "NULL plan");
   if (slot_bytes) *slot_bytes = P->lay.slot_bytes;

@@ -8,9 +8,12 @@ the plan's path:
   * dense state (paths a / b'): every rank holds the same D x fields state arrays; four
     all-reduces (int64 SUM, f64 SUM, int64 MIN, int64 MAX) combine them; every rank finalizes the
     same replicated result;
-  * hash path (b): each rank emits per-group partial states, buckets them by owner rank
-    (mulhi(fmix64(key), P), bits independent of the slot bits), exchanges them with an
-    all-to-all-v and merges what it owns; the result is distributed by key range.
+  * hash path (b), partials mode (default when the rank's rows outnumber the estimated groups):
+    each rank emits per-group partial states, buckets them by owner rank (mulhi(fmix64(key), P),
+    bits independent of the slot bits), exchanges them with an all-to-all-v and merges what it
+    owns; the result is distributed by key range;
+  * hash path (b), rows mode (est_groups >= rows per rank: partial states would be as large as
+    the rows): the raw rows are bucketed by owner, exchanged, and aggregated by their owner.
 
 The collective orchestration (`allreduce_dense_state`, `alltoallv_records`) only moves tensors; all
 GROUP BY arithmetic stays in libblugby.
@@ -48,9 +51,17 @@ def alltoallv_records(send: torch.Tensor, send_counts: List[int], words: int, gr
     return recv[: sum(recv_counts) * words]
 
 
-def dist_execute(plan, key_cols, val_cols, group=None, stream=None):
+def exchange_mode(plan, n_local: int, mode=None) -> str:
+    """'rows' when the estimate says partial states would not be smaller than the
+    rows (est_groups >= rows on this rank), else 'partials'; an explicit mode wins."""
+    if mode in ("rows", "partials"):
+        return mode
+    return "rows" if plan.info()["est_groups"] >= max(1, n_local) else "partials"
+
+
+def dist_execute(plan, key_cols, val_cols, group=None, stream=None, mode=None):
     """Whole-job GROUP BY of this rank's rows; returns (result, mode). Dense paths: replicated
-    finalized result; hash path: this rank's owned groups."""
+    finalized result; hash path: this rank's owned groups (mode 'partials' or 'rows')."""
     from . import blugby as bg
     P = dist.get_world_size(group)
     info = plan.info()
@@ -60,6 +71,13 @@ def dist_execute(plan, key_cols, val_cols, group=None, stream=None):
         if P > 1:
             allreduce_dense_state(st, group)
         return bg.blu_gby_finalize_dense_state(plan, st, stream=stream), "allreduce"
+    n_local = int(len(key_cols[0]))
+    if P > 1 and exchange_mode(plan, n_local, mode) == "rows":
+        words = plan.row_record_bytes // 8
+        send = torch.empty(max(1, n_local) * words, dtype=torch.int64, device=key_cols[0].device)
+        counts = bg.blu_gby_partition_rows(plan, key_cols, val_cols, P, send, stream=stream)
+        recv = alltoallv_records(send, counts, words, group)
+        return bg.blu_gby_execute_records(plan, recv, recv.numel() // words, stream=stream), "rows"
     part = bg.blu_gby_execute_partial(plan, key_cols, val_cols, stream=stream)
     if P == 1:
         return bg.blu_gby_merge(plan, [part], stream=stream), "local"
@@ -67,4 +85,4 @@ def dist_execute(plan, key_cols, val_cols, group=None, stream=None):
     send = torch.empty(max(1, part.n_groups) * words, dtype=torch.int64, device=key_cols[0].device)
     counts = bg.blu_gby_partition(plan, part, P, send, stream=stream)
     recv = alltoallv_records(send, counts, words, group)
-    return bg.blu_gby_merge_records(plan, recv, recv.numel() // words, stream=stream), "alltoall"
+    return bg.blu_gby_merge_records(plan, recv, recv.numel() // words, stream=stream), "partials"

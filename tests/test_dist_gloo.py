@@ -94,3 +94,22 @@ def test_bench_reference_arm_cpu():
     line = json.loads(out.stdout.strip().splitlines()[-1])
     assert line["impl"] == "reference" and line["value"] > 0 and line["unit"] == "rows/s"
     assert line["cpu_baseline"]["kind"] == "oracle" and line["e2e"]["h2d_bytes_per_step"] == 0
+
+
+def test_exchange_mode_rule():
+    """rows mode when est_groups >= rows on this rank, partials otherwise; an
+    explicit mode wins."""
+    bd = _dist_module()
+
+    class Stub:
+        def __init__(self, est):
+            self.est = est
+
+        def info(self):
+            return {"est_groups": self.est}
+
+    assert bd.exchange_mode(Stub(50_000_000), 500_000_000) == "partials"   # C5 at P = 8
+    assert bd.exchange_mode(Stub(50_000_000), 10_000_000) == "rows"        # as many groups as rows
+    assert bd.exchange_mode(Stub(10), 10) == "rows"
+    assert bd.exchange_mode(Stub(10**9), 5, mode="partials") == "partials"
+    assert bd.exchange_mode(Stub(1), 10**9, mode="rows") == "rows"

@@ -414,6 +414,54 @@ def test_partitioned_with_regrow(bg, oracles, monkeypatch, smem):
     assert_parity(gk, ga, o, w.schema)
 
 
+@pytest.mark.parametrize("name", ["C3", "C2", "C4"])
+def test_partition_rows_exchange(bg, oracles, name):
+    """S10 rows mode simulated on one GPU: each of P 'ranks' buckets its raw rows
+    by owner (blu_gby_partition_rows); each owner aggregates the row records it would receive
+    (blu_gby_execute_records). The union of the owners' results equals the full result — sparse
+    keys (C3) and dense composite keys (C2, C4: mixed-radix packed keys unpacked by the owner)."""
+    w, o = oracles(name)
+    kc, vc = blugen.device_columns(w)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    P = 4
+    cuts = np.linspace(0, w.n_rows, P + 1).astype(int)
+    rb = plan.row_record_bytes
+    assert rb == 8 * (1 + len(w.schema.vals))
+    inbox = [[] for _ in range(P)]
+    for r in range(P):
+        n = int(cuts[r + 1] - cuts[r])
+        buf = torch.empty(max(1, n) * rb // 8, dtype=torch.int64, device="cuda")
+        counts = bg.blu_gby_partition_rows(plan, [k[cuts[r]:cuts[r + 1]] for k in kc],
+                                           [v[cuts[r]:cuts[r + 1]] for v in vc], P, buf)
+        assert sum(counts) == n
+        off = 0
+        for dst in range(P):
+            inbox[dst].append(buf[off * rb // 8:(off + counts[dst]) * rb // 8])
+            off += counts[dst]
+    keys, aggs = [], []
+    for dst in range(P):
+        recs = torch.cat(inbox[dst])
+        res = bg.blu_gby_execute_records(plan, recs, recs.numel() * 8 // rb)
+        gk, ga = gpu_sorted(res, w.schema)
+        keys.append(gk)
+        aggs.append(ga)
+    allk = np.concatenate(keys)
+    order = np.lexsort(allk.T[::-1])
+    assert_parity(allk[order], [np.concatenate([a[i] for a in aggs])[order] for i in range(len(w.schema.aggs))],
+                  o, w.schema)
+
+
+def test_partition_rows_key_range(bg):
+    sch = blugen.Schema([(I32, 10)], [I64], [(COUNT, -1), (SUM, 0)])
+    k = np.array([1, 2, 10, 3], np.int32)  # 10 is outside the dictionary
+    dk, dv = _mk([k], [np.arange(4, dtype=np.int64)])
+    plan = bg.plan_for(sch, 4, 4)
+    buf = torch.empty(16 * 4, dtype=torch.int64, device="cuda")
+    with pytest.raises(bg.BluError) as e:
+        bg.blu_gby_partition_rows(plan, dk, dv, 2, buf)
+    assert e.value.status == bg.BLU_E_KEY_RANGE
+
+
 def _kmv_reference(keys_packed, k):
     """Independent numpy statement of the KMV estimate (same definition, no shared code):
     h = fmix64(packed ^ salt); est = (k-1) * 2^64 / (k-th smallest distinct h), exact if < k."""

@@ -22,11 +22,18 @@ if [ "$WHAT" = ncu ] || [ "$WHAT" = all ]; then
       env ITERS=3 python tools/phase_probe.py C3 > /dev/null 2>&1
   ncu --set full --clock-control none --import-source on -k regex:"blu_jit_global" -s 2 -c 1 -o $O/${TAG}_prof_C4 \
       env ITERS=3 python tools/phase_probe.py C4 > /dev/null 2>&1
+  # sort offload (NEXT-4): launch list and one radix downsweep (a level-2 pass: random digits)
+  ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/${TAG}_launches_S1.csv \
+      python bench.py --config S1 --steps 1 --warmup 3 --no-e2e --no-cpu > /dev/null 2>&1
+  ncu --set full --clock-control none --import-source on -k regex:"k_rs_downsweep" -s 40 -c 1 -o $O/${TAG}_prof_S1 \
+      python bench.py --config S1 --steps 1 --warmup 3 --no-e2e --no-cpu > /dev/null 2>&1
 fi
 if [ "$WHAT" = bench ] || [ "$WHAT" = all ]; then
   python bench.py --steps 200 --warmup 5 > $O/${TAG}_bench_C2.json 2> $O/${TAG}_bench_C2.err
   for c in C1 C3 C4 C5; do
     python bench.py --config $c --steps 10 --warmup 3 --no-e2e --no-cpu > $O/${TAG}_bench_$c.json 2>> $O/${TAG}_bench_$c.err
   done
+  python bench.py --config S1 --steps 10 --warmup 3 > $O/${TAG}_bench_S1.json 2> $O/${TAG}_bench_S1.err
   python bench.py --impl reference --steps 5 --warmup 3 > $O/${TAG}_bench_ref.json 2> $O/${TAG}_bench_ref.err
+  python bench.py --impl reference --config S1 --steps 3 --warmup 1 > $O/${TAG}_bench_ref_S1.json 2> $O/${TAG}_bench_ref_S1.err
 fi
