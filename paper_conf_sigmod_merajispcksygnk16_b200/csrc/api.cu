@@ -71,7 +71,7 @@ static uint64_t* pinned_scratch() {
   return p;
 }
 
-static void setup_pool() {
+void setup_pool() {
   static std::once_flag once;
   std::call_once(once, [] {
     int dev = 0;

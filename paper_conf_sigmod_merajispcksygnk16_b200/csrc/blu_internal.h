@@ -98,6 +98,7 @@ void count_launch(uint64_t n);
 // Workspace block cache (api.cu): cudaMalloc'd blocks reused across calls; a block may be put back
 // only after the stream that used it has been synchronised.
 cudaError_t cache_get(void** out, size_t bytes);
+void setup_pool();  // stream-ordered pool keeps its memory (release threshold = max)
 void cache_put(void* p);
 
 // NVRTC specialisation (jit.cpp)

@@ -442,7 +442,7 @@ struct DevBuf {  // stream-ordered scratch
 };
 
 // Per-launch CUDA events around the downsweeps (blu_sort_stats_t), read after the caller syncs.
-struct RsTiming {
+struct RsTiming {  // events are created once per thread and reused (creating them takes driver locks)
   std::vector<cudaEvent_t> ev;
   size_t used = 0;
   uint64_t bytes = 0;
@@ -454,10 +454,12 @@ struct RsTiming {
     }
     return ev[used++];
   }
-  ~RsTiming() {
-    for (auto e : ev) cudaEventDestroy(e);
+  void reset() {
+    used = 0;
+    bytes = 0;
   }
 };
+thread_local RsTiming t_rs;
 
 // Stable LSD radix sort of the low `bits` key bits: (kin, vin) -> (kout, vout); kt/vt scratch (n).
 template <typename KT>
@@ -468,8 +470,8 @@ cudaError_t radix_sort(const KT* kin, const uint32_t* vin, KT* kout, uint32_t* v
   int digits[8], passes = 0;
   {
     unsigned long long* oa = (unsigned long long*)(counts + (size_t)256 * (grid + 1));
-    const unsigned long long init[2] = {0ull, ~0ull};
-    cudaError_t e = cudaMemcpyAsync(oa, init, 16, cudaMemcpyHostToDevice, st);
+    cudaError_t e = cudaMemsetAsync(oa, 0, 8, st);
+    if (!e) e = cudaMemsetAsync(oa + 1, 0xFF, 8, st);
     if (e) return e;
     k_key_bits<KT><<<elem_grid(n), 256, 0, st>>>(kin, n, oa);
     count_launch(1);
@@ -524,13 +526,16 @@ blu_status_t cuda_err(cudaError_t e, const char* what) {
 template <typename KT>
 blu_status_t dup_pass(const KT* k, uint64_t m, const uint32_t* act_pos, uint32_t* next_pos, uint32_t* next_seg,
                       uint64_t* r_start, uint64_t* r_len, uint64_t cap, uint64_t* n_act, uint64_t* n_rng,
-                      cudaStream_t st) {
+                      cudaStream_t st, void* ws = nullptr) {
   *n_act = *n_rng = 0;
   if (m == 0) return BLU_OK;
   const uint64_t nb = (m + kDB - 1) / kDB;
   DevBuf w(st);
-  SCK(w.alloc(nb * 8 + 16), "dup workspace");
-  uint32_t* ca = (uint32_t*)w.p;
+  if (!ws) {
+    SCK(w.alloc(nb * 8 + 16), "dup workspace");
+    ws = w.p;
+  }
+  uint32_t* ca = (uint32_t*)ws;
   uint32_t* cs = ca + nb;
   uint32_t* tot = cs + nb;  // 2 totals
   k_dup_count<KT><<<(unsigned)nb, kDT, 0, st>>>(k, m, ca, cs);
@@ -584,6 +589,7 @@ blu_status_t blu_sort_pairs(const uint32_t* keys_in, const uint32_t* payload_in,
     return fail(BLU_E_INVALID, "outputs alias inputs");
   if (!n) return BLU_OK;
   cudaStream_t st = (cudaStream_t)stream;
+  setup_pool();
   const uint32_t grid = radix_grid();
   DevBuf w(st);
   SCK(w.alloc((size_t)n * 8 + (size_t)256 * (grid + 1) * 4 + 64), "sort workspace");
@@ -599,6 +605,7 @@ blu_status_t blu_sort_dup_ranges(const uint32_t* sorted_keys, uint64_t n, uint64
   if (!n_ranges || (n && !sorted_keys) || (cap && (!starts || !lens))) return fail(BLU_E_INVALID, "NULL pointer");
   if (n >= (1ull << 32)) return fail(BLU_E_INVALID, "n >= 2^32");
   uint64_t na = 0;
+  setup_pool();
   return dup_pass<uint32_t>(sorted_keys, n, nullptr, nullptr, nullptr, cap ? starts : nullptr, cap ? lens : nullptr, cap, &na,
                             n_ranges, (cudaStream_t)stream);
 }
@@ -612,11 +619,12 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
   if (!n) return BLU_OK;
   cudaStream_t st = (cudaStream_t)stream;
   const uint32_t grid = radix_grid();
-  cudaEvent_t e0 = nullptr, e1 = nullptr;
-  if (stats) {
+  static thread_local cudaEvent_t e0 = nullptr, e1 = nullptr;
+  if (stats && !e0) {
     cudaEventCreate(&e0);
     cudaEventCreate(&e1);
   }
+  setup_pool();
   auto level_time = [&](uint32_t l) {
     if (!stats || l >= 256) return;
     cudaEventRecord(e1, st);
@@ -633,7 +641,8 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
   };
   const double h0 = hnow();
   CachedBuf w;
-  const size_t need = (size_t)n * (4 + 4 + 8 + 8 + 8 + 4 + 4 + 4 + 4 * 4) + (size_t)256 * (grid + 1) * 4 + 256;
+  const size_t need = (size_t)n * (4 + 4 + 8 + 8 + 8 + 4 + 4 + 4 + 4 * 4) + (size_t)256 * (grid + 1) * 4 + 256 +
+                      ((n + kDB - 1) / kDB) * 8 + 64;
   SCK(w.alloc(need), "sort workspace");
   if (dbg) fprintf(stderr, "[blu_sort] workspace %.3f ms\n", hnow() - h0);
   uint8_t* q = (uint8_t*)w.p;
@@ -655,15 +664,17 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
   uint32_t* pos1 = (uint32_t*)take(n * 4);
   uint32_t* seg1 = (uint32_t*)take(n * 4);
   uint32_t* counts = (uint32_t*)take((size_t)256 * (grid + 1) * 4 + 64);
+  void* dws = take(((n + kDB - 1) / kDB) * 8 + 16);  // duplicate-range block counts
   if (stats) cudaEventRecord(e0, st);
   // level 0: the whole buffer is one job ("Initially there is only one job")
   k_partial_keys<uint32_t><<<elem_grid(n), 256, 0, st>>>(rows, n, W, 0, k32a, pa);
   count_launch(1);
-  RsTiming rtm;
+  RsTiming& rtm = t_rs;
+  rtm.reset();
   RsTiming* tm = stats ? &rtm : nullptr;
   SCK(radix_sort<uint32_t>(k32a, pa, k32b, perm_out, (uint32_t*)k64c, pc, n, 32, counts, grid, st, tm), "level 0 sort");
   uint64_t m = 0, nr = 0;
-  blu_status_t s = dup_pass<uint32_t>(k32b, n, nullptr, pos0, seg0, nullptr, nullptr, 0, &m, &nr, st);
+  blu_status_t s = dup_pass<uint32_t>(k32b, n, nullptr, pos0, seg0, nullptr, nullptr, 0, &m, &nr, st, dws);
   if (s != BLU_OK) return s;
   uint32_t level = 1;
   if (stats) {
@@ -683,7 +694,7 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
     k_level_scatter<<<elem_grid(m), 256, 0, st>>>(pos0, pb, m, perm_out);
     count_launch(1);
     uint64_t m2 = 0, nr2 = 0;
-    s = dup_pass<uint64_t>(k64b, m, pos0, pos1, seg1, nullptr, nullptr, 0, &m2, &nr2, st);
+    s = dup_pass<uint64_t>(k64b, m, pos0, pos1, seg1, nullptr, nullptr, 0, &m2, &nr2, st, dws);
     if (s != BLU_OK) return s;
     std::swap(pos0, pos1);
     std::swap(seg0, seg1);
@@ -698,8 +709,6 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
   }
   if (stats) {
     stats->levels = level;
-    cudaEventDestroy(e0);
-    cudaEventDestroy(e1);
     cudaStreamSynchronize(st);
     for (size_t i = 0; i + 1 < rtm.used; i += 2) {
       float x = 0;
