@@ -719,10 +719,16 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
         if (((uintptr_t)keys[k] & 15) != 0) vec = 0;
       }
       pk.vec_ok = (int32_t)vec;
+      // path (b'): a rank image when the bitmap of the domain fits the front's key region
+      const bool no_rank = getenv("BLU_GBY_NO_RANK_FRONT") != nullptr;
+      const uint64_t W = (L.domain + 31) / 32;
+      const uint32_t rank_words =
+          P->path == BLU_PATH_DIRECT_GLOBAL && !no_rank && L.domain > 0 && W <= base.front_slots ? (uint32_t)W : 0u;
       const uint64_t* front = nullptr;
-      int rc = launch_front_seed(pk, n, base.front_slots, ws, st, (int)P->sms, &front);
+      int rc = launch_front_seed(pk, n, base.front_slots, rank_words, ws, st, (int)P->sms, &front);
       if (rc) return (cudaError_t)rc;
       base.front_seed = front;
+      base.front_rank_words = rank_words;
     }
     if (P->path == BLU_PATH_HASH_GLOBAL && P->parts > 1 && n >= 4096 * (uint64_t)P->parts)
       return partitioned_feed(P, base, keys, vals, n, st, launches, w);

@@ -952,12 +952,29 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
     bool deduped = false;
     if constexpr (FRONT && SP::kStatic) {
       if constexpr (SP::DEDUPE) {  // opt-in (BLU_GBY_DEDUPE=1): pays off only for extreme skew
-        front_dedupe_rows<SP, NV, R, DIRECT>(p, sm, key, valid, v);
-        miss = 0;
-        deduped = true;
+        if (!p.front_rank_words) {
+          front_dedupe_rows<SP, NV, R, DIRECT>(p, sm, key, valid, v);
+          miss = 0;
+          deduped = true;
+        }
       }
     }
-    if (FRONT && !deduped) {
+    if (FRONT && DIRECT && p.front_rank_words && !deduped) {
+      // rank front: a dense key k is hot iff bit k%32 of word k/32 is set; its entry is the word's
+      // prefix plus the hot keys below it in the word. Converged, one LDS.64 per row, no probe loop.
+      const uint64_t* img = (const uint64_t*)(sm + p.key_off);
+      uint32_t fe[R];
+      uint32_t hit = 0;
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        const uint64_t x = (valid >> r & 1) ? img[key[r] >> 5] : 0ull;
+        const uint32_t b = (uint32_t)key[r] & 31u, bits = (uint32_t)x;
+        fe[r] = (uint32_t)(x >> 32) + __popc(bits & ((1u << b) - 1u));
+        hit |= (bits >> b & 1u) << r;
+      }
+      smem_apply_rows<SP, NV, R>(p, sm, fe, hit, v);
+      miss = valid & ~hit;
+    } else if (FRONT && !deduped) {
       // hot-key front: small open-addressing table per CTA in shared memory
       uint64_t* fk = (uint64_t*)(sm + p.key_off);
       const bool seeded = p.front_seed != nullptr;
@@ -1060,6 +1077,24 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
     __syncthreads();
     const uint64_t* fk = (const uint64_t*)(sm + p.key_off);
     const int cf = L.count_field;
+    if (DIRECT && p.front_rank_words) {  // rank front: entry prefix + j holds key 32w + (j-th set bit)
+      for (uint32_t w = threadIdx.x; w < p.front_rank_words; w += blockDim.x) {
+        const uint64_t x = fk[w];
+        uint32_t bits = (uint32_t)x, e = (uint32_t)(x >> 32);
+        for (; bits; bits &= bits - 1, ++e) {
+          if (s_read<FK_COUNT>(sm + p.soff[cf], e, S) == 0) continue;
+          const uint64_t g = (uint64_t)w * 32 + (uint64_t)(__ffs(bits) - 1);
+          for (int j = 0; j < L.n_fields; ++j) {
+            const uint8_t* b = sm + p.soff[j];
+            dispatch_kind(L.f[j].kind, [&](auto kc) {
+              constexpr int K = decltype(kc)::v;
+              d_upd<K, false>(dense_addr(p, j, g), s_read<K>(b, e, S));
+            });
+          }
+        }
+      }
+      return;
+    }
     for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) {
       const uint64_t key = fk[e];
       if (key == kEmpty) continue;

@@ -85,7 +85,7 @@ int launch_init_dense(const Layout& lay, void* const dense[4], uint64_t D, void*
                       uint32_t n_zero = 0);
 int launch_compact(const CompactParams& p, void* stream, uint32_t* launches);
 size_t front_seed_bytes(uint32_t S);
-int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, void* ws, void* stream, int sms,
+int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, uint32_t rank_words, void* ws, void* stream, int sms,
                       const uint64_t** front_out);
 int launch_read_roofline(const void* const* cols, const uint64_t* bytes, int n_cols, void* stream, uint64_t* out,
                          int sms);

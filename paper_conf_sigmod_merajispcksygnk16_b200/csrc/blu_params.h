@@ -122,6 +122,11 @@ struct AggParams {
   // front's open-addressing image; CTAs copy it and only look keys up (no inserts). NULL = the
   // front is filled first-come with CAS inserts.
   const uint64_t* front_seed;
+  // rank front (path b' only, dense domain D <= 32 * S): the seed is a rank image instead of a key
+  // table. Word w (< front_rank_words = ceil(D / 32)) holds in its low half the bitmap of the hot
+  // keys 32w..32w+31 and in its high half the number of hot keys below 32w, so a key's front entry is
+  // that prefix + popc(bits below it): one shared-memory load per row, no probing. 0 = hash front.
+  uint32_t front_rank_words;
   uint32_t prefetch;             // scatter: L2-prefetch the column bytes of the tile this many tiles ahead (0 = off)
   // partitioned pass 2 with bucket-local shared-memory tables (bucket_body): a bucket's rows are
   // cut into pieces of piece_rows rows (a multiple of the CTA tile); aux_off = byte offset of the

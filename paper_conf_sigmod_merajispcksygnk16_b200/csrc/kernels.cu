@@ -810,14 +810,51 @@ __global__ void __launch_bounds__(256) k_hh_build(HHParams h) {
   }
 }
 
+// Rank front (path b'): the hot keys' bits in the low halves of the image words (bit k%32 of word
+// k/32), then one CTA writes each word's prefix count of hot keys into its high half.
+__global__ void __launch_bounds__(256) k_hh_build_rank(HHParams h) {
+  const uint32_t t = h.ctl[0];
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < h.cap_s; i += (uint64_t)gridDim.x * blockDim.x) {
+    if (h.scnt[i] < t) continue;
+    if (atomicAdd(&h.ctl[1], 1u) >= h.K) continue;
+    const uint64_t key = h.skey[i];  // a valid dense code: < D <= 32 * rank_words
+    atomicOr((uint32_t*)(h.front + (key >> 5)), 1u << (key & 31));  // low half (little endian)
+  }
+}
+
+__global__ void __launch_bounds__(1024) k_hh_rank_scan(HHParams h, uint32_t words) {
+  __shared__ uint32_t wsum[32];
+  __shared__ uint32_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (uint32_t w0 = 0; w0 < words; w0 += blockDim.x) {
+    const uint32_t w = w0 + threadIdx.x;
+    const uint32_t c = w < words ? (uint32_t)__popc((uint32_t)h.front[w]) : 0u;
+    uint32_t inc = c;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+      if ((int)lane >= o) inc += y;
+    }
+    if (lane == 31) wsum[warp] = inc;
+    __syncthreads();
+    uint32_t before = carry;
+    for (unsigned q = 0; q < warp; ++q) before += wsum[q];
+    if (w < words) h.front[w] = (uint64_t)(uint32_t)h.front[w] | ((uint64_t)(before + inc - c) << 32);
+    __syncthreads();
+    if (threadIdx.x == blockDim.x - 1) carry = before + inc;
+    __syncthreads();
+  }
+}
+
 size_t front_seed_bytes(uint32_t S) { return (size_t)S * 8 + ((size_t)1 << 18) * 12 + kHHBins * 4 + 64; }
 
-int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, void* ws, void* stream, int sms,
-                      const uint64_t** front_out) {
+int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, uint32_t rank_words, void* ws, void* stream,
+                      int sms, const uint64_t** front_out) {
   cudaStream_t st = (cudaStream_t)stream;
   HHParams h{};
   h.S = S;
-  h.K = S / 2;
+  h.K = rank_words ? S : S / 2;  // the rank front has no load-factor slack
   h.cap_s = (uint64_t)1 << 18;
   uint8_t* w = (uint8_t*)ws;
   h.front = (uint64_t*)w;
@@ -832,13 +869,20 @@ int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, void* ws, v
   if (h.blocks <= 1) h.block_rows = n;
   k_fill_u64<<<grid_for((uint64_t)S + h.cap_s, 256, sms * 8), 256, 0, st>>>(h.front, (uint64_t)S + h.cap_s, kEmpty);
   cudaMemsetAsync(h.scnt, 0, h.cap_s * 4 + kHHBins * 4 + 64, st);
+  if (rank_words) cudaMemsetAsync(h.front, 0, (size_t)S * 8, st);  // empty bitmap, zero prefixes
   AggParams p = base;
   p.n_rows = n;
   k_hh_count<<<sms * 2, 512, 0, st>>>(p, h);
   k_hh_hist<<<sms, 256, 0, st>>>(h);
   k_hh_pick<<<1, 32, 0, st>>>(h);
-  k_hh_build<<<sms, 256, 0, st>>>(h);
-  count_launch(5);
+  if (rank_words) {
+    k_hh_build_rank<<<sms, 256, 0, st>>>(h);
+    k_hh_rank_scan<<<1, 1024, 0, st>>>(h, rank_words);
+    count_launch(6);
+  } else {
+    k_hh_build<<<sms, 256, 0, st>>>(h);
+    count_launch(5);
+  }
   *front_out = h.front;
   return (int)cudaGetLastError();
 }

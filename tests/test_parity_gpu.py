@@ -82,6 +82,40 @@ def test_forced_paths_identical(bg, oracles, monkeypatch, name, paths, front):
         assert_parity(gk, ga, o, w.schema)
 
 
+@pytest.mark.parametrize("rank", ["1", "0"])
+@pytest.mark.parametrize("dicts,n", [((13, 7), 200_003), ((64, 1024), 1_048_583), ((100, 20, 20), 700_001)])
+def test_rank_front(bg, monkeypatch, rank, dicts, n):
+    """Path (b') hot-key front as a rank image (bitmap + per-word prefix) vs the hash front: both equal
+    the oracle. D = 91, D = 32 * S exactly (S = 2048 front entries for this schema), D = 4 * 10^4.
+    Skewed keys so the seeded front fills up; rows of cold keys take the global REDs."""
+    rng = np.random.default_rng(sum(dicts) + n)
+    D = int(np.prod(dicts))
+    sch = blugen.Schema([(I32, d) for d in dicts], [I32, I64, F64], ALL(3))
+    r = np.minimum(rng.zipf(1.3, n) - 1, D - 1)          # heavy head, long tail, max code present
+    perm = rng.permutation(D)
+    g = perm[r]
+    g[:3] = [0, D - 1, D // 2]
+    kc, rem = [], g
+    for d in dicts:
+        kc.append((rem % d).astype(np.int32))
+        rem = rem // d
+    vc = [rng.integers(-(2**31), 2**31, n).astype(np.int32), rng.integers(-(2**62), 2**62, n).astype(np.int64),
+          rng.integers(-(2**20), 2**20, n) / 64.0]
+    o = oracle.groupby_arrays(sch, kc, vc)
+    monkeypatch.setenv("BLU_GBY_FORCE_PATH", "d")
+    monkeypatch.setenv("BLU_GBY_HOT_FRONT", "1")
+    if rank == "0":
+        monkeypatch.setenv("BLU_GBY_NO_RANK_FRONT", "1")
+    plan = bg.plan_for(sch, D, n)
+    info = plan.info()
+    assert info["hot_front"] == 1 and info["path"] == bg.BLU_PATH_DIRECT_GLOBAL
+    assert (D + 31) // 32 <= info["front_slots"]
+    dk, dv = _mk(kc, vc)
+    res = bg.blu_gby_execute(plan, dk, dv)
+    gk, ga = gpu_sorted(res, sch)
+    assert_parity(gk, ga, o, sch)
+
+
 @pytest.mark.parametrize("est", [1, 1000, 60_000, 2_000_003])
 def test_est_groups_invariance_and_regrow(bg, oracles, est):
     """Under-estimates take the error path: regrow and rerun, same exact result."""
