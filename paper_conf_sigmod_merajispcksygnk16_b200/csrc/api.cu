@@ -705,6 +705,9 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
   const bool single = n <= (((uint64_t)P->grid * (1ull << 30)) & ~3ull);
   Feeder feed = [&](AggParams& base, uint32_t* launches, Work& w, const FinalParams* fin) -> cudaError_t {
     base.jit_ok = L.key_words == 2 ? 0 : 1;
+    // path (b)/(b') one pass: each warp L2-prefetches its next tile (BLU_GBY_AGG_PREFETCH=0/1)
+    const char* ap = getenv("BLU_GBY_AGG_PREFETCH");
+    base.prefetch = ap ? (uint32_t)atoi(ap) : 0u;
     // hot-key front seeded with the heavy hitters of a row sample (needs a COUNT field to tell
     // seeded keys that received rows from those that did not)
     static const bool no_seed = getenv("BLU_GBY_NO_SEED") != nullptr;

@@ -255,6 +255,33 @@ __device__ __forceinline__ uint64_t enc(uint64_t x) {
   return x;
 }
 
+// Warp-level L2 prefetch of rows [r0, min(r0 + rows, n)) of every key and value column: lane l takes
+// the column's 128-byte lines l, l + 32, ... (C4: 3 i32 keys + i32 + 2 i64 values over 128 rows =
+// 32 lines, one per lane). Issued for the warp's next tile before it works on the current one.
+template <class SP>
+__device__ __forceinline__ void prefetch_warp_rows_l2(const AggParams& p, uint64_t r0, uint64_t rows, uint64_t n,
+                                                      unsigned lane) {
+  if (r0 >= n) return;
+  const uint64_t r1 = r0 + rows < n ? r0 + rows : n;
+  auto col = [&](const void* base, uint32_t w) {
+    const uintptr_t a0 = ((uintptr_t)base + r0 * w) & ~(uintptr_t)127, a1 = (uintptr_t)base + r1 * w;
+    for (uintptr_t a = a0 + (uintptr_t)lane * 128; a < a1; a += 32 * 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(a));
+  };
+  if constexpr (SP::kStatic) {
+    sfor<0, SP::NK>([&](auto kc) {
+      constexpr int k = decltype(kc)::v;
+      col(p.key[k], SP::KDT[k] == BLU_I32 ? 4u : 8u);
+    });
+    sfor<0, SP::NV>([&](auto cc) {
+      constexpr int c = decltype(cc)::v;
+      col(p.val[c], SP::VDT[c] == BLU_I32 ? 4u : 8u);
+    });
+  } else {
+    for (int k = 0; k < p.lay.n_keys; ++k) col(p.key[k], p.lay.key_dtype[k] == BLU_I32 ? 4u : 8u);
+    for (int c = 0; c < p.lay.n_vals; ++c) col(p.val[c], p.lay.val_dtype[c] == BLU_I32 ? 4u : 8u);
+  }
+}
+
 // Shared-memory table (path (a) and the hot-key front): SoA per field, S entries per field.
 // Encodings: COUNT u32; SUMI as two u32 arrays lo[S], hi[S] — native 32-bit ATOMS with an explicit
 // carry (64-bit shared atomics are CAS loops on sm_100a); SUMF f64 (CAS loop);
@@ -591,9 +618,103 @@ __device__ __forceinline__ void dense_finalize_block(const AggParams& p, const F
   if (threadIdx.x == 0) *fp.n_groups = base_s;
 }
 
+// ---- software-pipelined row stream (NVRTC-specialised kernels only: dense PIPE, global MODE 3) --
+// A warp issues the loads of its next tile before it unpacks and aggregates the current one, so the
+// HBM reads of tile t+1 are in flight during the work on tile t (without it, every tile waited the
+// full load latency right after issuing: 53% of C4's stall samples sat on the first use of a load).
+// Loaded words stay raw (i32 columns: one register; 8-byte columns: two) until the tile is unpacked.
+template <class SP, int R>
+struct RawTile {
+  static constexpr int NKC = SP::NK, NVC = SP::NV > 0 ? SP::NV : 1;
+  uint32_t klo[NKC][R], khi[NKC][R], vlo[NVC][R], vhi[NVC][R];
+};
+
+// Issue the loads of this lane's R rows of one column (PAIR mapping, R even); rows >= n read 0.
+template <int R, bool W64>
+__device__ __forceinline__ void load_raw(const void* base, uint64_t lb, uint64_t n, uint32_t vec, uint64_t pol,
+                                         uint32_t (&lo)[R], uint32_t (&hi)[R]) {
+#pragma unroll
+  for (int h = 0; h < R / 2; ++h) {
+    const uint64_t r0 = lb + (uint64_t)h * 64;
+    if (vec && r0 + 1 < n) {
+      if constexpr (W64) {
+        const int4 x = ld_stream_v4((const uint64_t*)base + r0, pol);
+        lo[2 * h] = (uint32_t)x.x, hi[2 * h] = (uint32_t)x.y, lo[2 * h + 1] = (uint32_t)x.z, hi[2 * h + 1] = (uint32_t)x.w;
+      } else {
+        const int2 x = ld_stream_v2((const int32_t*)base + r0, pol);
+        lo[2 * h] = (uint32_t)x.x, lo[2 * h + 1] = (uint32_t)x.y;
+      }
+    } else {
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        const uint64_t rr = r0 + q;
+        if constexpr (W64) {
+          const uint64_t x = rr < n ? ld_stream_u64((const uint64_t*)base + rr, pol) : 0ull;
+          lo[2 * h + q] = (uint32_t)x, hi[2 * h + q] = (uint32_t)(x >> 32);
+        } else {
+          lo[2 * h + q] = rr < n ? (uint32_t)ld_stream_s32((const int32_t*)base + rr, pol) : 0u;
+        }
+      }
+    }
+  }
+}
+
+template <class SP, int R>
+__device__ __forceinline__ void tile_load(const AggParams& p, uint64_t lb, uint64_t n, uint64_t pol, RawTile<SP, R>& T) {
+  sfor<0, SP::NK>([&](auto kc) {
+    constexpr int k = decltype(kc)::v;
+    load_raw<R, SP::KDT[k] != BLU_I32>(p.key[k], lb, n, p.vec_ok, pol, T.klo[k], T.khi[k]);
+  });
+  sfor<0, SP::NV>([&](auto cc) {
+    constexpr int c = decltype(cc)::v;
+    load_raw<R, SP::VDT[c] != BLU_I32>(p.val[c], lb, n, p.vec_ok, pol, T.vlo[c], T.vhi[c]);
+  });
+}
+
+// Raw words -> packed keys (S1, CCAT P:111, with the range check of pack_keys) and 64-bit values.
+template <class SP, int NV, int R>
+__device__ __forceinline__ uint32_t tile_unpack(const AggParams& p, const RawTile<SP, R>& T, uint64_t lb, uint64_t n,
+                                                uint64_t (&key)[R], uint64_t (&v)[NV][R]) {
+  uint32_t valid = 0, bad = 0;
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    key[r] = 0;
+    if (row_of<R>(lb, r) < n) valid |= 1u << r;
+  }
+  sfor<0, SP::NK>([&](auto kc) {
+    constexpr int k = decltype(kc)::v;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const uint64_t c = SP::KDT[k] == BLU_I32 ? (uint64_t)(int64_t)(int32_t)T.klo[k][r]
+                                               : ((uint64_t)T.khi[k][r] << 32 | T.klo[k][r]);
+      if constexpr (SP::SPARSE) {
+        key[r] = c;
+        if ((int64_t)c < 0) bad |= 1u << r;
+      } else {
+        if (c >= SP::DICT[k]) bad |= 1u << r;  // unsigned: negatives are huge
+        key[r] += c * SP::STRIDE[k];
+      }
+    }
+  });
+  bad &= valid;
+  if (bad) atomicOr(p.flags, FLAG_KEY_RANGE);
+#pragma unroll
+  for (int c = 0; c < NV; ++c)
+#pragma unroll
+    for (int r = 0; r < R; ++r) v[c][r] = 0;
+  sfor<0, SP::NV>([&](auto cc) {
+    constexpr int c = decltype(cc)::v;
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      v[c][r] = SP::VDT[c] == BLU_I32 ? (uint64_t)(int64_t)(int32_t)T.vlo[c][r]
+                                      : ((uint64_t)T.vhi[c][r] << 32 | T.vlo[c][r]);
+  });
+  return valid & ~bad;
+}
+
 // FUSE (small inputs, where launch latency dominates): S4 init and S8 compaction run inside this
 // kernel. Kept out of the large-input instantiation, whose register budget it would squeeze.
-template <class SP, int NV, int R, bool FUSE = false, bool PAIRMAP = false>
+template <class SP, int NV, int R, bool FUSE = false, bool PAIRMAP = false, bool PIPE = false>
 __device__ __forceinline__ void dense_body(const AggParams& p, const FinalParams& fp) {
   extern __shared__ __align__(16) uint8_t sm[];
   const Layout& L = p.lay;
@@ -613,7 +734,28 @@ __device__ __forceinline__ void dense_body(const AggParams& p, const FinalParams
   const uint64_t tile = (uint64_t)blockDim.x * R;
   const uint64_t ntiles = (n + tile - 1) / tile;
   uint32_t flag_seen = 0;
-  for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+  if constexpr (PIPE) {  // next tile's loads in flight during this tile's shared-memory updates
+    const unsigned warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    RawTile<SP, R> A, B;
+    uint64_t t = blockIdx.x;
+    if (t < ntiles) tile_load<SP, R>(p, lane_base<R>(t * tile, warp, lane), n, pol, A);
+    while (t < ntiles) {
+      const uint64_t tn = t + gridDim.x;
+      const uint32_t fl = *(volatile uint32_t*)p.flags;
+      if (tn < ntiles) tile_load<SP, R>(p, lane_base<R>(tn * tile, warp, lane), n, pol, B);
+      uint64_t key[R];
+      uint64_t v[NV][R];
+      const uint32_t valid = tile_unpack<SP, NV, R>(p, A, lane_base<R>(t * tile, warp, lane), n, key, v);
+      uint32_t e[R];
+#pragma unroll
+      for (int r = 0; r < R; ++r) e[r] = (uint32_t)key[r];
+      smem_apply_rows<SP, NV, R>(p, sm, e, valid, v);
+      if (__any_sync(0xffffffffu, fl)) break;
+      A = B;
+      t = tn;
+    }
+  }
+  for (uint64_t t = blockIdx.x; !PIPE && t < ntiles; t += gridDim.x) {
     if (flag_seen) break;
     flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);  // warp-uniform, seen next tile
     const uint64_t row = lane_base<R, PAIRMAP>(t * tile, threadIdx.x >> 5, threadIdx.x & 31);
@@ -836,6 +978,138 @@ __device__ __forceinline__ void front_dedupe_rows(const AggParams& p, uint8_t* s
   __syncwarp();
 }
 
+// One tile's rows after loading: hot-key front (rank image or hash table), then the global table
+// (path b: convergent probing; b': direct) for the rows the front did not take.
+template <class SP, int NV, int R, bool FRONT, bool DIRECT>
+__device__ __forceinline__ void process_rows(const AggParams& p, uint8_t* sm, uint64_t (&key)[R], uint32_t valid,
+                                             uint64_t (&v)[NV][R]) {
+  const Layout& L = p.lay;
+  const uint32_t S = p.S;
+  uint8_t* tb = (uint8_t*)p.table;
+  uint32_t miss = valid;
+  bool deduped = false;
+  if constexpr (FRONT && SP::kStatic) {
+    if constexpr (SP::DEDUPE) {  // opt-in (BLU_GBY_DEDUPE=1): pays off only for extreme skew
+      if (!p.front_rank_words) {
+        front_dedupe_rows<SP, NV, R, DIRECT>(p, sm, key, valid, v);
+        miss = 0;
+        deduped = true;
+      }
+    }
+  }
+  if (FRONT && DIRECT && p.front_rank_words && !deduped) {
+    // rank front: a dense key k is hot iff bit k%32 of word k/32 is set; its entry is the word's
+    // prefix plus the hot keys below it in the word. Converged, one LDS.64 per row, no probe loop.
+    const uint64_t* img = (const uint64_t*)(sm + p.key_off);
+    uint32_t fe[R];
+    uint32_t hit = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const uint64_t x = (valid >> r & 1) ? img[key[r] >> 5] : 0ull;
+      const uint32_t b = (uint32_t)key[r] & 31u, bits = (uint32_t)x;
+      fe[r] = (uint32_t)(x >> 32) + __popc(bits & ((1u << b) - 1u));
+      hit |= (bits >> b & 1u) << r;
+    }
+    smem_apply_rows<SP, NV, R>(p, sm, fe, hit, v);
+    miss = valid & ~hit;
+  } else if (FRONT && !deduped) {
+    // hot-key front: small open-addressing table per CTA in shared memory
+    uint64_t* fk = (uint64_t*)(sm + p.key_off);
+    const bool seeded = p.front_seed != nullptr;
+    uint32_t fe[R];
+    uint32_t hit = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      fe[r] = 0;
+      if (!(valid >> r & 1)) continue;
+      uint32_t s = front_home(key[r], S);
+      if (seeded) {  // read-only front (load <= 1/2): stop at the key or the first empty slot
+#pragma unroll 1
+        for (int q = 0; q < 8; ++q) {
+          const uint64_t cur = fk[s];
+          if (cur == key[r]) { hit |= 1u << r; break; }
+          if (cur == kEmpty) break;
+          s = (s + 1) & (S - 1);
+        }
+      } else {
+#pragma unroll 1
+        for (int q = 0; q < 8; ++q) {
+          uint64_t cur = *(volatile uint64_t*)(fk + s);
+          if (cur == key[r]) { hit |= 1u << r; break; }
+          if (cur == kEmpty) {
+            unsigned long long old = atomicCAS((unsigned long long*)(fk + s), (unsigned long long)kEmpty,
+                                               (unsigned long long)key[r]);
+            if (old == kEmpty || old == key[r]) { hit |= 1u << r; break; }
+          }
+          s = (s + 1) & (S - 1);
+        }
+      }
+      fe[r] = s;
+    }
+    __syncwarp();  // reconverge after the data-dependent probe loops (independent thread scheduling)
+    smem_apply_rows<SP, NV, R>(p, sm, fe, hit, v);
+    miss = valid & ~hit;
+  }
+  uint64_t slot[R];
+  if (DIRECT) {
+#pragma unroll
+    for (int r = 0; r < R; ++r) slot[r] = key[r];
+  } else {
+    // Convergent multi-row probe: every pending row of the lane advances one slot per iteration
+    // and all their key loads are issued together (memory-level parallelism); the warp stays
+    // converged (__any_sync), so the REDs that follow are warp-wide.
+    uint64_t cur[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      slot[r] = fmix64(key[r]) & p.cap_mask;
+      cur[r] = (miss >> r & 1) ? __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes)) : 0ull;
+    }
+    uint32_t pending = miss;
+    for (uint32_t it = 0;; ++it) {
+#pragma unroll
+      for (int r = 0; r < R; ++r) {
+        if (!(pending >> r & 1)) continue;
+        if (cur[r] == key[r]) {
+          pending &= ~(1u << r);
+        } else {
+          if (cur[r] == kEmpty) {
+            unsigned long long old = atomicCAS((unsigned long long*)(tb + slot[r] * L.slot_bytes),
+                                               (unsigned long long)kEmpty, (unsigned long long)key[r]);
+            if (old == kEmpty || old == key[r]) {
+              pending &= ~(1u << r);
+              continue;
+            }
+          }
+          slot[r] = (slot[r] + 1) & p.cap_mask;
+        }
+      }
+      if (!__any_sync(0xffffffffu, pending)) break;
+      if (it + 1 >= 4) {
+        // long tails (a few rows per warp): finish them one lane at a time, then reconverge
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (!(pending >> r & 1)) continue;
+          uint64_t sl;
+          const uint64_t c = __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes));
+          if (hash_locate(tb, p.cap_mask, L.slot_bytes, key[r], c, slot[r], p.max_probe, sl)) {
+            slot[r] = sl;
+          } else {  // the estimate was too small: flag, regrow, rerun
+            miss &= ~(1u << r);
+            atomicOr(p.flags, FLAG_OVERFLOW);
+          }
+        }
+        break;
+      }
+#pragma unroll
+      for (int r = 0; r < R; ++r)
+        if (pending >> r & 1) cur[r] = __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes));
+    }
+    __syncwarp();  // reconverge before the field reductions so each RED instruction is warp-wide
+  }
+  if (!DIRECT && L.lock_off) global_apply_rows_locked<SP, NV, R>(p, slot, miss, v);  // kernel 3
+  else global_apply_rows<SP, NV, R, DIRECT>(p, slot, miss, v);
+}
+
 // MODE 0: rows from columns; 1: records (merge of exchanged partials); 2: segments (pass 2 of the
 // partitioned mode: tiles enumerate the buckets in order, so at any moment all CTAs work inside
 // one bucket whose slice of the table is L2-resident).
@@ -843,7 +1117,7 @@ template <class SP, int NV, int R, bool FRONT, bool DIRECT, int MODE>
 __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs) {
   extern __shared__ __align__(16) uint8_t sm[];
   constexpr bool RECORDS = MODE == 1;
-  constexpr bool SEG = MODE == 2;
+  constexpr bool SEG = MODE == 2;  // MODE 3: rows from columns, software-pipelined (JIT only)
   if (p.gate && ((*(volatile const uint32_t*)p.gate != 0) != (p.gate_run_if != 0))) return;
   const Layout& L = p.lay;
   const uint32_t S = p.S;
@@ -895,7 +1169,25 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
     chunk_next = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;  // prefetched
     t = chunk * kGrab;
   }
-  while (t < ntiles) {
+  if constexpr (MODE == 3) {  // software-pipelined row stream (see RawTile)
+    const uint64_t n = p.n_rows;
+    const unsigned warp = threadIdx.x >> 5;
+    RawTile<SP, R> A, B;
+    if (t < ntiles) tile_load<SP, R>(p, lane_base<R>(t * tile, warp, lane), n, pol, A);
+    while (t < ntiles) {
+      const uint64_t tn = t + gridDim.x;
+      const uint32_t fl = *(volatile uint32_t*)p.flags;  // consumed after the tile: off the critical path
+      if (tn < ntiles) tile_load<SP, R>(p, lane_base<R>(tn * tile, warp, lane), n, pol, B);
+      uint64_t key[R];
+      uint64_t v[NV][R];
+      const uint32_t valid = tile_unpack<SP, NV, R>(p, A, lane_base<R>(t * tile, warp, lane), n, key, v);
+      process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v);
+      if (__any_sync(0xffffffffu, fl)) break;  // warp-uniform abort
+      A = B;
+      t = tn;
+    }
+  }
+  while (MODE != 3 && t < ntiles) {
     if (flag_seen) break;
     flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);  // warp-uniform abort
     uint64_t n = p.n_rows, row0 = t * tile, t_next = t + gridDim.x;
@@ -945,131 +1237,12 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
           }
       }
     } else {
+      if (!SEG && p.prefetch)  // the warp's next tile: in flight in L2 while this one is worked on
+        prefetch_warp_rows_l2<SP>(p, t_next * tile + (uint64_t)(threadIdx.x >> 5) * 32 * R, 32ull * R, n, lane);
       valid = pack_keys<SP, R>(p, row, n, pol, key);
       load_vals<SP, NV, R>(p, row, n, pol, v);
     }
-    uint32_t miss = valid;
-    bool deduped = false;
-    if constexpr (FRONT && SP::kStatic) {
-      if constexpr (SP::DEDUPE) {  // opt-in (BLU_GBY_DEDUPE=1): pays off only for extreme skew
-        if (!p.front_rank_words) {
-          front_dedupe_rows<SP, NV, R, DIRECT>(p, sm, key, valid, v);
-          miss = 0;
-          deduped = true;
-        }
-      }
-    }
-    if (FRONT && DIRECT && p.front_rank_words && !deduped) {
-      // rank front: a dense key k is hot iff bit k%32 of word k/32 is set; its entry is the word's
-      // prefix plus the hot keys below it in the word. Converged, one LDS.64 per row, no probe loop.
-      const uint64_t* img = (const uint64_t*)(sm + p.key_off);
-      uint32_t fe[R];
-      uint32_t hit = 0;
-#pragma unroll
-      for (int r = 0; r < R; ++r) {
-        const uint64_t x = (valid >> r & 1) ? img[key[r] >> 5] : 0ull;
-        const uint32_t b = (uint32_t)key[r] & 31u, bits = (uint32_t)x;
-        fe[r] = (uint32_t)(x >> 32) + __popc(bits & ((1u << b) - 1u));
-        hit |= (bits >> b & 1u) << r;
-      }
-      smem_apply_rows<SP, NV, R>(p, sm, fe, hit, v);
-      miss = valid & ~hit;
-    } else if (FRONT && !deduped) {
-      // hot-key front: small open-addressing table per CTA in shared memory
-      uint64_t* fk = (uint64_t*)(sm + p.key_off);
-      const bool seeded = p.front_seed != nullptr;
-      uint32_t fe[R];
-      uint32_t hit = 0;
-#pragma unroll
-      for (int r = 0; r < R; ++r) {
-        fe[r] = 0;
-        if (!(valid >> r & 1)) continue;
-        uint32_t s = front_home(key[r], S);
-        if (seeded) {  // read-only front (load <= 1/2): stop at the key or the first empty slot
-#pragma unroll 1
-          for (int q = 0; q < 8; ++q) {
-            const uint64_t cur = fk[s];
-            if (cur == key[r]) { hit |= 1u << r; break; }
-            if (cur == kEmpty) break;
-            s = (s + 1) & (S - 1);
-          }
-        } else {
-#pragma unroll 1
-          for (int q = 0; q < 8; ++q) {
-            uint64_t cur = *(volatile uint64_t*)(fk + s);
-            if (cur == key[r]) { hit |= 1u << r; break; }
-            if (cur == kEmpty) {
-              unsigned long long old = atomicCAS((unsigned long long*)(fk + s), (unsigned long long)kEmpty,
-                                                 (unsigned long long)key[r]);
-              if (old == kEmpty || old == key[r]) { hit |= 1u << r; break; }
-            }
-            s = (s + 1) & (S - 1);
-          }
-        }
-        fe[r] = s;
-      }
-      __syncwarp();  // reconverge after the data-dependent probe loops (independent thread scheduling)
-      smem_apply_rows<SP, NV, R>(p, sm, fe, hit, v);
-      miss = valid & ~hit;
-    }
-    uint64_t slot[R];
-    if (DIRECT) {
-#pragma unroll
-      for (int r = 0; r < R; ++r) slot[r] = key[r];
-    } else {
-      // Convergent multi-row probe: every pending row of the lane advances one slot per iteration
-      // and all their key loads are issued together (memory-level parallelism); the warp stays
-      // converged (__any_sync), so the REDs that follow are warp-wide.
-      uint64_t cur[R];
-#pragma unroll
-      for (int r = 0; r < R; ++r) {
-        slot[r] = fmix64(key[r]) & p.cap_mask;
-        cur[r] = (miss >> r & 1) ? __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes)) : 0ull;
-      }
-      uint32_t pending = miss;
-      for (uint32_t it = 0;; ++it) {
-#pragma unroll
-        for (int r = 0; r < R; ++r) {
-          if (!(pending >> r & 1)) continue;
-          if (cur[r] == key[r]) {
-            pending &= ~(1u << r);
-          } else {
-            if (cur[r] == kEmpty) {
-              unsigned long long old = atomicCAS((unsigned long long*)(tb + slot[r] * L.slot_bytes),
-                                                 (unsigned long long)kEmpty, (unsigned long long)key[r]);
-              if (old == kEmpty || old == key[r]) {
-                pending &= ~(1u << r);
-                continue;
-              }
-            }
-            slot[r] = (slot[r] + 1) & p.cap_mask;
-          }
-        }
-        if (!__any_sync(0xffffffffu, pending)) break;
-        if (it + 1 >= 4) {
-          // long tails (a few rows per warp): finish them one lane at a time, then reconverge
-#pragma unroll
-          for (int r = 0; r < R; ++r) {
-            if (!(pending >> r & 1)) continue;
-            uint64_t sl;
-            const uint64_t c = __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes));
-            if (hash_locate(tb, p.cap_mask, L.slot_bytes, key[r], c, slot[r], p.max_probe, sl)) {
-              slot[r] = sl;
-            } else {  // the estimate was too small: flag, regrow, rerun
-              miss &= ~(1u << r);
-              atomicOr(p.flags, FLAG_OVERFLOW);
-            }
-          }
-          break;
-        }
-#pragma unroll
-        for (int r = 0; r < R; ++r)
-          if (pending >> r & 1) cur[r] = __ldcg((const unsigned long long*)(tb + slot[r] * L.slot_bytes));
-      }
-      __syncwarp();  // reconverge before the field reductions so each RED instruction is warp-wide
-    }
-    if (!DIRECT && L.lock_off) global_apply_rows_locked<SP, NV, R>(p, slot, miss, v);  // kernel 3
-    else global_apply_rows<SP, NV, R, DIRECT>(p, slot, miss, v);
+    process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v);
     t = t_next;
   }
   if (FRONT) {

@@ -1030,14 +1030,29 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
       snprintf(name, sizeof name, "blu_jit_dense_%d_%d%s", nv, r, fuse ? "_fused" : "");
       snprintf(decl, sizeof decl, "%s(blu::AggParams p, blu::FinalParams fp)", name);
       const int pairmap = r == 4 && jit_env("BLU_GBY_DENSE_PAIR", 0);
-      snprintf(body, sizeof body, "blu::dense_body<blu::JitSpec, %d, %d, %s, %s>(p, fp);", nv, r, fuse ? "true" : "false",
-               pairmap ? "true" : "false");
+      // software-pipelined stream (BLU_GBY_DENSE_PIPE=0/1, rows per thread BLU_GBY_DENSE_PIPE_R)
+      // default on for the large-input kernel (C2: 0.704 -> 0.603 ms); the fused small-input kernel
+      // is launch-bound and measured slightly slower with it (C1: 18 -> 20 us)
+      const int pipe = !pairmap && jit_env("BLU_GBY_DENSE_PIPE", fuse ? 0 : 1);
+      if (pipe) {
+        r = jit_env("BLU_GBY_DENSE_PIPE_R", 2) >= 4 ? 4 : 2;
+        snprintf(name, sizeof name, "blu_jit_dense_%d_%d%s_p", nv, r, fuse ? "_fused" : "");
+        snprintf(decl, sizeof decl, "%s(blu::AggParams p, blu::FinalParams fp)", name);
+      }
+      snprintf(body, sizeof body, "blu::dense_body<blu::JitSpec, %d, %d, %s, %s, %s>(p, fp);", nv, r, fuse ? "true" : "false",
+               pairmap ? "true" : "false", pipe ? "true" : "false");
       FinalParams fpc = fin ? *fin : FinalParams{};
       void* args[] = {&pc, &fpc};
       // 2 CTAs x 512 threads per SM: <= 64 registers (one resident wave, see plan.cpp)
       if (launch_jit(body, decl, p, args, st, grid, block, smem, name, 2)) return 0;
     } else {
-      const int front = p.front_slots > 0, direct = path == BLU_PATH_DIRECT_GLOBAL, mode = p.seg_stride ? 2 : 0;
+      const int front = p.front_slots > 0, direct = path == BLU_PATH_DIRECT_GLOBAL;
+      // MODE 3: one-pass row stream with the next tile's loads issued before the current tile's
+      // work (BLU_GBY_PIPE=0/1, rows per thread BLU_GBY_PIPE_R, even)
+      // (default on: C4 14.2 -> 10.1 ms)
+      const int pipe = !p.seg_stride && jit_env("BLU_GBY_PIPE", 1);
+      const int mode = p.seg_stride ? 2 : pipe ? 3 : 0;
+      if (pipe) r = jit_env("BLU_GBY_PIPE_R", 2) >= 4 ? 4 : 2;
       snprintf(name, sizeof name, "blu_jit_global_%d_%d_%d_%d_%d", nv, r, front, direct, mode);
       snprintf(decl, sizeof decl, "%s(blu::AggParams p, blu::RecSrc rs)", name);
       snprintf(body, sizeof body, "blu::global_body<blu::JitSpec, %d, %d, %s, %s, %d>(p, rs);", nv, r,

@@ -55,11 +55,15 @@ def oracles():
     return get
 
 
-@pytest.mark.parametrize("jit", ["1", "0"])
+@pytest.mark.parametrize("jit", ["1", "0", "1-nopipe"])
 @pytest.mark.parametrize("name", ["C1", "C2", "C3", "C4", "C5"])
 def test_config_parity(bg, oracles, monkeypatch, name, jit):
-    """Both the NVRTC-specialised kernels (default) and the precompiled generic ones."""
-    monkeypatch.setenv("BLU_GBY_JIT", jit)
+    """The NVRTC-specialised kernels (default: software-pipelined row streams), the same without
+    the pipelining, and the precompiled generic ones."""
+    monkeypatch.setenv("BLU_GBY_JIT", jit[0])
+    if jit.endswith("nopipe"):
+        monkeypatch.setenv("BLU_GBY_PIPE", "0")
+        monkeypatch.setenv("BLU_GBY_DENSE_PIPE", "0")
     w, o = oracles(name)
     plan, res = run_gpu(bg, w)
     assert res.n_groups == o.n_groups
