@@ -629,6 +629,14 @@ struct RawTile {
   uint32_t klo[NKC][R], khi[NKC][R], vlo[NVC][R], vhi[NVC][R];
 };
 
+struct NoRawTile {};
+template <class SP, int R, bool PIPE>
+struct RawTileSel { using type = NoRawTile; };
+template <class SP, int R>
+struct RawTileSel<SP, R, true> { using type = RawTile<SP, R>; };
+template <class SP, int R, bool PIPE>
+using RawTileFor = typename RawTileSel<SP, R, PIPE>::type;
+
 // Issue the loads of this lane's R rows of one column (PAIR mapping, R even); rows >= n read 0.
 template <int R, bool W64>
 __device__ __forceinline__ void load_raw(const void* base, uint64_t lb, uint64_t n, uint32_t vec, uint64_t pol,
@@ -1117,11 +1125,13 @@ template <class SP, int NV, int R, bool FRONT, bool DIRECT, int MODE>
 __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs) {
   extern __shared__ __align__(16) uint8_t sm[];
   constexpr bool RECORDS = MODE == 1;
-  constexpr bool SEG = MODE == 2;  // MODE 3: rows from columns, software-pipelined (JIT only)
+  // MODE 3: rows from columns, MODE 4: segments, both software-pipelined (JIT only, see RawTile)
+  constexpr bool SEG = MODE == 2 || MODE == 4;
   if (p.gate && ((*(volatile const uint32_t*)p.gate != 0) != (p.gate_run_if != 0))) return;
   const Layout& L = p.lay;
   const uint32_t S = p.S;
   __shared__ uint64_t tpre[SEG ? 1025 : 1];
+  __shared__ uint64_t tend[MODE == 4 ? 1024 : 1];  // MODE 4: end row of each segment
   if constexpr (SEG) {  // warp-tile prefix over the buckets (warp 0)
     if (threadIdx.x < 32) {
       const uint64_t tile = 32ull * R;
@@ -1134,6 +1144,7 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
           if ((int)threadIdx.x >= o) inc += y;
         }
         if (b < p.n_segs) tpre[b] = carry + inc - x;
+        if (MODE == 4 && b < p.n_segs) tend[b] = (uint64_t)b * p.seg_stride + p.seg_count[b];
         carry += __shfl_sync(0xffffffffu, inc, 31);
       }
       if (threadIdx.x == 0) tpre[p.n_segs] = carry;
@@ -1187,7 +1198,51 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
       t = tn;
     }
   }
-  while (MODE != 3 && t < ntiles) {
+  if constexpr (MODE == 4) {  // segments, software-pipelined: tile coordinates from shared memory
+    auto coords = [&](uint64_t tt, uint64_t& lb, uint64_t& nn) {
+      uint32_t lo = 0, hi = p.n_segs - 1;
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi + 1) >> 1;
+        if (tpre[mid] <= tt) lo = mid; else hi = mid - 1;
+      }
+      lb = lane_base<R>((uint64_t)lo * p.seg_stride + (tt - tpre[lo]) * tile, 0, lane);
+      nn = tend[lo];
+    };
+    RawTile<SP, R> A, B;
+    uint64_t lbA = 0, nA = 0, lbB = 0, nB = 0;
+    if (t < ntiles) {
+      coords(t, lbA, nA);
+      tile_load<SP, R>(p, lbA, nA, pol, A);
+    }
+    while (t < ntiles) {
+      uint64_t t_next;
+      if (!dyn) {
+        t_next = t + (uint64_t)gridDim.x * (blockDim.x >> 5);
+      } else if (++k_in < kGrab) {
+        t_next = t + 1;
+      } else {
+        k_in = 0;
+        chunk = __shfl_sync(0xffffffffu, chunk_next, 0);
+        t_next = chunk * kGrab;
+        chunk_next = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;
+      }
+      const uint32_t fl = *(volatile uint32_t*)p.flags;
+      if (t_next < ntiles) {
+        coords(t_next, lbB, nB);
+        tile_load<SP, R>(p, lbB, nB, pol, B);
+      }
+      uint64_t key[R];
+      uint64_t v[NV][R];
+      const uint32_t valid = tile_unpack<SP, NV, R>(p, A, lbA, nA, key, v);
+      process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v);
+      if (__any_sync(0xffffffffu, fl)) break;
+      A = B;
+      lbA = lbB;
+      nA = nB;
+      t = t_next;
+    }
+  }
+  while (MODE != 3 && MODE != 4 && t < ntiles) {
     if (flag_seen) break;
     flag_seen = __any_sync(0xffffffffu, *(volatile uint32_t*)p.flags);  // warp-uniform abort
     uint64_t n = p.n_rows, row0 = t * tile, t_next = t + gridDim.x;
@@ -1510,7 +1565,9 @@ __device__ __forceinline__ void block_excl_scan(uint32_t* a, uint32_t* out, uint
   }
 }
 
-template <class SP, int NV, int R>
+// PIPE (NVRTC kernels only): the next tile's rows are loaded into registers as soon as the current
+// tile is staged in shared memory, so those HBM reads are in flight during its write-out phase.
+template <class SP, int NV, int R, bool PIPE = false>
 __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterParams& sp) {
   extern __shared__ __align__(16) uint8_t sm[];
   const Layout& L = p.lay;
@@ -1527,15 +1584,24 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
   const uint64_t pol = evict_first_policy();
   const uint64_t n = p.n_rows;
   const uint64_t ntiles = (n + TILE - 1) / TILE;
+  using Raw = RawTileFor<SP, R, PIPE>;
+  Raw T;
+  if constexpr (PIPE)
+    if (blockIdx.x < ntiles) tile_load<SP, R>(p, lane_base<R>(blockIdx.x * TILE, threadIdx.x >> 5, threadIdx.x & 31), n, pol, T);
   for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
     for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
     __syncthreads();
     const uint64_t row = lane_base<R>(t * TILE, threadIdx.x >> 5, threadIdx.x & 31);
     uint64_t key[R];
-    const uint32_t valid = pack_keys<SP, R>(p, row, n, pol, key);
     uint64_t v[NV][R];
-    load_vals<SP, NV, R>(p, row, n, pol, v);
-    if (p.prefetch) {  // a later tile of this CTA: in flight during the sort and the writes below
+    uint32_t valid;
+    if constexpr (PIPE) {
+      valid = tile_unpack<SP, NV, R>(p, T, row, n, key, v);
+    } else {
+      valid = pack_keys<SP, R>(p, row, n, pol, key);
+      load_vals<SP, NV, R>(p, row, n, pol, v);
+    }
+    if (!PIPE && p.prefetch) {  // a later tile of this CTA: in flight during the sort and the writes below
       const uint64_t nt = t + (uint64_t)gridDim.x * p.prefetch;
       prefetch_rows_l2<SP>(p, nt * TILE, nt * TILE + TILE < n ? nt * TILE + TILE : n);
     }
@@ -1565,6 +1631,10 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
 #pragma unroll
         for (int c = 0; c < NV; ++c) sval[(size_t)c * TILE + e] = v[c][r];
       }
+    if constexpr (PIPE) {  // this tile is in shared memory: the next one's loads go out now
+      const uint64_t tn = t + gridDim.x;
+      if (tn < ntiles) tile_load<SP, R>(p, lane_base<R>(tn * TILE, threadIdx.x >> 5, threadIdx.x & 31), n, pol, T);
+    }
     __syncthreads();
     const uint32_t tot = *total;
     for (uint32_t e = threadIdx.x; e < tot; e += blockDim.x) {

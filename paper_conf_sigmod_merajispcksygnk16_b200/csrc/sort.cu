@@ -165,21 +165,25 @@ __global__ void __launch_bounds__(kRT, 4) k_rs_downsweep(const KT* __restrict__ 
   }
   uint64_t t0, t1;
   tile_span((n + C::TILE - 1) / C::TILE, t0, t1);
+  // warp-striped tile: warp w owns keys [w * WARP_CHUNK, +WARP_CHUNK); item i of lane l is key
+  // i * 32 + l of that chunk, so (warp, i, lane) order is input order (stability)
+  KT k[C::ITEMS];
+  uint32_t v[C::ITEMS], rank[C::ITEMS];
+  auto load_tile = [&](uint64_t tt) {
+    const uint64_t bb = tt * C::TILE + (uint64_t)warp * C::WARP_CHUNK + lane;
+#pragma unroll
+    for (int i = 0; i < C::ITEMS; ++i) {
+      const uint64_t e = bb + (uint64_t)i * 32;
+      k[i] = e < n ? kin[e] : (KT)0;
+      v[i] = e < n ? vin[e] : 0u;
+    }
+  };
+  if (t0 < t1) load_tile(t0);
   for (uint64_t t = t0; t < t1; ++t) {
 #pragma unroll
     for (int w = 0; w < kRT / 32; ++w) wcnt[w][threadIdx.x] = 0;
     __syncthreads();
-    // warp-striped tile: warp w owns keys [w * WARP_CHUNK, +WARP_CHUNK); item i of lane l is key
-    // i * 32 + l of that chunk, so (warp, i, lane) order is input order (stability)
     const uint64_t b = t * C::TILE + (uint64_t)warp * C::WARP_CHUNK + lane;
-    KT k[C::ITEMS];
-    uint32_t v[C::ITEMS], rank[C::ITEMS];
-#pragma unroll
-    for (int i = 0; i < C::ITEMS; ++i) {
-      const uint64_t e = b + (uint64_t)i * 32;
-      k[i] = e < n ? kin[e] : (KT)0;
-      v[i] = e < n ? vin[e] : 0u;
-    }
 #pragma unroll
     for (int i = 0; i < C::ITEMS; ++i) {
       const bool valid = b + (uint64_t)i * 32 < n;
@@ -230,6 +234,8 @@ __global__ void __launch_bounds__(kRT, 4) k_rs_downsweep(const KT* __restrict__ 
       sk[lp] = k[i];
       sv[lp] = v[i];
     }
+    // the tile is staged: the next one's loads go out now and are in flight during the write-out
+    if (t + 1 < t1) load_tile(t + 1);
     __syncthreads();
     // ... then write it out: consecutive threads write consecutive addresses of each digit's run
     const uint64_t tile0 = t * C::TILE;
