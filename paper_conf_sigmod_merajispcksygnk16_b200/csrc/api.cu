@@ -333,24 +333,32 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       for (void* p : own->dev) cudaFreeAsync(p, st);
       delete own;
     };
-    cudaError_t ae = cudaSuccess;
-    auto t_oa = std::chrono::steady_clock::now();
-    for (int k = 0; k < lay.n_keys && ae == cudaSuccess; ++k) {
-      ae = U ? cudaMallocAsync(&okeys[k], U * dtype_bytes(lay.key_dtype[k]), st) : cudaSuccess;
-      if (okeys[k]) own->dev.push_back(okeys[k]);
-    }
-    for (int o = 0; o < os.n_out && ae == cudaSuccess; ++o) {
-      ae = U ? cudaMallocAsync(&ovals[o], U * dtype_bytes(os.out_dtype[o]), st) : cudaSuccess;
-      if (ovals[o]) own->dev.push_back(ovals[o]);
-    }
-    if (getenv("BLU_GBY_DEBUG_HOST"))
-      fprintf(stderr, "[blugby host] output alloc %.3f ms (%llu rows)\n",
-              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_oa).count(),
-              (unsigned long long)U);
-    if (ae != cudaSuccess) {
-      cudaGetLastError();
-      free_owner();
-      return cuda_fail(ae, "output alloc");
+    // Output allocation (stream-ordered). The fused kernel needs the pointers at launch; otherwise
+    // they are allocated after the aggregation launch, so this host work overlaps the kernel.
+    auto alloc_outputs = [&]() -> cudaError_t {
+      cudaError_t ae = cudaSuccess;
+      auto t_oa = std::chrono::steady_clock::now();
+      for (int k = 0; k < lay.n_keys && ae == cudaSuccess; ++k) {
+        ae = U ? cudaMallocAsync(&okeys[k], U * dtype_bytes(lay.key_dtype[k]), st) : cudaSuccess;
+        if (okeys[k]) own->dev.push_back(okeys[k]);
+      }
+      for (int o = 0; o < os.n_out && ae == cudaSuccess; ++o) {
+        ae = U ? cudaMallocAsync(&ovals[o], U * dtype_bytes(os.out_dtype[o]), st) : cudaSuccess;
+        if (ovals[o]) own->dev.push_back(ovals[o]);
+      }
+      if (getenv("BLU_GBY_DEBUG_HOST"))
+        fprintf(stderr, "[blugby host] output alloc %.3f ms (%llu rows)\n",
+                std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_oa).count(),
+                (unsigned long long)U);
+      if (ae != cudaSuccess) cudaGetLastError();
+      return ae;
+    };
+    if (fuse) {
+      cudaError_t ae = alloc_outputs();
+      if (ae != cudaSuccess) {
+        free_owner();
+        return cuda_fail(ae, "output alloc");
+      }
     }
     FinalParams fp{};
     if (fuse) {
@@ -377,6 +385,13 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       }
     }
     if (t_timing) cudaEventRecord(t_ev.e[2], st);
+    if (!fuse) {
+      cudaError_t ae = alloc_outputs();
+      if (ae != cudaSuccess) {
+        free_owner();
+        return cuda_fail(ae, "output alloc");
+      }
+    }
 
     if (U && !fuse) {
       CompactParams cp{};

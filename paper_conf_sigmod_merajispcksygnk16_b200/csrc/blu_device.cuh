@@ -467,7 +467,8 @@ template <class SP, int NV, int R>
 __device__ __forceinline__ void smem_apply_rows(const AggParams& p, uint8_t* sm, const uint32_t (&e)[R],
                                                 uint32_t mask, const uint64_t (&v)[NV][R]) {
   const uint32_t S = p.S;
-  if constexpr (SP::kStatic) {  // JIT: one straight-line update per (field, row)
+#ifdef BLU_FIELD_MAJOR  // experiment switch (BLU_GBY_JIT_DEFS): the previous field-major order
+  if constexpr (SP::kStatic) {
     sfor<0, SP::NF>([&](auto jc) {
       constexpr int j = decltype(jc)::v;
       constexpr int K = SP::KIND[j], c = SP::COL[j];
@@ -479,6 +480,21 @@ __device__ __forceinline__ void smem_apply_rows(const AggParams& p, uint8_t* sm,
           else s_upd<K, true>(b, e[r], S, v[c][r]);
         }
     });
+    return;
+  }
+#endif
+  if constexpr (SP::kStatic) {  // JIT: straight-line updates; one branch per row, not per (field, row)
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (mask >> r & 1) {
+        sfor<0, SP::NF>([&](auto jc) {
+          constexpr int j = decltype(jc)::v;
+          constexpr int K = SP::KIND[j], c = SP::COL[j];
+          uint8_t* b = sm + p.soff[j];
+          if constexpr (c < 0) s_upd<FK_COUNT, true>(b, e[r], S, 1ull);
+          else s_upd<K, true>(b, e[r], S, v[c][r]);
+        });
+      }
     return;
   }
   for (uint32_t m = p.cntmask; m; m &= m - 1) {
@@ -509,7 +525,8 @@ __device__ __forceinline__ void global_apply_rows(const AggParams& p, const uint
                                                   const uint64_t (&v)[NV][R]) {
   const Layout& L = p.lay;
   uint8_t* tb = (uint8_t*)p.table;
-  if constexpr (SP::kStatic) {  // JIT: slot size, field offsets and dense groups are constants
+#ifdef BLU_FIELD_MAJOR
+  if constexpr (SP::kStatic) {
     sfor<0, SP::NF>([&](auto jc) {
       constexpr int j = decltype(jc)::v;
       constexpr int K = SP::KIND[j], c = SP::COL[j], KK = c < 0 ? FK_COUNT : K;
@@ -523,6 +540,23 @@ __device__ __forceinline__ void global_apply_rows(const AggParams& p, const uint
           else g_upd<KK, true>(tb + slot[r] * slot_b + goff, x);
         }
     });
+    return;
+  }
+#endif
+  if constexpr (SP::kStatic) {  // JIT: slot size, field offsets and dense groups are constants
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+      if (mask >> r & 1) {  // one branch per row; its REDs go out back to back
+        sfor<0, SP::NF>([&](auto jc) {
+          constexpr int j = decltype(jc)::v;
+          constexpr int K = SP::KIND[j], c = SP::COL[j], KK = c < 0 ? FK_COUNT : K;
+          constexpr int sg = SP::SGROUP[j], goff = SP::GOFF[j];
+          constexpr uint64_t base = (uint64_t)SP::SIDX[j] * SP::DOMAIN, slot_b = SP::SLOT;
+          const uint64_t x = c < 0 ? 1ull : v[c < 0 ? 0 : c][r];
+          if constexpr (DIRECT) d_upd<KK, true>((uint64_t*)p.dense[sg] + base + slot[r], x);
+          else g_upd<KK, true>(tb + slot[r] * slot_b + goff, x);
+        });
+      }
     return;
   }
   for (uint32_t m = p.cntmask; m; m &= m - 1) {
@@ -698,6 +732,14 @@ __device__ __forceinline__ uint32_t tile_unpack(const AggParams& p, const RawTil
       if constexpr (SP::SPARSE) {
         key[r] = c;
         if ((int64_t)c < 0) bad |= 1u << r;
+#ifndef BLU_PACK64
+      } else if constexpr (SP::DOMAIN <= 0xFFFFFFFFull && SP::KDT[k] == BLU_I32 && SP::DICT[k] <= 0x80000000ull) {
+        // dense domain below 2^32: 32-bit mixed radix (one IMAD per column instead of a 64-bit one);
+        // a negative i32 code is >= 2^31 unsigned, so the same compare rejects it
+        const uint32_t c32 = T.klo[k][r];
+        if (c32 >= (uint32_t)SP::DICT[k]) bad |= 1u << r;
+        key[r] = (uint64_t)((uint32_t)key[r] + c32 * (uint32_t)SP::STRIDE[k]);
+#endif
       } else {
         if (c >= SP::DICT[k]) bad |= 1u << r;  // unsigned: negatives are huge
         key[r] += c * SP::STRIDE[k];

@@ -211,6 +211,24 @@ void jit_probe_begin(JitProbe* pr) { t_probe = pr; }
 void jit_probe_end() { t_probe = nullptr; }
 bool jit_probe_active() { return t_probe != nullptr; }
 
+// Experiment switches (benchmarks): BLU_GBY_JIT_DEFS=A,B compiles the kernels with #define A 1 ...
+static std::string jit_defs() {
+  std::string out;
+  const char* d = getenv("BLU_GBY_JIT_DEFS");
+  if (!d) return out;
+  std::string cur;
+  for (const char* c = d;; ++c) {
+    if (*c == ',' || *c == 0) {
+      if (!cur.empty()) out += "#define " + cur + " 1\n";
+      cur.clear();
+      if (!*c) break;
+    } else {
+      cur += *c;
+    }
+  }
+  return out;
+}
+
 // Compile-only probe (blu_gby_jit_probe): NVRTC compile of the program, no module load, no launch.
 static void probe_compile(const std::string& body) {
   JitProbe& pr = *t_probe;
@@ -220,7 +238,7 @@ static void probe_compile(const std::string& body) {
     pr.log += "NVRTC not found\n";
     return;
   }
-  std::string src = std::string(kPreamble) + kSrc_blu_params_h + "\n" + kSrc_blu_device_cuh + "\n" + body;
+  std::string src = std::string(kPreamble) + jit_defs() + kSrc_blu_params_h + "\n" + kSrc_blu_device_cuh + "\n" + body;
   std::vector<char> cubin;
   std::string log;
   if (!compile(src, cubin, log) || cubin.empty()) {
@@ -232,18 +250,18 @@ static void probe_compile(const std::string& body) {
 const void* jit_kernel(const std::string& spec_src, const std::string& entry_src, const char* entry) {
   if (!jit_enabled()) return nullptr;
   if (t_probe) {
-    probe_compile(spec_src + entry_src);
+    probe_compile(jit_defs() + spec_src + entry_src);
     return nullptr;
   }
   int dev = 0;
   cudaGetDevice(&dev);
-  const std::string body = spec_src + entry_src;
+  const std::string body = jit_defs() + spec_src + entry_src;
   const std::string key = std::to_string(dev) + "\n" + body;
   std::lock_guard<std::mutex> lk(g_mu);
   Entry& e = g_cache[key];
   if (e.failed) return nullptr;
   if (!e.lib) {
-    std::string src = std::string(kPreamble) + kSrc_blu_params_h + "\n" + kSrc_blu_device_cuh + "\n" + body;
+    std::string src = std::string(kPreamble) + jit_defs() + kSrc_blu_params_h + "\n" + kSrc_blu_device_cuh + "\n" + body;
     int major = 0, minor = 0;
     if (nvrtc()->ok && nvrtc()->version) nvrtc()->version(&major, &minor);
     const uint64_t h = fnv1a(src + std::to_string(major) + "." + std::to_string(minor));

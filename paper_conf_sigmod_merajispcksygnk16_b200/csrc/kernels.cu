@@ -21,6 +21,8 @@
 
 #include <algorithm>
 #include <atomic>
+#include <mutex>
+#include <unordered_map>
 
 #include "blu_internal.h"
 #include "blu_device.cuh"
@@ -52,7 +54,6 @@ static int jit_env(const char* k, int def) {
 static bool launch_jit(const char* body, const char* entry_decl, const AggParams& p, void** args, cudaStream_t st,
                        uint32_t grid, uint32_t block, uint32_t smem, const char* entry, int min_blocks = 1) {
   if (!p.jit_ok || !jit_enabled()) return false;
-  const std::string spec = jit_spec("JitSpec", p.lay);
   // 1024-thread CTAs (one per SM, wide hot-key front) keep the same 64-register budget
   const int maxt = block > 512 ? 1024 : 512, minb = block > 512 ? 1 : jit_env("BLU_GBY_JIT_MINB", min_blocks);
   std::string src = "extern \"C\" __global__ void __launch_bounds__(" + std::to_string(maxt) + ", " +
@@ -61,12 +62,51 @@ static bool launch_jit(const char* body, const char* entry_decl, const AggParams
   src += " { ";
   src += body;
   src += " }\n";
-  const void* k = jit_kernel(spec, src, entry);
-  if (jit_probe_active()) return true;  // compile-only probe: nothing is launched
-  if (!k) return false;
-  if (smem > 48 * 1024 && cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
-    cudaGetLastError();
-    return false;
+  // Launch-path cache: (layout bytes, entry source, device, experiment defines) -> kernel handle, so
+  // repeated executes of a plan skip building the spec source and the source-keyed lookup (host
+  // time the GPU would otherwise sit idle for). The layout bytes are compared on a hit.
+  struct Fast {
+    Layout lay;
+    std::string src;
+    const void* k;
+    uint32_t smem_ok;
+  };
+  static std::mutex fmu;
+  static std::unordered_map<uint64_t, Fast> fast;
+  const bool probe = jit_probe_active();
+  int dev = 0;
+  if (!probe) cudaGetDevice(&dev);
+  const char* defs = getenv("BLU_GBY_JIT_DEFS");
+  std::string tag = src + "|" + std::to_string(dev) + "|" + (defs ? defs : "");
+  uint64_t h = 1469598103934665603ull;
+  for (size_t i = 0; i < sizeof(Layout); ++i) h = (h ^ ((const uint8_t*)&p.lay)[i]) * 1099511628211ull;
+  for (char c : tag) h = (h ^ (uint8_t)c) * 1099511628211ull;
+  const void* k = nullptr;
+  uint32_t smem_ok = 0;
+  if (!probe) {
+    std::lock_guard<std::mutex> lk(fmu);
+    auto it = fast.find(h);
+    if (it != fast.end() && it->second.src == tag && memcmp(&it->second.lay, &p.lay, sizeof(Layout)) == 0) {
+      k = it->second.k;
+      smem_ok = it->second.smem_ok;
+    }
+  }
+  if (!k) {
+    k = jit_kernel(jit_spec("JitSpec", p.lay), src, entry);
+    if (probe) return true;  // compile-only probe: nothing is launched
+    if (!k) return false;
+  }
+  if (smem > 48 * 1024 && smem > smem_ok) {
+    if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
+      cudaGetLastError();
+      return false;
+    }
+    smem_ok = smem;
+  }
+  {
+    std::lock_guard<std::mutex> lk(fmu);
+    Fast& f = fast[h];
+    if (f.k != k || f.smem_ok < smem_ok || f.src != tag) f = Fast{p.lay, tag, k, smem_ok};
   }
   if (cudaLaunchKernel(k, dim3(grid), dim3(block), args, smem, st) != cudaSuccess) {
     cudaGetLastError();

@@ -194,6 +194,28 @@ def test_key_range_errors(bg):
     assert r.n_groups == 1 and int(r.aggs[0][0]) == 1000
 
 
+@pytest.mark.parametrize("path,front", [("a", "0"), ("d", "1"), ("d", "0"), ("b", "0")])
+def test_key_range_errors_large(bg, monkeypatch, path, front):
+    """Out-of-range codes caught by the software-pipelined kernels (tile_unpack) at sizes that take
+    the unfused, multi-tile launch; the bad row is the last one (ragged tail) or deep inside."""
+    n = 5_000_011
+    sch = blugen.Schema([(I32, 30), (I32, 40)], [I64], [(COUNT, -1), (SUM, 0)])
+    monkeypatch.setenv("BLU_GBY_FORCE_PATH", path)
+    monkeypatch.setenv("BLU_GBY_HOT_FRONT", front)
+    plan = bg.plan_for(sch, 1200, n)
+    k0 = torch.arange(n, dtype=torch.int64, device="cuda").remainder(30).to(torch.int32)
+    k1 = torch.arange(n, dtype=torch.int64, device="cuda").remainder(37).to(torch.int32)
+    v = torch.ones(n, dtype=torch.int64, device="cuda")
+    for col, pos, bad in ((0, n - 1, 30), (1, 3_333_333, -1), (1, 0, 40)):
+        ks = [k0.clone(), k1.clone()]
+        ks[col][pos] = bad
+        with pytest.raises(bg.BluError) as e:
+            bg.blu_gby_execute(plan, ks, [v])
+        assert e.value.status == bg.BLU_E_KEY_RANGE
+    r = bg.blu_gby_execute(plan, [k0, k1], [v])
+    assert r.n_groups == 30 * 37 and int(r.aggs[0].sum()) == n and int(r.aggs[1].sum()) == n
+
+
 def test_general_f64_within_tolerance(bg):
     """Non-dyadic doubles: SUM/AVG within 1e-12 * sum|v| of the oracle (reading A13)."""
     n = 1_000_003
