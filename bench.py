@@ -264,7 +264,8 @@ def run_sort(args):
     if os.path.exists(sp):  # DRAM bytes / algorithmic bytes of the captured downsweep, per average launch
         traffic = json.load(open(sp)).get("traffic_over_algorithmic", 0) * per_launch_bytes or None
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": traffic, "kernel": "k_rs_downsweep (radix pass: read + scatter of key, payload)",
+                "traffic": traffic,
+                "kernel": "k_rs_downsweep + k_seg_window_sort (sort passes: read + write of key, payload)",
                 "algorithmic_bytes_per_launch": per_launch_bytes, "avg_launch_ms": per_launch_ms,
                 "launches_per_step": sum(ds_launch) / args.steps,
                 "share_of_step": sum(ds_ms) / tot_ms, "peak_source": peak_src,

@@ -417,6 +417,150 @@ __global__ void k_level_scatter(const uint32_t* __restrict__ pos, const uint32_t
     perm[pos[j]] = rows_sorted[j];
 }
 
+// ---- segmented window sort (levels >= 1 whose duplicate ranges are all short) -------------------
+// The level's active list holds its ranges contiguously with consecutive range ids (seg), so sorting
+// the batched (seg << 32 | key) array only has to order elements WITHIN each range. When no range is
+// longer than kSW / 2, two passes of in-shared-memory sorts over fixed windows do it: windows
+// [w*kSW, (w+1)*kSW), then windows shifted by kSW / 2. A range inside a first-pass window is sorted
+// by it; a range across a first-pass boundary lies inside one shifted window (length <= kSW / 2),
+// and a shifted window re-sorting already sorted parts leaves them in place. Each window is a stable
+// LSD radix sort in shared memory on (seg - first seg in window, key): 12 + 32 bits, 8-bit digits,
+// digits that are constant across the window skipped. Replaces the 6-7 global radix passes of such
+// a level (S1 level 2: ~915K ranges of ~109 rows) by two reads and writes of the level's keys.
+// Window size kSW elements, kST = kSW / 4 threads (4 elements each); 2048-element windows fit three
+// CTAs per SM, 4096-element windows one (BLU_SORT_SEG_W).
+template <int kSW>
+constexpr size_t seg_smem() { return (size_t)kSW * (8 + 8 + 4 + 4) + (kSW / 128) * 256 * 4 + 2 * 256 * 4 + 64; }
+
+template <int kSW>
+__global__ void __launch_bounds__(kSW / 4) k_seg_window_sort(uint64_t* __restrict__ keys, uint32_t* __restrict__ rows,
+                                                             uint64_t m, uint64_t off) {
+  constexpr int kST = kSW / 4, kNW = kST / 32;
+  extern __shared__ __align__(16) uint8_t smraw[];
+  uint64_t* ka = (uint64_t*)smraw;
+  uint64_t* kb = ka + kSW;
+  uint32_t* ra = (uint32_t*)(kb + kSW);
+  uint32_t* rb = ra + kSW;
+  uint32_t (*wcnt)[256] = (uint32_t(*)[256])(rb + kSW);
+  uint32_t* tot = (uint32_t*)(wcnt + kNW);
+  uint32_t* dstart = tot + 256;
+  uint32_t* misc = dstart + 256;  // [0] OR lo, [1] OR hi, [2] AND lo, [3] AND hi, [4..11] warp sums
+  const unsigned tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t lt_mask = (1u << lane) - 1u;
+  for (uint64_t b0 = off + (uint64_t)blockIdx.x * kSW; b0 < m; b0 += (uint64_t)gridDim.x * kSW) {
+    const uint32_t cnt = (uint32_t)(m - b0 < (uint64_t)kSW ? m - b0 : (uint64_t)kSW);
+    const uint32_t seg0 = (uint32_t)(keys[b0] >> 32);
+    if (tid == 0) {
+      misc[0] = misc[1] = 0u;
+      misc[2] = misc[3] = ~0u;
+    }
+    __syncthreads();
+    uint32_t o0 = 0, o1 = 0, a0 = ~0u, a1 = ~0u;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const uint32_t e = warp * 128 + i * 32 + lane;
+      if (e < cnt) {
+        const uint64_t k = keys[b0 + e];
+        const uint64_t lk = ((uint64_t)((uint32_t)(k >> 32) - seg0) << 32) | (k & 0xFFFFFFFFull);
+        ka[e] = lk;
+        ra[e] = rows[b0 + e];
+        o0 |= (uint32_t)lk, o1 |= (uint32_t)(lk >> 32), a0 &= (uint32_t)lk, a1 &= (uint32_t)(lk >> 32);
+      }
+    }
+    o0 = __reduce_or_sync(0xffffffffu, o0), o1 = __reduce_or_sync(0xffffffffu, o1);
+    a0 = __reduce_and_sync(0xffffffffu, a0), a1 = __reduce_and_sync(0xffffffffu, a1);
+    if (lane == 0) {
+      atomicOr(&misc[0], o0), atomicOr(&misc[1], o1);
+      atomicAnd(&misc[2], a0), atomicAnd(&misc[3], a1);
+    }
+    __syncthreads();
+    const uint64_t vary = ((uint64_t)(misc[1] ^ misc[3]) << 32) | (misc[0] ^ misc[2]);
+    uint64_t* ks = ka;
+    uint64_t* kd = kb;
+    uint32_t* rs = ra;
+    uint32_t* rd = rb;
+    for (uint32_t shift = 0; shift < 48; shift += 8) {
+      if (((vary >> shift) & 255ull) == 0) continue;  // constant digit: the pass is the identity
+#pragma unroll
+      for (int q = 0; q < 8; ++q) wcnt[warp][q * 32 + lane] = 0u;
+      __syncthreads();
+      uint32_t dg[4], rk[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const uint32_t e = warp * 128 + i * 32 + lane;
+        const bool valid = e < cnt;
+        const uint32_t d = valid ? (uint32_t)(ks[e] >> shift) & 255u : 256u + lane;
+        const uint32_t peers = __match_any_sync(0xffffffffu, d);
+        const int leader = __ffs(peers) - 1;
+        uint32_t c = 0;
+        if (valid && (int)lane == leader) {
+          c = wcnt[warp][d];
+          wcnt[warp][d] = c + (uint32_t)__popc(peers);
+        }
+        c = __shfl_sync(0xffffffffu, c, leader);
+        dg[i] = d;
+        rk[i] = c + (uint32_t)__popc(peers & lt_mask);
+        __syncwarp();
+      }
+      __syncthreads();
+      if (tid < 256) {  // per digit: exclusive prefix over the warps, and the digit total
+        uint32_t run = 0;
+        for (int w = 0; w < kNW; ++w) {
+          const uint32_t x = wcnt[w][tid];
+          wcnt[w][tid] = run;
+          run += x;
+        }
+        uint32_t inc = run;  // exclusive scan of the 256 digit totals (8 warps)
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+          if ((int)lane >= o) inc += y;
+        }
+        if (lane == 31) misc[4 + warp] = inc;
+        tot[tid] = inc - run;
+      }
+      __syncthreads();
+      if (tid < 256) {
+        uint32_t before = 0;
+        for (unsigned q = 0; q < warp; ++q) before += misc[4 + q];
+        dstart[tid] = before + tot[tid];
+      }
+      __syncthreads();
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const uint32_t e = warp * 128 + i * 32 + lane;
+        if (e < cnt) {
+          const uint32_t pos = dstart[dg[i]] + wcnt[warp][dg[i]] + rk[i];
+          kd[pos] = ks[e];
+          rd[pos] = rs[e];
+        }
+      }
+      __syncthreads();
+      uint64_t* tk = ks; ks = kd; kd = tk;
+      uint32_t* tr = rs; rs = rd; rd = tr;
+    }
+    for (uint32_t e = tid; e < cnt; e += kST) {
+      const uint64_t lk = ks[e];
+      keys[b0 + e] = ((uint64_t)((uint32_t)(lk >> 32) + seg0) << 32) | (lk & 0xFFFFFFFFull);
+      rows[b0 + e] = rs[e];
+    }
+    __syncthreads();
+  }
+}
+
+// Longest run of equal range ids in seg[0..m): run starts (per range id) then run lengths.
+__global__ void k_seg_starts(const uint32_t* __restrict__ seg, uint64_t m, uint32_t* __restrict__ starts) {
+  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < m; j += (uint64_t)gridDim.x * blockDim.x)
+    if (j == 0 || seg[j] != seg[j - 1]) starts[seg[j]] = (uint32_t)j;
+}
+__global__ void k_seg_maxlen(const uint32_t* __restrict__ seg, uint64_t m, const uint32_t* __restrict__ starts,
+                             uint32_t* __restrict__ mx) {
+  uint32_t best = 0;
+  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < m; j += (uint64_t)gridDim.x * blockDim.x)
+    if (j + 1 == m || seg[j] != seg[j + 1]) best = max(best, (uint32_t)(j + 1) - starts[seg[j]]);
+  best = __reduce_max_sync(0xffffffffu, best);
+  if ((threadIdx.x & 31) == 0 && best) atomicMax(mx, best);
+}
+
 int sms_now() {
   int dev = 0, s = 148;
   cudaGetDevice(&dev);
@@ -640,6 +784,9 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
   // workspace: level-0 keys/payload scratch (u32) + level keys (u64 x3) + payload x3 + pos/seg x2;
   // from the block cache (every level ends with a synchronisation, so it is idle on return)
   static const bool dbg = getenv("BLU_SORT_DEBUG") != nullptr;
+  const bool no_seg = getenv("BLU_SORT_NO_SEG") != nullptr;  // always the batched global radix sort
+  const char* sgw = getenv("BLU_SORT_SEG_W");
+  const int seg_w = sgw ? atoi(sgw) : 2048;
   auto hnow = [] {
     timespec ts;
     clock_gettime(CLOCK_MONOTONIC, &ts);
@@ -696,11 +843,55 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
     while (bits_seg < 32 && (1ull << bits_seg) < nr) ++bits_seg;
     k_level_keys<<<elem_grid(m), 256, 0, st>>>(rows, W, word, pos0, seg0, perm_out, m, k64a, pa);
     count_launch(1);
-    SCK(radix_sort<uint64_t>(k64a, pa, k64b, pb, k64c, pc, m, 32 + bits_seg, counts, grid, st, tm), "level sort");
-    k_level_scatter<<<elem_grid(m), 256, 0, st>>>(pos0, pb, m, perm_out);
+    // all ranges short (<= kSW / 2): two passes of shared-memory window sorts, in place
+    uint32_t maxlen = ~0u;
+    const int sw = seg_w == 2048 ? 2048 : 4096;
+    if (!no_seg) {
+      uint32_t* mx = counts + (size_t)256 * (grid + 1) + 8;
+      SCK(cudaMemsetAsync(mx, 0, 4, st), "seg maxlen");
+      k_seg_starts<<<elem_grid(m), 256, 0, st>>>(seg0, m, seg1);
+      k_seg_maxlen<<<elem_grid(m), 256, 0, st>>>(seg0, m, seg1, mx);
+      count_launch(2);
+      SCK(cudaMemcpyAsync(&maxlen, mx, 4, cudaMemcpyDeviceToHost, st), "seg maxlen D2H");
+      SCK(cudaStreamSynchronize(st), "seg maxlen sync");
+    }
+    const uint64_t* lk = k64b;
+    const uint32_t* lrows = pb;
+    if (maxlen <= (uint32_t)sw / 2) {
+      static bool attr = false;
+      if (!attr) {
+        SCK(cudaFuncSetAttribute(k_seg_window_sort<4096>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)seg_smem<4096>()), "seg sort smem");
+        SCK(cudaFuncSetAttribute(k_seg_window_sort<2048>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)seg_smem<2048>()), "seg sort smem");
+        attr = true;
+      }
+      const uint32_t per_sm = sw == 2048 ? 3 : 1;
+      const uint32_t wg =
+          (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>((m + sw - 1) / sw, (uint64_t)sms_now() * per_sm));
+      if (tm) cudaEventRecord(tm->next(), st);
+      if (sw == 2048) {
+        k_seg_window_sort<2048><<<wg, 512, seg_smem<2048>(), st>>>(k64a, pa, m, 0);
+        if (m > 1024) k_seg_window_sort<2048><<<wg, 512, seg_smem<2048>(), st>>>(k64a, pa, m, 1024);
+      } else {
+        k_seg_window_sort<4096><<<wg, 1024, seg_smem<4096>(), st>>>(k64a, pa, m, 0);
+        if (m > 2048) k_seg_window_sort<4096><<<wg, 1024, seg_smem<4096>(), st>>>(k64a, pa, m, 2048);
+      }
+      if (tm) {
+        cudaEventRecord(tm->next(), st);
+        tm->bytes += 2ull * 2 * m * (8 + 4);
+      }
+      count_launch(2);
+      SCK(cudaGetLastError(), "seg window sort");
+      lk = k64a;
+      lrows = pa;
+    } else {
+      SCK(radix_sort<uint64_t>(k64a, pa, k64b, pb, k64c, pc, m, 32 + bits_seg, counts, grid, st, tm), "level sort");
+    }
+    k_level_scatter<<<elem_grid(m), 256, 0, st>>>(pos0, lrows, m, perm_out);
     count_launch(1);
     uint64_t m2 = 0, nr2 = 0;
-    s = dup_pass<uint64_t>(k64b, m, pos0, pos1, seg1, nullptr, nullptr, 0, &m2, &nr2, st, dws);
+    s = dup_pass<uint64_t>(lk, m, pos0, pos1, seg1, nullptr, nullptr, 0, &m2, &nr2, st, dws);
     if (s != BLU_OK) return s;
     std::swap(pos0, pos1);
     std::swap(seg0, seg1);

@@ -60,9 +60,13 @@ def test_dup_ranges(bg, n, card):
     assert np.array_equal(st.cpu().numpy(), est) and np.array_equal(ln.cpu().numpy(), eln)
 
 
+@pytest.mark.parametrize("seg", ["1", "0"])
 @pytest.mark.parametrize("n,W", [(0, 8), (1, 8), (2, 4), (4097, 8), (300_007, 16), (1_000_003, 12), (2_000_000, 16)])
-def test_sort_rows(bg, n, W):
-    """The completed sort: identical permutation (stable lexicographic order)."""
+def test_sort_rows(bg, monkeypatch, n, W, seg):
+    """The completed sort: identical permutation (stable lexicographic order), with short
+    ranges sorted by the shared-memory window sort (default) or by the batched radix sort."""
+    if seg == "0":
+        monkeypatch.setenv("BLU_SORT_NO_SEG", "1")
     rows = blugen.sort_rows(n, W, seed=n + W)
     perm, stats = bg.blu_sort_rows(torch.from_numpy(rows).cuda())
     assert np.array_equal(u32(perm), oracle.sort_rows(rows))
@@ -88,3 +92,24 @@ def test_sort_rows_special_cases(bg):
     rev = np.stack([np.frombuffer(int(x).to_bytes(W, "big"), np.uint8) for x in range(n)])[::-1].copy()
     perm, stats = bg.blu_sort_rows(torch.from_numpy(rev).cuda())
     assert np.array_equal(u32(perm), np.arange(n, dtype=np.uint32)[::-1])
+
+
+@pytest.mark.parametrize("sw", ["2048", "4096"])
+@pytest.mark.parametrize("run", [1, 2, 7, 300, 1024, 1025, 2048, 2049, 5000])
+def test_sort_rows_window_boundaries(bg, monkeypatch, run, sw):
+    """Level-1 ranges of a fixed length (word 0 = row // run) whose level-1 keys are random with many
+    ties (word 1 from {0..3}): ranges of up to sw/2 rows straddle the sw-row windows at every offset
+    and take the window sort; longer ones take the batched radix sort. Word 2 = row id reversed keeps
+    a third level for the tied rows."""
+    monkeypatch.setenv("BLU_SORT_SEG_W", sw)
+    n = 60_001
+    rng = np.random.default_rng(run)
+    i = np.arange(n, dtype=np.uint64)
+    w0 = (i // run).astype(np.uint32)
+    w1 = rng.integers(0, 4, n).astype(np.uint32)
+    w2 = (n - i).astype(np.uint32)
+    rows = np.stack([w0, w1, w2], 1).astype(">u4").view(np.uint8).reshape(n, 12).copy()
+    perm, stats = bg.blu_sort_rows(torch.from_numpy(rows).cuda())
+    assert np.array_equal(u32(perm), oracle.sort_rows(rows))
+    if run > 1:
+        assert stats["levels"] >= 2
