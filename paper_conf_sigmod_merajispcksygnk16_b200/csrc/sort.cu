@@ -393,20 +393,40 @@ __global__ void k_range_lens(const uint64_t* __restrict__ r_start, uint64_t* __r
 
 // One batched level: key = (range id << 32) | partial key `word` of the row at buffer position
 // pos[j]; payload = that row id.
+// The row reads are random 4-byte gathers: each thread keeps 4 of them in flight (elements j,
+// j + stride, j + 2 stride, j + 3 stride) instead of one.
 __global__ void k_level_keys(const uint8_t* __restrict__ rows, uint32_t W, uint32_t word, const uint32_t* __restrict__ pos,
                              const uint32_t* __restrict__ seg, const uint32_t* __restrict__ perm, uint64_t m,
                              uint64_t* __restrict__ keys, uint32_t* __restrict__ payload) {
-  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < m; j += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t row = perm[pos[j]];
-    const uint32_t p = 4 * word;
-    uint32_t k = 0;
-    if ((W & 3) == 0 && p + 4 <= W && ((uintptr_t)rows & 3) == 0) {
-      k = __byte_perm(__ldg((const unsigned int*)(rows + (uint64_t)row * W + p)), 0, 0x0123);
-    } else {
-      for (uint32_t q = 0; q < 4; ++q) k = (k << 8) | (p + q < W ? rows[(uint64_t)row * W + p + q] : 0u);
+  const uint32_t p = 4 * word;
+  const bool aligned = (W & 3) == 0 && p + 4 <= W && ((uintptr_t)rows & 3) == 0;
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  for (uint64_t j0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j0 < m; j0 += 4 * stride) {
+    uint32_t row[4], k[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint64_t j = j0 + u * stride;
+      row[u] = j < m ? __ldg(perm + __ldg(pos + j)) : 0u;
     }
-    keys[j] = ((uint64_t)seg[j] << 32) | k;
-    payload[j] = row;
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint64_t j = j0 + u * stride;
+      k[u] = 0;
+      if (j >= m) continue;
+      if (aligned) {
+        k[u] = __ldg((const unsigned int*)(rows + (uint64_t)row[u] * W + p));
+      } else {
+        for (uint32_t q = 0; q < 4; ++q) k[u] = (k[u] << 8) | (p + q < W ? rows[(uint64_t)row[u] * W + p + q] : 0u);
+        k[u] = __byte_perm(k[u], 0, 0x0123);  // undone below: both branches yield big-endian order
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint64_t j = j0 + u * stride;
+      if (j >= m) continue;
+      keys[j] = ((uint64_t)__ldg(seg + j) << 32) | __byte_perm(k[u], 0, 0x0123);
+      payload[j] = row[u];
+    }
   }
 }
 
@@ -544,6 +564,81 @@ __global__ void __launch_bounds__(kSW / 4) k_seg_window_sort(uint64_t* __restric
       rows[b0 + e] = rs[e];
     }
     __syncthreads();
+  }
+}
+
+// ---- warp-per-range sort (levels whose ranges are all <= 256 rows) -------------------------------
+// One warp sorts one range in registers with a bitonic network over (key << 32 | index in range):
+// the index makes every element distinct, so the order is the stable one. N = 32 R elements,
+// element i = r * 32 + lane in register r; partners at distance >= 32 are in the same lane
+// (registers r, r ^ j/32), closer ones in lane ^ j (shuffle). Rows follow their index after the sort.
+template <int R>
+__device__ __forceinline__ void warp_range_sort(uint64_t* __restrict__ keys, uint32_t* __restrict__ rows,
+                                                uint32_t start, uint32_t len, unsigned lane) {
+  constexpr int N = 32 * R;
+  uint64_t v[R];
+  const uint32_t seg = (uint32_t)(keys[start] >> 32);
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const uint32_t i = r * 32 + lane;
+    v[r] = i < len ? (keys[start + i] << 32) | i : ~0ull;
+  }
+#pragma unroll
+  for (int k = 2; k <= N; k <<= 1) {
+#pragma unroll
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      if (j >= 32) {
+        const int jr = j / 32;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          if (r & jr) continue;
+          const uint32_t i = r * 32 + lane;
+          const bool up = (i & k) == 0;
+          const uint64_t a = v[r], b = v[r + jr];
+          if ((a > b) == up) {
+            v[r] = b;
+            v[r + jr] = a;
+          }
+        }
+      } else {
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+          const uint32_t i = r * 32 + lane;
+          const uint64_t o = __shfl_xor_sync(0xffffffffu, v[r], j);
+          const bool up = (i & k) == 0, low = (lane & j) == 0;
+          v[r] = (low == up) ? (v[r] < o ? v[r] : o) : (v[r] > o ? v[r] : o);
+        }
+      }
+    }
+  }
+  uint32_t rr[R];
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const uint32_t i = r * 32 + lane;
+    rr[r] = i < len ? rows[start + (uint32_t)(v[r] & 0xFFFFFFFFull)] : 0u;
+  }
+  __syncwarp();
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const uint32_t i = r * 32 + lane;
+    if (i < len) {
+      keys[start + i] = ((uint64_t)seg << 32) | (v[r] >> 32);
+      rows[start + i] = rr[r];
+    }
+  }
+}
+
+__global__ void __launch_bounds__(256) k_seg_warp_sort(uint64_t* __restrict__ keys, uint32_t* __restrict__ rows,
+                                                      const uint32_t* __restrict__ starts, uint64_t nr, uint64_t m) {
+  const unsigned lane = threadIdx.x & 31;
+  const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
+  for (uint64_t s = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); s < nr; s += nwarps) {
+    const uint32_t start = starts[s], end = s + 1 < nr ? starts[s + 1] : (uint32_t)m, len = end - start;
+    if (len <= 1) continue;
+    if (len <= 32) warp_range_sort<1>(keys, rows, start, len, lane);
+    else if (len <= 64) warp_range_sort<2>(keys, rows, start, len, lane);
+    else if (len <= 128) warp_range_sort<4>(keys, rows, start, len, lane);
+    else warp_range_sort<8>(keys, rows, start, len, lane);
   }
 }
 
@@ -785,6 +880,7 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
   // from the block cache (every level ends with a synchronisation, so it is idle on return)
   static const bool dbg = getenv("BLU_SORT_DEBUG") != nullptr;
   const bool no_seg = getenv("BLU_SORT_NO_SEG") != nullptr;  // always the batched global radix sort
+  const bool no_warp = getenv("BLU_SORT_NO_WARP") != nullptr;  // window sort even for ranges <= 256
   const char* sgw = getenv("BLU_SORT_SEG_W");
   const int seg_w = sgw ? atoi(sgw) : 2048;
   auto hnow = [] {
@@ -857,7 +953,18 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
     }
     const uint64_t* lk = k64b;
     const uint32_t* lrows = pb;
-    if (maxlen <= (uint32_t)sw / 2) {
+    if (maxlen <= 256 && !no_warp) {  // one warp per range, bitonic in registers
+      if (tm) cudaEventRecord(tm->next(), st);
+      k_seg_warp_sort<<<(uint32_t)sms_now() * 8, 256, 0, st>>>(k64a, pa, seg1, nr, m);
+      if (tm) {
+        cudaEventRecord(tm->next(), st);
+        tm->bytes += 2ull * m * (8 + 4);
+      }
+      count_launch(1);
+      SCK(cudaGetLastError(), "seg warp sort");
+      lk = k64a;
+      lrows = pa;
+    } else if (maxlen <= (uint32_t)sw / 2) {
       static bool attr = false;
       if (!attr) {
         SCK(cudaFuncSetAttribute(k_seg_window_sort<4096>, cudaFuncAttributeMaxDynamicSharedMemorySize,

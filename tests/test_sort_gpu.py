@@ -94,14 +94,17 @@ def test_sort_rows_special_cases(bg):
     assert np.array_equal(u32(perm), np.arange(n, dtype=np.uint32)[::-1])
 
 
-@pytest.mark.parametrize("sw", ["2048", "4096"])
-@pytest.mark.parametrize("run", [1, 2, 7, 300, 1024, 1025, 2048, 2049, 5000])
+@pytest.mark.parametrize("sw", ["2048", "4096", "2048-nowarp"])
+@pytest.mark.parametrize("run", [1, 2, 7, 33, 100, 256, 257, 300, 1024, 1025, 2048, 2049, 5000])
 def test_sort_rows_window_boundaries(bg, monkeypatch, run, sw):
     """Level-1 ranges of a fixed length (word 0 = row // run) whose level-1 keys are random with many
-    ties (word 1 from {0..3}): ranges of up to sw/2 rows straddle the sw-row windows at every offset
-    and take the window sort; longer ones take the batched radix sort. Word 2 = row id reversed keeps
+    ties (word 1 from {0..3}): ranges of up to 256 rows take the warp sort (every network size), up to
+    sw/2 rows the window sort (straddling the sw-row windows at every offset), longer ones the batched
+    radix sort. Word 2 = row id reversed keeps
     a third level for the tied rows."""
-    monkeypatch.setenv("BLU_SORT_SEG_W", sw)
+    monkeypatch.setenv("BLU_SORT_SEG_W", sw[:4])
+    if sw.endswith("nowarp"):  # ranges <= 256 rows take the window sort instead of the warp sort
+        monkeypatch.setenv("BLU_SORT_NO_WARP", "1")
     n = 60_001
     rng = np.random.default_rng(run)
     i = np.arange(n, dtype=np.uint64)

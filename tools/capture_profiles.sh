@@ -25,7 +25,9 @@ if [ "$WHAT" = ncu ] || [ "$WHAT" = all ]; then
   # sort offload (NEXT-4): launch list and one radix downsweep (a level-2 pass: random digits)
   ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/${TAG}_launches_S1.csv \
       python bench.py --config S1 --steps 1 --warmup 3 --no-e2e --no-cpu > /dev/null 2>&1
-  ncu --set full --clock-control none --import-source on -k regex:"k_rs_downsweep" -s 40 -c 1 -o $O/${TAG}_prof_S1 \
+  ncu --set full --clock-control none --import-source on -k regex:"k_rs_downsweep<unsigned long>" -s 6 -c 1 -o $O/${TAG}_prof_S1 \
+      python bench.py --config S1 --steps 1 --warmup 3 --no-e2e --no-cpu > /dev/null 2>&1
+  ncu --set full --clock-control none --import-source on -k regex:"k_seg_warp_sort" -s 2 -c 1 -o $O/${TAG}_prof_S1w \
       python bench.py --config S1 --steps 1 --warmup 3 --no-e2e --no-cpu > /dev/null 2>&1
 fi
 if [ "$WHAT" = bench ] || [ "$WHAT" = all ]; then
