@@ -205,6 +205,23 @@ def run_sort_reference(args):
     return 0
 
 
+def init_dist(torch, dist):
+    """One process per GPU (torchrun env), NCCL process group for N > 1. Test-only overrides:
+    BLU_BENCH_DIST_BACKEND=gloo and BLU_BENCH_DEVICE=<index> run every rank on one GPU, to exercise the
+    N > 1 code path (partition, exchange, merge, max-over-ranks timing) where only one GPU exists."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("BLU_BENCH_DEVICE", os.environ.get("LOCAL_RANK", "0")))
+    torch.cuda.set_device(local)
+    if world > 1:
+        backend = os.environ.get("BLU_BENCH_DIST_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+    return world, rank, local
+
+
 def run_sort(args):
     import torch
     import torch.distributed as dist
@@ -212,12 +229,7 @@ def run_sort(args):
     import blugen
     from paper_conf_sigmod_merajispcksygnk16_b200 import blugby as bg
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    world, rank, local = init_dist(torch, dist)
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream(dev)
     n = args.rows or SORT_N
@@ -335,13 +347,8 @@ def main():
     from paper_conf_sigmod_merajispcksygnk16_b200 import blugby as bg
     from paper_conf_sigmod_merajispcksygnk16_b200 import dist as bdist
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
+    world, rank, local = init_dist(torch, dist)
     bg.blu_gby_bind_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream(dev)
 
@@ -389,7 +396,7 @@ def main():
         ev[i][0].record(stream)
         r = step()
         ev[i][1].record(stream)
-        t = bg.blu_gby_last_timing()
+        t = getattr(r, "agg_timing", None) or bg.blu_gby_last_timing()  # N > 1: the rank-local aggregation
         agg_ms.append(t["aggregate_ms"] / max(1, t["aggregate_launches"]))
         agg_kernel = t["kernel"]
         part_t.append((t["scatter_ms"], t["pass2_ms"], t["part_chunks"]))

@@ -1007,12 +1007,26 @@ blu_status_t blu_gby_execute_dense_state(blu_gby_plan_t P, const void* const* ke
   base.flags = (uint32_t*)small;
   fill_smem_layout(base, P->path == BLU_PATH_DENSE_SMEM ? (uint32_t)L.domain : base.front_slots, base.front_slots > 0);
   base.jit_ok = L.key_words == 2 ? 0 : 1;
-  CK(agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, nullptr), "aggregate");
+  uint32_t launches = 0;
+  if (t_timing) {
+    t_ev.make();
+    cudaEventRecord(t_ev.e[1], st);
+  }
+  CK(agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, &launches), "aggregate");
+  if (t_timing) cudaEventRecord(t_ev.e[2], st);
   uint64_t* hs = pinned_scratch();
   uint64_t hb[2] = {0, 0};
   uint64_t* dst = hs ? hs : hb;
   CK(cudaMemcpyAsync(dst, small, 8, cudaMemcpyDeviceToHost, st), "flags D2H");
   CK(cudaStreamSynchronize(st), "sync");
+  if (t_timing) {  // the aggregation launches of this call (multi-GPU path (a): the per-rank kernel)
+    blu_gby_timing_t tm{};
+    cudaEventElapsedTime(&tm.aggregate_ms, t_ev.e[1], t_ev.e[2]);
+    tm.aggregate_launches = launches;
+    tm.total_ms = tm.aggregate_ms;
+    memcpy(tm.kernel, t_last_kernel, sizeof tm.kernel);
+    t_last = tm;
+  }
   if ((uint32_t)dst[0] & FLAG_KEY_RANGE) return fail(BLU_E_KEY_RANGE, "a key code is outside [0, dict_size)");
   return BLU_OK;
 }

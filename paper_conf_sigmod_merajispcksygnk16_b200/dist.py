@@ -65,24 +65,36 @@ def dist_execute(plan, key_cols, val_cols, group=None, stream=None, mode=None):
     from . import blugby as bg
     P = dist.get_world_size(group)
     info = plan.info()
+    # res.agg_timing: blu_gby_last_timing() of the rank-local aggregation (the kernel that scales),
+    # taken before the exchange and merge calls overwrite it (None unless timing is enabled)
     if info["path"] != bg.BLU_PATH_HASH_GLOBAL:
         st = bg.dense_state_arrays(plan, device=key_cols[0].device)
         bg.blu_gby_execute_dense_state(plan, key_cols, val_cols, st, init=True, stream=stream)
+        t = bg.blu_gby_last_timing()
         if P > 1:
             allreduce_dense_state(st, group)
-        return bg.blu_gby_finalize_dense_state(plan, st, stream=stream), "allreduce"
+        res = bg.blu_gby_finalize_dense_state(plan, st, stream=stream)
+        res.agg_timing = t
+        return res, "allreduce"
     n_local = int(len(key_cols[0]))
     if P > 1 and exchange_mode(plan, n_local, mode) == "rows":
         words = plan.row_record_bytes // 8
         send = torch.empty(max(1, n_local) * words, dtype=torch.int64, device=key_cols[0].device)
         counts = bg.blu_gby_partition_rows(plan, key_cols, val_cols, P, send, stream=stream)
         recv = alltoallv_records(send, counts, words, group)
-        return bg.blu_gby_execute_records(plan, recv, recv.numel() // words, stream=stream), "rows"
+        res = bg.blu_gby_execute_records(plan, recv, recv.numel() // words, stream=stream)
+        res.agg_timing = bg.blu_gby_last_timing()
+        return res, "rows"
     part = bg.blu_gby_execute_partial(plan, key_cols, val_cols, stream=stream)
+    t = bg.blu_gby_last_timing()
     if P == 1:
-        return bg.blu_gby_merge(plan, [part], stream=stream), "local"
+        res = bg.blu_gby_merge(plan, [part], stream=stream)
+        res.agg_timing = t
+        return res, "local"
     words = plan.record_bytes // 8
     send = torch.empty(max(1, part.n_groups) * words, dtype=torch.int64, device=key_cols[0].device)
     counts = bg.blu_gby_partition(plan, part, P, send, stream=stream)
     recv = alltoallv_records(send, counts, words, group)
-    return bg.blu_gby_merge_records(plan, recv, recv.numel() // words, stream=stream), "partials"
+    res = bg.blu_gby_merge_records(plan, recv, recv.numel() // words, stream=stream)
+    res.agg_timing = t
+    return res, "partials"
