@@ -432,8 +432,13 @@ def main():
         sc_ms = statistics.mean(a for a, _, _ in part_t) / chunks
         p2_ms = statistics.mean(b for _, b, _ in part_t) / chunks
         rows_per_launch = n / chunks
-        sc_alg, p2_alg = rows_per_launch * (bpr + rec_bytes), rows_per_launch * rec_bytes
-        tr_sc, tr_rows_sc = load_traffic(args.config, "scatter")
+        # shared-memory bucket tables with >= 256 buckets: the scatter phase is two scatters (input ->
+        # 32 buckets, then each bucket -> its sub-buckets), i.e. the records are written twice
+        two_level = (info["part_smem"] == 1 and info["partitions"] >= 256
+                     and os.environ.get("BLU_GBY_PART_2LEVEL", "1") != "0")
+        sc_alg = rows_per_launch * (bpr + rec_bytes + (2 * rec_bytes if two_level else 0))
+        p2_alg = rows_per_launch * rec_bytes
+        tr_sc, tr_rows_sc = load_traffic(args.config, "scatter2" if two_level else "scatter")
         tr_p2, tr_rows_p2 = load_traffic(args.config, "pass2")
         phases = {
             "scatter": {"avg_launch_ms": sc_ms, "algorithmic_bytes_per_launch": sc_alg,
@@ -448,7 +453,8 @@ def main():
         agg_avg_ms = phases[dom]["avg_launch_ms"]
         alg_bytes = phases[dom]["algorithmic_bytes_per_launch"]
         traffic = phases[dom]["traffic"]
-        agg_kernel = f"{dom}: " + (agg_kernel if dom == "pass2" else "blu_jit_scatter")
+        agg_kernel = f"{dom}: " + (agg_kernel if dom == "pass2" else
+                                   "blu_jit_scatter x2 levels" if two_level else "blu_jit_scatter")
         achieved = alg_bytes / (agg_avg_ms / 1000.0) / 1e9
     else:
         achieved = alg_bytes / (agg_avg_ms / 1000.0) / 1e9
@@ -507,6 +513,7 @@ def main():
             "scaling": scaling, "vs_baseline": None, "dtype": "int64+f64", "data": "synthetic",
             "config": {"workload": f"{args.config}: {w.note}", "rows_per_gpu": n, "groups": n_groups,
                        "bytes_per_row": bpr, "path": info["path_name"], "hot_front": info["hot_front"],
+                       "partitions": info["partitions"], "bucket_tables": info["part_smem"],
                        "grid": info["grid"], "block": info["block"], "smem_bytes": info["smem_bytes"],
                        "parallelism": f"rows sharded x{world}" + (" + NCCL allreduce" if world > 1 and info["path"] != 1 else
                                                                    " + NCCL all-to-all" if world > 1 else ""),

@@ -293,6 +293,12 @@ blu_status_t blu_gby_read_roofline(const void* const* cols, const uint64_t* byte
  * GPU: pass the local rank). */
 blu_status_t blu_gby_bind_device(int32_t device);
 
+/* Workspace (hash tables, dense state, partition buffers) is kept in a per-process cache of device
+ * blocks reused by later calls (the "single large memory segment" of P:62). This frees the idle
+ * blocks of the current device back to CUDA (after a device synchronisation); blocks in use by a
+ * call on another thread stay. Returns the bytes freed in *freed (may be NULL). */
+blu_status_t blu_gby_release_workspace(uint64_t* freed);
+
 void blu_gby_result_free(blu_gby_result_t* r, void* stream);
 void blu_gby_plan_destroy(blu_gby_plan_t plan);
 const char* blu_gby_status_str(blu_status_t s);

@@ -111,6 +111,7 @@ def _load():
         "blu_gby_read_roofline": ([P(vp), P(u64), i32, vp, vp], i32),
         "blu_gby_jit_probe": ([vp, ctypes.c_char_p, u32, P(i32)], i32),
         "blu_gby_bind_device": ([i32], i32),
+        "blu_gby_release_workspace": ([P(u64)], i32),
         "blu_gby_result_free": ([P(ResultC), vp], None),
         "blu_gby_plan_destroy": ([vp], None),
         "blu_gby_status_str": ([i32], ctypes.c_char_p),
@@ -506,6 +507,13 @@ def blu_gby_read_roofline(cols, out, stream=None):
 
 def blu_gby_bind_device(device: int):
     _check(lib.blu_gby_bind_device(int(device)))
+
+
+def blu_gby_release_workspace() -> int:
+    """Free the library's idle cached workspace blocks on the current device; returns bytes freed."""
+    freed = ctypes.c_uint64()
+    _check(lib.blu_gby_release_workspace(ctypes.byref(freed)))
+    return int(freed.value)
 
 
 # ---- sort offload (include/blu_sort.h; PAPER.md §3, P:76-88) ----------------------------------------

@@ -572,6 +572,12 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     M = std::max<uint64_t>(budget_rows, 1ull << 22);
     P->part_chunk.store(M);
   }
+  // two-level scatter (bucket tables with >= 256 buckets; BLU_GBY_PART_2LEVEL=0 disables): B1 first-level buckets, each split
+  // into B / B1 second-level buckets by a second scatter, instead of one B-way scatter (a 2048-way
+  // scatter writes ~2 rows per bucket per tile); needs a second set of partition buffers
+  const char* tl = getenv("BLU_GBY_PART_2LEVEL");
+  const uint32_t B1 = (P->part_smem && !(tl && tl[0] == '0') && B >= 256) ? 32u : 0u;
+  if (B1) M = std::max<uint64_t>(M / 2, 1ull << 22);
   M = std::min<uint64_t>(n, M);
   if (const char* cr = getenv("BLU_GBY_PART_CHUNK")) M = std::min<uint64_t>(n, std::max<uint64_t>(1024, strtoull(cr, 0, 10)));
   // bucket capacity: the mean plus slack for the spread of the number of GROUPS per bucket (keys
@@ -587,6 +593,21 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   cudaError_t e = w.alloc(&kbuf, rows_alloc * 8);
   for (int c = 0; c < L.n_vals && e == cudaSuccess; ++c) e = w.alloc(&vbuf[c], rows_alloc * dtype_bytes(L.val_dtype[c]));
   if (e == cudaSuccess) e = w.alloc(&meta, (size_t)B * 16 + 64);
+  // first-level buffers of the two-level scatter
+  uint64_t seg_cap1 = 0;
+  void* kbuf1 = nullptr;
+  void* vbuf1[kMaxVals] = {};
+  uint64_t* d_cursor1 = nullptr;
+  if (B1 && e == cudaSuccess) {
+    const double gpb1 = std::max(1.0, (double)P->est_groups / (double)B1);
+    const double slack1 = 1.03 + std::min(1.0, 6.0 / std::sqrt(gpb1));
+    seg_cap1 = ((uint64_t)((double)((M + B1 - 1) / B1) * slack1) + 4096 + 63) & ~63ull;
+    e = w.alloc(&kbuf1, seg_cap1 * B1 * 8);
+    for (int c = 0; c < L.n_vals && e == cudaSuccess; ++c) e = w.alloc(&vbuf1[c], seg_cap1 * B1 * dtype_bytes(L.val_dtype[c]));
+    void* m1 = nullptr;
+    if (e == cudaSuccess) e = w.alloc(&m1, (size_t)B1 * 8 + 64);
+    d_cursor1 = (uint64_t*)m1;
+  }
   if (e != cudaSuccess) return e;
   const double h1 = now();
   uint64_t* d_cursor = (uint64_t*)meta;  // B cursors, gate, tile counter
@@ -643,8 +664,54 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       cudaEventRecord(tev[0], st);
     }
     int le = 0;
-    le = launch_scatter(p1, sp, st, sgrid);
-    if (le) return (cudaError_t)le;
+    if (!B1) {
+      le = launch_scatter(p1, sp, st, sgrid);
+      if (le) return (cudaError_t)le;
+    } else {
+      uint32_t lc = (uint32_t)__builtin_popcountll(base.cap_mask), lb1 = 0, lb2 = 0;
+      while ((1u << lb1) < B1) ++lb1;
+      while ((1u << lb2) < B / B1) ++lb2;
+      const uint32_t shift1 = lc > lb1 ? lc - lb1 : 0;
+      if ((e = cudaMemsetAsync(d_cursor1, 0, (size_t)B1 * 8, st))) return e;
+      ScatterParams s1 = sp;
+      s1.B = B1;
+      s1.shift = shift1;
+      s1.seg_stride = seg_cap1;
+      s1.seg_cap = seg_cap1;
+      s1.cursor = d_cursor1;
+      s1.out_key = (uint64_t*)kbuf1;
+      for (int c = 0; c < L.n_vals; ++c) s1.out_val[c] = vbuf1[c];
+      le = launch_scatter(p1, s1, st, scatter_grid((uint32_t)P->sms, B1));
+      if (le) return (cudaError_t)le;
+      uint64_t* hc = B1 <= 32 ? pinned_scratch() : nullptr;  // 256 pinned bytes
+      std::vector<uint64_t> cnt1(B1);
+      if ((e = cudaMemcpyAsync(hc ? (void*)hc : (void*)cnt1.data(), d_cursor1, (size_t)B1 * 8, cudaMemcpyDeviceToHost, st)))
+        return e;
+      if ((e = cudaStreamSynchronize(st))) return e;
+      if (hc) memcpy(cnt1.data(), hc, (size_t)B1 * 8);
+      const uint32_t B2 = B / B1;
+      for (uint32_t b1 = 0; b1 < B1; ++b1) {
+        const uint64_t c1 = std::min(cnt1[b1], seg_cap1);  // an overflowed bucket set the gate: fallback
+        if (!c1) continue;
+        AggParams q = base;
+        q.lay = L2;
+        q.key[0] = (const uint8_t*)kbuf1 + b1 * seg_cap1 * 8;
+        for (int c = 0; c < L.n_vals; ++c) q.val[c] = (const uint8_t*)vbuf1[c] + b1 * seg_cap1 * dtype_bytes(L.val_dtype[c]);
+        q.vec_ok = 3;  // segments start at multiples of 64 rows
+        q.n_rows = c1;
+        q.prefetch = 0;
+        q.cap_mask = shift1 >= 64 ? ~0ull : ((1ull << shift1) - 1);  // the slot bits below the first level's
+        ScatterParams s2 = sp;
+        s2.B = B2;
+        s2.shift = shift1 > lb2 ? shift1 - lb2 : 0;
+        s2.cursor = d_cursor + (size_t)b1 * B2;
+        s2.out_key = (uint64_t*)kbuf + (size_t)b1 * B2 * seg_cap;
+        for (int c = 0; c < L.n_vals; ++c)
+          s2.out_val[c] = (uint8_t*)vbuf[c] + (size_t)b1 * B2 * seg_cap * dtype_bytes(L.val_dtype[c]);
+        le = launch_scatter(q, s2, st, scatter_grid((uint32_t)P->sms, B2));
+        if (le) return (cudaError_t)le;
+      }
+    }
     if (dbg) cudaEventRecord(ev[1], st);
     if (t_timing) cudaEventRecord(tev[1], st);
     // pass 2 (runs if no bucket overflowed)
@@ -772,6 +839,31 @@ blu_status_t blu_gby_last_timing(blu_gby_timing_t* out) {
 }
 
 uint64_t blu_gby_launch_count(void) { return launches_total(); }
+
+blu_status_t blu_gby_release_workspace(uint64_t* freed) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  cudaError_t se = cudaDeviceSynchronize();
+  if (se != cudaSuccess) {
+    cudaGetLastError();
+    return fail(BLU_E_CUDA, "release workspace: %s", cudaGetErrorString(se));
+  }
+  uint64_t t = 0;
+  {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    for (auto it = g_cache.begin(); it != g_cache.end();) {
+      if (!it->busy && it->dev == dev) {
+        t += it->bytes;
+        cudaFree(it->p);
+        it = g_cache.erase(it);
+      } else {
+        ++it;
+      }
+    }
+  }
+  if (freed) *freed = t;
+  return BLU_OK;
+}
 
 blu_status_t blu_gby_jit_probe(blu_gby_plan_t P, char* log, uint32_t log_cap, int32_t* n_programs) {
   if (!P) return fail(BLU_E_INVALID, "NULL plan");

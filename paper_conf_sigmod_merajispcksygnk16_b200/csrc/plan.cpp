@@ -431,24 +431,38 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     uint64_t budget = (uint64_t)kPartBudgetMB << 20;
     if (const char* pm = env("BLU_GBY_PART_MB")) budget = (uint64_t)atoi(pm) << 20;
     uint64_t tbytes = P->cap * (uint64_t)L.slot_bytes;
-    // shared-memory bucket tables are opt-in: measured on C3 (10^9 rows, 10^7 groups) they need
-    // >= 2048 buckets, whose scatter costs 32 ms against 10 ms for the 32-bucket L2 mode
+    // Shared-memory bucket tables: C3 (10^9 rows, 10^7 groups) needs 2048 buckets. Scattered in one
+    // pass that costs 31 ms against 9.4 ms for the 32-bucket L2 mode; in two passes (32 x 64, api.cu)
+    // 19.4 ms, and pass 2 drops from 25.4 to 12.5 ms: 32.5 vs 35.7 ms. So the mode is
+    // the default when the estimated groups fit >= 256 buckets of at most kMaxBuckets (two-level
+    // scatter); C5's 5*10^7 groups do not fit and keep the L2 mode. BLU_GBY_PART_SMEM=0/1 overrides.
+    auto S_of = [&](uint32_t b) {
+      uint32_t S = 16;
+      while (bucket_smem_bytes(L, S + 16, b) <= kSmemMax) S += 16;
+      return S;
+    };
+    // smallest B whose buckets hold <= kBucketLoad * S groups on average, within the scatter's
+    // shared memory and <= kMaxBuckets; the records' layout has the same fields as L
+    auto smem_B = [&]() {
+      uint64_t b = 2;
+      while (b < kMaxBuckets && (double)P->est_groups > kBucketLoad * S_of((uint32_t)b) * (double)b &&
+             scatter_smem(L.n_vals, (uint32_t)b * 2) <= kSmemMax && b * 2 <= P->cap / 1024)
+        b <<= 1;
+      return b;
+    };
     bool smem_mode = false;
-    if (const char* ps = env("BLU_GBY_PART_SMEM")) smem_mode = !L.lock_off && ps[0] == '1';
+    if (const char* ps = env("BLU_GBY_PART_SMEM")) {
+      smem_mode = !L.lock_off && ps[0] == '1';
+    } else if (!L.lock_off && budget && tbytes > budget && !env("BLU_GBY_PARTS")) {
+      const uint64_t b = smem_B();
+      const char* tl = env("BLU_GBY_PART_2LEVEL");
+      smem_mode = b >= 256 && (double)P->est_groups <= kBucketLoad * S_of((uint32_t)b) * (double)b &&
+                  !(tl && tl[0] == '0');
+    }
     uint64_t B = 1;
     const char* forced = env("BLU_GBY_PARTS");
     if (smem_mode && ((budget && tbytes > budget) || (forced && atoi(forced) > 1))) {
-      // smallest B whose buckets hold <= kBucketLoad * S groups on average, within the scatter's
-      // shared memory and <= kMaxBuckets; the records' layout has the same fields as L
-      auto S_of = [&](uint32_t b) {
-        uint32_t S = 16;
-        while (bucket_smem_bytes(L, S + 16, b) <= kSmemMax) S += 16;
-        return S;
-      };
-      B = 2;
-      while (B < kMaxBuckets && (double)P->est_groups > kBucketLoad * S_of((uint32_t)B) * (double)B &&
-             scatter_smem(L.n_vals, (uint32_t)B * 2) <= kSmemMax && B * 2 <= P->cap / 1024)
-        B <<= 1;
+      B = smem_B();
       if (forced) B = std::max(2, std::min((int)kMaxBuckets, atoi(forced)));
       while (B > 2 && scatter_smem(L.n_vals, (uint32_t)B) > kSmemMax) B >>= 1;
       P->part_smem = 1;

@@ -93,14 +93,26 @@ def test_planner_paths_for_the_five_configs(bg):
     c5 = _plan(bg, blugen.workload("C5")).info()
     assert c1["path"] == c2["path"] == bg.BLU_PATH_DENSE_SMEM
     assert c1["capacity"] == 16 and c2["capacity"] == 1024
-    # C3: 537 MB at load 0.6 exceeds the L2 budget -> partitioned mode, sized at load <= 0.5
-    assert c3["path"] == bg.BLU_PATH_HASH_GLOBAL and c3["capacity"] == 2**25 and c3["slot_bytes"] == 32
-    assert c3["part_smem"] == 0
-    assert c3["partitions"] >= 16 and c3["capacity"] * 32 // c3["partitions"] <= 48 * 2**20
+    # C3: 537 MB at load 0.6 exceeds the L2 budget -> partitioned mode; its 10^7 groups fit 2048
+    # shared-memory bucket tables (two-level scatter), so that mode is the default
+    assert c3["path"] == bg.BLU_PATH_HASH_GLOBAL and c3["capacity"] == 2**24 and c3["slot_bytes"] == 32
+    assert c3["part_smem"] == 1 and c3["partitions"] == 2048
     assert c3["hot_front"] == 0
     assert c4["path"] == bg.BLU_PATH_DIRECT_GLOBAL and c4["capacity"] == 100_000 and c4["hot_front"] == 1
     assert c5["path"] == bg.BLU_PATH_HASH_GLOBAL and c5["capacity"] == 2**27 and c5["partitions"] >= 64
     assert c1["partitions"] == c2["partitions"] == c4["partitions"] == 1
+
+
+def test_planner_partitioned_l2_mode(bg, monkeypatch):
+    """BLU_GBY_PART_SMEM=0 (and C5, whose 5*10^7 groups do not fit the bucket tables): pass 2 into
+    L2-resident slices of the global table, sized at load <= 0.5."""
+    c5 = _plan(bg, blugen.workload("C5")).info()
+    assert c5["part_smem"] == 0 and c5["partitions"] >= 64
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "0")
+    c3 = _plan(bg, blugen.workload("C3")).info()
+    assert c3["path"] == bg.BLU_PATH_HASH_GLOBAL and c3["capacity"] == 2**25 and c3["slot_bytes"] == 32
+    assert c3["part_smem"] == 0
+    assert c3["partitions"] >= 16 and c3["capacity"] * 32 // c3["partitions"] <= 48 * 2**20
 
 
 def test_planner_partitioned_smem_mode(bg, monkeypatch):
@@ -127,8 +139,10 @@ def test_capacity_rounding(bg, monkeypatch, est, cap):
     assert p.info()["capacity"] == cap and p.info()["partitions"] == 1
     monkeypatch.delenv("BLU_GBY_PART_MB")
     p2 = bg.blu_gby_plan([(I64, 0)], [I64], [(SUM, 0)], est, 10**10)
-    if p2.info()["partitions"] > 1:  # L2-resident slices: load <= 0.5
+    if p2.info()["partitions"] > 1 and not p2.info()["part_smem"]:  # L2-resident slices: load <= 0.5
         assert p2.info()["capacity"] >= 2 * est
+    if p2.info()["part_smem"]:  # default shared-memory bucket tables: the global table keeps load <= 0.7
+        assert p2.info()["capacity"] == cap and p2.info()["partitions"] >= 256
     monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
     p3 = bg.blu_gby_plan([(I64, 0)], [I64], [(SUM, 0)], est, 10**10)
     if p3.info()["partitions"] > 1:  # shared-memory bucket tables: the global table keeps load <= 0.7

@@ -418,14 +418,17 @@ def test_partitioned_two_pass(bg, oracles, monkeypatch, parts, chunk, div, smem)
     assert_parity(gk, ga, o, w.schema)
 
 
+@pytest.mark.parametrize("two_level", ["0", "1"])
 @pytest.mark.parametrize("parts", [None, "4096"])
-def test_partitioned_wide_fanout(bg, monkeypatch, parts):
+def test_partitioned_wide_fanout(bg, monkeypatch, parts, two_level):
     """Shared-memory bucket tables as planned for 2M groups (several hundred buckets, the 1024-thread
-    wide scatter) and with a forced 4096-way scatter, at 20M rows, against the oracle."""
+    wide scatter) and with a forced 4096-way scatter, at 20M rows, against the oracle; in one B-way
+    scatter or in two levels (32 first-level buckets, each scattered again into B / 32)."""
     w = blugen.workload("C3", n_rows=20_000_003, n_groups=2_000_000)
     o = oracle.groupby_generated(w)
     kc, vc = blugen.device_columns(w)
     monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
+    monkeypatch.setenv("BLU_GBY_PART_2LEVEL", two_level)
     if parts:
         monkeypatch.setenv("BLU_GBY_PARTS", parts)
     plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
@@ -462,12 +465,13 @@ def test_partitioned_skew_falls_back(bg, monkeypatch, smem):
     assert_parity(gk, ga, o, sch)
 
 
-@pytest.mark.parametrize("smem", ["1", "0"])
+@pytest.mark.parametrize("smem", ["1", "0", "2level"])
 def test_partitioned_with_regrow(bg, oracles, monkeypatch, smem):
     w, o = oracles("C5")
     kc, vc = blugen.device_columns(w)
-    monkeypatch.setenv("BLU_GBY_PARTS", "4")
-    monkeypatch.setenv("BLU_GBY_PART_SMEM", smem)
+    monkeypatch.setenv("BLU_GBY_PARTS", "4" if smem != "2level" else "512")
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "1" if smem == "2level" else smem)
+    monkeypatch.setenv("BLU_GBY_PART_2LEVEL", "1" if smem == "2level" else "0")
     plan = bg.plan_for(w.schema, 1000, w.n_rows)  # under-estimate: partitioned + regrow
     res = bg.blu_gby_execute(plan, kc, vc)
     gk, ga = gpu_sorted(res, w.schema)

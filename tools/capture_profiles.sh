@@ -18,8 +18,14 @@ if [ "$WHAT" = ncu ] || [ "$WHAT" = all ]; then
       python bench.py --config C1 --steps 1 --warmup 3 --no-e2e --no-cpu > /dev/null 2>&1
   ncu --set full --clock-control none --import-source on -k regex:"blu_jit_global" -s 2 -c 1 -o $O/${TAG}_prof_C3p2 \
       env ITERS=3 python tools/phase_probe.py C3 > /dev/null 2>&1
-  ncu --set full --clock-control none --import-source on -k regex:"blu_jit_scatter" -s 2 -c 1 -o $O/${TAG}_prof_C3sc \
-      env ITERS=3 python tools/phase_probe.py C3 > /dev/null 2>&1
+  # C3's default two-level scatter: launch 0 = first level (input -> 32 buckets), launch 1 = one of the
+  # 32 second-level launches (a bucket -> its 64 sub-buckets)
+  ncu --set full --clock-control none --import-source on -k regex:"blu_jit_scatter" -s 0 -c 1 -o $O/${TAG}_prof_C3sc \
+      env ITERS=1 python tools/phase_probe.py C3 > /dev/null 2>&1
+  ncu --set full --clock-control none --import-source on -k regex:"blu_jit_scatter" -s 1 -c 1 -o $O/${TAG}_prof_C3sc2 \
+      env ITERS=1 python tools/phase_probe.py C3 > /dev/null 2>&1
+  ncu --set full --clock-control none --import-source on -k regex:"blu_jit_bucket" -s 0 -c 1 -o $O/${TAG}_prof_C3bk \
+      env ITERS=1 python tools/phase_probe.py C3 > /dev/null 2>&1
   ncu --set full --clock-control none --import-source on -k regex:"blu_jit_global" -s 2 -c 1 -o $O/${TAG}_prof_C4 \
       env ITERS=3 python tools/phase_probe.py C4 > /dev/null 2>&1
   # sort offload (NEXT-4): launch list and one radix downsweep (a level-2 pass: random digits)
