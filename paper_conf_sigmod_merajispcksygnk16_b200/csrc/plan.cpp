@@ -59,6 +59,7 @@ constexpr uint64_t kRowLockRatio = 16;          // kernel 3 when rows/groups <= 
 constexpr uint32_t kPartBudgetMB = 48;          // L2 slice per bucket (126 MB L2)
 constexpr uint32_t kSmemMax = 232448;           // dynamic shared memory per CTA (227 KB opt-in)
 constexpr uint32_t kMaxBuckets = 4096;          // one-pass scatter fan-out
+constexpr uint32_t kMaxBuckets2 = 16384;        // two-level scatter (32 x 512)
 constexpr double kBucketLoad = 0.7;             // mean groups per bucket / bucket table entries
 
 static bool field_q(int kind) { return kind == FK_SUMQ || kind == FK_MINQ || kind == FK_MAXQ; }
@@ -443,28 +444,33 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     };
     // smallest B whose buckets hold <= kBucketLoad * S groups on average, within the scatter's
     // shared memory and <= kMaxBuckets; the records' layout has the same fields as L
-    auto smem_B = [&]() {
+    // two_level: the fan-outs are 32 and b / 32 (api.cu), so b may exceed the one-pass limit
+    auto smem_B = [&](bool two_level) {
+      const uint64_t max_b = two_level ? kMaxBuckets2 : kMaxBuckets;
       uint64_t b = 2;
-      while (b < kMaxBuckets && (double)P->est_groups > kBucketLoad * S_of((uint32_t)b) * (double)b &&
-             scatter_smem(L.n_vals, (uint32_t)b * 2) <= kSmemMax && b * 2 <= P->cap / 1024)
+      while (b < max_b && (double)P->est_groups > kBucketLoad * S_of((uint32_t)b) * (double)b &&
+             scatter_smem(L.n_vals, (uint32_t)(two_level && b >= 256 ? std::max<uint64_t>(64, 2 * b / 32) : b * 2)) <=
+                 kSmemMax &&
+             b * 2 <= P->cap / 1024)
         b <<= 1;
       return b;
     };
+    const char* tl = env("BLU_GBY_PART_2LEVEL");
+    const bool two_ok = !(tl && tl[0] == '0');
     bool smem_mode = false;
     if (const char* ps = env("BLU_GBY_PART_SMEM")) {
       smem_mode = !L.lock_off && ps[0] == '1';
-    } else if (!L.lock_off && budget && tbytes > budget && !env("BLU_GBY_PARTS")) {
-      const uint64_t b = smem_B();
-      const char* tl = env("BLU_GBY_PART_2LEVEL");
-      smem_mode = b >= 256 && (double)P->est_groups <= kBucketLoad * S_of((uint32_t)b) * (double)b &&
-                  !(tl && tl[0] == '0');
+    } else if (!L.lock_off && budget && tbytes > budget && !env("BLU_GBY_PARTS") && two_ok) {
+      const uint64_t b = smem_B(true);
+      smem_mode = b >= 256 && (double)P->est_groups <= kBucketLoad * S_of((uint32_t)b) * (double)b;
     }
     uint64_t B = 1;
     const char* forced = env("BLU_GBY_PARTS");
     if (smem_mode && ((budget && tbytes > budget) || (forced && atoi(forced) > 1))) {
-      B = smem_B();
-      if (forced) B = std::max(2, std::min((int)kMaxBuckets, atoi(forced)));
-      while (B > 2 && scatter_smem(L.n_vals, (uint32_t)B) > kSmemMax) B >>= 1;
+      B = smem_B(two_ok);
+      if (forced) B = std::max(2, std::min((int)(two_ok ? kMaxBuckets2 : kMaxBuckets), atoi(forced)));
+      auto widest = [&](uint64_t b) { return (uint32_t)(two_ok && b >= 256 ? std::max<uint64_t>(32, b / 32) : b); };
+      while (B > 2 && scatter_smem(L.n_vals, widest(B)) > kSmemMax) B >>= 1;
       P->part_smem = 1;
       P->bucket_S = S_of((uint32_t)B);
       P->bucket_smem = bucket_smem_bytes(L, P->bucket_S, (uint32_t)B);

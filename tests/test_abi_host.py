@@ -104,11 +104,17 @@ def test_planner_paths_for_the_five_configs(bg):
 
 
 def test_planner_partitioned_l2_mode(bg, monkeypatch):
-    """BLU_GBY_PART_SMEM=0 (and C5, whose 5*10^7 groups do not fit the bucket tables): pass 2 into
-    L2-resident slices of the global table, sized at load <= 0.5."""
+    """C5's 5*10^7 groups fit 16384 bucket tables of the two-level scatter (default); with
+    BLU_GBY_PART_SMEM=0 pass 2 goes into L2-resident slices of the global table, sized at load <= 0.5;
+    K3's 8-field states do not fit and keep the L2 mode."""
+    c5 = _plan(bg, blugen.workload("C5")).info()
+    assert c5["part_smem"] == 1 and c5["partitions"] == 16384
+    assert 5 * 10**7 / c5["partitions"] <= 0.7 * c5["bucket_entries"]
+    k3 = _plan(bg, blugen.workload("K3")).info()
+    assert k3["part_smem"] == 0 and k3["partitions"] > 1
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "0")
     c5 = _plan(bg, blugen.workload("C5")).info()
     assert c5["part_smem"] == 0 and c5["partitions"] >= 64
-    monkeypatch.setenv("BLU_GBY_PART_SMEM", "0")
     c3 = _plan(bg, blugen.workload("C3")).info()
     assert c3["path"] == bg.BLU_PATH_HASH_GLOBAL and c3["capacity"] == 2**25 and c3["slot_bytes"] == 32
     assert c3["part_smem"] == 0
@@ -118,12 +124,15 @@ def test_planner_partitioned_l2_mode(bg, monkeypatch):
 def test_planner_partitioned_smem_mode(bg, monkeypatch):
     """BLU_GBY_PART_SMEM=1: pass 2 in per-CTA shared-memory bucket tables; buckets hold <= 0.7 x the
     table's entries on average (C3: 10^7 / 2048 = 4883 of 8000); the global table keeps load <= 0.7;
-    the one-pass scatter fans out to at most 4096 buckets (C5)."""
+    the two-level scatter (32 x 512) allows 16384 buckets (C5), a one-level scatter at most 4096."""
     monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
     c3 = _plan(bg, blugen.workload("C3")).info()
     assert c3["part_smem"] == 1 and c3["capacity"] == 2**24
     assert c3["partitions"] == 2048 and c3["bucket_entries"] >= 7900
     assert 10**7 / c3["partitions"] <= 0.7 * c3["bucket_entries"]
+    c5 = _plan(bg, blugen.workload("C5")).info()
+    assert c5["part_smem"] == 1 and c5["partitions"] == 16384
+    monkeypatch.setenv("BLU_GBY_PART_2LEVEL", "0")
     c5 = _plan(bg, blugen.workload("C5")).info()
     assert c5["part_smem"] == 1 and c5["partitions"] == 4096
 
