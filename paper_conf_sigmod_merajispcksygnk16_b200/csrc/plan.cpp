@@ -445,8 +445,8 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     // smallest B whose buckets hold <= kBucketLoad * S groups on average, within the scatter's
     // shared memory and <= kMaxBuckets; the records' layout has the same fields as L
     // two_level: the fan-outs are 32 and b / 32 (api.cu), so b may exceed the one-pass limit
-    auto smem_B = [&](bool two_level) {
-      const uint64_t max_b = two_level ? kMaxBuckets2 : kMaxBuckets;
+    auto smem_B = [&](bool two_level, bool cap_default = false) {
+      const uint64_t max_b = two_level && !cap_default ? kMaxBuckets2 : kMaxBuckets;
       uint64_t b = 2;
       while (b < max_b && (double)P->est_groups > kBucketLoad * S_of((uint32_t)b) * (double)b &&
              scatter_smem(L.n_vals, (uint32_t)(two_level && b >= 256 ? std::max<uint64_t>(64, 2 * b / 32) : b * 2)) <=
@@ -461,13 +461,16 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     if (const char* ps = env("BLU_GBY_PART_SMEM")) {
       smem_mode = !L.lock_off && ps[0] == '1';
     } else if (!L.lock_off && budget && tbytes > budget && !env("BLU_GBY_PARTS") && two_ok) {
-      const uint64_t b = smem_B(true);
+      // default only up to kMaxBuckets: C5 (5*10^7 groups) in 16384 tables behind a 32 x 512 scatter
+      // measured 45.5 ms per 10^9 rows against 36.7 ms in the L2-slice mode (the 512-way second level
+      // and the smaller tables cost more than the L2 atomics they save)
+      const uint64_t b = smem_B(true, true);
       smem_mode = b >= 256 && (double)P->est_groups <= kBucketLoad * S_of((uint32_t)b) * (double)b;
     }
     uint64_t B = 1;
     const char* forced = env("BLU_GBY_PARTS");
     if (smem_mode && ((budget && tbytes > budget) || (forced && atoi(forced) > 1))) {
-      B = smem_B(two_ok);
+      B = smem_B(two_ok, !env("BLU_GBY_PART_SMEM"));
       if (forced) B = std::max(2, std::min((int)(two_ok ? kMaxBuckets2 : kMaxBuckets), atoi(forced)));
       auto widest = [&](uint64_t b) { return (uint32_t)(two_ok && b >= 256 ? std::max<uint64_t>(32, b / 32) : b); };
       while (B > 2 && scatter_smem(L.n_vals, widest(B)) > kSmemMax) B >>= 1;

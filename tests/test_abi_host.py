@@ -104,12 +104,11 @@ def test_planner_paths_for_the_five_configs(bg):
 
 
 def test_planner_partitioned_l2_mode(bg, monkeypatch):
-    """C5's 5*10^7 groups fit 16384 bucket tables of the two-level scatter (default); with
-    BLU_GBY_PART_SMEM=0 pass 2 goes into L2-resident slices of the global table, sized at load <= 0.5;
-    K3's 8-field states do not fit and keep the L2 mode."""
+    """C5's 5*10^7 groups need more than 4096 bucket tables (16384 measured slower than the L2 mode)
+    and K3's 8-field states do not fit either: both keep pass 2 in L2-resident slices of the global
+    table, sized at load <= 0.5; BLU_GBY_PART_SMEM=0 forces that mode for C3 too."""
     c5 = _plan(bg, blugen.workload("C5")).info()
-    assert c5["part_smem"] == 1 and c5["partitions"] == 16384
-    assert 5 * 10**7 / c5["partitions"] <= 0.7 * c5["bucket_entries"]
+    assert c5["part_smem"] == 0 and c5["partitions"] >= 64
     k3 = _plan(bg, blugen.workload("K3")).info()
     assert k3["part_smem"] == 0 and k3["partitions"] > 1
     monkeypatch.setenv("BLU_GBY_PART_SMEM", "0")
