@@ -139,8 +139,13 @@ ALL = lambda nv: [(COUNT, -1)] + [(op, c) for c in range(nv) for op in (SUM, MIN
 
 
 @pytest.mark.parametrize("n", [0, 1, 3, 31, 33, 4095, 4097, 65_537])
-@pytest.mark.parametrize("path", ["a", "b", "d"])
+@pytest.mark.parametrize("path", ["a", "a-nofuse", "b", "d"])
 def test_small_and_ragged(bg, monkeypatch, n, path):
+    """Tiny and ragged sizes on every path; "a-nofuse" takes the unfused, software-pipelined dense
+    kernel (the one large inputs use) instead of the fused small-input one."""
+    if path == "a-nofuse":
+        monkeypatch.setenv("BLU_GBY_NO_FUSE", "1")
+        path = "a"
     rng = np.random.default_rng(n + 7)
     sch = blugen.Schema([(I32, 13), (I64, 7)], [I32, I64, F64], ALL(3))
     kc = [rng.integers(0, 13, n).astype(np.int32), rng.integers(0, 7, n).astype(np.int64)]
@@ -198,6 +203,7 @@ def test_key_range_errors(bg):
 def test_key_range_errors_large(bg, monkeypatch, path, front):
     """Out-of-range codes caught by the software-pipelined kernels (tile_unpack) at sizes that take
     the unfused, multi-tile launch; the bad row is the last one (ragged tail) or deep inside."""
+    monkeypatch.setenv("BLU_GBY_NO_FUSE", "1")  # path (a): the pipelined kernel, not the fused one
     n = 5_000_011
     sch = blugen.Schema([(I32, 30), (I32, 40)], [I64], [(COUNT, -1), (SUM, 0)])
     monkeypatch.setenv("BLU_GBY_FORCE_PATH", path)
