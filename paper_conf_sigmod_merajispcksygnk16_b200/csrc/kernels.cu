@@ -55,7 +55,8 @@ static bool launch_jit(const char* body, const char* entry_decl, const AggParams
                        uint32_t grid, uint32_t block, uint32_t smem, const char* entry, int min_blocks = 1) {
   if (!p.jit_ok || !jit_enabled()) return false;
   // 1024-thread CTAs (one per SM, wide hot-key front) keep the same 64-register budget
-  const int maxt = block > 512 ? 1024 : 512, minb = block > 512 ? 1 : jit_env("BLU_GBY_JIT_MINB", min_blocks);
+  // (a 768-thread CTA gets 80 registers: __launch_bounds__(768, 1))
+  const int maxt = block > 512 ? (int)block : 512, minb = block > 512 ? 1 : jit_env("BLU_GBY_JIT_MINB", min_blocks);
   std::string src = "extern \"C\" __global__ void __launch_bounds__(" + std::to_string(maxt) + ", " +
                     std::to_string(minb) + ") ";
   src += entry_decl;
@@ -1099,7 +1100,8 @@ static int launch_agg_nv(const blu_gby_plan_s* P, int path, const AggParams& p, 
       // MODE 4: the same for pass 2 of the partitioned path (BLU_GBY_SEG_PIPE=0/1)
       const int pipe = p.seg_stride ? jit_env("BLU_GBY_SEG_PIPE", 0) : jit_env("BLU_GBY_PIPE", 1);
       const int mode = p.seg_stride ? (pipe ? 4 : 2) : pipe ? 3 : 0;
-      if (pipe) r = jit_env("BLU_GBY_PIPE_R", 2) >= 4 ? 4 : 2;
+      // rows per thread double-buffered: 4 when the CTA has 513..768 threads (>= 80 registers), else 2
+      if (pipe) r = jit_env("BLU_GBY_PIPE_R", block > 512 && block <= 768 ? 4 : 2) >= 4 ? 4 : 2;
       snprintf(name, sizeof name, "blu_jit_global_%d_%d_%d_%d_%d", nv, r, front, direct, mode);
       snprintf(decl, sizeof decl, "%s(blu::AggParams p, blu::RecSrc rs)", name);
       snprintf(body, sizeof body, "blu::global_body<blu::JitSpec, %d, %d, %s, %s, %d>(p, rs);", nv, r,
