@@ -1443,7 +1443,7 @@ __device__ __forceinline__ void bucket_flush_entry(const AggParams& p, uint8_t* 
   fk[e] = kEmpty;
 }
 
-template <class SP, int NV, int R>
+template <class SP, int NV, int R, bool PIPE = false>
 __device__ __forceinline__ void bucket_body(const AggParams& p) {
   extern __shared__ __align__(16) uint8_t sm[];
   if (p.gate && ((*(volatile const uint32_t*)p.gate != 0) != (p.gate_run_if != 0))) return;
@@ -1495,12 +1495,24 @@ __device__ __forceinline__ void bucket_body(const AggParams& p) {
     const uint64_t r0 = seg0 + (uint64_t)(item - ppre[lo]) * piece;
     const uint64_t cnt = p.seg_count[lo];
     const uint64_t r1 = seg0 + ((uint64_t)(item - ppre[lo]) * piece + piece < cnt ? (uint64_t)(item - ppre[lo]) * piece + piece : cnt);
+    // PIPE (NVRTC kernels): the piece's next tile is loaded into registers before this one is probed
+    using Raw = RawTileFor<SP, R, PIPE>;
+    Raw A, Bt;
+    if constexpr (PIPE)
+      if (r0 < r1) tile_load<SP, R>(p, lane_base<R>(r0, warp, lane), r1, pol, A);
     for (uint64_t row0 = r0; row0 < r1; row0 += tile) {
       const uint64_t row = lane_base<R>(row0, warp, lane);
       uint64_t key[R];
       uint64_t v[NV][R];
-      const uint32_t valid = pack_keys<SP, R>(p, row, r1, pol, key);
-      load_vals<SP, NV, R>(p, row, r1, pol, v);
+      uint32_t valid;
+      if constexpr (PIPE) {
+        if (row0 + tile < r1) tile_load<SP, R>(p, lane_base<R>(row0 + tile, warp, lane), r1, pol, Bt);
+        valid = tile_unpack<SP, NV, R>(p, A, row, r1, key, v);
+        A = Bt;
+      } else {
+        valid = pack_keys<SP, R>(p, row, r1, pol, key);
+        load_vals<SP, NV, R>(p, row, r1, pol, v);
+      }
       // convergent probe of the shared table: every pending row inspects one 4-entry bucket per step
       const uint32_t nbk = S >> 2;
       uint32_t e[R], h[R];

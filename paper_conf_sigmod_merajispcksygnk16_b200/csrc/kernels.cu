@@ -226,12 +226,15 @@ template <int NV, int R>
 static int launch_bucket_nv(const AggParams& p, cudaStream_t st, uint32_t grid, uint32_t smem) {
   if (p.jit_ok) {
     char body[160], decl[160], name[64];
-    snprintf(name, sizeof name, "blu_jit_bucket_%d_%d", NV, R);
+    // BLU_GBY_BUCKET_PIPE=1: 768 threads x 80 registers with the tile loads double-buffered
+    const int pipe = jit_env("BLU_GBY_BUCKET_PIPE", 0) && R % 2 == 0;
+    const uint32_t threads = pipe ? (uint32_t)jit_env("BLU_GBY_BUCKET_THREADS", 768) : 1024u;
+    snprintf(name, sizeof name, "blu_jit_bucket_%d_%d%s", NV, R, pipe ? "_p" : "");
     snprintf(decl, sizeof decl, "%s(blu::AggParams p)", name);
-    snprintf(body, sizeof body, "blu::bucket_body<blu::JitSpec, %d, %d>(p);", NV, R);
+    snprintf(body, sizeof body, "blu::bucket_body<blu::JitSpec, %d, %d, %s>(p);", NV, R, pipe ? "true" : "false");
     AggParams pc = p;
     void* args[] = {&pc};
-    if (launch_jit(body, decl, p, args, st, grid, 1024, smem, name, 1)) return 0;
+    if (launch_jit(body, decl, p, args, st, grid, threads, smem, name, 1)) return 0;
   }
   auto k = k_agg_bucket<NV, R>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
