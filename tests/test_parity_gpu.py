@@ -449,17 +449,19 @@ def test_partitioned_wide_fanout(bg, monkeypatch, parts, two_level):
     assert_parity(gk, ga, o, w.schema)
 
 
-@pytest.mark.parametrize("smem", ["1", "0"])
+@pytest.mark.parametrize("smem", ["1", "0", "2level"])
 def test_partitioned_skew_falls_back(bg, monkeypatch, smem):
-    """A bucket overflow (every row in one bucket) takes the device-side fallback: still exact."""
-    n = 600_000
+    """A bucket overflow (every row in one bucket) takes the device-side fallback: still exact; with the
+    two-level scatter the first level overflows and the second level sees truncated buckets (the
+    partitioned path needs >= 4096 rows per bucket: 512 buckets -> 2.2M rows)."""
+    n = 2_200_000 if smem == "2level" else 600_000
     rng = np.random.default_rng(3)
     sch = blugen.Schema([(I64, 0)], [I64, F64], [(COUNT, -1), (SUM, 0), (AVG, 1), (MIN, 0), (MAX, 1)])
     k = np.where(rng.random(n) < 0.9, 77, rng.integers(0, 5000, n)).astype(np.int64)
     v = [rng.integers(-(2**40), 2**40, n), rng.integers(-(2**20), 2**20, n) / 64.0]
     o = oracle.groupby_arrays(sch, [k], v)
-    monkeypatch.setenv("BLU_GBY_PARTS", "16")
-    monkeypatch.setenv("BLU_GBY_PART_SMEM", smem)
+    monkeypatch.setenv("BLU_GBY_PARTS", "512" if smem == "2level" else "16")
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "1" if smem == "2level" else smem)
     dk, dv = _mk([k], v)
     plan = bg.plan_for(sch, 5000, n)
     bg.blu_gby_set_timing(True)
