@@ -484,15 +484,24 @@ __device__ __forceinline__ void smem_apply_rows(const AggParams& p, uint8_t* sm,
   }
 #endif
   if constexpr (SP::kStatic) {  // JIT: straight-line updates; one branch per row, not per (field, row)
+#ifndef BLU_SOFF_PARAM  // table entries and field offsets are compile-time constants of the launch
+    constexpr uint32_t ST = SP::STAB;
+#else
+    const uint32_t ST = S;
+#endif
 #pragma unroll
     for (int r = 0; r < R; ++r)
       if (mask >> r & 1) {
         sfor<0, SP::NF>([&](auto jc) {
           constexpr int j = decltype(jc)::v;
           constexpr int K = SP::KIND[j], c = SP::COL[j];
+#ifndef BLU_SOFF_PARAM
+          uint8_t* b = sm + SP::SOFF[j];
+#else
           uint8_t* b = sm + p.soff[j];
-          if constexpr (c < 0) s_upd<FK_COUNT, true>(b, e[r], S, 1ull);
-          else s_upd<K, true>(b, e[r], S, v[c][r]);
+#endif
+          if constexpr (c < 0) s_upd<FK_COUNT, true>(b, e[r], ST, 1ull);
+          else s_upd<K, true>(b, e[r], ST, v[c][r]);
         });
       }
     return;

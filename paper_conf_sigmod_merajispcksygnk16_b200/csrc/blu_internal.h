@@ -111,7 +111,7 @@ void jit_probe_begin(JitProbe* pr);
 void jit_probe_end();
 bool jit_probe_active();
 const void* jit_kernel(const std::string& spec_src, const std::string& entry_src, const char* entry);
-std::string jit_spec(const char* name, const Layout& L);
+std::string jit_spec(const char* name, const Layout& L, uint32_t S, const uint32_t* soff);
 
 // Planner helpers (plan.cpp)
 uint32_t smem_entry_bytes(const Layout& lay);

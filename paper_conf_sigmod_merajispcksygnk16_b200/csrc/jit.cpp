@@ -102,7 +102,7 @@ std::string arru(const uint64_t* a, int n, int pad) {
   return s + "}";
 }
 
-std::string spec_source(const char* name, const Layout& L) {
+std::string spec_source(const char* name, const Layout& L, uint32_t S, const uint32_t* soff) {
   int kdt[kMaxKeys], vdt[kMaxVals], kind[kMaxFields], col[kMaxFields], goff[kMaxFields], sg[kMaxFields], si[kMaxFields];
   for (int k = 0; k < L.n_keys; ++k) kdt[k] = L.key_dtype[k];
   for (int c = 0; c < L.n_vals; ++c) vdt[c] = L.val_dtype[c];
@@ -132,6 +132,12 @@ std::string spec_source(const char* name, const Layout& L) {
   s += "  static constexpr unsigned long long SLOT = " + std::to_string(L.slot_bytes) + "ULL;\n";
   s += "  static constexpr unsigned long long DOMAIN = " + std::to_string((unsigned long long)L.domain) + "ULL;\n";
   s += "  static constexpr int LOCKOFF = " + std::to_string(L.lock_off) + ";\n";
+  // the launch's shared-memory table (path (a) dense table, hot-key front or bucket table): entries
+  // and per-field byte offsets, so field addresses are immediates instead of parameter loads
+  int so[kMaxFields];
+  for (int j = 0; j < L.n_fields; ++j) so[j] = soff ? (int)soff[j] : 0;
+  s += "  static constexpr unsigned STAB = " + std::to_string(S) + "u;\n";
+  s += "  static constexpr int SOFF[24] = " + arr(so, L.n_fields, 24) + ";\n";
   const char* dd = getenv("BLU_GBY_DEDUPE");
   s += std::string("  static constexpr int DEDUPE = ") + (dd && dd[0] == '1' ? "1" : "0") + ";\n";
   s += "};\n}  // namespace blu\n";
@@ -309,6 +315,8 @@ const void* jit_kernel(const std::string& spec_src, const std::string& entry_src
   return (const void*)k;
 }
 
-std::string jit_spec(const char* name, const Layout& L) { return spec_source(name, L); }
+std::string jit_spec(const char* name, const Layout& L, uint32_t S, const uint32_t* soff) {
+  return spec_source(name, L, S, soff);
+}
 
 }  // namespace blu

@@ -78,7 +78,8 @@ static bool launch_jit(const char* body, const char* entry_decl, const AggParams
   int dev = 0;
   if (!probe) cudaGetDevice(&dev);
   const char* defs = getenv("BLU_GBY_JIT_DEFS");
-  std::string tag = src + "|" + std::to_string(dev) + "|" + (defs ? defs : "");
+  std::string tag = src + "|" + std::to_string(dev) + "|" + (defs ? defs : "") + "|" + std::to_string(p.S);
+  for (int j = 0; j < p.lay.n_fields; ++j) tag += "," + std::to_string(p.soff[j]);
   uint64_t h = 1469598103934665603ull;
   for (size_t i = 0; i < sizeof(Layout); ++i) h = (h ^ ((const uint8_t*)&p.lay)[i]) * 1099511628211ull;
   for (char c : tag) h = (h ^ (uint8_t)c) * 1099511628211ull;
@@ -93,7 +94,7 @@ static bool launch_jit(const char* body, const char* entry_decl, const AggParams
     }
   }
   if (!k) {
-    k = jit_kernel(jit_spec("JitSpec", p.lay), src, entry);
+    k = jit_kernel(jit_spec("JitSpec", p.lay, p.S, p.soff), src, entry);
     if (probe) return true;  // compile-only probe: nothing is launched
     if (!k) return false;
   }
