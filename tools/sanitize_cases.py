@@ -6,12 +6,15 @@ from paper_conf_sigmod_merajispcksygnk16_b200 import blugby as bg
 cases = [("C1", dict(n_rows=100_003), None), ("C2", dict(n_rows=200_011), None), ("C2", dict(n_rows=100_000), "b"),
          ("C3", dict(n_rows=300_003, n_groups=20_000), None), ("C4", dict(n_rows=300_017), None),
          ("C3", dict(n_rows=300_003, n_groups=20_000), "parts"),
-         ("C3", dict(n_rows=300_003, n_groups=20_000), "parts_smem")]
+         ("C3", dict(n_rows=300_003, n_groups=20_000), "parts_smem"),
+         ("C4", dict(n_rows=300_017), "front"),
+         ("C3", dict(n_rows=1_000_003, n_groups=300_000), "parts_smem")]
 for name, kw, mode in cases:
     env = {}
     if mode == "b": os.environ["BLU_GBY_FORCE_PATH"] = "b"
     if mode in ("parts", "parts_smem"): os.environ["BLU_GBY_PARTS"] = "8"
     if mode == "parts_smem": os.environ["BLU_GBY_PART_SMEM"] = "1"
+    if mode == "front": os.environ["BLU_GBY_FORCE_PATH"], os.environ["BLU_GBY_HOT_FRONT"] = "d", "1"
     w = blugen.workload(name, **kw)
     kc, vc = blugen.device_columns(w)
     plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
@@ -19,8 +22,10 @@ for name, kw, mode in cases:
     p = bg.blu_gby_execute_partial(plan, kc, vc)
     m = bg.blu_gby_merge(plan, [p, p])
     torch.cuda.synchronize()
-    print(name, mode, plan.info()["path_name"], r.n_groups, m.n_groups, flush=True)
+    inf = plan.info()
+    print(name, mode, inf["path_name"], inf.get("hot_front"), inf.get("parts"), inf.get("bucket_S"), r.n_groups, m.n_groups, flush=True)
     os.environ.pop("BLU_GBY_FORCE_PATH", None); os.environ.pop("BLU_GBY_PARTS", None); os.environ.pop("BLU_GBY_PART_SMEM", None)
+    os.environ.pop("BLU_GBY_HOT_FRONT", None)
 est, ex = bg.blu_gby_estimate_groups(w.schema.keys, kc, k=256)
 print("kmv", est, ex)
 
