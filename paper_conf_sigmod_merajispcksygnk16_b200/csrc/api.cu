@@ -810,8 +810,11 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
       const uint32_t rank_words =
           P->path == BLU_PATH_DIRECT_GLOBAL && !no_rank && L.domain > 0 && W <= base.front_slots ? (uint32_t)W : 0u;
       const uint64_t* front = nullptr;
-      int rc = launch_front_seed(pk, n, base.front_slots, rank_words, ws, st, (int)P->sms, &front);
+      const uint64_t* hot = nullptr;
+      int rc = launch_front_seed(pk, n, base.front_slots, rank_words, ws, st, (int)P->sms, &front,
+                                 rank_words && jit_hot_reg() ? &hot : nullptr);
       if (rc) return (cudaError_t)rc;
+      base.hot_key = hot;
       base.front_seed = front;
       base.front_rank_words = rank_words;
     }

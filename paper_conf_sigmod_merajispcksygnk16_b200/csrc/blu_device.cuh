@@ -16,6 +16,7 @@ namespace blu {
 // Schema read from AggParams::lay at run time.
 struct GenericSpec {
   static constexpr bool kStatic = false;
+  static constexpr int HOTREG = 0;
 };
 
 // ------------------------------------------------------------------------------------------------
@@ -1037,11 +1038,101 @@ __device__ __forceinline__ void front_dedupe_rows(const AggParams& p, uint8_t* s
   __syncwarp();
 }
 
+// Register accumulator of the rank front's hottest key (SP::HOTREG, JIT only): that key's rows are
+// combined per thread in registers (encoded like the shared table) and flushed once at the end, so
+// the key that most often collides with itself inside a warp costs no shared-memory atomics.
+template <class SP, int H>
+struct HotAccT {
+  __device__ __forceinline__ void init(const uint64_t*) {}
+};
+template <class SP, int H>
+struct HotAccT2 {
+  uint64_t key[H];
+  uint64_t a[H][SP::NF];
+  template <int j>
+  static constexpr int kind() { return SP::COL[j] < 0 ? FK_COUNT : SP::KIND[j]; }
+  __device__ __forceinline__ void init(const uint64_t* hk) {
+#pragma unroll
+    for (int h = 0; h < H; ++h) {
+      key[h] = hk ? __ldg((const unsigned long long*)hk + h) : kEmpty;
+      sfor<0, SP::NF>([&](auto jc) {
+        constexpr int j = decltype(jc)::v;
+        a[h][j] = identity64(kind<j>());
+      });
+    }
+  }
+  template <int NV, int R>
+  __device__ __forceinline__ void add(int h, const uint64_t (&v)[NV][R], int r) {
+    sfor<0, SP::NF>([&](auto jc) {
+      constexpr int j = decltype(jc)::v;
+      constexpr int K = kind<j>(), c = SP::COL[j];
+      uint64_t& acc = a[h][j];
+      if constexpr (c < 0) {
+        acc += 1;
+      } else {
+        const uint64_t x = enc<K, true>(v[c][r]);
+        if constexpr (K == FK_COUNT || K == FK_SUMI) acc += x;
+        else if constexpr (K == FK_SUMF)
+          acc = (uint64_t)__double_as_longlong(__longlong_as_double((long long)acc) + __longlong_as_double((long long)x));
+        else if constexpr (K == FK_MINI32) acc = (int)x < (int)acc ? (uint64_t)(int64_t)(int)x : acc;
+        else if constexpr (K == FK_MAXI32) acc = (int)x > (int)acc ? (uint64_t)(int64_t)(int)x : acc;
+        else if constexpr (K == FK_MINI64 || K == FK_MINF64) acc = (long long)x < (long long)acc ? x : acc;
+        else acc = (long long)x > (long long)acc ? x : acc;
+      }
+    });
+  }
+  // take the rows of the hot keys out of `valid` (their fields go to registers)
+  template <int NV, int R>
+  __device__ __forceinline__ void take(const uint64_t (&k)[R], uint32_t& valid, const uint64_t (&v)[NV][R]) {
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+#pragma unroll
+      for (int h = 0; h < H; ++h)
+        if ((valid >> r & 1) && k[r] == key[h]) {
+          add(h, v, r);
+          valid &= ~(1u << r);
+        }
+  }
+  // into the key's rank-front entry, or straight into the dense state if the key is not in the front
+  __device__ __forceinline__ void flush(const AggParams& p, uint8_t* sm) {
+#pragma unroll
+    for (int h = 0; h < H; ++h) {
+      const uint64_t kh = key[h];
+      if (kh == kEmpty || count(h) == 0) continue;
+      const uint64_t x = ((const uint64_t*)(sm + p.key_off))[kh >> 5];
+      const uint32_t b = (uint32_t)kh & 31u, bits = (uint32_t)x;
+      const bool in_front = bits >> b & 1u;
+      const uint32_t e = (uint32_t)(x >> 32) + __popc(bits & ((1u << b) - 1u));
+      sfor<0, SP::NF>([&](auto jc) {
+        constexpr int j = decltype(jc)::v;
+        constexpr int K = kind<j>();
+        if (in_front) s_upd<K, false>(sm + p.soff[j], e, p.S, a[h][j]);
+        else d_upd<K, false>(dense_addr(p, j, kh), a[h][j]);
+      });
+    }
+  }
+  __device__ __forceinline__ uint64_t count(int h) const {
+    uint64_t c = 0;
+    sfor<0, SP::NF>([&](auto jc) {
+      constexpr int j = decltype(jc)::v;
+      if constexpr (kind<j>() == FK_COUNT) c = a[h][j];
+    });
+    return c;
+  }
+};
+template <class SP> struct HotAccT<SP, 1> : HotAccT2<SP, 1> {};
+template <class SP> struct HotAccT<SP, 2> : HotAccT2<SP, 2> {};
+template <class SP>
+using HotAcc = HotAccT<SP, SP::HOTREG>;
+
 // One tile's rows after loading: hot-key front (rank image or hash table), then the global table
 // (path b: convergent probing; b': direct) for the rows the front did not take.
 template <class SP, int NV, int R, bool FRONT, bool DIRECT>
 __device__ __forceinline__ void process_rows(const AggParams& p, uint8_t* sm, uint64_t (&key)[R], uint32_t valid,
-                                             uint64_t (&v)[NV][R]) {
+                                             uint64_t (&v)[NV][R], HotAcc<SP>& ha) {
+  if constexpr (FRONT && DIRECT && SP::HOTREG != 0) {  // the hottest key: registers (see HotAccT)
+    ha.take(key, valid, v);
+  }
   const Layout& L = p.lay;
   const uint32_t S = p.S;
   uint8_t* tb = (uint8_t*)p.table;
@@ -1210,6 +1301,8 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
       for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) smem_init_entry(sm + p.soff[j], L.f[j].kind, e, S);
     __syncthreads();
   }
+  HotAcc<SP> ha;
+  ha.init(FRONT && DIRECT && p.front_rank_words ? p.hot_key : nullptr);
   const uint64_t pol = evict_first_policy();
   // SEG: warp tiles (32*R rows) handed out in bucket order by a global counter, so every warp of
   // the grid stays inside the same one or two buckets (their table slices L2-resident); static
@@ -1243,7 +1336,7 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
       uint64_t key[R];
       uint64_t v[NV][R];
       const uint32_t valid = tile_unpack<SP, NV, R>(p, A, lane_base<R>(t * tile, warp, lane), n, key, v);
-      process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v);
+      process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v, ha);
       if (__any_sync(0xffffffffu, fl)) break;  // warp-uniform abort
       A = B;
       t = tn;
@@ -1285,7 +1378,7 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
       uint64_t key[R];
       uint64_t v[NV][R];
       const uint32_t valid = tile_unpack<SP, NV, R>(p, A, lbA, nA, key, v);
-      process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v);
+      process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v, ha);
       if (__any_sync(0xffffffffu, fl)) break;
       A = B;
       lbA = lbB;
@@ -1348,9 +1441,10 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
       valid = pack_keys<SP, R>(p, row, n, pol, key);
       load_vals<SP, NV, R>(p, row, n, pol, v);
     }
-    process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v);
+    process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v, ha);
     t = t_next;
   }
+  if constexpr (FRONT && DIRECT && SP::HOTREG != 0) ha.flush(p, sm);
   if (FRONT) {
     // merge the front into the global table
     __syncthreads();

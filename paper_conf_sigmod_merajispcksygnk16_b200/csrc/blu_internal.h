@@ -86,7 +86,7 @@ int launch_init_dense(const Layout& lay, void* const dense[4], uint64_t D, void*
 int launch_compact(const CompactParams& p, void* stream, uint32_t* launches);
 size_t front_seed_bytes(uint32_t S);
 int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, uint32_t rank_words, void* ws, void* stream, int sms,
-                      const uint64_t** front_out);
+                      const uint64_t** front_out, const uint64_t** hot_out = nullptr);
 int launch_read_roofline(const void* const* cols, const uint64_t* bytes, int n_cols, void* stream, uint64_t* out,
                          int sms);
 int launch_partition(const Layout& lay, const void* const* key_cols, const void* const* state_cols,
@@ -103,6 +103,7 @@ void cache_put(void* p);
 
 // NVRTC specialisation (jit.cpp)
 bool jit_enabled();
+int jit_hot_reg();
 struct JitProbe {  // compile-only mode of the JIT (blu_gby_jit_probe)
   int programs = 0, failed = 0;
   std::string log;

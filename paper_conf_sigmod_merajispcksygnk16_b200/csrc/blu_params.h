@@ -127,6 +127,10 @@ struct AggParams {
   // keys 32w..32w+31 and in its high half the number of hot keys below 32w, so a key's front entry is
   // that prefix + popc(bits below it): one shared-memory load per row, no probing. 0 = hash front.
   uint32_t front_rank_words;
+  // rank front: the sample's most frequent key (device word written by the seed kernels; ~0 = none).
+  // With SP::HOTREG each thread sums that key's rows in registers and flushes them once at the end,
+  // so the hottest key (13% of C4's Zipf(1.1) rows) costs no shared-memory atomics. NULL = off.
+  const uint64_t* hot_key;
   uint32_t prefetch;             // scatter: L2-prefetch the column bytes of the tile this many tiles ahead (0 = off)
   // partitioned pass 2 with bucket-local shared-memory tables (bucket_body): a bucket's rows are
   // cut into pieces of piece_rows rows (a multiple of the CTA tile); aux_off = byte offset of the

@@ -138,6 +138,7 @@ std::string spec_source(const char* name, const Layout& L, uint32_t S, const uin
   for (int j = 0; j < L.n_fields; ++j) so[j] = soff ? (int)soff[j] : 0;
   s += "  static constexpr unsigned STAB = " + std::to_string(S) + "u;\n";
   s += "  static constexpr int SOFF[24] = " + arr(so, L.n_fields, 24) + ";\n";
+  s += "  static constexpr int HOTREG = " + std::to_string(jit_hot_reg()) + ";\n";
   const char* dd = getenv("BLU_GBY_DEDUPE");
   s += std::string("  static constexpr int DEDUPE = ") + (dd && dd[0] == '1' ? "1" : "0") + ";\n";
   s += "};\n}  // namespace blu\n";
@@ -204,6 +205,13 @@ bool compile(const std::string& src, std::vector<char>& cubin, std::string& log)
 }
 
 }  // namespace
+
+// The rank front's 0, 1 or 2 hottest keys summed in registers (BLU_GBY_HOT_REG=0/1/2)
+int jit_hot_reg() {
+  const char* e = getenv("BLU_GBY_HOT_REG");  // read per plan execution (tests switch it)
+  const int h = e ? atoi(e) : 0;
+  return jit_enabled() ? (h < 0 ? 0 : h > 2 ? 2 : h) : 0;
+}
 
 bool jit_enabled() {
   const char* e = getenv("BLU_GBY_JIT");

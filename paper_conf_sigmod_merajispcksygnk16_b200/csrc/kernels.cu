@@ -78,7 +78,8 @@ static bool launch_jit(const char* body, const char* entry_decl, const AggParams
   int dev = 0;
   if (!probe) cudaGetDevice(&dev);
   const char* defs = getenv("BLU_GBY_JIT_DEFS");
-  std::string tag = src + "|" + std::to_string(dev) + "|" + (defs ? defs : "") + "|" + std::to_string(p.S);
+  std::string tag = src + "|" + std::to_string(dev) + "|" + (defs ? defs : "") + "|" + std::to_string(p.S) +
+                    "|hot" + std::to_string(jit_hot_reg());
   for (int j = 0; j < p.lay.n_fields; ++j) tag += "," + std::to_string(p.soff[j]);
   uint64_t h = 1469598103934665603ull;
   for (size_t i = 0; i < sizeof(Layout); ++i) h = (h ^ ((const uint8_t*)&p.lay)[i]) * 1099511628211ull;
@@ -898,10 +899,39 @@ __global__ void __launch_bounds__(1024) k_hh_rank_scan(HHParams h, uint32_t word
   }
 }
 
+// the sample's `top` most frequent keys -> (uint64_t*)(ctl + 2)[0..top) (~0 where the sample has
+// fewer keys); one CTA, one argmax pass per key
+__global__ void __launch_bounds__(1024) k_hh_top(HHParams h, int top) {
+  __shared__ unsigned long long wbest[32];
+  __shared__ unsigned long long taken[4];
+  uint64_t* out = (uint64_t*)(h.ctl + 2);
+  for (int q = 0; q < top; ++q) {
+    unsigned long long best = 0;  // (count << 32) | slot
+    for (uint64_t i = threadIdx.x; i < h.cap_s; i += blockDim.x) {
+      bool skip = false;
+      for (int u = 0; u < q; ++u) skip |= taken[u] == i;
+      const unsigned long long c = skip ? 0ull : ((unsigned long long)h.scnt[i] << 32) | (unsigned long long)i;
+      best = c > best ? c : best;
+    }
+    for (int o = 16; o; o >>= 1) {
+      const unsigned long long y = __shfl_xor_sync(0xffffffffu, best, o);
+      best = y > best ? y : best;
+    }
+    if ((threadIdx.x & 31) == 0) wbest[threadIdx.x >> 5] = best;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      for (unsigned w = 0; w < (blockDim.x >> 5); ++w) best = wbest[w] > best ? wbest[w] : best;
+      taken[q] = (best >> 32) ? (best & 0xffffffffull) : ~0ull;
+      out[q] = (best >> 32) ? h.skey[best & 0xffffffffull] : kEmpty;
+    }
+    __syncthreads();
+  }
+}
+
 size_t front_seed_bytes(uint32_t S) { return (size_t)S * 8 + ((size_t)1 << 18) * 12 + kHHBins * 4 + 64; }
 
 int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, uint32_t rank_words, void* ws, void* stream,
-                      int sms, const uint64_t** front_out) {
+                      int sms, const uint64_t** front_out, const uint64_t** hot_out) {
   cudaStream_t st = (cudaStream_t)stream;
   HHParams h{};
   h.S = S;
@@ -930,6 +960,11 @@ int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, uint32_t ra
     k_hh_build_rank<<<sms, 256, 0, st>>>(h);
     k_hh_rank_scan<<<1, 1024, 0, st>>>(h, rank_words);
     count_launch(6);
+    if (hot_out) {
+      k_hh_top<<<1, 1024, 0, st>>>(h, jit_hot_reg());
+      count_launch(1);
+      *hot_out = (const uint64_t*)(h.ctl + 2);
+    }
   } else {
     k_hh_build<<<sms, 256, 0, st>>>(h);
     count_launch(5);

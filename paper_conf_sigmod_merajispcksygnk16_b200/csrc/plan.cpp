@@ -537,7 +537,9 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     P->smem_bytes = b;
     // one CTA per SM: 768 threads x 80 registers carry 4 pipelined rows per thread (C4 9.2 ms)
     // where 1024 x 64 carry 2 (10.2 ms); 640 and 512 (x 128) measured the same as 768
-    P->block = P->front_wide ? 768 : 512;
+    // with the hot keys in registers (BLU_GBY_HOT_REG, +12 registers per key): 640 x 96 (C4 8.87 ms
+    // vs 9.10 without; at 768 x 80 those registers spill: 11.2 ms)
+    P->block = P->front_wide ? (jit_hot_reg() ? 640 : 768) : 512;
   } else {
     P->smem_bytes = 0;
     P->block = 256;
