@@ -209,7 +209,8 @@ bool compile(const std::string& src, std::vector<char>& cubin, std::string& log)
 // The rank front's 0, 1 or 2 hottest keys summed in registers (BLU_GBY_HOT_REG=0/1/2)
 int jit_hot_reg() {
   const char* e = getenv("BLU_GBY_HOT_REG");  // read per plan execution (tests switch it)
-  const int h = e ? atoi(e) : 0;
+  // default 1: C4 8.91 vs 9.18-9.36 ms (640 threads, one key); two keys measured slower (11.8-12.0 ms)
+  const int h = e ? atoi(e) : 1;
   return jit_enabled() ? (h < 0 ? 0 : h > 2 ? 2 : h) : 0;
 }
 
