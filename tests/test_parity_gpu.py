@@ -141,6 +141,36 @@ def _mk(keys_np, vals_np):
 ALL = lambda nv: [(COUNT, -1)] + [(op, c) for c in range(nv) for op in (SUM, MIN, MAX, AVG)]
 
 
+@pytest.mark.parametrize("seed", [1, 2, 3, 4])
+def test_hot_reg_key_outside_front(bg, monkeypatch, seed):
+    """Hottest key in registers when the seeded front cannot hold every heavy hitter: a 64-entry rank
+    front, 100 keys each far above the sample histogram's top bin, so the front takes 64 of them
+    first come and the sample's argmax key may be left out; its register partial then goes straight
+    to the dense state instead of a front entry. Either way the result equals the oracle."""
+    rng = np.random.default_rng(seed)
+    n, D = 2_000_003, 2048
+    sch = blugen.Schema([(I32, D)], [I32, I64, F64], ALL(3))
+    hot = rng.choice(D, 100, replace=False)
+    g = hot[rng.integers(0, 100, n)]
+    cold = rng.random(n) < 0.05
+    g[cold] = rng.integers(0, D, int(cold.sum()))
+    kc = [g.astype(np.int32)]
+    vc = [rng.integers(-(2**31), 2**31, n).astype(np.int32), rng.integers(-(2**62), 2**62, n).astype(np.int64),
+          rng.integers(-(2**20), 2**20, n) / 64.0]
+    o = oracle.groupby_arrays(sch, kc, vc)
+    monkeypatch.setenv("BLU_GBY_FORCE_PATH", "d")
+    monkeypatch.setenv("BLU_GBY_HOT_FRONT", "1")
+    monkeypatch.setenv("BLU_GBY_FRONT_SLOTS", "64")
+    monkeypatch.setenv("BLU_GBY_HOT_REG", "1")
+    plan = bg.plan_for(sch, D, n)
+    info = plan.info()
+    assert info["hot_front"] == 1 and info["front_slots"] == 64
+    dk, dv = _mk(kc, vc)
+    res = bg.blu_gby_execute(plan, dk, dv)
+    gk, ga = gpu_sorted(res, sch)
+    assert_parity(gk, ga, o, sch)
+
+
 @pytest.mark.parametrize("n", [0, 1, 3, 31, 33, 4095, 4097, 65_537])
 @pytest.mark.parametrize("path", ["a", "a-nofuse", "b", "d"])
 def test_small_and_ragged(bg, monkeypatch, n, path):
