@@ -1061,8 +1061,8 @@ struct HotAccT2 {
       });
     }
   }
-  template <int NV, int R>
-  __device__ __forceinline__ void add(int h, const uint64_t (&v)[NV][R], int r) {
+  template <int h, int NV, int R>
+  __device__ __forceinline__ void add(const uint64_t (&v)[NV][R], int r) {
     sfor<0, SP::NF>([&](auto jc) {
       constexpr int j = decltype(jc)::v;
       constexpr int K = kind<j>(), c = SP::COL[j];
@@ -1086,12 +1086,13 @@ struct HotAccT2 {
   __device__ __forceinline__ void take(const uint64_t (&k)[R], uint32_t& valid, const uint64_t (&v)[NV][R]) {
 #pragma unroll
     for (int r = 0; r < R; ++r)
-#pragma unroll
-      for (int h = 0; h < H; ++h)
+      sfor<0, H>([&](auto hc) {  // h a compile-time index: the partials stay in registers
+        constexpr int h = decltype(hc)::v;
         if ((valid >> r & 1) && k[r] == key[h]) {
-          add(h, v, r);
+          add<h>(v, r);
           valid &= ~(1u << r);
         }
+      });
   }
   // into the key's rank-front entry, or straight into the dense state if the key is not in the front
   __device__ __forceinline__ void flush(const AggParams& p, uint8_t* sm) {
