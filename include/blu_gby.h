@@ -116,12 +116,16 @@ typedef struct {
     void* _owner;        /* library-private                                                     */
 } blu_gby_result_t;
 
-/* ---- plan (host only; never touches the GPU) -------------------------------------------------
+/* ---- plan (host only; launches no GPU work) --------------------------------------------------
+ * The first plan of a process queries the current device's SM count (cudaDeviceGetAttribute) to
+ * size the grid; nothing is allocated or launched.
  * Validates the schema and freezes the plan: path, hash-table capacity ("slightly larger than the
  * estimated number of groups": cap = next_pow2(ceil(max(est,1)/0.7)), >= 1024), slot
  * layout (key + state fields padded to a power of two, "1, 2, 4, 8 or 16 byte aligned"),
  * shared-memory bytes and grid. est_groups is clamped to [1, n_rows]; n_rows is the exact row
- * count and may be 0. Errors: BLU_E_INVALID (NULL / bad schema), BLU_E_UNSUPPORTED.
+ * count and may be 0. Errors: BLU_E_INVALID (NULL / bad schema), BLU_E_UNSUPPORTED (a key
+ * tuple wider than 128 bits, or an AoS slot of more than 256 bytes, e.g. 16 aggregates over 128-bit
+ * payloads).
  * Environment overrides for tests and benchmarks only: BLU_GBY_FORCE_PATH=a|b|d,
  * BLU_GBY_HOT_FRONT=0|1. */
 blu_status_t blu_gby_plan(const blu_gby_schema_t* schema, uint64_t est_groups, uint64_t n_rows,

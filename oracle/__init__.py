@@ -65,6 +65,10 @@ def lib():
         L.oracle_dup_ranges.restype = u64
         L.oracle_sort_rows.argtypes = [vp, u64, ctypes.c_uint32, vp]
         L.oracle_sort_rows.restype = None
+        L.oracle_kmv.argtypes = [vp, vp, vp, ctypes.c_int32, u64, ctypes.c_uint32, vp]
+        L.oracle_kmv.restype = ctypes.c_double
+        L.oracle_fmix64_export.argtypes = [u64]
+        L.oracle_fmix64_export.restype = u64
         _lib = L
     return _lib
 
@@ -189,3 +193,24 @@ def sort_rows(rows: np.ndarray) -> np.ndarray:
     out = np.zeros(n, np.uint32)
     lib().oracle_sort_rows(rows.ctypes.data, n, W, out.ctypes.data)
     return out
+
+
+# ---- KMV group-count estimate (oracle/kmv_oracle.cpp) --------------------------------
+def kmv(key_cols: Sequence[np.ndarray], dict_sizes: Sequence[int], k: int):
+    """(estimate, exact) of the number of distinct key tuples: the k-th smallest distinct
+    fmix64(concatenated key ^ salt), est = (k - 1) * 2^64 / U_(k); exact count below k."""
+    cols = [np.ascontiguousarray(c) for c in key_cols]
+    for c in cols:
+        assert c.dtype in (np.int32, np.int64), c.dtype
+    n = len(cols[0]) if cols else 0
+    kp = (ctypes.c_void_p * max(1, len(cols)))(*[c.ctypes.data for c in cols])
+    is64 = (ctypes.c_int32 * max(1, len(cols)))(*[1 if c.dtype == np.int64 else 0 for c in cols])
+    ds = (ctypes.c_uint64 * max(1, len(cols)))(*[int(d) for d in dict_sizes])
+    ex = ctypes.c_int32(0)
+    est = lib().oracle_kmv(kp, is64, ds, len(cols), n, k, ctypes.byref(ex))
+    return float(est), bool(ex.value)
+
+
+def fmix64(x: int) -> int:
+    """The oracle's Murmur3 finalizer (for its bijectivity pin)."""
+    return int(lib().oracle_fmix64_export(x))

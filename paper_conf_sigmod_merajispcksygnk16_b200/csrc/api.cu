@@ -179,12 +179,15 @@ void cache_put(void* p) {
     if (b.p == p) b.busy = false;
 }
 
-// Scratch of one execute; released (to the cache) when destroyed, after the stream has been
-// synchronised by the caller.
+// Scratch of one execute; released (to the cache) when destroyed. A block may only go back once
+// the kernels queued on `st` that use it have finished: the success paths synchronise `st` and call
+// drained(); on an early error return the destructor synchronises `st` itself before releasing.
 struct Work {
   cudaStream_t st;
   std::vector<void*> ptrs;
+  bool synced = false;
   explicit Work(cudaStream_t s) : st(s) {}
+  void drained() { synced = true; }
   cudaError_t alloc(void** p, size_t bytes) {
     *p = nullptr;
     if (!bytes) return cudaSuccess;
@@ -193,6 +196,10 @@ struct Work {
     return e;
   }
   ~Work() {
+    if (!ptrs.empty() && !synced) {
+      cudaStreamSynchronize(st);  // error path: queued kernels may still write these blocks
+      cudaGetLastError();
+    }
     for (void* p : ptrs) cache_put(p);
   }
 };
@@ -427,6 +434,7 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     auto t_sync0 = std::chrono::steady_clock::now();
     cudaError_t ce = cudaMemcpyAsync(dst, small, 16, cudaMemcpyDeviceToHost, st);
     if (ce == cudaSuccess) ce = cudaStreamSynchronize(st);
+    if (ce == cudaSuccess) w.drained();
     if (hdbg)
       fprintf(stderr, "[blugby host] final sync waited %.3f ms\n",
               std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_sync0).count());
@@ -951,6 +959,7 @@ blu_status_t blu_gby_execute_host(blu_gby_plan_t P, const void* const* hkeys, co
   cudaStream_t cs = nullptr;
   cudaEvent_t ready[2] = {nullptr, nullptr}, freed[2] = {nullptr, nullptr}, t0 = nullptr, t1 = nullptr;
   auto cleanup = [&]() {
+    if (cs) cudaStreamSynchronize(cs);  // H2D copies still queued on cs must land before the frees
     for (int b = 0; b < 2; ++b) {
       if (stage[b]) cudaFreeAsync(stage[b], st);
       if (ready[b]) cudaEventDestroy(ready[b]);
@@ -1114,6 +1123,7 @@ blu_status_t blu_gby_execute_dense_state(blu_gby_plan_t P, const void* const* ke
   uint64_t* dst = hs ? hs : hb;
   CK(cudaMemcpyAsync(dst, small, 8, cudaMemcpyDeviceToHost, st), "flags D2H");
   CK(cudaStreamSynchronize(st), "sync");
+  w.drained();
   if (t_timing) {  // the aggregation launches of this call (multi-GPU path (a): the per-rank kernel)
     blu_gby_timing_t tm{};
     cudaEventElapsedTime(&tm.aggregate_ms, t_ev.e[1], t_ev.e[2]);
@@ -1187,6 +1197,7 @@ blu_status_t blu_gby_partition_rows(blu_gby_plan_t P, const void* const* key_col
   CK(cudaMemcpyAsync(send_counts, d_counts, 8 * (size_t)n_parts, cudaMemcpyDeviceToHost, st), "counts D2H");
   CK(cudaMemcpyAsync(&flags, d_flags, 4, cudaMemcpyDeviceToHost, st), "flags D2H");
   CK(cudaStreamSynchronize(st), "sync");
+  w.drained();
   if (flags & FLAG_KEY_RANGE) return fail(BLU_E_KEY_RANGE, "a key code is outside its dictionary (or negative)");
   return BLU_OK;
 }
@@ -1214,6 +1225,7 @@ blu_status_t blu_gby_partition(blu_gby_plan_t P, const blu_gby_result_t* partial
      "partition");
   CK(cudaMemcpyAsync(send_counts, d_counts, 8 * (size_t)n_parts, cudaMemcpyDeviceToHost, st), "counts D2H");
   CK(cudaStreamSynchronize(st), "sync");
+  w.drained();
   return BLU_OK;
 }
 

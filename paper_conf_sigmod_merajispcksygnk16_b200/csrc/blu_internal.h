@@ -114,6 +114,10 @@ bool jit_probe_active();
 const void* jit_kernel(const std::string& spec_src, const std::string& entry_src, const char* entry);
 std::string jit_spec(const char* name, const Layout& L, uint32_t S, const uint32_t* soff);
 
+// Own LSD radix sort of u64 keys (sort.cu), used by the KMV estimate (kmv.cu)
+size_t sort_u64_scratch_bytes(uint64_t n);
+cudaError_t sort_u64_keys(const uint64_t* kin, uint64_t* kout, uint64_t n, void* ws, cudaStream_t st);
+
 // Planner helpers (plan.cpp)
 uint32_t smem_entry_bytes(const Layout& lay);
 void build_slot_template(const Layout& lay, uint8_t* out);

@@ -7,14 +7,13 @@
 //   h(row) = fmix64(packed_key ^ kKmvSalt)            (independent of the table's slot hash)
 //   L      = the k smallest DISTINCT values of h over all rows
 //   est    = (k - 1) * 2^64 / L[k-1]                   (exact distinct count if fewer than k)
+// (the same definition is written out plainly in oracle/kmv_oracle.cpp, which the tests compare with)
 // Each CTA keeps its k smallest distinct hashes in shared memory (a row survives only if it is below
 // the CTA's current k-th value; survivors are buffered and merged with a bitonic sort); the per-CTA
-// lists are then merged by one device sort. The result depends only on the SET of keys, not on the
+// lists are then merged by one device sort (the repo's own LSD radix sort, sort.cu). The result depends only on the SET of keys, not on the
 // row order or the launch shape.
 #include <cuda_runtime.h>
 #include <stdint.h>
-
-#include <cub/cub.cuh>
 
 #include "blu_internal.h"
 #include "blu_device.cuh"
@@ -187,8 +186,7 @@ extern "C" blu_status_t blu_gby_estimate_groups(const blu_key_desc_t* keys, int3
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const uint32_t grid = (uint32_t)sms;
   const uint64_t m = (uint64_t)grid * k;
-  size_t tmp_bytes = 0;
-  cub::DeviceRadixSort::SortKeys(nullptr, tmp_bytes, (const uint64_t*)nullptr, (uint64_t*)nullptr, (int)m, 0, 64, st);
+  const size_t tmp_bytes = sort_u64_scratch_bytes(m);
   void* ws = nullptr;
   const size_t bytes = 64 + 2 * m * 8 + tmp_bytes;
   if (cudaMallocAsync(&ws, bytes, st) != cudaSuccess) {
@@ -205,9 +203,15 @@ extern "C" blu_status_t blu_gby_estimate_groups(const blu_key_desc_t* keys, int3
   const size_t smem = kKmvSort * 8;
   cudaFuncSetAttribute(k_kmv_local, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   k_kmv_local<<<grid, 512, smem, st>>>(p, k, cand);
-  cub::DeviceRadixSort::SortKeys(tmp, tmp_bytes, cand, sorted, (int)m, 0, 64, st);
+  count_launch(1);
+  cudaError_t se = sort_u64_keys(cand, sorted, m, tmp, st);
+  if (se != cudaSuccess) {
+    cudaGetLastError();
+    cudaFreeAsync(ws, st);
+    return fail(BLU_E_CUDA, "estimate sort: %s", cudaGetErrorString(se));
+  }
   k_kmv_select<<<1, 32, 0, st>>>(sorted, m, k, res);
-  count_launch(3);
+  count_launch(1);
   uint64_t h[4] = {0, 0, 0, 0};
   cudaMemcpyAsync(h, ws, 32, cudaMemcpyDeviceToHost, st);
   cudaError_t e = cudaStreamSynchronize(st);

@@ -61,6 +61,7 @@ constexpr uint32_t kSmemMax = 232448;           // dynamic shared memory per CTA
 constexpr uint32_t kMaxBuckets = 4096;          // one-pass scatter fan-out
 constexpr uint32_t kMaxBuckets2 = 16384;        // two-level scatter (32 x 512)
 constexpr double kBucketLoad = 0.7;             // mean groups per bucket / bucket table entries
+constexpr uint32_t kMaxSlotBytes = 256;         // AoS slot limit (init template size)
 
 static bool field_q(int kind) { return kind == FK_SUMQ || kind == FK_MINQ || kind == FK_MAXQ; }
 static int32_t field_gsize(int kind) {
@@ -277,7 +278,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     bool over = false;
     for (int k = 0; k < s->n_keys && !sparse; ++k) {
       const uint64_t d = s->keys[k].dict_size;
-      if (Dt > ((1ull << 62) / d)) over = true;
+      if (Dt > ((1ull << 62) - 1) / d) over = true;  // one word only while D < 2^62 (strict)
       else Dt *= d;
     }
     wide = (sparse && s->n_keys > 1) || over;
@@ -301,7 +302,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
       if (!d) continue;
       int t = -1;
       for (int c = 0; c < 2 && t < 0; ++c)
-        if (!full[c] && prod[c] <= ((1ull << 62) / d)) t = c;
+        if (!full[c] && prod[c] <= ((1ull << 62) - 1) / d) t = c;  // per-word product < 2^62
       if (t < 0) return fail(BLU_E_UNSUPPORTED, "key tuple does not fit in 128 bits");
       kword[k] = t;
       kstride[k] = prod[t];
@@ -376,12 +377,13 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   uint32_t entry_with_count = L.smem_entry_bytes + (L.count_field < 0 ? 4u : 0u);
   L.sparse = sparse ? 1 : 0;
   int path;
-  if (!sparse && D * (uint64_t)entry_with_count <= kSmemDenseMax) path = BLU_PATH_DENSE_SMEM;
+  // division form: D * entry bytes can wrap u64 for D near 2^62
+  if (!sparse && D <= kSmemDenseMax / entry_with_count) path = BLU_PATH_DENSE_SMEM;
   else if (!sparse && D <= std::max<uint64_t>(2 * cap_est, kDirectMin)) path = BLU_PATH_DIRECT_GLOBAL;
   else path = BLU_PATH_HASH_GLOBAL;
   if (const char* fp = env("BLU_GBY_FORCE_PATH")) {
     int want = fp[0] == 'a' ? BLU_PATH_DENSE_SMEM : fp[0] == 'd' ? BLU_PATH_DIRECT_GLOBAL : BLU_PATH_HASH_GLOBAL;
-    if (want == BLU_PATH_DENSE_SMEM && (sparse || D * (uint64_t)entry_with_count > 200 * 1024)) {
+    if (want == BLU_PATH_DENSE_SMEM && (sparse || D > (200u * 1024u) / entry_with_count)) {
       delete P;
       return fail(BLU_E_UNSUPPORTED, "BLU_GBY_FORCE_PATH=a: dense domain does not fit in shared memory");
     }
@@ -392,6 +394,10 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     path = want;
   }
   if (L.key_words == 2) path = BLU_PATH_HASH_GLOBAL;  // wide keys: 16-byte key CAS, hash path only
+  if (L.slot_bytes > kMaxSlotBytes) {  // the init template (kernels.cu SlotTemplate) holds 256 bytes
+    delete P;
+    return fail(BLU_E_UNSUPPORTED, "slot of %u bytes (key + state fields) exceeds %u bytes", L.slot_bytes, kMaxSlotBytes);
+  }
   if (L.has_q) path = BLU_PATH_HASH_GLOBAL;            // 128-bit payloads: 16-byte global fields only
   P->path = path;
   if (path != BLU_PATH_HASH_GLOBAL && L.count_field < 0) {  // dense occupancy = COUNT > 0
@@ -415,6 +421,10 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     if (lock) {
       L.lock_off = 1;  // placeholder: finish_layout assigns the real offset
       finish_layout(L);
+      if (L.slot_bytes > kMaxSlotBytes) {
+        delete P;
+        return fail(BLU_E_UNSUPPORTED, "slot with row lock exceeds %u bytes", kMaxSlotBytes);
+      }
     }
   }
 

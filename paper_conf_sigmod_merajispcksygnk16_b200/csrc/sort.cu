@@ -755,6 +755,7 @@ cudaError_t radix_sort(const KT* kin, const uint32_t* vin, KT* kout, uint32_t* v
 
 uint32_t radix_grid() { return (uint32_t)sms_now() * 8; }  // 8 x 256 threads per SM
 
+
 blu_status_t cuda_err(cudaError_t e, const char* what) {
   cudaGetLastError();
   if (e == cudaErrorMemoryAllocation) return fail(BLU_E_OOM, "%s: %s", what, cudaGetErrorString(e));
@@ -808,6 +809,22 @@ blu_status_t dup_pass(const KT* k, uint64_t m, const uint32_t* act_pos, uint32_t
 }
 
 }  // namespace
+
+// Ascending sort of n u64 keys with the radix sort above (the KMV estimate's candidate merge, kmv.cu).
+// ws: caller-owned device scratch of sort_u64_scratch_bytes(n) bytes, released stream-ordered by the
+// caller. Synchronises `st` once (the constant-digit check).
+size_t sort_u64_scratch_bytes(uint64_t n) { return (size_t)n * (8 + 3 * 4) + (size_t)256 * (radix_grid() + 1) * 4 + 64; }
+cudaError_t sort_u64_keys(const uint64_t* kin, uint64_t* kout, uint64_t n, void* ws, cudaStream_t st) {
+  if (!n) return cudaSuccess;
+  const uint32_t grid = radix_grid();
+  uint64_t* kt = (uint64_t*)ws;
+  uint32_t* vin = (uint32_t*)(kt + n);  // payloads are not used: any content
+  uint32_t* vout = vin + n;
+  uint32_t* vt = vout + n;
+  uint32_t* counts = vt + n;
+  return radix_sort<uint64_t>(kin, vin, kout, vout, kt, vt, n, 64, counts, grid, st);
+}
+
 }  // namespace blu
 
 using namespace blu;

@@ -283,3 +283,28 @@ def test_i128_plan_and_mask(bg):
     with pytest.raises(bg.BluError) as e:            # 128-bit payloads with two-word keys
         bg.blu_gby_plan([(I64, 0), (I64, 0)], [I128], [(SUM, 0)], 100, 1000)
     assert e.value.status == bg.BLU_E_UNSUPPORTED
+
+
+def test_planner_no_u64_wrap_near_2_pow_62(bg):
+    """two i32 keys of dict_size 2^31 give D = 2^62; D * entry bytes wrapped u64 to 0
+    and the planner chose the shared-memory path with 0 bytes. The one-word packing now requires
+    D < 2^62 strictly, so this tuple takes two key words (hash path); D just below 2^62 stays one word
+    on the hash/direct path, never path (a)."""
+    d = bg.blu_gby_plan([(I32, 2**31), (I32, 2**31)], [], [(COUNT, -1)], 1000, 10**6).info()
+    assert d["path"] == bg.BLU_PATH_HASH_GLOBAL and d["slot_bytes"] >= 24  # two-word key
+    d = bg.blu_gby_plan([(I32, 2**31), (I32, 2**31 - 1)], [], [(COUNT, -1)], 1000, 10**6).info()
+    assert d["path"] == bg.BLU_PATH_HASH_GLOBAL and d["slot_bytes"] == 16 and d["capacity"] >= 1024
+    # the largest dense domain path (a) takes still fits its 96 KB shared-memory budget
+    d = bg.blu_gby_plan([(I32, 4096)], [], [(COUNT, -1)], 1000, 10**6).info()
+    assert d["path"] == bg.BLU_PATH_DENSE_SMEM and 0 < d["smem_bytes"] <= 96 * 1024
+
+
+def test_planner_rejects_slots_over_256_bytes(bg):
+    """16 SUMs over 16 i128 columns need a 320-byte slot, more than the init
+    template holds; the planner reports BLU_E_UNSUPPORTED instead of overflowing it."""
+    from blugen import I128
+    with pytest.raises(bg.BluError) as e:
+        bg.blu_gby_plan([(I64, 0)], [I128] * 16, [(SUM, c) for c in range(16)], 1000, 10**6)
+    assert e.value.status == bg.BLU_E_UNSUPPORTED
+    ok = bg.blu_gby_plan([(I64, 0)], [I128] * 15, [(SUM, c) for c in range(15)], 1000, 10**6).info()
+    assert ok["slot_bytes"] == 256

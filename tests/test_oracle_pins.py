@@ -80,6 +80,15 @@ def assert_matches_brute(schema, kc, vc, exact_f64=True):
         assert int(o.count[gi]) == cnt
         for a, (kind, val, sa) in enumerate(res):
             got = o.aggs[a][gi]
+            if sa is not None:
+                # the oracle's sum|v| sets the A13 tolerance of every f64 SUM/AVG parity check: pin it
+                # to the correctly rounded math.fsum of |v| (long double accumulation: <= n * 2^-64 rel.)
+                osa = float(o.sumabs[a][gi])
+                assert abs(osa - sa) <= 4e-16 * sa * max(1, cnt) + 0.0, (gi, a, osa, sa)
+                if exact_f64:
+                    assert osa == sa, (gi, a, osa, sa)
+            else:
+                assert o.sumabs[a] is None or schema.aggs[a][0] not in (SUM, AVG), (gi, a)
             if kind == "i":
                 assert int(got) == val, (gi, a, got, val)
             elif exact_f64 or sa is None:
@@ -459,3 +468,75 @@ def test_sort_rows_special_cases_and_invariants():
             nxt += [(a + int(x), a + int(x) + int(y)) for x, y in zip(st, ln)]
         ranges = nxt
     assert np.array_equal(order, perm)
+
+
+# ---- KMV group-count estimate (oracle/kmv_oracle.cpp; NEXT-3) --------------------------
+def test_kmv_exact_below_k_equals_distinct_tuples():
+    """Fewer than k distinct tuples: the estimate is exact and equals a Python set's size (fmix64 is a
+    bijection and the mixed-radix concatenation is injective on in-dictionary codes)."""
+    rng = np.random.default_rng(77)
+    for dicts, n in (((7, 5, 3), 5000), ((16,), 100), ((1,), 50), ((300,), 4000)):
+        cols = [rng.integers(0, d, n).astype(np.int32) for d in dicts]
+        est, exact = oracle.kmv(cols, dicts, k=512)
+        assert exact and est == len(set(zip(*[c.tolist() for c in cols])))
+    sparse = rng.integers(0, 2**62, 200).astype(np.int64)[rng.integers(0, 200, 3000)]
+    est, exact = oracle.kmv([sparse], [0], k=1024)
+    assert exact and est == len(set(sparse.tolist()))
+    est, exact = oracle.kmv([np.zeros(0, np.int64)], [0], k=16)
+    assert exact and est == 0
+
+
+def test_kmv_kth_value_matches_python_sort():
+    """U_(k) is the k-th smallest DISTINCT hash (Python sorted() of a set, not std::set) and
+    est = (k - 1) * 2^64 / U_(k) (the estimator of the paper's KMV reference [2])."""
+    rng = np.random.default_rng(5)
+    keys = rng.integers(0, 2**62, 300).astype(np.int64)
+    rows = keys[rng.integers(0, 300, 2000)]
+    salt = 0x6B6D765F73616C74  # "kmv_salt"
+    hs = sorted({oracle.fmix64(int(x) ^ salt) for x in rows.tolist()} - {2**64 - 1})
+    for k in (16, 64, 255):
+        est, exact = oracle.kmv([rows], [0], k=k)
+        assert not exact and est == (k - 1) * 18446744073709551616.0 / float(hs[k - 1])
+
+
+def test_kmv_relative_error_bound_over_seeds():
+    """KMV is unbiased with relative standard error ~ 1/sqrt(k - 2): over 30 independent key sets of
+    G = 20000 groups every estimate is within 5 sd and the mean within 4 sd / sqrt(30)."""
+    G, k = 20000, 256
+    sd = 1.0 / math.sqrt(k - 2)
+    ratios = []
+    for seed in range(30):
+        rng = np.random.default_rng(9000 + seed)
+        keys = np.unique(rng.integers(0, 2**62, G + 64).astype(np.int64))[:G]
+        rows = keys[rng.integers(0, G, 3 * G)]
+        rows = np.concatenate([keys, rows])  # every key present
+        est, exact = oracle.kmv([rows], [0], k=k)
+        assert not exact
+        ratios.append(est / G)
+        assert abs(est / G - 1) <= 5 * sd, (seed, est)
+    assert abs(float(np.mean(ratios)) - 1) <= 4 * sd / math.sqrt(30), np.mean(ratios)
+
+
+def test_kmv_invariant_to_row_order_and_duplicates():
+    rng = np.random.default_rng(11)
+    cols = [rng.integers(0, 100, 50000).astype(np.int32), rng.integers(0, 50, 50000).astype(np.int32)]
+    est, _ = oracle.kmv(cols, [100, 50], k=128)
+    perm = rng.permutation(50000)
+    est_p, _ = oracle.kmv([c[perm] for c in cols], [100, 50], k=128)
+    est_d, _ = oracle.kmv([np.concatenate([c, c[:777]]) for c in cols], [100, 50], k=128)
+    assert est == est_p == est_d
+
+
+def test_kmv_hash_is_a_bijective_avalanching_mix():
+    """fmix64 (Murmur3 finalizer): 0 -> 0, no collisions on 2^16 consecutive inputs, and one flipped
+    input bit flips ~half of the output bits (a dropped xorshift or multiply fails one of these)."""
+    assert oracle.fmix64(0) == 0
+    outs = {oracle.fmix64(i) for i in range(1 << 16)}
+    assert len(outs) == 1 << 16
+    rng = np.random.default_rng(3)
+    flips = []
+    for _ in range(2000):
+        x = int(rng.integers(0, 2**63))
+        b = int(rng.integers(0, 64))
+        flips.append(bin(oracle.fmix64(x) ^ oracle.fmix64(x ^ (1 << b))).count("1"))
+    assert 31.0 <= float(np.mean(flips)) <= 33.0

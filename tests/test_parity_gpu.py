@@ -567,24 +567,6 @@ def test_partition_rows_key_range(bg):
     assert e.value.status == bg.BLU_E_KEY_RANGE
 
 
-def _kmv_reference(keys_packed, k):
-    """Independent numpy statement of the KMV estimate (same definition, no shared code):
-    h = fmix64(packed ^ salt); est = (k-1) * 2^64 / (k-th smallest distinct h), exact if < k."""
-    M = (1 << 64) - 1
-    h = (keys_packed.astype(np.uint64) ^ np.uint64(0x6b6d765f73616c74))
-    with np.errstate(over="ignore"):
-        h ^= h >> np.uint64(33)
-        h *= np.uint64(0xff51afd7ed558ccd)
-        h ^= h >> np.uint64(33)
-        h *= np.uint64(0xc4ceb9fe1a85ec53)
-        h ^= h >> np.uint64(33)
-    u = np.unique(h)
-    u = u[u != np.uint64(M)]
-    if u.size < k:
-        return float(u.size), True
-    return (k - 1) * 18446744073709551616.0 / float(int(u[k - 1])), False
-
-
 @pytest.mark.parametrize("G,n,k", [(700, 200_000, 2048), (50_000, 3_000_000, 2048), (1_000_000, 4_000_000, 1024)])
 def test_kmv_estimate(bg, G, n, k):
     """NEXT-3: on-GPU KMV estimate equals the numpy statement of the same definition,
@@ -593,7 +575,7 @@ def test_kmv_estimate(bg, G, n, k):
     kc, _ = blugen.device_columns(w)
     est, exact = bg.blu_gby_estimate_groups(w.schema.keys, kc, k=k)
     host = kc[0].cpu().numpy()
-    ref, ref_exact = _kmv_reference(host, k)
+    ref, ref_exact = oracle.kmv([host], [0], k)  # oracle/kmv_oracle.cpp: the plain definition
     true = len(np.unique(host))
     assert exact == ref_exact and est == ref
     if exact:
@@ -611,7 +593,7 @@ def test_kmv_dense_composite_keys(bg):
     kc, _ = blugen.device_columns(w)
     est, exact = bg.blu_gby_estimate_groups(w.schema.keys, kc, k=2048)
     packed = kc[0].long() + 100 * kc[1].long() + 5000 * kc[2].long()
-    ref, ref_exact = _kmv_reference(packed.cpu().numpy(), 2048)
+    ref, ref_exact = oracle.kmv([c.cpu().numpy() for c in kc], [d for _, d in w.schema.keys], 2048)
     assert est == ref and exact == ref_exact
     true = int(torch.unique(packed).numel())
     assert abs(est - true) <= 5 * true / np.sqrt(2046)
