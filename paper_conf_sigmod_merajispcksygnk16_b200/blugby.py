@@ -473,8 +473,18 @@ def blu_gby_init_table(plan: Plan, dev_table, n_slots: int, stream=None):
     _check(lib.blu_gby_init_table(plan.handle, _ptr(dev_table), int(n_slots), _stream_handle(stream)))
 
 
+_timing_on = False
+
+
 def blu_gby_set_timing(enable: bool):
+    global _timing_on
+    _timing_on = bool(enable)
     lib.blu_gby_set_timing(1 if enable else 0)
+
+
+def timing_enabled() -> bool:
+    """Whether blu_gby_set_timing(True) is in effect in this process (per-phase events in dist.py)."""
+    return _timing_on
 
 
 def blu_gby_last_timing() -> dict:

@@ -5,9 +5,9 @@ partitioning, "the input data is partitioned ... sent to some numb
 GPU devices ... The results are then merged together in the final step"). The merge is chosen by
 the plan's path:
 
-  * dense state (paths a / b'): every rank holds the same D x fields state arrays; four
-    all-reduces (int64 SUM, f64 SUM, int64 MIN, int64 MAX) combine them; every rank finalizes the
-    same replicated result;
+  * dense state (paths a / b'): every rank holds the same D x fields state arrays; three
+    all-reduces issued back to back (int64 SUM, f64 SUM, and int64 MIN over MIN ++ ~MAX) combine
+    them; every rank finalizes the same replicated result;
   * hash path (b), partials mode (default when the rank's rows outnumber the estimated groups):
     each rank emits per-group partial states, buckets them by owner rank (mulhi(fmix64(key), P),
     bits independent of the slot bits), exchanges them with an all-to-all-v and merges what it
@@ -26,12 +26,55 @@ import torch
 import torch.distributed as dist
 
 
+class _Phases:
+    """CUDA events around the local, exchange and merge phases of one dist_execute (on the launching
+    stream); read after the call's own synchronisation. Off unless timing is enabled."""
+
+    def __init__(self, on: bool, stream):
+        self.on = on
+        self.stream = stream
+        self.ev = []
+
+    def mark(self, name: str):
+        if self.on:
+            e = torch.cuda.Event(enable_timing=True)
+            e.record(self.stream)
+            self.ev.append((name, e))
+
+    def result(self) -> dict:
+        if not self.on or len(self.ev) < 2:
+            return {}
+        self.ev[-1][1].synchronize()
+        out = {}
+        for (_, a), (name, b) in zip(self.ev, self.ev[1:]):
+            out[name + "_ms"] = out.get(name + "_ms", 0.0) + a.elapsed_time(b)
+        return out
+
+
 def allreduce_dense_state(state_arrays: Sequence[torch.Tensor], group=None) -> None:
-    """[int64 SUM group, f64 SUM group, int64 MIN group, int64 MAX group] in place."""
-    ops = (dist.ReduceOp.SUM, dist.ReduceOp.SUM, dist.ReduceOp.MIN, dist.ReduceOp.MAX)
-    for t, op in zip(state_arrays, ops):
-        if t.numel():
-            dist.all_reduce(t, op=op, group=group)
+    """[int64 SUM group, f64 SUM group, int64 MIN group, int64 MAX group] in place, with three
+    collectives issued back to back (no host wait between them): int64 SUM, f64 SUM, and one int64
+    MIN over the MIN group concatenated with the bitwise complement of the MAX group (~ reverses the
+    order of two's-complement integers, so max(x) = ~min(~x) with no overflow at INT64_MIN)."""
+    isum, fsum, mn, mx = state_arrays
+    works = []
+    if isum.numel():
+        works.append(dist.all_reduce(isum, op=dist.ReduceOp.SUM, group=group, async_op=True))
+    if fsum.numel():
+        works.append(dist.all_reduce(fsum, op=dist.ReduceOp.SUM, group=group, async_op=True))
+    mm = None
+    if mn.numel() or mx.numel():
+        mm = torch.cat([mn.reshape(-1), torch.bitwise_not(mx.reshape(-1))])
+        works.append(dist.all_reduce(mm, op=dist.ReduceOp.MIN, group=group, async_op=True))
+    for w in works:
+        w.wait()
+    if mm is not None:
+        a = mn.numel()
+        if a:
+            mn.copy_(mm[:a].reshape(mn.shape))
+        if mx.numel():
+            torch.bitwise_not(mm[a:], out=mm[a:])
+            mx.copy_(mm[a:].reshape(mx.shape))
 
 
 def alltoallv_records(send: torch.Tensor, send_counts: List[int], words: int, group=None) -> torch.Tensor:
@@ -61,40 +104,62 @@ def exchange_mode(plan, n_local: int, mode=None) -> str:
 
 def dist_execute(plan, key_cols, val_cols, group=None, stream=None, mode=None):
     """Whole-job GROUP BY of this rank's rows; returns (result, mode). Dense paths: replicated
-    finalized result; hash path: this rank's owned groups (mode 'partials' or 'rows')."""
+    finalized result; hash path: this rank's owned groups (mode 'partials' or 'rows').
+    With timing on (blu_gby_set_timing), res.agg_timing holds the rank-local aggregation's
+    blu_gby_last_timing() and res.phase_ms the CUDA-event times of the local / exchange / merge
+    phases on this rank."""
     from . import blugby as bg
     P = dist.get_world_size(group)
     info = plan.info()
-    # res.agg_timing: blu_gby_last_timing() of the rank-local aggregation (the kernel that scales),
-    # taken before the exchange and merge calls overwrite it (None unless timing is enabled)
+    if stream is None:
+        stream = torch.cuda.current_stream(key_cols[0].device) if key_cols[0].is_cuda else None
+    ph = _Phases(bool(bg.timing_enabled()) and stream is not None, stream)
+    ph.mark("start")
     if info["path"] != bg.BLU_PATH_HASH_GLOBAL:
         st = bg.dense_state_arrays(plan, device=key_cols[0].device)
         bg.blu_gby_execute_dense_state(plan, key_cols, val_cols, st, init=True, stream=stream)
         t = bg.blu_gby_last_timing()
+        ph.mark("local")
         if P > 1:
             allreduce_dense_state(st, group)
+        ph.mark("exchange")
         res = bg.blu_gby_finalize_dense_state(plan, st, stream=stream)
+        ph.mark("merge")
         res.agg_timing = t
+        res.phase_ms = ph.result()
         return res, "allreduce"
     n_local = int(len(key_cols[0]))
     if P > 1 and exchange_mode(plan, n_local, mode) == "rows":
         words = plan.row_record_bytes // 8
         send = torch.empty(max(1, n_local) * words, dtype=torch.int64, device=key_cols[0].device)
         counts = bg.blu_gby_partition_rows(plan, key_cols, val_cols, P, send, stream=stream)
+        ph.mark("local")
         recv = alltoallv_records(send, counts, words, group)
+        ph.mark("exchange")
         res = bg.blu_gby_execute_records(plan, recv, recv.numel() // words, stream=stream)
         res.agg_timing = bg.blu_gby_last_timing()
+        ph.mark("merge")
+        res.phase_ms = ph.result()
         return res, "rows"
     part = bg.blu_gby_execute_partial(plan, key_cols, val_cols, stream=stream)
     t = bg.blu_gby_last_timing()
     if P == 1:
+        ph.mark("local")
         res = bg.blu_gby_merge(plan, [part], stream=stream)
+        ph.mark("merge")
         res.agg_timing = t
+        res.phase_ms = ph.result()
         return res, "local"
     words = plan.record_bytes // 8
     send = torch.empty(max(1, part.n_groups) * words, dtype=torch.int64, device=key_cols[0].device)
     counts = bg.blu_gby_partition(plan, part, P, send, stream=stream)
+    del part
+    ph.mark("local")
     recv = alltoallv_records(send, counts, words, group)
+    del send
+    ph.mark("exchange")
     res = bg.blu_gby_merge_records(plan, recv, recv.numel() // words, stream=stream)
+    ph.mark("merge")
     res.agg_timing = t
+    res.phase_ms = ph.result()
     return res, "partials"
