@@ -160,15 +160,19 @@ def oracle_sliced(config, row0, n, P):
 
 
 def sample_rows(config, P, seconds):
-    """Rows of a bounded sample that keeps the key-sliced oracle busy for about `seconds`."""
+    """Rows of a bounded sample that keeps the key-sliced oracle busy for about `seconds` (calibrated on
+    growing samples so the worker start-up does not distort the rate)."""
     import blugen
-    n_cal = 400_000
-    rate, dt, _ = oracle_sliced(config, 0, n_cal, P)
     full = blugen.workload(config).n_rows
-    return int(max(n_cal, min(full, rate * seconds)))
+    n = 2_000_000
+    while True:
+        _, dt, _ = oracle_sliced(config, 0, n, P)
+        if dt >= seconds / 4 or n >= full:
+            return int(max(1, min(full, n * seconds / max(dt, 1e-3))))
+        n = min(full, n * 4)
 
 
-def cpu_baseline(config, seconds=15.0):
+def cpu_baseline(config, seconds=12.0):
     """The oracle as it stands on the host cores (key-sliced, one process per core) on a bounded
     sample: the first R rows of the workload, R sized for ~`seconds` of wall time."""
     P = max(1, os.cpu_count() or 1)

@@ -25,7 +25,7 @@ CASES = {
     "dense_a_C2": ("C2", 600_001, None, "allreduce"),
     "dense_bprime_C4": ("C4", 800_003, None, "allreduce"),
     "partials_C5": ("C5", 1_200_007, 20_000, "partials"),
-    "rows_C3": ("C3", 900_001, 400_000, "rows"),
+    "rows_C3": ("C3", 900_001, 600_000, "rows"),  # est 600K >= rows per rank (450K at P = 2)
 }
 
 

@@ -202,6 +202,7 @@ struct RP {
   uint32_t Tp, S, NP, CW;
   uint32_t* flags;
   uint32_t mode;
+  uint32_t l2frac;  // keys whose hash byte is below this go straight to the global table (L2 REDs)
 };
 
 __device__ __forceinline__ uint32_t home4(uint64_t key, uint32_t nbk) {
@@ -221,11 +222,15 @@ template <int R>
 __device__ __forceinline__ void tbl_apply(const Tbl& T, const RP& p, const uint64_t (&key)[R], const uint64_t (&v0)[R],
                                           const double (&v1)[R], uint32_t valid) {
   uint32_t h[R], e[R];
+  uint32_t glob = 0;
 #pragma unroll
   for (int r = 0; r < R; ++r) {
-    h[r] = home4(key[r], T.nbk);
+    const uint64_t hh = fmix64(key[r] ^ 0x2545F4914F6CDD1Dull);
+    h[r] = (uint32_t)(((hh >> 32) * (uint64_t)T.nbk) >> 32);
+    if ((uint32_t)(hh & 255) < p.l2frac) glob |= 1u << r;
     e[r] = 0;
   }
+  valid &= ~glob;
   uint32_t pending = valid, hit = 0;
   for (int it = 0; it < 32 && pending; ++it) {
 #pragma unroll
@@ -262,7 +267,7 @@ __device__ __forceinline__ void tbl_apply(const Tbl& T, const RP& p, const uint6
       const uint32_t carry = (old + lo) < old ? 1u : 0u;
       if (hi + carry) atomicAdd(&T.hi[x], hi + carry);
       atomicAdd(&T.f[x], v1[r]);
-    } else if (pending >> r & 1) {
+    } else if ((pending | glob) >> r & 1) {
       uint64_t sl;
       if (g_locate(p.table, p.mask, key[r], sl)) {
         atomicAdd(&p.table[sl].cnt, 1ull);
@@ -540,6 +545,7 @@ int main(int argc, char** argv) {
   const int NBUF = argc > 10 ? atoi(argv[10]) : 3;
   const uint32_t mode = argc > 11 ? atoi(argv[11]) : 0;
   const int reps = argc > 12 ? atoi(argv[12]) : 2;
+  const uint32_t l2frac = argc > 13 ? atoi(argv[13]) : 0;
   int sms = 0;
   CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
   const uint64_t cap = 1ull << cb, mask = cap - 1;
@@ -615,11 +621,12 @@ int main(int argc, char** argv) {
   p.CW = CW;
   p.flags = flags;
   p.mode = mode;
+  p.l2frac = l2frac;
   const uint32_t block = (NP + 4 + CW) * 32;
   const size_t smem = (size_t)6 * Tp * 8 + (size_t)S * 28 + (B1 + 1) * 4 + (size_t)NBUF * sms * 4 + 16 + 64;
-  printf("v3: G %llu rows %llu B1 %u Tp %u S %u NP %u CW %u CAPP %u NBUF %d block %u smem %zu sub %.1f MB mode %u\n",
+  printf("v3: G %llu rows %llu B1 %u Tp %u S %u NP %u CW %u CAPP %u NBUF %d block %u smem %zu sub %.1f MB mode %u l2frac %u\n",
          (unsigned long long)G, (unsigned long long)tot, B1, Tp, S, NP, CW, CAPP, NBUF, block, smem,
-         (double)NBUF * sms * sms * CAPP * 32 / 1e6, mode);
+         (double)NBUF * sms * sms * CAPP * 32 / 1e6, mode, l2frac);
   if (smem > 232448 || block > 1024) {
     printf("v3: does not fit\n");
     return 1;

@@ -258,6 +258,155 @@ __global__ void __launch_bounds__(1024, 1) k_agg3(uint64_t rows_per_cta, uint32_
   atomicAdd(out, acc);
 }
 
+
+// v4: atomic-free aggregation. Per tile of 1024 x R rows: warp-level multisplit of the rows by owner
+// warp (32 table partitions by hash bits; match_any ranks, per-warp counters, one block scan; no
+// atomics), rows staged in shared memory by owner, then every warp aggregates its own rows into its
+// own partition: probe (2 x LDS.128 per 4-entry bucket), equal entries grouped with match_any and
+// combined by shuffles, then plain loads/stores by the group leader. Only claiming an empty entry is
+// an atomic (CAS: once per group per table lifetime).
+template <int R>
+__global__ void __launch_bounds__(1024, 1) k_agg4(uint64_t rows_per_cta, uint32_t G, uint32_t S, unsigned long long* out) {
+  extern __shared__ __align__(16) uint8_t sm[];
+  const uint32_t T = blockDim.x * R;  // rows per tile
+  uint64_t* tkey = (uint64_t*)sm;     // S
+  uint64_t* ts0 = tkey + S;           // S  (int64 sum, plain RMW)
+  double* ts1 = (double*)(ts0 + S);   // S
+  uint32_t* tcnt = (uint32_t*)(ts1 + S);  // S
+  uint64_t* sk = (uint64_t*)(tcnt + S);   // T staged keys
+  uint64_t* sa = sk + T;                  // T
+  double* sc = (double*)(sa + T);         // T
+  uint32_t* wcnt = (uint32_t*)(sc + T);   // [32 dest][32 warp]
+  uint32_t* wtot = wcnt + 1024;           // 32 + 1
+  for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) {
+    tkey[e] = kEmpty;
+    ts0[e] = 0;
+    ts1[e] = 0.0;
+    tcnt[e] = 0;
+  }
+  const uint32_t lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const uint32_t P = S >> 5;   // entries per warp partition
+  const uint32_t nbk = P >> 2;
+  const uint32_t lt = (1u << lane) - 1;
+  __syncthreads();
+  for (uint64_t j0 = 0; j0 < rows_per_cta; j0 += T) {
+    uint64_t key[R], v0[R];
+    double v1[R];
+    uint32_t d[R], rk[R];
+    wcnt[threadIdx.x] = 0;  // blockDim == 1024 == 32 x 32 counters
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      synth(blockIdx.x, j0 + (uint64_t)r * blockDim.x + threadIdx.x, G, key[r], v0[r], v1[r]);
+      d[r] = (uint32_t)(fmix64(key[r] ^ 0x2545F4914F6CDD1Dull) >> 59);  // owner warp (top 5 hash bits)
+      const uint32_t m = __match_any_sync(0xffffffffu, d[r]);
+      const uint32_t before = wcnt[d[r] * 32 + w];  // this warp's count for d so far (only this warp writes it)
+      rk[r] = before + __popc(m & lt);
+      __syncwarp();
+      if ((m & lt) == 0) wcnt[d[r] * 32 + w] = before + __popc(m);
+      __syncwarp();
+    }
+    __syncthreads();
+    {  // exclusive scan of the 1024 counters in (dest, warp) order: thread t holds element t
+      const uint32_t x = wcnt[threadIdx.x];
+      uint32_t inc = x;
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if ((int)lane >= o) inc += y;
+      }
+      if (lane == 31) wtot[w] = inc;
+      __syncthreads();
+      if (w == 0) {
+        const uint32_t v = wtot[lane];
+        uint32_t vi = v;
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t y = __shfl_up_sync(0xffffffffu, vi, o);
+          if ((int)lane >= o) vi += y;
+        }
+        wtot[lane] = vi - v;  // exclusive prefix of dest block `lane` (dest-major: row = dest)
+        if (lane == 31) wtot[32] = vi;
+      }
+      __syncthreads();
+      wcnt[threadIdx.x] = wtot[w] + inc - x;  // element (dest = w_row, warp = lane) -> its offset
+    }
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const uint32_t pos = wcnt[d[r] * 32 + w] + rk[r];
+      sk[pos] = key[r];
+      sa[pos] = v0[r];
+      sc[pos] = v1[r];
+    }
+    __syncthreads();
+    // warp w aggregates destination block w: rows [start, end)
+    const uint32_t start = wcnt[w * 32], end = (w == 31) ? wtot[32] : wcnt[(w + 1) * 32];
+    uint64_t* pk = tkey + (size_t)P * w;
+    for (uint32_t i0 = start; i0 < end; i0 += 32) {
+      const uint32_t i = i0 + lane;
+      const bool ok = i < end;
+      const uint64_t kk = ok ? sk[i] : kEmpty;
+      const uint64_t a = ok ? sa[i] : 0;
+      const double c = ok ? sc[i] : 0.0;
+      uint32_t h = ok ? (uint32_t)(((fmix64(kk ^ 0x2545F4914F6CDD1Dull) >> 27 & 0xFFFFFFFFull) * nbk) >> 32) : 0u;
+      int e = -1;
+      bool pend = ok;
+      for (int it = 0; it < 32 && __any_sync(0xffffffffu, pend); ++it) {
+        if (pend) {
+          const uint64_t* q = pk + 4 * h;
+          uint64_t k0, k1, k2, k3;
+          lds128v(q, k0, k1);
+          lds128v(q + 2, k2, k3);
+          int m = k0 == kk ? 0 : k1 == kk ? 1 : k2 == kk ? 2 : k3 == kk ? 3 : -1;
+          if (m < 0) {
+            const int z = k0 == kEmpty ? 0 : k1 == kEmpty ? 1 : k2 == kEmpty ? 2 : k3 == kEmpty ? 3 : -1;
+            if (z >= 0) {
+              const unsigned long long old = atomicCAS((unsigned long long*)(q + z), kEmpty, (unsigned long long)kk);
+              if (old == kEmpty || old == kk) m = z;
+            } else {
+              h = h + 1 == nbk ? 0u : h + 1;
+            }
+          }
+          if (m >= 0) {
+            e = (int)(4 * h + m);
+            pend = false;
+          }
+        }
+      }
+      // group equal entries, combine in the leader, plain read-modify-write
+      const uint32_t g = __match_any_sync(0xffffffffu, (uint32_t)e);
+      const uint32_t leader = __ffs(g) - 1;
+      uint64_t s0 = a;
+      double s1 = c;
+      if (__any_sync(0xffffffffu, __popc(g) > 1)) {
+        uint32_t rest = g & ~(1u << leader);
+        s0 = lane == leader ? a : 0;
+        s1 = lane == leader ? c : 0.0;
+        while (__any_sync(0xffffffffu, rest)) {
+          const uint32_t src = rest ? __ffs(rest) - 1 : lane;
+          const uint64_t x = __shfl_sync(0xffffffffu, a, src);
+          const double y = __shfl_sync(0xffffffffu, c, src);
+          if (rest && lane == leader) {
+            s0 += x;
+            s1 += y;
+          }
+          if (rest) rest &= rest - 1;
+        }
+      }
+      if (e >= 0 && lane == leader) {
+        const uint32_t x = P * w + (uint32_t)e;
+        ts0[x] += s0;
+        ts1[x] += s1;
+        tcnt[x] += __popc(g);
+      }
+    }
+    __syncthreads();
+  }
+  __syncthreads();
+  unsigned long long acc = 0;
+  for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) acc += tcnt[e];
+  atomicAdd(out, acc);
+}
+
 int main(int argc, char** argv) {
   const uint64_t rows = argc > 1 ? strtoull(argv[1], 0, 10) : 1000000000ull;
   const uint32_t G = argc > 2 ? atoi(argv[2]) : 2111;
@@ -268,7 +417,7 @@ int main(int argc, char** argv) {
   unsigned long long* out;
   CK(cudaMalloc(&out, 8));
   const uint64_t per = rows / sms / (block * 4) * (block * 4);
-  const size_t smem = (size_t)S * (8 + 8 + 4 + 4 + 4 + 8);
+  const size_t smem = (size_t)S * (8 + 8 + 4 + 4 + 4 + 8) + (size_t)1024 * 2 * 24 + 4096 + 256;
   cudaEvent_t e0, e1;
   cudaEventCreate(&e0);
   cudaEventCreate(&e1);
@@ -293,8 +442,7 @@ int main(int argc, char** argv) {
   run(k_agg<4, 1>, "v1 atomics, 2xLDS.128 probe");
   run(k_agg<4, 2>, "v2 match_any + 3 atomics");
   run(k_agg<2, 1>, "v1 R=2");
-  run(k_agg3<4, 0>, "v3 warp-exclusive, plain RMW");
-  run(k_agg3<4, 1>, "v3 synth only");
-  run(k_agg3<4, 2>, "v3 synth + probe");
+  run(k_agg4<2>, "v4 multisplit, no atomics R=2");
+
   return 0;
 }
