@@ -1742,22 +1742,33 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
   const uint64_t pol = evict_first_policy();
   const uint64_t n = p.n_rows;
   const uint64_t ntiles = (n + TILE - 1) / TILE;
+  // segmented input (second scatter level): rows [s * in_seg, s * in_seg + in_count[s]) of every
+  // first-level bucket s; in_seg is a multiple of TILE, so a tile lies in one bucket
+  auto tile_lim = [&](uint64_t t) -> uint64_t {
+    if (!sp.in_seg) return n;
+    const uint64_t s0 = (t * TILE) / sp.in_seg;
+    const uint64_t c = sp.in_count[s0];
+    return s0 * sp.in_seg + (c < sp.in_seg ? c : sp.in_seg);
+  };
   using Raw = RawTileFor<SP, R, PIPE>;
   Raw T;
   if constexpr (PIPE)
-    if (blockIdx.x < ntiles) tile_load<SP, R>(p, lane_base<R>(blockIdx.x * TILE, threadIdx.x >> 5, threadIdx.x & 31), n, pol, T);
+    if (blockIdx.x < ntiles)
+      tile_load<SP, R>(p, lane_base<R>(blockIdx.x * TILE, threadIdx.x >> 5, threadIdx.x & 31), tile_lim(blockIdx.x), pol, T);
   for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
     for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
     __syncthreads();
     const uint64_t row = lane_base<R>(t * TILE, threadIdx.x >> 5, threadIdx.x & 31);
+    const uint64_t lim = tile_lim(t);
+    const uint32_t bbase = sp.in_seg ? (uint32_t)((t * TILE) / sp.in_seg) * sp.in_B2 : 0u;
     uint64_t key[R];
     uint64_t v[NV][R];
     uint32_t valid;
     if constexpr (PIPE) {
-      valid = tile_unpack<SP, NV, R>(p, T, row, n, key, v);
+      valid = tile_unpack<SP, NV, R>(p, T, row, lim, key, v);
     } else {
-      valid = pack_keys<SP, R>(p, row, n, pol, key);
-      load_vals<SP, NV, R>(p, row, n, pol, v);
+      valid = pack_keys<SP, R>(p, row, lim, pol, key);
+      load_vals<SP, NV, R>(p, row, lim, pol, v);
     }
     if (!PIPE && p.prefetch) {  // a later tile of this CTA: in flight during the sort and the writes below
       const uint64_t nt = t + (uint64_t)gridDim.x * p.prefetch;
@@ -1766,7 +1777,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
     uint32_t bb[R], pos[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-      bb[r] = (uint32_t)((fmix64(key[r]) & p.cap_mask) >> sp.shift);
+      bb[r] = bbase + (uint32_t)((fmix64(key[r]) & p.cap_mask) >> sp.shift);
       pos[r] = (valid >> r & 1) ? atomicAdd(&hist[bb[r]], 1u) : 0u;
     }
     __syncthreads();
@@ -1791,7 +1802,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
       }
     if constexpr (PIPE) {  // this tile is in shared memory: the next one's loads go out now
       const uint64_t tn = t + gridDim.x;
-      if (tn < ntiles) tile_load<SP, R>(p, lane_base<R>(tn * TILE, threadIdx.x >> 5, threadIdx.x & 31), n, pol, T);
+      if (tn < ntiles) tile_load<SP, R>(p, lane_base<R>(tn * TILE, threadIdx.x >> 5, threadIdx.x & 31), tile_lim(tn), pol, T);
     }
     __syncthreads();
     const uint32_t tot = *total;

@@ -162,6 +162,13 @@ struct ScatterParams {
   uint64_t* out_key;         // packed keys (u64)
   void* out_val[kMaxVals];   // value columns, input dtypes
   uint32_t* gate;            // set to 1 if any bucket overflows (pass 2 then falls back)
+  // segmented input (the second level of a two-level scatter, one launch over every first-level
+  // bucket): first-level bucket s holds rows [s * in_seg, s * in_seg + in_count[s]) of the input
+  // (in_seg a multiple of the tile); its rows go to buckets s * in_B2 + ((h & cap_mask) >> shift).
+  // in_seg = 0: plain input rows [0, n).
+  uint64_t in_seg;
+  const uint64_t* in_count;
+  uint32_t in_B2;
 };
 
 enum : uint32_t { FLAG_OVERFLOW = 1u, FLAG_KEY_RANGE = 2u };

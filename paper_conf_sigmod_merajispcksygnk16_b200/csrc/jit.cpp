@@ -264,6 +264,22 @@ static void probe_compile(const std::string& body) {
 
 const void* jit_kernel(const std::string& spec_src, const std::string& entry_src, const char* entry) {
   if (!jit_enabled()) return nullptr;
+  if (const char* dump = getenv("BLU_GBY_JIT_DUMP")) {  // write the program text (SASS inspection offline)
+    std::string fn = std::string(dump) + "/" + entry + ".cu";
+    std::string src = std::string(kPreamble) + jit_defs() + kSrc_blu_params_h + "\n" + kSrc_blu_device_cuh + "\n" +
+                      spec_src + entry_src;
+    if (FILE* f = fopen(fn.c_str(), "w")) {
+      fwrite(src.data(), 1, src.size(), f);
+      fclose(f);
+    }
+    std::vector<char> cubin;
+    std::string log;
+    if (compile(src, cubin, log))
+      if (FILE* f = fopen((std::string(dump) + "/" + entry + ".cubin").c_str(), "wb")) {
+        fwrite(cubin.data(), 1, cubin.size(), f);
+        fclose(f);
+      }
+  }
   if (t_probe) {
     probe_compile(jit_defs() + spec_src + entry_src);
     return nullptr;
