@@ -700,7 +700,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       q.lay = L2;
       q.key[0] = kbuf1;
       for (int c = 0; c < L.n_vals; ++c) q.val[c] = vbuf1[c];
-      q.vec_ok = 3;  // segments start at multiples of 4096 rows
+      q.vec_ok = 3;  // segments start at multiples of 4096 rows (>= the second level's tile)
       q.n_rows = (uint64_t)B1 * seg_cap1;
       q.prefetch = 0;
       q.cap_mask = shift1 >= 64 ? ~0ull : ((1ull << shift1) - 1);  // the slot bits below the first level's
@@ -710,7 +710,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       s2.in_seg = seg_cap1;
       s2.in_count = d_cursor1;
       s2.in_B2 = B2;
-      le = launch_scatter(q, s2, st, scatter_grid((uint32_t)P->sms, B));
+      le = launch_scatter(q, s2, st, scatter_grid((uint32_t)P->sms, B2));
       if (le) return (cudaError_t)le;
     }
     if (dbg) cudaEventRecord(ev[1], st);

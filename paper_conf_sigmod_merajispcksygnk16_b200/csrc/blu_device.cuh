@@ -1729,7 +1729,9 @@ template <class SP, int NV, int R, bool PIPE = false>
 __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterParams& sp) {
   extern __shared__ __align__(16) uint8_t sm[];
   const Layout& L = p.lay;
-  const uint32_t B = sp.B;
+  // histogram bins: the buckets one tile can reach (segmented input: the B2 buckets of its first-level
+  // bucket, global index bbase + local bin)
+  const uint32_t B = sp.in_seg ? sp.in_B2 : sp.B;
   const uint32_t TILE = blockDim.x * R;
   uint64_t* skey = (uint64_t*)sm;                       // TILE
   uint64_t* sval = skey + TILE;                         // NV x TILE
@@ -1777,7 +1779,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
     uint32_t bb[R], pos[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) {
-      bb[r] = bbase + (uint32_t)((fmix64(key[r]) & p.cap_mask) >> sp.shift);
+      bb[r] = (uint32_t)((fmix64(key[r]) & p.cap_mask) >> sp.shift);
       pos[r] = (valid >> r & 1) ? atomicAdd(&hist[bb[r]], 1u) : 0u;
     }
     __syncthreads();
@@ -1785,7 +1787,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
     for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
       uint32_t h = hist[b];
       if (h) {
-        uint64_t g = atomicAdd((unsigned long long*)&sp.cursor[b], (unsigned long long)h);
+        uint64_t g = atomicAdd((unsigned long long*)&sp.cursor[bbase + b], (unsigned long long)h);
         gpos[b] = g;
         if (g + h > sp.seg_cap) atomicExch(sp.gate, 1u);
       }
@@ -1810,7 +1812,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
       const uint32_t b = sbid[e];
       const uint64_t g = gpos[b] + (e - lstart[b]);
       if (g >= sp.seg_cap) continue;
-      const uint64_t idx = (uint64_t)b * sp.seg_stride + g;
+      const uint64_t idx = (uint64_t)(bbase + b) * sp.seg_stride + g;
       sp.out_key[idx] = skey[e];
 #pragma unroll
       for (int c = 0; c < NV; ++c)

@@ -184,8 +184,9 @@ size_t scatter_smem(int nv, uint32_t B) {
 
 template <int NV, int R>
 static int launch_scatter_nv(const AggParams& p, const ScatterParams& sp, cudaStream_t st, uint32_t grid) {
-  const uint32_t block = scatter_block(sp.B);
-  const size_t smem = scatter_smem(p.lay.n_vals, sp.B);
+  const uint32_t bins = sp.in_seg ? sp.in_B2 : sp.B;  // histogram bins of one tile
+  const uint32_t block = scatter_block(bins);
+  const size_t smem = scatter_smem(p.lay.n_vals, bins);
   if (p.jit_ok && jit_env("BLU_GBY_JIT_SCATTER", 1)) {
     char body[160], decl[160], name[64];
     // register-pipelined tile loads instead of the L2 prefetch (C3 scatter 10.07 -> 9.48 ms)

@@ -459,7 +459,8 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
       const uint64_t max_b = two_level && !cap_default ? kMaxBuckets2 : kMaxBuckets;
       uint64_t b = 2;
       while (b < max_b && (double)P->est_groups > kBucketLoad * S_of((uint32_t)b) * (double)b &&
-             scatter_smem(L.n_vals, (uint32_t)(b * 2)) <= kSmemMax &&  // the second level has every bucket's bin
+             scatter_smem(L.n_vals, (uint32_t)(two_level && b >= 256 ? std::max<uint64_t>(64, 2 * b / 32) : b * 2)) <=
+                 kSmemMax &&
              b * 2 <= P->cap / 1024)
         b <<= 1;
       return b;
@@ -481,7 +482,8 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     if (smem_mode && ((budget && tbytes > budget) || (forced && atoi(forced) > 1))) {
       B = smem_B(two_ok, !env("BLU_GBY_PART_SMEM"));
       if (forced) B = std::max(2, std::min((int)(two_ok ? kMaxBuckets2 : kMaxBuckets), atoi(forced)));
-      while (B > 2 && scatter_smem(L.n_vals, (uint32_t)B) > kSmemMax) B >>= 1;  // one-launch second level: B bins
+      auto widest = [&](uint64_t b) { return (uint32_t)(two_ok && b >= 256 ? std::max<uint64_t>(32, b / 32) : b); };
+      while (B > 2 && scatter_smem(L.n_vals, widest(B)) > kSmemMax) B >>= 1;  // histogram bins per tile
       P->part_smem = 1;
       P->bucket_S = S_of((uint32_t)B);
       P->bucket_smem = bucket_smem_bytes(L, P->bucket_S, (uint32_t)B);

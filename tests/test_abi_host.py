@@ -123,15 +123,15 @@ def test_planner_partitioned_l2_mode(bg, monkeypatch):
 def test_planner_partitioned_smem_mode(bg, monkeypatch):
     """BLU_GBY_PART_SMEM=1: pass 2 in per-CTA shared-memory bucket tables; buckets hold <= 0.7 x the
     table's entries on average (C3: 10^7 / 2048 = 4883 of 8000); the global table keeps load <= 0.7;
-    the two-level scatter's second level is one launch whose shared-memory histogram holds every bucket,
-    so C5's records allow at most 4096 buckets either way (the planner never defaults C5 to this mode)."""
+    the two-level scatter (32 x 512; the second level one launch with 512 bins per tile) allows 16384
+    buckets (C5), a one-level scatter at most 4096."""
     monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
     c3 = _plan(bg, blugen.workload("C3")).info()
     assert c3["part_smem"] == 1 and c3["capacity"] == 2**24
     assert c3["partitions"] == 2048 and c3["bucket_entries"] >= 7900
     assert 10**7 / c3["partitions"] <= 0.7 * c3["bucket_entries"]
     c5 = _plan(bg, blugen.workload("C5")).info()
-    assert c5["part_smem"] == 1 and c5["partitions"] == 4096
+    assert c5["part_smem"] == 1 and c5["partitions"] == 16384
     monkeypatch.setenv("BLU_GBY_PART_2LEVEL", "0")
     c5 = _plan(bg, blugen.workload("C5")).info()
     assert c5["part_smem"] == 1 and c5["partitions"] == 4096
