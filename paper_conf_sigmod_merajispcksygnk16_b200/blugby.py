@@ -278,6 +278,17 @@ class _DevArray:
                                          "version": 3, "strides": None}
 
 
+class _HostArray:
+    """__array_interface__ provider for a host result column: numpy views it without a copy and keeps
+    the result's owner (which frees the library's host memory) alive while any view exists."""
+
+    def __init__(self, owner: _Owner, ptr: int, n: int, dt: int):
+        typestr = {BLU_I32: "<i4", BLU_I64: "<i8", BLU_F64: "<f8", BLU_I128: "<i8"}[dt]
+        self._owner = owner
+        shape = (n, 2) if dt == BLU_I128 else (n,)
+        self.__array_interface__ = {"shape": shape, "typestr": typestr, "data": (ptr, False), "version": 3}
+
+
 class Result:
     """A blu_gby_result_t. keys / aggs / states are torch tensors (device, zero-copy) or numpy
     arrays (host results). Library memory is released when this object and every view are gone."""
@@ -304,9 +315,7 @@ class Result:
             w = 2 if dt == BLU_I128 else 1
             if n == 0:
                 return np.zeros((0, 2) if w == 2 else 0, npdt)
-            buf = (ctypes.c_char * (n * w * np.dtype(npdt).itemsize)).from_address(ptr)
-            a = np.frombuffer(buf, npdt).copy()  # host results are small; copy and free below
-            return a.reshape(n, 2) if w == 2 else a
+            return np.asarray(_HostArray(self._owner, ptr, n, dt))  # zero-copy view of the library's host memory
         import torch
         if n == 0:
             return torch.zeros((0, 2) if dt == BLU_I128 else 0, dtype=_torch_dtype(dt), device=device or "cuda")
@@ -373,9 +382,7 @@ def blu_gby_execute_host(plan: Plan, key_cols, val_cols, n_rows: Optional[int] =
     s = _stream_handle(stream)
     rc = ResultC()
     _check(lib.blu_gby_execute_host(plan.handle, _ptrs(key_cols), _ptrs(val_cols), n, s, ctypes.byref(rc)))
-    r = Result(rc, _key_dtypes(plan), _out_dtypes(plan, False), s)
-    r.free()  # numpy copies were taken
-    return r
+    return Result(rc, _key_dtypes(plan), _out_dtypes(plan, False), s)
 
 
 def _results_array(partials: Sequence[Result]):

@@ -282,6 +282,57 @@ static cudaError_t agg_batch(const blu_gby_plan_s* P, int path, AggParams p, con
   return cudaSuccess;
 }
 
+// Device -> pageable host copies through two pinned bounce buffers (allocated once per thread): the
+// copy engine writes pinned memory at the PCIe rate while the host copies the previous chunk out.
+static cudaError_t d2h_staged(const std::vector<std::pair<void*, const void*>>& cols, const std::vector<size_t>& sizes,
+                              cudaStream_t st) {
+  constexpr size_t kChunk = 32u << 20;
+  static thread_local uint8_t* pin[2] = {nullptr, nullptr};
+  static thread_local cudaEvent_t done[2] = {nullptr, nullptr};
+  size_t total = 0;
+  for (size_t b : sizes) total += b;
+  if (total <= kChunk / 8 || (!pin[0] && (cudaMallocHost((void**)&pin[0], kChunk) != cudaSuccess ||
+                                          cudaMallocHost((void**)&pin[1], kChunk) != cudaSuccess))) {
+    cudaGetLastError();
+    for (size_t i = 0; i < cols.size(); ++i)  // small result (or no pinned memory): direct copies
+      if (sizes[i]) {
+        cudaError_t e = cudaMemcpyAsync(cols[i].first, cols[i].second, sizes[i], cudaMemcpyDeviceToHost, st);
+        if (e) return e;
+      }
+    return cudaSuccess;
+  }
+  if (!done[0]) {
+    cudaEventCreateWithFlags(&done[0], cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&done[1], cudaEventDisableTiming);
+  }
+  struct Pending {
+    uint8_t* dst = nullptr;
+    size_t n = 0;
+  } pend[2];
+  int slot = 0;
+  auto drain = [&](int b) -> cudaError_t {
+    if (!pend[b].n) return cudaSuccess;
+    cudaError_t e = cudaEventSynchronize(done[b]);
+    if (e) return e;
+    memcpy(pend[b].dst, pin[b], pend[b].n);
+    pend[b].n = 0;
+    return cudaSuccess;
+  };
+  for (size_t i = 0; i < cols.size(); ++i)
+    for (size_t off = 0; off < sizes[i]; off += kChunk) {
+      const size_t n = std::min(kChunk, sizes[i] - off);
+      cudaError_t e = drain(slot);  // this bounce buffer's previous chunk
+      if (!e) e = cudaMemcpyAsync(pin[slot], (const uint8_t*)cols[i].second + off, n, cudaMemcpyDeviceToHost, st);
+      if (!e) e = cudaEventRecord(done[slot], st);
+      if (e) return e;
+      pend[slot] = Pending{(uint8_t*)cols[i].first + off, n};
+      slot ^= 1;
+    }
+  cudaError_t e = drain(slot);
+  if (!e) e = drain(slot ^ 1);
+  return e;
+}
+
 // The core: init -> feed -> compact -> one sync -> regrow on overflow.
 static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int path, bool front, uint64_t cap0,
                              uint64_t total_rows, const Feeder& feed, bool partial, cudaStream_t st,
@@ -487,23 +538,29 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     for (int k = 0; k < lay.n_keys; ++k) kc[k] = okeys[k];
     for (int o = 0; o < os.n_out; ++o) vc[o] = ovals[o];
     if (host_out) {
-      // copy to host and release the device outputs
+      // copy to host (pageable memory owned by the result) through two pinned bounce buffers, so the
+      // D2H runs at the pinned rate and overlaps the host-side copies; release the device outputs
       Owner* hown = new Owner();
+      std::vector<std::pair<void*, const void*>> cols;
+      std::vector<size_t> sizes;
       for (int k = 0; k < lay.n_keys; ++k) {
         size_t b = ng * dtype_bytes(lay.key_dtype[k]);
         void* h = malloc(std::max<size_t>(b, 1));
-        if (b) cudaMemcpyAsync(h, okeys[k], b, cudaMemcpyDeviceToHost, st);
         hown->host.push_back(h);
         kc[k] = h;
+        cols.push_back({h, okeys[k]});
+        sizes.push_back(b);
       }
       for (int o = 0; o < os.n_out; ++o) {
         size_t b = ng * dtype_bytes(os.out_dtype[o]);
         void* h = malloc(std::max<size_t>(b, 1));
-        if (b) cudaMemcpyAsync(h, ovals[o], b, cudaMemcpyDeviceToHost, st);
         hown->host.push_back(h);
         vc[o] = h;
+        cols.push_back({h, ovals[o]});
+        sizes.push_back(b);
       }
-      cudaError_t se = cudaStreamSynchronize(st);
+      cudaError_t se = d2h_staged(cols, sizes, st);
+      if (se == cudaSuccess) se = cudaStreamSynchronize(st);
       free_owner();
       own = hown;
       if (se != cudaSuccess) {

@@ -1758,10 +1758,17 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
     if (blockIdx.x < ntiles)
       tile_load<SP, R>(p, lane_base<R>(blockIdx.x * TILE, threadIdx.x >> 5, threadIdx.x & 31), tile_lim(blockIdx.x), pol, T);
   for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    const uint64_t lim = tile_lim(t);
+    if (sp.in_seg && lim <= t * TILE) {  // past its first-level bucket's rows (the segment's slack)
+      if constexpr (PIPE) {
+        const uint64_t tn = t + gridDim.x;
+        if (tn < ntiles) tile_load<SP, R>(p, lane_base<R>(tn * TILE, threadIdx.x >> 5, threadIdx.x & 31), tile_lim(tn), pol, T);
+      }
+      continue;
+    }
     for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
     __syncthreads();
     const uint64_t row = lane_base<R>(t * TILE, threadIdx.x >> 5, threadIdx.x & 31);
-    const uint64_t lim = tile_lim(t);
     const uint32_t bbase = sp.in_seg ? (uint32_t)((t * TILE) / sp.in_seg) * sp.in_B2 : 0u;
     uint64_t key[R];
     uint64_t v[NV][R];
