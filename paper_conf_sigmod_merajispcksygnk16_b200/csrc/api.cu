@@ -784,6 +784,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     p2.seg_count = d_cursor;
     p2.n_segs = B;
     p2.tile_ctr = getenv("BLU_GBY_DYN") && atoi(getenv("BLU_GBY_DYN")) == 0 ? nullptr : (uint64_t*)(d_cursor + B + 1);
+    if (const char* g = getenv("BLU_GBY_GRAB")) p2.grab = (uint32_t)atoi(g);
     p2.gate = d_gate;
     p2.gate_run_if = 0;
     p2.front_slots = 0;

@@ -1313,8 +1313,10 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
   const unsigned lane = threadIdx.x & 31;
   uint8_t* tb = (uint8_t*)p.table;
   uint32_t flag_seen = 0;
-  // SEG: a warp claims kGrab consecutive warp tiles per atomic (one counter for the whole grid)
-  constexpr uint32_t kGrab = 16;
+  // SEG: a warp claims kGrab consecutive warp tiles per atomic (one counter for the whole grid). The
+  // rows in flight span (warps x kGrab x tile) rows in bucket order, i.e. that fraction of the table
+  // (p.grab, 0 = 16; 1-4 keep C5's table window in L2 but measured no faster)
+  const uint32_t kGrab = p.grab ? p.grab : 16u;
   uint64_t t = blockIdx.x, chunk = 0, chunk_next = 0;
   uint32_t k_in = 0;
   const bool dyn = SEG && p.tile_ctr != nullptr;

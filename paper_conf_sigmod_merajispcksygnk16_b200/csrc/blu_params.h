@@ -137,6 +137,8 @@ struct AggParams {
   // per-bucket piece prefix (n_segs + 1 u32) behind the S-entry table in dynamic shared memory.
   uint64_t piece_rows;
   uint32_t aux_off;
+  // partitioned pass 2 in the L2-slice mode: warp tiles claimed per atomic on tile_ctr (0 = 16)
+  uint32_t grab;
 };
 
 // Path (a) in-kernel compaction (S8 fused into S5a/S7 for small dense domains).
