@@ -1725,15 +1725,17 @@ __device__ __forceinline__ void block_excl_scan(uint32_t* a, uint32_t* out, uint
   }
 }
 
+constexpr uint32_t kMaxInSeg = 64;  // first-level buckets of a two-level scatter (the planner uses 32)
+
 // PIPE (NVRTC kernels only): the next tile's rows are loaded into registers as soon as the current
 // tile is staged in shared memory, so those HBM reads are in flight during its write-out phase.
-template <class SP, int NV, int R, bool PIPE = false>
+template <class SP, int NV, int R, bool PIPE = false, bool SEGIN = false>
 __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterParams& sp) {
   extern __shared__ __align__(16) uint8_t sm[];
   const Layout& L = p.lay;
   // histogram bins: the buckets one tile can reach (segmented input: the B2 buckets of its first-level
   // bucket, global index bbase + local bin)
-  const uint32_t B = sp.in_seg ? sp.in_B2 : sp.B;
+  const uint32_t B = SEGIN ? sp.in_B2 : sp.B;
   const uint32_t TILE = blockDim.x * R;
   uint64_t* skey = (uint64_t*)sm;                       // TILE
   uint64_t* sval = skey + TILE;                         // NV x TILE
@@ -1748,11 +1750,18 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
   const uint64_t ntiles = (n + TILE - 1) / TILE;
   // segmented input (second scatter level): rows [s * in_seg, s * in_seg + in_count[s]) of every
   // first-level bucket s; in_seg is a multiple of TILE, so a tile lies in one bucket
+  __shared__ uint64_t seg_end[SEGIN ? kMaxInSeg : 1];  // end row of each first-level bucket
+  if constexpr (SEGIN) {
+    const uint32_t nseg = (uint32_t)((n + sp.in_seg - 1) / sp.in_seg);
+    for (uint32_t s0 = threadIdx.x; s0 < nseg && s0 < kMaxInSeg; s0 += blockDim.x) {
+      const uint64_t c = sp.in_count[s0];
+      seg_end[s0] = s0 * sp.in_seg + (c < sp.in_seg ? c : sp.in_seg);
+    }
+    __syncthreads();
+  }
   auto tile_lim = [&](uint64_t t) -> uint64_t {
-    if (!sp.in_seg) return n;
-    const uint64_t s0 = (t * TILE) / sp.in_seg;
-    const uint64_t c = sp.in_count[s0];
-    return s0 * sp.in_seg + (c < sp.in_seg ? c : sp.in_seg);
+    if constexpr (SEGIN) return seg_end[(t * TILE) / sp.in_seg];
+    return n;
   };
   using Raw = RawTileFor<SP, R, PIPE>;
   Raw T;
@@ -1761,7 +1770,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
       tile_load<SP, R>(p, lane_base<R>(blockIdx.x * TILE, threadIdx.x >> 5, threadIdx.x & 31), tile_lim(blockIdx.x), pol, T);
   for (uint64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
     const uint64_t lim = tile_lim(t);
-    if (sp.in_seg && lim <= t * TILE) {  // past its first-level bucket's rows (the segment's slack)
+    if (SEGIN && lim <= t * TILE) {  // past its first-level bucket's rows (the segment's slack)
       if constexpr (PIPE) {
         const uint64_t tn = t + gridDim.x;
         if (tn < ntiles) tile_load<SP, R>(p, lane_base<R>(tn * TILE, threadIdx.x >> 5, threadIdx.x & 31), tile_lim(tn), pol, T);
@@ -1771,7 +1780,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
     for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
     __syncthreads();
     const uint64_t row = lane_base<R>(t * TILE, threadIdx.x >> 5, threadIdx.x & 31);
-    const uint32_t bbase = sp.in_seg ? (uint32_t)((t * TILE) / sp.in_seg) * sp.in_B2 : 0u;
+    const uint32_t bbase = SEGIN ? (uint32_t)((t * TILE) / sp.in_seg) * sp.in_B2 : 0u;
     uint64_t key[R];
     uint64_t v[NV][R];
     uint32_t valid;

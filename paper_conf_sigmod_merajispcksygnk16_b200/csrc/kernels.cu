@@ -160,16 +160,16 @@ __global__ void __launch_bounds__(512, 2) k_agg_global(AggParams p, RecSrc rs) {
   global_body<GenericSpec, NV, R, FRONT, DIRECT, MODE>(p, rs);
 }
 
-template <int NV, int R>
+template <int NV, int R, bool SEGIN>
 __global__ void __launch_bounds__(512, 2) k_scatter(AggParams p, ScatterParams sp) {
-  scatter_body<GenericSpec, NV, R>(p, sp);
+  scatter_body<GenericSpec, NV, R, false, SEGIN>(p, sp);
 }
 
 // wide fan-out (B > 512): one 1024-thread CTA per SM, a tile twice as long (more rows per bucket
 // per cursor reservation)
-template <int NV, int R>
+template <int NV, int R, bool SEGIN>
 __global__ void __launch_bounds__(1024, 1) k_scatter_wide(AggParams p, ScatterParams sp) {
-  scatter_body<GenericSpec, NV, R>(p, sp);
+  scatter_body<GenericSpec, NV, R, false, SEGIN>(p, sp);
 }
 
 uint32_t scatter_block(uint32_t B) { return B > 512 ? 1024u : 512u; }
@@ -191,15 +191,18 @@ static int launch_scatter_nv(const AggParams& p, const ScatterParams& sp, cudaSt
     char body[160], decl[160], name[64];
     // register-pipelined tile loads instead of the L2 prefetch (C3 scatter 10.07 -> 9.48 ms)
     const int pipe = jit_env("BLU_GBY_SCATTER_PIPE", 1);
-    snprintf(name, sizeof name, "blu_jit_scatter_%d_%d%s", NV, R, pipe ? "_p" : "");
+    const bool seg = sp.in_seg != 0;
+    snprintf(name, sizeof name, "blu_jit_scatter_%d_%d%s%s", NV, R, pipe ? "_p" : "", seg ? "_s" : "");
     snprintf(decl, sizeof decl, "%s(blu::AggParams p, blu::ScatterParams sp)", name);
-    snprintf(body, sizeof body, "blu::scatter_body<blu::JitSpec, %d, %d, %s>(p, sp);", NV, R, pipe ? "true" : "false");
+    snprintf(body, sizeof body, "blu::scatter_body<blu::JitSpec, %d, %d, %s, %s>(p, sp);", NV, R, pipe ? "true" : "false",
+             seg ? "true" : "false");
     AggParams pc = p;
     ScatterParams sc = sp;
     void* args[] = {&pc, &sc};
     if (launch_jit(body, decl, p, args, st, grid, block, (uint32_t)smem, name, 2)) return 0;
   }
-  auto k = block > 512 ? k_scatter_wide<NV, R> : k_scatter<NV, R>;
+  auto k = sp.in_seg ? (block > 512 ? k_scatter_wide<NV, R, true> : k_scatter<NV, R, true>)
+                     : (block > 512 ? k_scatter_wide<NV, R, false> : k_scatter<NV, R, false>);
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e) return (int)e;
   k<<<grid, block, smem, st>>>(p, sp);

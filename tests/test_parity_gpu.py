@@ -457,17 +457,19 @@ def test_partitioned_two_pass(bg, oracles, monkeypatch, parts, chunk, div, smem)
     assert_parity(gk, ga, o, w.schema)
 
 
-@pytest.mark.parametrize("two_level", ["0", "1"])
+@pytest.mark.parametrize("two_level", ["0", "1", "1-one"])
 @pytest.mark.parametrize("parts", [None, "4096"])
 def test_partitioned_wide_fanout(bg, monkeypatch, parts, two_level):
     """Shared-memory bucket tables as planned for 2M groups (several hundred buckets, the 1024-thread
     wide scatter) and with a forced 4096-way scatter, at 20M rows, against the oracle; in one B-way
-    scatter or in two levels (32 first-level buckets, each scattered again into B / 32)."""
+    scatter or in two levels (32 first-level buckets, each scattered again into B / 32: one launch per
+    first-level bucket, or '1-one': all of them in one launch over the segmented first-level output)."""
     w = blugen.workload("C3", n_rows=20_000_003, n_groups=2_000_000)
     o = oracle.groupby_generated(w)
     kc, vc = blugen.device_columns(w)
     monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
-    monkeypatch.setenv("BLU_GBY_PART_2LEVEL", two_level)
+    monkeypatch.setenv("BLU_GBY_PART_2LEVEL", two_level[0])
+    monkeypatch.setenv("BLU_GBY_2LEVEL_ONE", "1" if two_level.endswith("one") else "0")
     if parts:
         monkeypatch.setenv("BLU_GBY_PARTS", parts)
     plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
