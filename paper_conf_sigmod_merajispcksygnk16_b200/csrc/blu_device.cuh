@@ -1832,13 +1832,22 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
       if (g >= sp.seg_cap) continue;
       const uint64_t idx = (uint64_t)(bbase + b) * sp.seg_stride + g;
       sp.out_key[idx] = skey[e];
-#pragma unroll
-      for (int c = 0; c < NV; ++c)
-        if (c < L.n_vals) {
+      if constexpr (SP::kStatic) {  // JIT: the value columns and their widths are compile-time
+        sfor<0, SP::NV>([&](auto cc) {
+          constexpr int c = decltype(cc)::v;
           const uint64_t x = sval[(size_t)c * TILE + e];
-          if (L.val_dtype[c] == BLU_I32) ((int32_t*)sp.out_val[c])[idx] = (int32_t)(uint32_t)x;
+          if constexpr (SP::VDT[c] == BLU_I32) ((int32_t*)sp.out_val[c])[idx] = (int32_t)(uint32_t)x;
           else ((uint64_t*)sp.out_val[c])[idx] = x;
-        }
+        });
+      } else {
+#pragma unroll
+        for (int c = 0; c < NV; ++c)
+          if (c < L.n_vals) {
+            const uint64_t x = sval[(size_t)c * TILE + e];
+            if (L.val_dtype[c] == BLU_I32) ((int32_t*)sp.out_val[c])[idx] = (int32_t)(uint32_t)x;
+            else ((uint64_t*)sp.out_val[c])[idx] = x;
+          }
+      }
     }
     __syncthreads();
   }
