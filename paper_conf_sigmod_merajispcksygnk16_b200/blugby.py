@@ -298,15 +298,34 @@ class Result:
         self.n_groups = int(rc.n_groups)
         self.is_partial = bool(rc.is_partial)
         self.is_host = bool(rc.is_host)
-        n = self.n_groups
-        cols = rc.state_cols if self.is_partial else rc.agg_cols
-        n_out = rc.n_states if self.is_partial else rc.n_aggs
-        self.keys = [self._wrap(rc.key_cols[k], n, key_dtypes[k], device) for k in range(rc.n_keys)]
-        vals = [self._wrap(cols[o], n, out_dtypes[o], device) for o in range(n_out)]
-        if self.is_partial:
-            self.states, self.aggs = vals, None
-        else:
-            self.aggs, self.states = vals, None
+        self._spec = (key_dtypes, out_dtypes, device)
+        self._cols = None  # the column views are built on first access (a caller that only needs
+                           # n_groups pays no view construction)
+
+    def _views(self):
+        if self._cols is None:
+            key_dtypes, out_dtypes, device = self._spec
+            rc, n = self._owner.rc, self.n_groups
+            if rc is None:
+                raise BluError(BLU_E_INVALID, "result already freed")
+            cols = rc.state_cols if self.is_partial else rc.agg_cols
+            n_out = rc.n_states if self.is_partial else rc.n_aggs
+            keys = [self._wrap(rc.key_cols[k], n, key_dtypes[k], device) for k in range(rc.n_keys)]
+            vals = [self._wrap(cols[o], n, out_dtypes[o], device) for o in range(n_out)]
+            self._cols = (keys, vals)
+        return self._cols
+
+    @property
+    def keys(self):
+        return self._views()[0]
+
+    @property
+    def aggs(self):
+        return None if self.is_partial else self._views()[1]
+
+    @property
+    def states(self):
+        return self._views()[1] if self.is_partial else None
 
     def _wrap(self, ptr, n, dt, device):
         if self.is_host:

@@ -337,6 +337,10 @@ static cudaError_t d2h_staged(const std::vector<std::pair<void*, const void*>>& 
 static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int path, bool front, uint64_t cap0,
                              uint64_t total_rows, const Feeder& feed, bool partial, cudaStream_t st,
                              blu_gby_result_t* out, bool host_out, float* h2d_ms_acc, bool fuse_req = false) {
+  static const bool hprof = getenv("BLU_GBY_DEBUG_HOST") != nullptr;  // host-time breakdown per execute
+  auto hnow = [] { return std::chrono::steady_clock::now(); };
+  const auto h_entry = hnow();
+  std::chrono::steady_clock::time_point h_init{}, h_feed{}, h_alloc{}, h_compact{}, h_sync{};
   setup_pool();
   memset(out, 0, sizeof *out);
   const bool dense = path != BLU_PATH_HASH_GLOBAL;
@@ -372,6 +376,7 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       CK(launch_init_slots(lay, table, cap, st, (uint64_t*)small, 8), "init slots");  // + flags
     }
     if (t_timing) cudaEventRecord(t_ev.e[1], st);
+    if (hprof) h_init = hnow();
 
     AggParams base{};
     base.lay = lay;
@@ -395,7 +400,6 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     // they are allocated after the aggregation launch, so this host work overlaps the kernel.
     auto alloc_outputs = [&]() -> cudaError_t {
       cudaError_t ae = cudaSuccess;
-      auto t_oa = std::chrono::steady_clock::now();
       for (int k = 0; k < lay.n_keys && ae == cudaSuccess; ++k) {
         ae = U ? cudaMallocAsync(&okeys[k], U * dtype_bytes(lay.key_dtype[k]), st) : cudaSuccess;
         if (okeys[k]) own->dev.push_back(okeys[k]);
@@ -404,10 +408,6 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
         ae = U ? cudaMallocAsync(&ovals[o], U * dtype_bytes(os.out_dtype[o]), st) : cudaSuccess;
         if (ovals[o]) own->dev.push_back(ovals[o]);
       }
-      if (getenv("BLU_GBY_DEBUG_HOST"))
-        fprintf(stderr, "[blugby host] output alloc %.3f ms (%llu rows)\n",
-                std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_oa).count(),
-                (unsigned long long)U);
       if (ae != cudaSuccess) cudaGetLastError();
       return ae;
     };
@@ -443,6 +443,7 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       }
     }
     if (t_timing) cudaEventRecord(t_ev.e[2], st);
+    if (hprof) h_feed = hnow();
     if (!fuse) {
       cudaError_t ae = alloc_outputs();
       if (ae != cudaSuccess) {
@@ -451,6 +452,7 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       }
     }
 
+    if (hprof) h_alloc = hnow();
     if (U && !fuse) {
       CompactParams cp{};
       cp.lay = lay;
@@ -478,17 +480,13 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       }
     }
     if (t_timing) cudaEventRecord(t_ev.e[3], st);
+    if (hprof) h_compact = hnow();
     uint64_t* hs = pinned_scratch();
     uint64_t hbuf[2] = {0, 0};
     uint64_t* dst = hs ? hs : hbuf;
-    static const bool hdbg = getenv("BLU_GBY_DEBUG_HOST") != nullptr;
-    auto t_sync0 = std::chrono::steady_clock::now();
     cudaError_t ce = cudaMemcpyAsync(dst, small, 16, cudaMemcpyDeviceToHost, st);
     if (ce == cudaSuccess) ce = cudaStreamSynchronize(st);
     if (ce == cudaSuccess) w.drained();
-    if (hdbg)
-      fprintf(stderr, "[blugby host] final sync waited %.3f ms\n",
-              std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_sync0).count());
     if (ce != cudaSuccess) {
       cudaGetLastError();
       free_owner();
@@ -496,6 +494,14 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     }
     uint32_t flags = (uint32_t)dst[0];
     uint64_t ng = dst[1];
+    if (hprof) {
+      h_sync = hnow();
+      auto us = [](std::chrono::steady_clock::time_point a, std::chrono::steady_clock::time_point b) {
+        return std::chrono::duration<double, std::micro>(b - a).count();
+      };
+      fprintf(stderr, "[blugby host] us: init %.1f | feed %.1f | out-alloc %.1f | compact %.1f | sync-wait %.1f\n",
+              us(h_entry, h_init), us(h_init, h_feed), us(h_feed, h_alloc), us(h_alloc, h_compact), us(h_compact, h_sync));
+    }
     if (t_timing) {
       float a = 0, b = 0, c = 0;
       cudaEventElapsedTime(&a, t_ev.e[0], t_ev.e[1]);
