@@ -1038,6 +1038,61 @@ __device__ __forceinline__ void front_dedupe_rows(const AggParams& p, uint8_t* s
   __syncwarp();
 }
 
+// Rank front with warp-level combining (SP::DEDUPE, JIT only): for each of the lane's R rows, lanes
+// whose rows hit the same front entry (__match_any_sync on the entry) combine every field's value
+// onto the lowest such lane with a successor-doubling shuffle tree, and only that lane updates the
+// shared table (COUNT adds the group size). Under Zipf skew the second, third, ... hottest keys
+// repeat inside a warp; each repeat is a same-address lane in every shared atomic of the row.
+template <class SP, int NV, int R>
+__device__ __forceinline__ void rank_dedupe_apply(const AggParams& p, uint8_t* sm, const uint32_t (&fe)[R],
+                                                  uint32_t hit, const uint64_t (&v)[NV][R]) {
+  const unsigned lane = threadIdx.x & 31;
+#ifndef BLU_SOFF_PARAM
+  constexpr uint32_t ST = SP::STAB;
+#else
+  const uint32_t ST = p.S;
+#endif
+#pragma unroll
+  for (int r = 0; r < R; ++r) {
+    const bool hr = hit >> r & 1;
+    const uint32_t peers = __match_any_sync(0xffffffffu, hr ? fe[r] : (0x80000000u | lane));
+    const uint32_t np = __popc(peers);
+    const uint32_t maxnp = __reduce_max_sync(0xffffffffu, hr ? np : 1u);
+    uint64_t xr[SP::NF];
+    sfor<0, SP::NF>([&](auto jc) {
+      constexpr int j = decltype(jc)::v;
+      constexpr int c = SP::COL[j];
+      xr[j] = c < 0 ? (uint64_t)np : v[c < 0 ? 0 : c][r];
+    });
+    if (maxnp > 1) {
+      const uint32_t rank = __popc(peers & ((1u << lane) - 1u));
+      const uint32_t above = lane == 31 ? 0u : (peers & (0xffffffffu << (lane + 1)));
+      int sk = above ? __ffs(above) - 1 : -1;  // next member of this lane's group
+      for (uint32_t k = 1; k < maxnp; k <<= 1) {
+        const int src = sk < 0 ? (int)lane : sk;
+        const bool take = sk >= 0 && (rank & (2 * k - 1)) == 0;
+        sfor<0, SP::NF>([&](auto jc) {
+          constexpr int j = decltype(jc)::v;
+          constexpr int c = SP::COL[j], K = SP::KIND[j];
+          if constexpr (c >= 0) {
+            const uint64_t y = __shfl_sync(0xffffffffu, xr[j], src);
+            if (take) xr[j] = combine_vals<K>(xr[j], y);
+          }
+        });
+        const int s2 = __shfl_sync(0xffffffffu, sk, src);
+        sk = sk < 0 ? -1 : s2;
+      }
+      if (rank != 0) continue;  // a non-leader's row is in its leader's combined values
+    }
+    if (!hr) continue;
+    sfor<0, SP::NF>([&](auto jc) {
+      constexpr int j = decltype(jc)::v;
+      constexpr int KK = SP::COL[j] < 0 ? FK_COUNT : SP::KIND[j];
+      s_upd<KK, true>(sm + SP::SOFF[j], fe[r], ST, xr[j]);
+    });
+  }
+}
+
 // Register accumulator of the rank front's hottest key (SP::HOTREG, JIT only): that key's rows are
 // combined per thread in registers (encoded like the shared table) and flushed once at the end, so
 // the key that most often collides with itself inside a warp costs no shared-memory atomics.
@@ -1161,7 +1216,14 @@ __device__ __forceinline__ void process_rows(const AggParams& p, uint8_t* sm, ui
       fe[r] = (uint32_t)(x >> 32) + __popc(bits & ((1u << b) - 1u));
       hit |= (bits >> b & 1u) << r;
     }
-    smem_apply_rows<SP, NV, R>(p, sm, fe, hit, v);
+    bool done = false;
+    if constexpr (SP::kStatic) {
+      if constexpr (SP::DEDUPE) {  // opt-in (BLU_GBY_DEDUPE=1): warp-level combining of equal entries
+        rank_dedupe_apply<SP, NV, R>(p, sm, fe, hit, v);
+        done = true;
+      }
+    }
+    if (!done) smem_apply_rows<SP, NV, R>(p, sm, fe, hit, v);
     miss = valid & ~hit;
   } else if (FRONT && !deduped) {
     // hot-key front: small open-addressing table per CTA in shared memory

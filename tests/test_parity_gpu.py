@@ -86,15 +86,17 @@ def test_forced_paths_identical(bg, oracles, monkeypatch, name, paths, front):
         assert_parity(gk, ga, o, w.schema)
 
 
-@pytest.mark.parametrize("rank", ["1", "1-hotreg", "0"])
+@pytest.mark.parametrize("rank", ["1", "1-hotreg", "0", "1-dedupe", "1-hotreg-dedupe"])
 @pytest.mark.parametrize("dicts,n", [((13, 7), 200_003), ((64, 1024), 1_048_583), ((100, 20, 20), 700_001)])
 def test_rank_front(bg, monkeypatch, rank, dicts, n):
     """Path (b') hot-key front as a rank image (bitmap + per-word prefix) vs the hash front: both equal
     the oracle. D = 91, D = 32 * S exactly (S = 2048 front entries for this schema), D = 4 * 10^4.
-    Skewed keys so the seeded front fills up; rows of cold keys take the global REDs. "1-hotreg": the
+    Skewed keys so the seeded front fills up; rows of cold keys take the global REDs. "hotreg": the
     sample's hottest key summed in per-thread registers (BLU_GBY_HOT_REG=1) for every field kind of
-    ALL(3) (i32/i64/f64 SUM, MIN, MAX, COUNT)."""
-    monkeypatch.setenv("BLU_GBY_HOT_REG", "1" if rank == "1-hotreg" else "0")
+    ALL(3) (i32/i64/f64 SUM, MIN, MAX, COUNT); "dedupe": lanes hitting the same front entry combined
+    with __match_any_sync + a shuffle tree before the shared-memory update (BLU_GBY_DEDUPE=1)."""
+    monkeypatch.setenv("BLU_GBY_HOT_REG", "1" if "hotreg" in rank else "0")
+    monkeypatch.setenv("BLU_GBY_DEDUPE", "1" if "dedupe" in rank else "0")
     rng = np.random.default_rng(sum(dicts) + n)
     D = int(np.prod(dicts))
     sch = blugen.Schema([(I32, d) for d in dicts], [I32, I64, F64], ALL(3))
