@@ -654,8 +654,23 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   // bucket capacity: the mean plus slack for the spread of the number of GROUPS per bucket (keys
   // hash uniformly: relative sd 1/sqrt(est/B); 6 sd) and of rows per group; heavier skew overflows a
   // bucket and takes the gated one-pass fallback
+  // TMA bulk write-out of the staged runs (every value column 8 bytes; BLU_GBY_SCATTER_TMA=0 turns it
+  // off): each (tile, bucket) run is padded to an even row count with an empty-key record the readers
+  // skip. C3 scatter 19.4 -> 18.2 ms, C5 22.1 -> 20.0 ms per chunk
+  bool tma = true;
+  {
+    const char* tm = getenv("BLU_GBY_SCATTER_TMA");
+    if (tm && tm[0] == '0') tma = false;
+    for (int c = 0; c < L.n_vals; ++c) tma = tma && dtype_bytes(L.val_dtype[c]) == 8;
+    // the padded staging must fit the scatter's shared memory at the widest histogram of this plan
+    const uint32_t bins = B1 ? std::max<uint32_t>(B1, B / B1) : B;
+    tma = tma && scatter_smem(L.n_vals, bins, true) <= 232448;
+  }
   const double gpb = std::max(1.0, (double)P->est_groups / (double)B);
-  const double slack = 1.03 + std::min(1.0, 6.0 / std::sqrt(gpb));
+  // padding: at most one row per (tile, bucket) run, i.e. a fraction ~ bins / (2 x tile rows) of a
+  // bucket's rows; reserve twice that (tiles hold >= 2048 rows)
+  const double pad = tma ? (double)(B1 ? B / B1 : B) / 2048.0 : 0.0;
+  const double slack = 1.03 + std::min(1.0, 6.0 / std::sqrt(gpb)) + pad;
   uint64_t seg_cap = ((uint64_t)((double)((M + B - 1) / B) * slack) + 4096 + 63) & ~63ull;
   uint64_t rows_alloc = seg_cap * B;
   void* kbuf = nullptr;
@@ -671,7 +686,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   uint64_t* d_cursor1 = nullptr;
   if (B1 && e == cudaSuccess) {
     const double gpb1 = std::max(1.0, (double)P->est_groups / (double)B1);
-    const double slack1 = 1.03 + std::min(1.0, 6.0 / std::sqrt(gpb1));
+    const double slack1 = 1.03 + std::min(1.0, 6.0 / std::sqrt(gpb1)) + (tma ? (double)B1 / 2048.0 : 0.0);  // as above
     // a multiple of the second-level scatter's tile (1024 threads x up to 4 rows): every tile of the
     // one-launch second level lies inside one first-level bucket
     seg_cap1 = ((uint64_t)((double)((M + B1 - 1) / B1) * slack1) + 4096 + 4095) & ~4095ull;
@@ -690,6 +705,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   L2.n_keys = 1;
   L2.sparse = 1;
   L2.key_dtype[0] = BLU_I64;
+  L2.pad_keys = 1;  // records: empty-key padding rows (TMA write-out) are skipped
   for (uint64_t r0 = 0; r0 < n; r0 += M) {
     const uint64_t m = std::min(M, n - r0);
     if ((e = cudaMemsetAsync(d_cursor, 0, (size_t)B * 8 + 16, st))) return e;
@@ -725,6 +741,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     sp.out_key = (uint64_t*)kbuf;
     for (int c = 0; c < L.n_vals; ++c) sp.out_val[c] = vbuf[c];
     sp.gate = d_gate;
+    sp.tma = tma ? 1u : 0u;
     static const bool dbg = getenv("BLU_GBY_DEBUG_PART") != nullptr;
     cudaEvent_t ev[4];
     if (dbg) {

@@ -405,6 +405,9 @@ __device__ __forceinline__ uint32_t pack_keys(const AggParams& p, uint64_t row, 
 #pragma unroll
       for (int r = 0; r < R; ++r) {
         key[r] = c[r];
+        if constexpr (SP::PADK) {
+          if (c[r] == kEmpty) valid &= ~(1u << r);  // padding record
+        }
         if ((int64_t)c[r] < 0) bad |= 1u << r;
       }
     } else {
@@ -427,6 +430,7 @@ __device__ __forceinline__ uint32_t pack_keys(const AggParams& p, uint64_t row, 
 #pragma unroll
     for (int r = 0; r < R; ++r) {
       key[r] = c[r];
+      if (p.lay.pad_keys && c[r] == kEmpty) valid &= ~(1u << r);  // padding record
       if ((int64_t)c[r] < 0) bad |= 1u << r;
     }
   } else {
@@ -741,6 +745,9 @@ __device__ __forceinline__ uint32_t tile_unpack(const AggParams& p, const RawTil
                                                : ((uint64_t)T.khi[k][r] << 32 | T.klo[k][r]);
       if constexpr (SP::SPARSE) {
         key[r] = c;
+        if constexpr (SP::PADK) {
+          if (c == kEmpty) valid &= ~(1u << r);  // padding record
+        }
         if ((int64_t)c < 0) bad |= 1u << r;
 #ifndef BLU_PACK64
       } else if constexpr (SP::DOMAIN <= 0xFFFFFFFFull && SP::KDT[k] == BLU_I32 && SP::DICT[k] <= 0x80000000ull) {
@@ -1791,7 +1798,7 @@ constexpr uint32_t kMaxInSeg = 64;  // first-level buckets of a two-level scatte
 
 // PIPE (NVRTC kernels only): the next tile's rows are loaded into registers as soon as the current
 // tile is staged in shared memory, so those HBM reads are in flight during its write-out phase.
-template <class SP, int NV, int R, bool PIPE = false, bool SEGIN = false>
+template <class SP, int NV, int R, bool PIPE = false, bool SEGIN = false, bool TMAS = false>
 __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterParams& sp) {
   extern __shared__ __align__(16) uint8_t sm[];
   const Layout& L = p.lay;
@@ -1799,14 +1806,17 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
   // bucket, global index bbase + local bin)
   const uint32_t B = SEGIN ? sp.in_B2 : sp.B;
   const uint32_t TILE = blockDim.x * R;
-  uint64_t* skey = (uint64_t*)sm;                       // TILE
-  uint64_t* sval = skey + TILE;                         // NV x TILE
-  uint64_t* gpos = sval + (size_t)NV * TILE;            // B
+  // staging stride: TMAS pads every bucket's run to an even length, up to B rows more than the tile
+  const uint32_t TS = TMAS ? TILE + ((B + 1u) & ~1u) : TILE;
+  uint64_t* skey = (uint64_t*)sm;                       // TS
+  uint64_t* sval = skey + TS;                           // NV x TS
+  uint64_t* gpos = sval + (size_t)NV * TS;              // B
   uint32_t* hist = (uint32_t*)(gpos + B);               // B
   uint32_t* lstart = hist + B;                          // B
   uint32_t* wtot = lstart + B;                          // 32
   uint32_t* total = wtot + 32;                          // 1
   uint16_t* sbid = (uint16_t*)(total + 4);              // TILE
+  uint32_t* hcnt = (uint32_t*)(sbid + TILE);            // B (TMAS: rows per bucket before padding)
   const uint64_t pol = evict_first_policy();
   const uint64_t n = p.n_rows;
   const uint64_t ntiles = (n + TILE - 1) / TILE;
@@ -1863,6 +1873,14 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
       pos[r] = (valid >> r & 1) ? atomicAdd(&hist[bb[r]], 1u) : 0u;
     }
     __syncthreads();
+    if constexpr (TMAS) {  // bulk copies move whole 16-byte units: runs padded to an even row count
+      for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
+        const uint32_t h = hist[b];
+        hcnt[b] = h;
+        hist[b] = (h + 1u) & ~1u;
+      }
+      __syncthreads();
+    }
     block_excl_scan(hist, lstart, B, wtot, total);
     for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
       uint32_t h = hist[b];
@@ -1870,6 +1888,9 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
         uint64_t g = atomicAdd((unsigned long long*)&sp.cursor[bbase + b], (unsigned long long)h);
         gpos[b] = g;
         if (g + h > sp.seg_cap) atomicExch(sp.gate, 1u);
+        if constexpr (TMAS) {
+          if (hcnt[b] & 1u) skey[lstart[b] + hcnt[b]] = kEmpty;  // the padding record
+        }
       }
     }
     __syncthreads();  // lstart and gpos visible to every thread
@@ -1880,11 +1901,32 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
         skey[e] = key[r];
         sbid[e] = (uint16_t)bb[r];
 #pragma unroll
-        for (int c = 0; c < NV; ++c) sval[(size_t)c * TILE + e] = v[c][r];
+        for (int c = 0; c < NV; ++c) sval[(size_t)c * TS + e] = v[c][r];
       }
     if constexpr (PIPE) {  // this tile is in shared memory: the next one's loads go out now
       const uint64_t tn = t + gridDim.x;
       if (tn < ntiles) tile_load<SP, R>(p, lane_base<R>(tn * TILE, threadIdx.x >> 5, threadIdx.x & 31), tile_lim(tn), pol, T);
+    }
+    if constexpr (TMAS) {
+      // every bucket's run of every column leaves shared memory in one bulk copy (TMA engine; no
+      // per-element loads and stores): thread t copies column t / B of bucket t % B
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // staged writes -> async proxy
+      __syncthreads();
+      for (uint32_t t2 = threadIdx.x; t2 < B * (1u + (uint32_t)NV); t2 += blockDim.x) {
+        const uint32_t col = t2 / B, b = t2 - col * B;
+        const uint32_t hp = hist[b];
+        if (!hp || (col > 0 && (int)col > L.n_vals) || gpos[b] + hp > sp.seg_cap) continue;
+        const uint64_t row = (uint64_t)(bbase + b) * sp.seg_stride + gpos[b];
+        const uint64_t* src = (col == 0 ? skey : sval + (size_t)(col - 1) * TS) + lstart[b];
+        uint64_t* dst = (col == 0 ? sp.out_key : (uint64_t*)sp.out_val[col - 1]) + row;
+        asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst),
+                     "r"((uint32_t)__cvta_generic_to_shared(src)), "r"(hp * 8u)
+                     : "memory");
+      }
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // sources read: staging reusable
+      __syncthreads();
+      continue;
     }
     __syncthreads();
     const uint32_t tot = *total;
@@ -1897,7 +1939,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
       if constexpr (SP::kStatic) {  // JIT: the value columns and their widths are compile-time
         sfor<0, SP::NV>([&](auto cc) {
           constexpr int c = decltype(cc)::v;
-          const uint64_t x = sval[(size_t)c * TILE + e];
+          const uint64_t x = sval[(size_t)c * TS + e];
           if constexpr (SP::VDT[c] == BLU_I32) ((int32_t*)sp.out_val[c])[idx] = (int32_t)(uint32_t)x;
           else ((uint64_t*)sp.out_val[c])[idx] = x;
         });
@@ -1905,7 +1947,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
 #pragma unroll
         for (int c = 0; c < NV; ++c)
           if (c < L.n_vals) {
-            const uint64_t x = sval[(size_t)c * TILE + e];
+            const uint64_t x = sval[(size_t)c * TS + e];
             if (L.val_dtype[c] == BLU_I32) ((int32_t*)sp.out_val[c])[idx] = (int32_t)(uint32_t)x;
             else ((uint64_t*)sp.out_val[c])[idx] = x;
           }
@@ -1913,6 +1955,8 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
     }
     __syncthreads();
   }
+  if constexpr (TMAS) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // bulk writes complete
 }
+
 
 }  // namespace blu

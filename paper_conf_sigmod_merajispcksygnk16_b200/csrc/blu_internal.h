@@ -73,7 +73,7 @@ uint64_t launches_total();
 int launch_scatter(const AggParams& p, const ScatterParams& s, void* stream, uint32_t grid);
 uint32_t scatter_block(uint32_t B);
 uint32_t scatter_grid(uint32_t sms, uint32_t B);
-size_t scatter_smem(int nv, uint32_t B);
+size_t scatter_smem(int nv, uint32_t B, bool tma = false);
 int launch_bucket(const AggParams& p, void* stream, uint32_t grid, uint32_t smem);
 // bucket table sizing: bytes of an S-entry table (keys + SoA fields) and the kernel's total smem
 uint32_t bucket_table_bytes(const Layout& L, uint32_t S);

@@ -77,6 +77,9 @@ struct Layout {
   int32_t key_words;
   int32_t kword[kMaxKeys];
   int32_t has_q;  // 1: some value column is i128 / some field is 128-bit (generic k_agg_q kernel)
+  // partition records (pass 2 / second scatter level): a sparse key equal to the empty mark is a
+  // padding record written to keep bulk-copied runs 16-byte aligned; it is skipped, not an error
+  int32_t pad_keys;
 };
 
 // ---------------------------------------------------------------------------------------------
@@ -171,6 +174,9 @@ struct ScatterParams {
   uint64_t in_seg;
   const uint64_t* in_count;
   uint32_t in_B2;
+  // 1: bucket runs leave shared memory by TMA bulk copies (cp.async.bulk), padded to an even number of
+  // rows with empty-key records (all value columns 8 bytes; JIT kernels)
+  uint32_t tma;
 };
 
 enum : uint32_t { FLAG_OVERFLOW = 1u, FLAG_KEY_RANGE = 2u };

@@ -118,6 +118,7 @@ std::string spec_source(const char* name, const Layout& L, uint32_t S, const uin
   s += " {\n  static constexpr bool kStatic = true;\n";
   s += "  static constexpr int NK = " + std::to_string(L.n_keys) + ";\n";
   s += "  static constexpr int SPARSE = " + std::to_string(L.sparse) + ";\n";
+  s += "  static constexpr int PADK = " + std::to_string(L.pad_keys) + ";\n";
   s += "  static constexpr int KDT[8] = " + arr(kdt, L.n_keys, 8) + ";\n";
   s += "  static constexpr unsigned long long DICT[8] = " + arru(L.dict, L.n_keys, 8) + ";\n";
   s += "  static constexpr unsigned long long STRIDE[8] = " + arru(L.stride, L.n_keys, 8) + ";\n";

@@ -175,27 +175,29 @@ __global__ void __launch_bounds__(1024, 1) k_scatter_wide(AggParams p, ScatterPa
 uint32_t scatter_block(uint32_t B) { return B > 512 ? 1024u : 512u; }
 uint32_t scatter_grid(uint32_t sms, uint32_t B) { return B > 512 ? sms : 2 * sms; }  // resident CTAs
 
-size_t scatter_smem(int nv, uint32_t B) {
+size_t scatter_smem(int nv, uint32_t B, bool tma) {
   const int R = rows_per_thread(nv);
   const size_t NV = nv <= 1 ? 1 : nv <= 2 ? 2 : nv <= 4 ? 4 : nv <= 8 ? 8 : 16;
   const size_t TILE = (size_t)scatter_block(B) * R;
-  return TILE * 8 * (1 + NV) + (size_t)B * 16 + 36 * 4 + 16 + TILE * 2;
+  // the TMA write-out pads every bucket's run to an even length: staging rows TILE + B
+  const size_t TS = tma ? TILE + ((B + 1) & ~1u) : TILE;
+  return TS * 8 * (1 + NV) + (size_t)B * 16 + 36 * 4 + 16 + TILE * 2 + (size_t)B * 4;
 }
 
 template <int NV, int R>
 static int launch_scatter_nv(const AggParams& p, const ScatterParams& sp, cudaStream_t st, uint32_t grid) {
   const uint32_t bins = sp.in_seg ? sp.in_B2 : sp.B;  // histogram bins of one tile
   const uint32_t block = scatter_block(bins);
-  const size_t smem = scatter_smem(p.lay.n_vals, bins);
+  const size_t smem = scatter_smem(p.lay.n_vals, bins, sp.tma != 0);
   if (p.jit_ok && jit_env("BLU_GBY_JIT_SCATTER", 1)) {
     char body[160], decl[160], name[64];
     // register-pipelined tile loads instead of the L2 prefetch (C3 scatter 10.07 -> 9.48 ms)
     const int pipe = jit_env("BLU_GBY_SCATTER_PIPE", 1);
-    const bool seg = sp.in_seg != 0;
-    snprintf(name, sizeof name, "blu_jit_scatter_%d_%d%s%s", NV, R, pipe ? "_p" : "", seg ? "_s" : "");
+    const bool seg = sp.in_seg != 0, tma = sp.tma != 0;
+    snprintf(name, sizeof name, "blu_jit_scatter_%d_%d%s%s%s", NV, R, pipe ? "_p" : "", seg ? "_s" : "", tma ? "_t" : "");
     snprintf(decl, sizeof decl, "%s(blu::AggParams p, blu::ScatterParams sp)", name);
-    snprintf(body, sizeof body, "blu::scatter_body<blu::JitSpec, %d, %d, %s, %s>(p, sp);", NV, R, pipe ? "true" : "false",
-             seg ? "true" : "false");
+    snprintf(body, sizeof body, "blu::scatter_body<blu::JitSpec, %d, %d, %s, %s, %s>(p, sp);", NV, R,
+             pipe ? "true" : "false", seg ? "true" : "false", tma ? "true" : "false");
     AggParams pc = p;
     ScatterParams sc = sp;
     void* args[] = {&pc, &sc};

@@ -459,6 +459,33 @@ def test_partitioned_two_pass(bg, oracles, monkeypatch, parts, chunk, div, smem)
     assert_parity(gk, ga, o, w.schema)
 
 
+@pytest.mark.parametrize("tma", ["1", "0"])
+@pytest.mark.parametrize("shape", [("C3", 3_000_017, 200_000, None), ("C3", 2_000_003, 30_000, "1"),
+                                   ("C5", 4_000_037, 400_000, None)])
+def test_scatter_tma_write_out(bg, monkeypatch, tma, shape):
+    """Partitioned path (b) with the scatter's staged bucket runs leaving shared memory by TMA bulk
+    copies (cp.async.bulk, runs padded to even lengths with empty-key records that pass 2 and the second
+    scatter level skip) and with the per-element write-out: both equal the oracle, one level (L2-slice
+    pass 2) and two levels (shared-memory bucket tables)."""
+    name, n, G, smem = shape
+    w = blugen.workload(name, n_rows=n, n_groups=G)
+    o = oracle.groupby_generated(w)
+    kc, vc = blugen.device_columns(w)
+    monkeypatch.setenv("BLU_GBY_SCATTER_TMA", tma)
+    monkeypatch.setenv("BLU_GBY_PARTS", "256" if smem else "64")
+    if smem:
+        monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    assert plan.info()["partitions"] > 1
+    bg.blu_gby_set_timing(True)
+    res = bg.blu_gby_execute(plan, kc, vc)
+    t = bg.blu_gby_last_timing()
+    bg.blu_gby_set_timing(False)
+    assert t["part_chunks"] >= 1 and t["part_fallbacks"] == 0, t
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
 @pytest.mark.parametrize("two_level", ["0", "1", "1-one"])
 @pytest.mark.parametrize("parts", [None, "4096"])
 def test_partitioned_wide_fanout(bg, monkeypatch, parts, two_level):
