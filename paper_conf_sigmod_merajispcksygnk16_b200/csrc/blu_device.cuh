@@ -1811,8 +1811,8 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
   uint64_t* skey = (uint64_t*)sm;                       // TS
   uint64_t* sval = skey + TS;                           // NV x TS
   uint64_t* gpos = sval + (size_t)NV * TS;              // B
-  uint32_t* hist = (uint32_t*)(gpos + B);               // B
-  uint32_t* lstart = hist + B;                          // B
+  uint32_t* histbuf = (uint32_t*)(gpos + B);            // 2 x B: tiles alternate (zeroed one tile ahead)
+  uint32_t* lstart = histbuf + 2 * B;                   // B
   uint32_t* wtot = lstart + B;                          // 32
   uint32_t* total = wtot + 32;                          // 1
   uint16_t* sbid = (uint16_t*)(total + 4);              // TILE
@@ -1835,6 +1835,9 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
     if constexpr (SEGIN) return seg_end[(t * TILE) / sp.in_seg];
     return n;
   };
+  for (uint32_t b = threadIdx.x; b < 2 * B; b += blockDim.x) histbuf[b] = 0;
+  __syncthreads();
+  uint32_t kt = 0;  // tiles processed by this CTA (selects the histogram buffer)
   using Raw = RawTileFor<SP, R, PIPE>;
   Raw T;
   if constexpr (PIPE)
@@ -1849,8 +1852,12 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
       }
       continue;
     }
-    for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
-    __syncthreads();
+    // No barrier at the top of a tile: the previous tile's readers of the staging, lstart and gpos are
+    // ordered before this tile's writers by the barrier after the rank atomics below, and this tile's
+    // histogram buffer was zeroed during the previous tile.
+    uint32_t* hist = histbuf + (kt & 1u) * B;
+    uint32_t* hnext = histbuf + ((kt + 1u) & 1u) * B;
+    ++kt;
     const uint64_t row = lane_base<R>(t * TILE, threadIdx.x >> 5, threadIdx.x & 31);
     const uint32_t bbase = SEGIN ? (uint32_t)((t * TILE) / sp.in_seg) * sp.in_B2 : 0u;
     uint64_t key[R];
@@ -1883,6 +1890,7 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
     }
     block_excl_scan(hist, lstart, B, wtot, total);
     for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
+      hnext[b] = 0;  // every thread is past the previous tile (its last reader of this buffer)
       uint32_t h = hist[b];
       if (h) {
         uint64_t g = atomicAdd((unsigned long long*)&sp.cursor[bbase + b], (unsigned long long)h);
@@ -1925,7 +1933,6 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
       }
       asm volatile("cp.async.bulk.commit_group;" ::: "memory");
       asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // sources read: staging reusable
-      __syncthreads();
       continue;
     }
     __syncthreads();
@@ -1953,7 +1960,6 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
           }
       }
     }
-    __syncthreads();
   }
   if constexpr (TMAS) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // bulk writes complete
 }

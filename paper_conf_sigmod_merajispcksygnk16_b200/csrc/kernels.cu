@@ -181,7 +181,7 @@ size_t scatter_smem(int nv, uint32_t B, bool tma) {
   const size_t TILE = (size_t)scatter_block(B) * R;
   // the TMA write-out pads every bucket's run to an even length: staging rows TILE + B
   const size_t TS = tma ? TILE + ((B + 1) & ~1u) : TILE;
-  return TS * 8 * (1 + NV) + (size_t)B * 16 + 36 * 4 + 16 + TILE * 2 + (size_t)B * 4;
+  return TS * 8 * (1 + NV) + (size_t)B * 20 + 36 * 4 + 16 + TILE * 2 + (size_t)B * 4;  // hist x 2
 }
 
 template <int NV, int R>
