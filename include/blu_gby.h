@@ -27,8 +27,9 @@
  *     device; "host" pointers are ordinary host memory (pinned memory is faster).
  *   - Input columns are BORROWED: they must stay valid and unchanged until the call returns
  *     (execute* synchronize `stream` before returning).
- *   - Results are LIBRARY-OWNED (device memory from cudaMallocAsync on `stream`, or host memory
- *     for blu_gby_execute_host); release them with blu_gby_result_free.
+ *   - Results are LIBRARY-OWNED (device memory from cudaMallocAsync on `stream`, or pinned host
+ *     memory for blu_gby_execute_host, taken from a per-process cache of pinned blocks that
+ *     blu_gby_result_free returns them to); release them with blu_gby_result_free.
  *   - stream is a cudaStream_t passed as void* (0 = legacy default stream).
  *   - Plans are immutable and may be shared by threads; concurrent executes on different streams
  *     are safe.
@@ -298,9 +299,10 @@ blu_status_t blu_gby_read_roofline(const void* const* cols, const uint64_t* byte
 blu_status_t blu_gby_bind_device(int32_t device);
 
 /* Workspace (hash tables, dense state, partition buffers) is kept in a per-process cache of device
- * blocks reused by later calls (the "single large memory segment" of P:62). This frees the idle
- * blocks of the current device back to CUDA (after a device synchronisation); blocks in use by a
- * call on another thread stay. Returns the bytes freed in *freed (may be NULL). */
+ * blocks reused by later calls (the "single large memory segment" of P:62), and host results in a
+ * cache of pinned host blocks. This frees the idle blocks of the current device and the idle pinned
+ * host blocks back to CUDA (after a device synchronisation); blocks in use (a live result, a call on
+ * another thread) stay. Returns the bytes freed in *freed (may be NULL). */
 blu_status_t blu_gby_release_workspace(uint64_t* freed);
 
 void blu_gby_result_free(blu_gby_result_t* r, void* stream);

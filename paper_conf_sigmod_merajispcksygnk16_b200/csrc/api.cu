@@ -107,8 +107,51 @@ static blu_status_t cuda_fail(cudaError_t e, const char* what) {
 // Owner record behind blu_gby_result_t::_owner.
 struct Owner {
   std::vector<void*> dev;
-  std::vector<void*> host;
+  std::vector<void*> host;  // pinned blocks of the host-result cache (released with host_put)
 };
+
+// Pinned host blocks for host results (blu_gby_execute_host), kept and reused across queries — the
+// paper's "single large memory segment" pinned once and reused: results are copied at the
+// pinned D2H rate with no page-locking, page faults or bounce copy per query. A block returns to the
+// cache when its result is freed.
+struct HostBlock {
+  void* p;
+  size_t bytes;
+  bool busy;
+};
+static std::mutex g_hcache_mu;
+static std::vector<HostBlock> g_hcache;
+
+static void* host_get(size_t bytes) {
+  bytes = std::max<size_t>((bytes + 4095) & ~(size_t)4095, 4096);
+  {
+    std::lock_guard<std::mutex> lk(g_hcache_mu);
+    int best = -1;
+    for (int i = 0; i < (int)g_hcache.size(); ++i) {
+      const HostBlock& b = g_hcache[i];
+      if (b.busy || b.bytes < bytes || b.bytes > 2 * bytes + (16u << 20)) continue;
+      if (best < 0 || b.bytes < g_hcache[best].bytes) best = i;
+    }
+    if (best >= 0) {
+      g_hcache[best].busy = true;
+      return g_hcache[best].p;
+    }
+  }
+  void* p = nullptr;
+  if (cudaMallocHost(&p, bytes) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  std::lock_guard<std::mutex> lk(g_hcache_mu);
+  g_hcache.push_back(HostBlock{p, bytes, true});
+  return p;
+}
+
+static void host_put(void* p) {
+  std::lock_guard<std::mutex> lk(g_hcache_mu);
+  for (auto& b : g_hcache)
+    if (b.p == p) b.busy = false;
+}
 
 static size_t dtype_bytes(int dt) { return dt == BLU_I32 ? 4 : dt == BLU_I128 ? 16 : 8; }
 
@@ -280,57 +323,6 @@ static cudaError_t agg_batch(const blu_gby_plan_s* P, int path, AggParams p, con
     if (launches) ++*launches;
   }
   return cudaSuccess;
-}
-
-// Device -> pageable host copies through two pinned bounce buffers (allocated once per thread): the
-// copy engine writes pinned memory at the PCIe rate while the host copies the previous chunk out.
-static cudaError_t d2h_staged(const std::vector<std::pair<void*, const void*>>& cols, const std::vector<size_t>& sizes,
-                              cudaStream_t st) {
-  constexpr size_t kChunk = 32u << 20;
-  static thread_local uint8_t* pin[2] = {nullptr, nullptr};
-  static thread_local cudaEvent_t done[2] = {nullptr, nullptr};
-  size_t total = 0;
-  for (size_t b : sizes) total += b;
-  if (total <= kChunk / 8 || (!pin[0] && (cudaMallocHost((void**)&pin[0], kChunk) != cudaSuccess ||
-                                          cudaMallocHost((void**)&pin[1], kChunk) != cudaSuccess))) {
-    cudaGetLastError();
-    for (size_t i = 0; i < cols.size(); ++i)  // small result (or no pinned memory): direct copies
-      if (sizes[i]) {
-        cudaError_t e = cudaMemcpyAsync(cols[i].first, cols[i].second, sizes[i], cudaMemcpyDeviceToHost, st);
-        if (e) return e;
-      }
-    return cudaSuccess;
-  }
-  if (!done[0]) {
-    cudaEventCreateWithFlags(&done[0], cudaEventDisableTiming);
-    cudaEventCreateWithFlags(&done[1], cudaEventDisableTiming);
-  }
-  struct Pending {
-    uint8_t* dst = nullptr;
-    size_t n = 0;
-  } pend[2];
-  int slot = 0;
-  auto drain = [&](int b) -> cudaError_t {
-    if (!pend[b].n) return cudaSuccess;
-    cudaError_t e = cudaEventSynchronize(done[b]);
-    if (e) return e;
-    memcpy(pend[b].dst, pin[b], pend[b].n);
-    pend[b].n = 0;
-    return cudaSuccess;
-  };
-  for (size_t i = 0; i < cols.size(); ++i)
-    for (size_t off = 0; off < sizes[i]; off += kChunk) {
-      const size_t n = std::min(kChunk, sizes[i] - off);
-      cudaError_t e = drain(slot);  // this bounce buffer's previous chunk
-      if (!e) e = cudaMemcpyAsync(pin[slot], (const uint8_t*)cols[i].second + off, n, cudaMemcpyDeviceToHost, st);
-      if (!e) e = cudaEventRecord(done[slot], st);
-      if (e) return e;
-      pend[slot] = Pending{(uint8_t*)cols[i].first + off, n};
-      slot ^= 1;
-    }
-  cudaError_t e = drain(slot);
-  if (!e) e = drain(slot ^ 1);
-  return e;
 }
 
 // The core: init -> feed -> compact -> one sync -> regrow on overflow.
@@ -547,30 +539,24 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
       // copy to host (pageable memory owned by the result) through two pinned bounce buffers, so the
       // D2H runs at the pinned rate and overlaps the host-side copies; release the device outputs
       Owner* hown = new Owner();
-      std::vector<std::pair<void*, const void*>> cols;
-      std::vector<size_t> sizes;
-      for (int k = 0; k < lay.n_keys; ++k) {
-        size_t b = ng * dtype_bytes(lay.key_dtype[k]);
-        void* h = malloc(std::max<size_t>(b, 1));
+      cudaError_t se = cudaSuccess;
+      auto take = [&](const void* dsrc, size_t b) -> void* {
+        void* h = host_get(b);
+        if (!h) {
+          se = cudaErrorMemoryAllocation;
+          return nullptr;
+        }
         hown->host.push_back(h);
-        kc[k] = h;
-        cols.push_back({h, okeys[k]});
-        sizes.push_back(b);
-      }
-      for (int o = 0; o < os.n_out; ++o) {
-        size_t b = ng * dtype_bytes(os.out_dtype[o]);
-        void* h = malloc(std::max<size_t>(b, 1));
-        hown->host.push_back(h);
-        vc[o] = h;
-        cols.push_back({h, ovals[o]});
-        sizes.push_back(b);
-      }
-      cudaError_t se = d2h_staged(cols, sizes, st);
+        if (b && se == cudaSuccess) se = cudaMemcpyAsync(h, dsrc, b, cudaMemcpyDeviceToHost, st);
+        return h;
+      };
+      for (int k = 0; k < lay.n_keys; ++k) kc[k] = take(okeys[k], ng * dtype_bytes(lay.key_dtype[k]));
+      for (int o = 0; o < os.n_out; ++o) vc[o] = take(ovals[o], ng * dtype_bytes(os.out_dtype[o]));
       if (se == cudaSuccess) se = cudaStreamSynchronize(st);
       free_owner();
       own = hown;
       if (se != cudaSuccess) {
-        for (void* h : hown->host) free(h);
+        for (void* h : hown->host) host_put(h);
         delete hown;
         free(kc);
         free(vc);
@@ -981,6 +967,18 @@ blu_status_t blu_gby_release_workspace(uint64_t* freed) {
       }
     }
   }
+  {  // idle pinned host-result blocks too
+    std::lock_guard<std::mutex> lk(g_hcache_mu);
+    for (auto it = g_hcache.begin(); it != g_hcache.end();) {
+      if (!it->busy) {
+        t += it->bytes;
+        cudaFreeHost(it->p);
+        it = g_hcache.erase(it);
+      } else {
+        ++it;
+      }
+    }
+  }
   if (freed) *freed = t;
   return BLU_OK;
 }
@@ -1354,7 +1352,7 @@ void blu_gby_result_free(blu_gby_result_t* r, void* stream) {
   Owner* o = (Owner*)r->_owner;
   if (o) {
     for (void* p : o->dev) cudaFreeAsync(p, (cudaStream_t)stream);
-    for (void* h : o->host) free(h);
+    for (void* h : o->host) host_put(h);
     delete o;
   }
   free(r->key_cols);
