@@ -881,7 +881,8 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
 
 // Schema column pointers -> kernel columns (the layout's value columns are the schema's).
 static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* keys, const void* const* vals,
-                                   uint64_t n, cudaStream_t st, bool partial, blu_gby_result_t* out) {
+                                   uint64_t n, cudaStream_t st, bool partial, blu_gby_result_t* out,
+                                   bool host_out = false) {
   if (!P || !out) return fail(BLU_E_INVALID, "NULL plan or out");
   if (n && (!nonnull_cols(keys, P->lay.n_keys) || !nonnull_cols(vals, P->lay.n_vals)))
     return fail(BLU_E_INVALID, "NULL column pointer");
@@ -926,7 +927,7 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
     return agg_batch(P, P->path, base, keys, vals, n, nullptr, st, P->grid, P->block, P->smem_bytes, launches, fin);
   };
   // fusion only pays where launch latency dominates (<= 16M rows)
-  return run_core(P, L, P->path, P->hot_front != 0, P->cap, n, feed, partial, st, out, false, nullptr,
+  return run_core(P, L, P->path, P->hot_front != 0, P->cap, n, feed, partial, st, out, host_out, nullptr,
                   single && n > 0 && n <= (16ull << 20));
 }
 
@@ -1054,10 +1055,46 @@ blu_status_t blu_gby_execute_host(blu_gby_plan_t P, const void* const* hkeys, co
     return fail(BLU_E_INVALID, "NULL column pointer");
   cudaStream_t st = (cudaStream_t)stream;
   const Layout& L = P->lay;
-  // chunk: ~256 MB of rows per staging buffer, a multiple of 4 rows
   size_t row_bytes = 0;
   for (int k = 0; k < L.n_keys; ++k) row_bytes += dtype_bytes(L.key_dtype[k]);
   for (int c = 0; c < L.n_vals; ++c) row_bytes += dtype_bytes(L.val_dtype[c]);
+  // Partitioned hash plans (tables larger than L2): a streamed one-pass aggregation would update a
+  // DRAM-resident table at random, so when the columns fit in a quarter of the free device memory they
+  // are copied whole (pinned-rate H2D) and the query runs as on device columns (scatter + pass 2).
+  if (n && P->path == BLU_PATH_HASH_GLOBAL && P->parts > 1 && !L.has_q && L.key_words == 1) {
+    size_t free_b = 0, total_b = 0;
+    cudaMemGetInfo(&free_b, &total_b);
+    cudaGetLastError();
+    if ((double)n * (double)row_bytes < 0.25 * (double)(free_b + cache_idle_bytes())) {
+      setup_pool();
+      std::vector<void*> dk(L.n_keys, nullptr), dv(L.n_vals, nullptr);
+      auto release = [&]() {
+        for (void* q : dk) if (q) cudaFreeAsync(q, st);
+        for (void* q : dv) if (q) cudaFreeAsync(q, st);
+      };
+      cudaError_t e = cudaSuccess;
+      for (int k = 0; k < L.n_keys && !e; ++k) {
+        const size_t b = n * dtype_bytes(L.key_dtype[k]);
+        e = cudaMallocAsync(&dk[k], b, st);
+        if (!e) e = cudaMemcpyAsync(dk[k], hkeys[k], b, cudaMemcpyHostToDevice, st);
+      }
+      for (int c = 0; c < L.n_vals && !e; ++c) {
+        const size_t b = n * dtype_bytes(L.val_dtype[c]);
+        e = cudaMallocAsync(&dv[c], b, st);
+        if (!e) e = cudaMemcpyAsync(dv[c], hvals[c], b, cudaMemcpyHostToDevice, st);
+      }
+      if (e) {
+        cudaGetLastError();
+        release();
+        cudaStreamSynchronize(st);
+        return cuda_fail(e, "host columns to device");
+      }
+      blu_status_t s = execute_device(P, dk.data(), dv.data(), n, st, false, out, true);
+      release();
+      return s;
+    }
+  }
+  // otherwise: chunks of ~256 MB of rows through two staging buffers, a multiple of 4 rows
   uint64_t chunk = std::max<uint64_t>(4, ((256ull << 20) / std::max<size_t>(row_bytes, 1)) & ~3ull);
   if (chunk > n) chunk = (n + 3) & ~3ull;
   const int ncols = L.n_keys + L.n_vals;
