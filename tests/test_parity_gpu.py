@@ -356,17 +356,26 @@ def test_dense_state_accumulate_and_finalize(bg, oracles, name):
     assert_parity(gk, ga, o, w.schema)
 
 
-@pytest.mark.parametrize("name", ["C1", "C3"])
-def test_execute_host_columns(bg, oracles, name):
-    """Host columns in (chunked H2D overlapped with aggregation), host result out."""
-    w, o = oracles(name)
+@pytest.mark.parametrize("name", ["C1", "C3", "C3-parts"])
+def test_execute_host_columns(bg, oracles, monkeypatch, name):
+    """Host columns in, host result out (pinned result blocks, reused after the result is released):
+    chunked H2D overlapped with aggregation (C1, C3 one pass), or — for a partitioned plan — the whole
+    input copied to the device and run through the scatter + pass 2 ('C3-parts'). Twice, so the second
+    call reuses the first result's pinned blocks."""
+    w, o = oracles(name.split("-")[0])
+    if name.endswith("parts"):
+        monkeypatch.setenv("BLU_GBY_PARTS", "16")
     hk, hv = blugen.host_columns(w)
     hk = [torch.from_numpy(k).pin_memory() for k in hk]
     hv = [torch.from_numpy(v).pin_memory() for v in hv]
     plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
-    res = bg.blu_gby_execute_host(plan, hk, hv)
-    gk, ga = host_sorted(res, w.schema)
-    assert_parity(gk, ga, o, w.schema)
+    if name.endswith("parts"):
+        assert plan.info()["partitions"] == 16
+    for _ in range(2):
+        res = bg.blu_gby_execute_host(plan, hk, hv)
+        gk, ga = host_sorted(res, w.schema)
+        assert_parity(gk, ga, o, w.schema)
+        del res
 
 
 def test_init_table_matches_table1(bg):
