@@ -1002,6 +1002,12 @@ blu_status_t blu_gby_jit_probe(blu_gby_plan_t P, char* log, uint32_t log_cap, in
     ScatterParams sp{};
     sp.B = P->parts;
     if (!rc) rc = launch_scatter(p, sp, nullptr, P->grid);
+    bool wide8 = true;  // the TMA write-out variant (8-byte value columns)
+    for (int c = 0; c < P->lay.n_vals; ++c) wide8 = wide8 && dtype_bytes(P->lay.val_dtype[c]) == 8;
+    if (wide8) {
+      sp.tma = 1;
+      if (!rc) rc = launch_scatter(p, sp, nullptr, P->grid);
+    }
     AggParams p2 = p;
     p2.lay.n_keys = 1;
     p2.lay.sparse = 1;
