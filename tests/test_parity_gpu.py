@@ -495,6 +495,48 @@ def test_scatter_tma_write_out(bg, monkeypatch, tma, shape):
     assert_parity(gk, ga, o, w.schema)
 
 
+@pytest.mark.parametrize("n,parts,chunk", [(4097, "2", None), (65_537, "16", "8192"), (1_000_003, "64", "300001"),
+                                          (300_007, "256", "65536")])
+def test_scatter_tma_edges(bg, monkeypatch, n, parts, chunk):
+    """TMA write-out edge cases: ragged sizes, 2 to 256 buckets, several chunks (padding records in every
+    chunk's partition buffers), the smallest inputs the partitioned mode accepts; equal to the oracle."""
+    w = blugen.workload("C5", n_rows=n, n_groups=max(16, n // 50))
+    o = oracle.groupby_generated(w)
+    kc, vc = blugen.device_columns(w)
+    monkeypatch.setenv("BLU_GBY_SCATTER_TMA", "1")
+    monkeypatch.setenv("BLU_GBY_PARTS", parts)
+    if chunk:
+        monkeypatch.setenv("BLU_GBY_PART_CHUNK", chunk)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    bg.blu_gby_set_timing(True)
+    res = bg.blu_gby_execute(plan, kc, vc)
+    t = bg.blu_gby_last_timing()
+    bg.blu_gby_set_timing(False)
+    if n >= 4096 * int(parts):
+        assert t["part_chunks"] >= 1 and t["part_fallbacks"] == 0, t
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
+def test_host_results_pinned_reuse(bg, oracles):
+    """Host results of different sizes one after another, some kept alive while others are freed: each
+    takes its own pinned blocks from the cache (never one still referenced) and stays intact."""
+    held = []
+    for name, n in (("C3", 400_003), ("C1", 10_007), ("C3", 900_001), ("C2", 50_001)):
+        w = blugen.workload(name, n_rows=n)
+        o = oracle.groupby_generated(w)
+        hk, hv = blugen.host_columns(w)
+        plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+        res = bg.blu_gby_execute_host(plan, [torch.from_numpy(k).pin_memory() for k in hk],
+                                      [torch.from_numpy(v).pin_memory() for v in hv])
+        held.append((res, o, w.schema))
+        if len(held) == 3:
+            held.pop(0)  # free one result while two stay alive
+    for res, o, sch in held:
+        gk, ga = host_sorted(res, sch)
+        assert_parity(gk, ga, o, sch)
+
+
 @pytest.mark.parametrize("two_level", ["0", "1", "1-one"])
 @pytest.mark.parametrize("parts", [None, "4096"])
 def test_partitioned_wide_fanout(bg, monkeypatch, parts, two_level):
