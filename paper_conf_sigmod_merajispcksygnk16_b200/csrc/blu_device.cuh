@@ -17,6 +17,7 @@ namespace blu {
 struct GenericSpec {
   static constexpr bool kStatic = false;
   static constexpr int HOTREG = 0;
+  static constexpr int MMBOUND = 0;
 };
 
 // ------------------------------------------------------------------------------------------------
@@ -467,8 +468,150 @@ __device__ __forceinline__ void load_vals(const AggParams& p, uint64_t row, uint
   }
 }
 
+// MIN/MAX skip bounds of a shared-memory table (SP::MMBOUND, JIT only, opt-in: measured no faster on
+// C2, slower on C4 — DESIGN.md §7h). For each MIN field the CTA
+// publishes B >= max over the table's live entries of their current (encoded) MIN; a row whose value
+// is >= B cannot lower the MIN of any entry, so it skips the read-before-atomic of s_upd (MAX
+// symmetric). An entry's MIN only ever decreases, so every value ever computed from it stays an
+// upper bound of its current MIN: a bound may be stale, never wrong, and concurrent publishers need
+// no ordering. Every warp, every kMMRefresh of its own tiles, takes the max over its 1/nwarps slice
+// of the entries (part[warp]) and publishes the max over all warps' parts; no warp carries more of
+// this work than another (tiles are assigned statically, so one busy warp would hold the CTA at its
+// final barrier). Parts start at the identity: nothing is skipped until every warp has refreshed.
+constexpr int kMMRefresh = 16;
+template <class SP>
+constexpr int mm_count() {
+  int n = 0;
+  for (int j = 0; j < SP::NF; ++j)
+    if (SP::COL[j] >= 0 && (SP::KIND[j] >= FK_MINI32 && SP::KIND[j] <= FK_MAXF64)) ++n;
+  return n;
+}
+template <class SP>
+constexpr int mm_slot(int j) {  // index of MIN/MAX field j among the table's MIN/MAX fields
+  int n = 0;
+  for (int i = 0; i < j; ++i)
+    if (SP::COL[i] >= 0 && (SP::KIND[i] >= FK_MINI32 && SP::KIND[i] <= FK_MAXF64)) ++n;
+  return n;
+}
+template <int K>
+constexpr bool is_min_kind() { return K == FK_MINI32 || K == FK_MINI64 || K == FK_MINF64; }
+template <int K>
+constexpr bool is_max_kind() { return K == FK_MAXI32 || K == FK_MAXI64 || K == FK_MAXF64; }
+template <class SP>
+struct MMShared {
+  static constexpr int N = mm_count<SP>() > 0 ? mm_count<SP>() : 1;
+  long long pub[N];
+  long long part[32][N];
+};
+template <class SP>
+__device__ __forceinline__ MMShared<SP>& mm_shared() {
+  __shared__ MMShared<SP> m;
+  return m;
+}
+template <class SP>
+constexpr bool mm_on() {  // path (a) dense tables: BLU_GBY_MMBOUND >= 1
+  if constexpr (SP::kStatic) return SP::MMBOUND != 0 && mm_count<SP>() > 0;
+  else return false;
+}
+template <class SP>
+constexpr bool mm_front_on() {  // rank front: BLU_GBY_MMBOUND=2 only (C4: spills at 96 registers)
+  if constexpr (SP::kStatic) return SP::MMBOUND >= 2 && mm_count<SP>() > 0;
+  else return false;
+}
+
+// MIN/MAX update of an encoded value x behind the skip bound: the read-before-atomic is a
+// predicated shared load (no branch around it); a skipped read leaves `cur` at the value that makes
+// the row "no better", so only an improving row reaches the atomic.
+template <int K>
+__device__ __forceinline__ void s_mm_bounded(uint8_t* base, uint32_t e, uint64_t x, long long bnd) {
+  constexpr bool MN = is_min_kind<K>();
+  const uint32_t pass = MN ? (long long)x < bnd : (long long)x > bnd;
+  if constexpr (K == FK_MINI32 || K == FK_MAXI32) {
+    int* q = (int*)base + e;
+    int cur = MN ? INT32_MIN : INT32_MAX;
+    asm volatile("{ .reg .pred p; setp.ne.b32 p, %2, 0; @p ld.volatile.shared.b32 %0, [%1]; }"
+                 : "+r"(cur) : "r"((uint32_t)__cvta_generic_to_shared(q)), "r"(pass));
+    if (MN ? (int)x < cur : (int)x > cur) {
+      if (MN) atomicMin(q, (int)x); else atomicMax(q, (int)x);
+    }
+  } else {
+    long long* q = (long long*)base + e;
+    long long cur = MN ? INT64_MIN : INT64_MAX;
+    asm volatile("{ .reg .pred p; setp.ne.b32 p, %2, 0; @p ld.volatile.shared.b64 %0, [%1]; }"
+                 : "+l"(cur) : "r"((uint32_t)__cvta_generic_to_shared(q)), "r"(pass));
+    if (MN ? (long long)x < cur : (long long)x > cur) {
+      if (MN) atomicMin(q, (long long)x); else atomicMax(q, (long long)x);
+    }
+  }
+}
+
+// before the CTA's first tile (ordered by the barrier after the table initialisation)
+template <class SP, bool ON>
+__device__ __forceinline__ void mm_init() {
+  if constexpr (ON) {
+    MMShared<SP>& m = mm_shared<SP>();
+    sfor<0, SP::NF>([&](auto jc) {
+      constexpr int j = decltype(jc)::v;
+      if constexpr (SP::COL[j] >= 0 && (is_min_kind<SP::KIND[j]>() || is_max_kind<SP::KIND[j]>())) {
+        constexpr int q = mm_slot<SP>(j);
+        const long long id = (long long)identity64(SP::KIND[j]);
+        if (threadIdx.x < 32) m.part[threadIdx.x][q] = id;
+        if (threadIdx.x == 0) m.pub[q] = id;
+      }
+    });
+  }
+}
+
+// The calling warp (converged): refresh its part over entries of its slice of [0, n) except `skip0`,
+// `skip1` (entries whose rows bypass the table, e.g. the rank front's register-held hottest keys),
+// then publish the max (MIN fields) / min (MAX fields) over all warps' parts.
+#ifdef BLU_MM_INLINE
+#define BLU_MM_REFRESH_ATTR __forceinline__
+#else
+#define BLU_MM_REFRESH_ATTR __noinline__
+#endif
+template <class SP>
+__device__ BLU_MM_REFRESH_ATTR void mm_refresh(const uint8_t* sm, uint32_t n, uint32_t skip0, uint32_t skip1) {
+  if constexpr (mm_on<SP>()) {
+    MMShared<SP>& m = mm_shared<SP>();
+    const unsigned lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const uint32_t lo = (uint32_t)((uint64_t)n * warp / nw), hi = (uint32_t)((uint64_t)n * (warp + 1) / nw);
+    sfor<0, SP::NF>([&](auto jc) {
+      constexpr int j = decltype(jc)::v;
+      constexpr int K = SP::KIND[j];
+      if constexpr (SP::COL[j] >= 0 && (is_min_kind<K>() || is_max_kind<K>())) {
+        constexpr int q = mm_slot<SP>(j);
+        constexpr bool MN = is_min_kind<K>();
+        const uint8_t* b = sm + SP::SOFF[j];
+        long long acc = (long long)identity64(MN ? FK_MAXI64 : FK_MINI64);
+        for (uint32_t e = lo + lane; e < hi; e += 32) {
+          if (e == skip0 || e == skip1) continue;
+          const long long x = (K == FK_MINI32 || K == FK_MAXI32) ? (long long)((const volatile int*)b)[e]
+                                                                  : ((const volatile long long*)b)[e];
+          acc = MN ? max(acc, x) : min(acc, x);
+        }
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+          const long long y = __shfl_xor_sync(0xffffffffu, acc, o);
+          acc = MN ? max(acc, y) : min(acc, y);
+        }
+        if (lane == 0) ((volatile long long*)m.part[warp])[q] = acc;
+        __syncwarp();
+        long long all = lane < nw ? ((const volatile long long*)m.part[lane])[q]
+                                  : (long long)identity64(MN ? FK_MAXI64 : FK_MINI64);
+#pragma unroll
+        for (int o = 16; o; o >>= 1) {
+          const long long y = __shfl_xor_sync(0xffffffffu, all, o);
+          all = MN ? max(all, y) : min(all, y);
+        }
+        if (lane == 0) ((volatile long long*)m.pub)[q] = all;
+      }
+    });
+  }
+}
+
 // Apply every field to the rows in `mask` of a shared-memory table at entries e[r].
-template <class SP, int NV, int R>
+template <class SP, int NV, int R, bool MMB = false>
 __device__ __forceinline__ void smem_apply_rows(const AggParams& p, uint8_t* sm, const uint32_t (&e)[R],
                                                 uint32_t mask, const uint64_t (&v)[NV][R]) {
   const uint32_t S = p.S;
@@ -494,6 +637,12 @@ __device__ __forceinline__ void smem_apply_rows(const AggParams& p, uint8_t* sm,
 #else
     const uint32_t ST = S;
 #endif
+    long long bnd[SP::NF > 0 ? SP::NF : 1];
+    sfor<0, SP::NF>([&](auto jc) {
+      constexpr int j = decltype(jc)::v;
+      if constexpr (MMB && SP::COL[j] >= 0 && (is_min_kind<SP::KIND[j]>() || is_max_kind<SP::KIND[j]>()))
+        bnd[j] = ((const volatile long long*)mm_shared<SP>().pub)[mm_slot<SP>(j)];
+    });
 #pragma unroll
     for (int r = 0; r < R; ++r)
       if (mask >> r & 1) {
@@ -505,8 +654,15 @@ __device__ __forceinline__ void smem_apply_rows(const AggParams& p, uint8_t* sm,
 #else
           uint8_t* b = sm + p.soff[j];
 #endif
-          if constexpr (c < 0) s_upd<FK_COUNT, true>(b, e[r], ST, 1ull);
-          else s_upd<K, true>(b, e[r], ST, v[c][r]);
+          if constexpr (c < 0) {
+            s_upd<FK_COUNT, true>(b, e[r], ST, 1ull);
+          } else if constexpr (MMB && is_min_kind<K>()) {
+            s_mm_bounded<K>(b, e[r], enc<K, true>(v[c][r]), bnd[j]);
+          } else if constexpr (MMB && is_max_kind<K>()) {
+            s_mm_bounded<K>(b, e[r], enc<K, true>(v[c][r]), bnd[j]);
+          } else {
+            s_upd<K, true>(b, e[r], ST, v[c][r]);
+          }
         });
       }
     return;
@@ -794,6 +950,7 @@ __device__ __forceinline__ void dense_body(const AggParams& p, const FinalParams
   }
   for (int j = 0; j < L.n_fields; ++j)
     for (uint32_t e = threadIdx.x; e < D; e += blockDim.x) smem_init_entry(sm + p.soff[j], L.f[j].kind, e, D);
+  mm_init<SP, mm_on<SP>()>();
   __syncthreads();
 
   const uint64_t pol = evict_first_policy();
@@ -801,6 +958,7 @@ __device__ __forceinline__ void dense_body(const AggParams& p, const FinalParams
   const uint64_t tile = (uint64_t)blockDim.x * R;
   const uint64_t ntiles = (n + tile - 1) / tile;
   uint32_t flag_seen = 0;
+  uint32_t mm_it = 0;  // this warp's tiles since its last MIN/MAX bound refresh
   if constexpr (PIPE) {  // next tile's loads in flight during this tile's shared-memory updates
     const unsigned warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     RawTile<SP, R> A, B;
@@ -816,7 +974,8 @@ __device__ __forceinline__ void dense_body(const AggParams& p, const FinalParams
       uint32_t e[R];
 #pragma unroll
       for (int r = 0; r < R; ++r) e[r] = (uint32_t)key[r];
-      smem_apply_rows<SP, NV, R>(p, sm, e, valid, v);
+      smem_apply_rows<SP, NV, R, mm_on<SP>()>(p, sm, e, valid, v);
+      if (mm_on<SP>() && ++mm_it % kMMRefresh == 0) mm_refresh<SP>(sm, D, ~0u, ~0u);
       if (__any_sync(0xffffffffu, fl)) break;
       A = B;
       t = tn;
@@ -833,7 +992,8 @@ __device__ __forceinline__ void dense_body(const AggParams& p, const FinalParams
     uint32_t e[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) e[r] = (uint32_t)key[r];
-    smem_apply_rows<SP, NV, R>(p, sm, e, valid, v);
+    smem_apply_rows<SP, NV, R, mm_on<SP>()>(p, sm, e, valid, v);
+    if (mm_on<SP>() && ++mm_it % kMMRefresh == 0) mm_refresh<SP>(sm, D, ~0u, ~0u);
   }
   __syncthreads();
   if (FUSE && p.fuse_init) {  // the dense state must be initialised before this CTA flushes into it
@@ -1174,6 +1334,14 @@ struct HotAccT2 {
       });
     }
   }
+  // rank-front entry of hot key h, or ~0u (empty key or not in the front)
+  __device__ __forceinline__ uint32_t entry(const AggParams& p, const uint8_t* sm, int h) const {
+    const uint64_t kh = key[h];
+    if (kh == kEmpty) return ~0u;
+    const uint64_t x = ((const uint64_t*)(sm + p.key_off))[kh >> 5];
+    const uint32_t b = (uint32_t)kh & 31u, bits = (uint32_t)x;
+    return (bits >> b & 1u) ? (uint32_t)(x >> 32) + __popc(bits & ((1u << b) - 1u)) : ~0u;
+  }
   __device__ __forceinline__ uint64_t count(int h) const {
     uint64_t c = 0;
     sfor<0, SP::NF>([&](auto jc) {
@@ -1230,7 +1398,7 @@ __device__ __forceinline__ void process_rows(const AggParams& p, uint8_t* sm, ui
         done = true;
       }
     }
-    if (!done) smem_apply_rows<SP, NV, R>(p, sm, fe, hit, v);
+    if (!done) smem_apply_rows<SP, NV, R, mm_front_on<SP>()>(p, sm, fe, hit, v);
     miss = valid & ~hit;
   } else if (FRONT && !deduped) {
     // hot-key front: small open-addressing table per CTA in shared memory
@@ -1369,10 +1537,32 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
       ((uint64_t*)(sm + p.key_off))[e] = seed ? __ldg((const unsigned long long*)seed + e) : kEmpty;
     for (int j = 0; j < L.n_fields; ++j)
       for (uint32_t e = threadIdx.x; e < S; e += blockDim.x) smem_init_entry(sm + p.soff[j], L.f[j].kind, e, S);
+    mm_init<SP, FRONT && DIRECT && mm_front_on<SP>()>();
     __syncthreads();
   }
   HotAcc<SP> ha;
   ha.init(FRONT && DIRECT && p.front_rank_words ? p.hot_key : nullptr);
+  // rank front: every warp refreshes the MIN/MAX skip bounds over its slice of the hot entries (the
+  // register-held hottest keys' entries excluded: their rows never reach the table before the flush)
+  uint32_t mm_it = 0;
+  auto mm_front = [&]() {
+    if constexpr (FRONT && DIRECT) {
+      if constexpr (mm_front_on<SP>()) {
+#ifndef BLU_MM_NOREFRESH
+        if (p.front_rank_words && ++mm_it % kMMRefresh == 0) {
+#else
+        if (false) {
+#endif
+          const uint64_t xl = ((const uint64_t*)(sm + p.key_off))[p.front_rank_words - 1];
+          const uint32_t nh = (uint32_t)(xl >> 32) + __popc((uint32_t)xl);
+          uint32_t s0 = ~0u, s1 = ~0u;
+          if constexpr (SP::HOTREG >= 1) s0 = ha.entry(p, sm, 0);
+          if constexpr (SP::HOTREG >= 2) s1 = ha.entry(p, sm, 1);
+          mm_refresh<SP>(sm, nh, s0, s1);
+        }
+      }
+    }
+  };
   const uint64_t pol = evict_first_policy();
   // SEG: warp tiles (32*R rows) handed out in bucket order by a global counter, so every warp of
   // the grid stays inside the same one or two buckets (their table slices L2-resident); static
@@ -1409,6 +1599,7 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
       uint64_t v[NV][R];
       const uint32_t valid = tile_unpack<SP, NV, R>(p, A, lane_base<R>(t * tile, warp, lane), n, key, v);
       process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v, ha);
+      mm_front();
       if (__any_sync(0xffffffffu, fl)) break;  // warp-uniform abort
       A = B;
       t = tn;
@@ -1514,6 +1705,7 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
       load_vals<SP, NV, R>(p, row, n, pol, v);
     }
     process_rows<SP, NV, R, FRONT, DIRECT>(p, sm, key, valid, v, ha);
+    mm_front();
     t = t_next;
   }
   if constexpr (FRONT && DIRECT && SP::HOTREG != 0) ha.flush(p, sm);

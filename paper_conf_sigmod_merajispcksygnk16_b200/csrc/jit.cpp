@@ -140,6 +140,9 @@ std::string spec_source(const char* name, const Layout& L, uint32_t S, const uin
   s += "  static constexpr unsigned STAB = " + std::to_string(S) + "u;\n";
   s += "  static constexpr int SOFF[24] = " + arr(so, L.n_fields, 24) + ";\n";
   s += "  static constexpr int HOTREG = " + std::to_string(jit_hot_reg()) + ";\n";
+  // MIN/MAX skip bounds (opt-in): 1 = path (a) dense tables, 2 = also the rank front
+  const char* mb = getenv("BLU_GBY_MMBOUND");
+  s += std::string("  static constexpr int MMBOUND = ") + (mb && (mb[0] == '1' || mb[0] == '2') ? mb[0] : '0') + ";\n";
   const char* dd = getenv("BLU_GBY_DEDUPE");
   s += std::string("  static constexpr int DEDUPE = ") + (dd && dd[0] == '1' ? "1" : "0") + ";\n";
   s += "};\n}  // namespace blu\n";

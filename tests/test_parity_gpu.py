@@ -173,6 +173,63 @@ def test_hot_reg_key_outside_front(bg, monkeypatch, seed):
     assert_parity(gk, ga, o, sch)
 
 
+@pytest.mark.parametrize("mmb", ["2", "1", "0"])
+@pytest.mark.parametrize("recipe", ["group-offset", "trend", "late-extremes"])
+@pytest.mark.parametrize("path", ["a", "d-rank", "d-rank-hotreg"])
+def test_minmax_skip_bounds(bg, monkeypatch, mmb, recipe, path):
+    """MIN/MAX skip bounds of the shared-memory tables (BLU_GBY_MMBOUND): a row skips
+    the read-before-atomic only when its value cannot beat the largest current MIN (smallest MAX) of
+    any live entry. Adversarial value recipes: per-group offsets far apart (the bound is the highest
+    group's MIN, so low groups must never be skipped), a monotone trend over the rows (every row is
+    a new MIN of its group in one column and a new MAX in another), and the column extremes placed
+    in the last 1% of the rows (after the bound has converged). i32 / i64 / f64 (negative values:
+    the order-preserving encoding) MIN and MAX, on path (a) and the rank front with and without the
+    register-held hottest key; equal to the oracle bit for bit with the bounds off (0), on path (a)
+    only (1) and also on the rank front (2)."""
+    monkeypatch.setenv("BLU_GBY_MMBOUND", mmb)
+    monkeypatch.setenv("BLU_GBY_HOT_REG", "1" if "hotreg" in path else "0")
+    rng = np.random.default_rng(len(recipe) * 7 + len(path))
+    n = 3_000_017
+    D = 1024 if path == "a" else 20_000
+    if path == "a":
+        g = rng.integers(0, D, n)
+    else:
+        g = np.minimum(rng.zipf(1.2, n) - 1, D - 1)
+        g = rng.permutation(D)[g]
+    i = np.arange(n, dtype=np.int64)
+    if recipe == "group-offset":
+        off = rng.permutation(D).astype(np.int64) * 1_000_000
+        v1 = off[g] + rng.integers(0, 1000, n)
+    elif recipe == "trend":
+        v1 = -i * 3 + rng.integers(0, 2, n)
+    else:
+        v1 = rng.integers(-10**6, 10**6, n)
+        late = rng.random(n) < 0.01
+        late[: n * 99 // 100] = False
+        v1[late] = rng.choice([-(10**9), 10**9], int(late.sum())) + rng.integers(-5, 5, int(late.sum()))
+    v0 = np.clip(v1 // 1000, -(2**31), 2**31 - 1).astype(np.int32)
+    if recipe == "trend":
+        v0 = (i // 3 - 2**20).astype(np.int32)  # rising: every row a new MAX of its group
+    v2 = (v1 % (2**20) - 2**19) / 64.0 - (i if recipe == "trend" else 0) / 2.0
+    sch = blugen.Schema([(I32, D)], [I32, I64, F64], ALL(3))
+    kc = [g.astype(np.int32)]
+    vc = [v0, v1.astype(np.int64), v2]
+    o = oracle.groupby_arrays(sch, kc, vc)
+    if path == "a":
+        monkeypatch.setenv("BLU_GBY_FORCE_PATH", "a")
+        monkeypatch.setenv("BLU_GBY_NO_FUSE", "1")
+    else:
+        monkeypatch.setenv("BLU_GBY_FORCE_PATH", "d")
+        monkeypatch.setenv("BLU_GBY_HOT_FRONT", "1")
+    plan = bg.plan_for(sch, D, n)
+    if path != "a":
+        assert plan.info()["hot_front"] == 1
+    dk, dv = _mk(kc, vc)
+    res = bg.blu_gby_execute(plan, dk, dv)
+    gk, ga = gpu_sorted(res, sch)
+    assert_parity(gk, ga, o, sch)
+
+
 @pytest.mark.parametrize("n", [0, 1, 3, 31, 33, 4095, 4097, 65_537])
 @pytest.mark.parametrize("path", ["a", "a-nofuse", "b", "d"])
 def test_small_and_ragged(bg, monkeypatch, n, path):
