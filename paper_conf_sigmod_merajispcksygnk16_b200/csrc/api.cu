@@ -82,7 +82,7 @@ void setup_pool() {
       cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
     }
     // L2 fetch granularity for the random slot traffic of path (b) (a hint; 0 keeps the default)
-    if (const char* g = getenv("BLU_GBY_L2_FETCH")) {
+    if (const char* g = benv("BLU_GBY_L2_FETCH")) {
       int v = atoi(g);
       if (v > 0) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, (size_t)v);
     }
@@ -283,7 +283,7 @@ using Feeder = std::function<cudaError_t(AggParams& base, uint32_t* launches, Wo
 
 static bool ptr_aligned(const void* p) { return ((uintptr_t)p & 15) == 0; }
 static uint32_t prefetch_enabled() {  // scatter prefetch distance in tiles (BLU_GBY_PREFETCH, default 1)
-  static const uint32_t d = getenv("BLU_GBY_PREFETCH") ? (uint32_t)atoi(getenv("BLU_GBY_PREFETCH")) : 1u;
+  static const uint32_t d = benv("BLU_GBY_PREFETCH") ? (uint32_t)atoi(benv("BLU_GBY_PREFETCH")) : 1u;
   return d;
 }
 
@@ -329,7 +329,7 @@ static cudaError_t agg_batch(const blu_gby_plan_s* P, int path, AggParams p, con
 static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int path, bool front, uint64_t cap0,
                              uint64_t total_rows, const Feeder& feed, bool partial, cudaStream_t st,
                              blu_gby_result_t* out, bool host_out, float* h2d_ms_acc, bool fuse_req = false) {
-  static const bool hprof = getenv("BLU_GBY_DEBUG_HOST") != nullptr;  // host-time breakdown per execute
+  static const bool hprof = benv("BLU_GBY_DEBUG_HOST") != nullptr;  // host-time breakdown per execute
   auto hnow = [] { return std::chrono::steady_clock::now(); };
   const auto h_entry = hnow();
   std::chrono::steady_clock::time_point h_init{}, h_feed{}, h_alloc{}, h_compact{}, h_sync{};
@@ -350,7 +350,7 @@ static blu_status_t run_core(const blu_gby_plan_s* P, const Layout& lay, int pat
     if (t_timing) cudaEventRecord(t_ev.e[0], st);
     // path (a) with a small domain: init (S4) and compaction (S8) fused into the aggregation kernel
     const bool fuse = fuse_req && path == BLU_PATH_DENSE_SMEM && D <= 65536 && !partial && !host_out &&
-                      !getenv("BLU_GBY_NO_FUSE");
+                      !benv("BLU_GBY_NO_FUSE");
     const uint64_t n_entries = dense ? D : cap;
     const uint64_t nb = (n_entries + 4095) / 4096;
     void* small = nullptr;
@@ -600,7 +600,7 @@ static bool nonnull_cols(const void* const* cols, int n) {
 static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, const void* const* keys,
                                     const void* const* vals, uint64_t n, cudaStream_t st, uint32_t* launches,
                                     Work& w) {
-  static const bool hdbg = getenv("BLU_GBY_DEBUG_HOST") != nullptr;
+  static const bool hdbg = benv("BLU_GBY_DEBUG_HOST") != nullptr;
   auto now = [] { return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count(); };
   const double h0 = now();
   const Layout& L = P->lay;
@@ -632,11 +632,11 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   // two-level scatter (bucket tables with >= 256 buckets; BLU_GBY_PART_2LEVEL=0 disables): B1 first-level buckets, each split
   // into B / B1 second-level buckets by a second scatter, instead of one B-way scatter (a 2048-way
   // scatter writes ~2 rows per bucket per tile); needs a second set of partition buffers
-  const char* tl = getenv("BLU_GBY_PART_2LEVEL");
+  const char* tl = benv("BLU_GBY_PART_2LEVEL");
   const uint32_t B1 = (P->part_smem && !(tl && tl[0] == '0') && B >= 256) ? 32u : 0u;
   if (B1) M = std::max<uint64_t>(M / 2, 1ull << 22);
   M = std::min<uint64_t>(n, M);
-  if (const char* cr = getenv("BLU_GBY_PART_CHUNK")) M = std::min<uint64_t>(n, std::max<uint64_t>(1024, strtoull(cr, 0, 10)));
+  if (const char* cr = benv("BLU_GBY_PART_CHUNK")) M = std::min<uint64_t>(n, std::max<uint64_t>(1024, strtoull(cr, 0, 10)));
   // bucket capacity: the mean plus slack for the spread of the number of GROUPS per bucket (keys
   // hash uniformly: relative sd 1/sqrt(est/B); 6 sd) and of rows per group; heavier skew overflows a
   // bucket and takes the gated one-pass fallback
@@ -645,7 +645,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   // skip. C3 scatter 19.4 -> 18.2 ms, C5 22.1 -> 20.0 ms per chunk
   bool tma = true;
   {
-    const char* tm = getenv("BLU_GBY_SCATTER_TMA");
+    const char* tm = benv("BLU_GBY_SCATTER_TMA");
     if (tm && tm[0] == '0') tma = false;
     for (int c = 0; c < L.n_vals; ++c) tma = tma && dtype_bytes(L.val_dtype[c]) == 8;
     // the padded staging must fit the scatter's shared memory at the widest histogram of this plan
@@ -728,7 +728,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     for (int c = 0; c < L.n_vals; ++c) sp.out_val[c] = vbuf[c];
     sp.gate = d_gate;
     sp.tma = tma ? 1u : 0u;
-    static const bool dbg = getenv("BLU_GBY_DEBUG_PART") != nullptr;
+    static const bool dbg = benv("BLU_GBY_DEBUG_PART") != nullptr;
     cudaEvent_t ev[4];
     if (dbg) {
       for (auto& x : ev) cudaEventCreate(&x);
@@ -760,7 +760,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       le = launch_scatter(p1, s1, st, scatter_grid((uint32_t)P->sms, B1));
       if (le) return (cudaError_t)le;
       const uint32_t B2 = B / B1;
-      const bool one_launch = getenv("BLU_GBY_2LEVEL_ONE") && atoi(getenv("BLU_GBY_2LEVEL_ONE")) == 1;
+      const bool one_launch = benv("BLU_GBY_2LEVEL_ONE") && atoi(benv("BLU_GBY_2LEVEL_ONE")) == 1;
       if (one_launch) {
         // second level as ONE launch over every first-level bucket (segmented input; the first-level
         // counts stay on the device, no host round trip): bucket b1's rows go to [b1 * B2, b1 * B2 + B2).
@@ -827,14 +827,14 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     p2.seg_stride = seg_cap;
     p2.seg_count = d_cursor;
     p2.n_segs = B;
-    p2.tile_ctr = getenv("BLU_GBY_DYN") && atoi(getenv("BLU_GBY_DYN")) == 0 ? nullptr : (uint64_t*)(d_cursor + B + 1);
-    if (const char* g = getenv("BLU_GBY_GRAB")) p2.grab = (uint32_t)atoi(g);
+    p2.tile_ctr = benv("BLU_GBY_DYN") && atoi(benv("BLU_GBY_DYN")) == 0 ? nullptr : (uint64_t*)(d_cursor + B + 1);
+    if (const char* g = benv("BLU_GBY_GRAB")) p2.grab = (uint32_t)atoi(g);
     p2.gate = d_gate;
     p2.gate_run_if = 0;
     p2.front_slots = 0;
     if (P->part_smem) {
       // bucket-local shared-memory tables: pieces of ~1/div of the mean bucket, whole 4096-row tiles
-      const uint64_t div = getenv("BLU_GBY_PIECE_DIV") ? std::max(1, atoi(getenv("BLU_GBY_PIECE_DIV"))) : 2;
+      const uint64_t div = benv("BLU_GBY_PIECE_DIV") ? std::max(1, atoi(benv("BLU_GBY_PIECE_DIV"))) : 2;
       const uint64_t mean = (m + B - 1) / B;
       uint64_t piece = ((mean + div - 1) / div + 4095) / 4096 * 4096;
       piece = std::min<uint64_t>(std::max<uint64_t>(piece, 4096), 1ull << 30);
@@ -892,11 +892,11 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
   Feeder feed = [&](AggParams& base, uint32_t* launches, Work& w, const FinalParams* fin) -> cudaError_t {
     base.jit_ok = L.key_words == 2 ? 0 : 1;
     // path (b)/(b') one pass: each warp L2-prefetches its next tile (BLU_GBY_AGG_PREFETCH=0/1)
-    const char* ap = getenv("BLU_GBY_AGG_PREFETCH");
+    const char* ap = benv("BLU_GBY_AGG_PREFETCH");
     base.prefetch = ap ? (uint32_t)atoi(ap) : 0u;
     // hot-key front seeded with the heavy hitters of a row sample (needs a COUNT field to tell
     // seeded keys that received rows from those that did not)
-    static const bool no_seed = getenv("BLU_GBY_NO_SEED") != nullptr;
+    static const bool no_seed = benv("BLU_GBY_NO_SEED") != nullptr;
     if (base.front_slots > 0 && L.count_field >= 0 && !no_seed && n >= (1u << 16)) {
       void* ws = nullptr;
       cudaError_t e = w.alloc(&ws, front_seed_bytes(base.front_slots));
@@ -909,7 +909,7 @@ static blu_status_t execute_device(const blu_gby_plan_s* P, const void* const* k
       }
       pk.vec_ok = (int32_t)vec;
       // path (b'): a rank image when the bitmap of the domain fits the front's key region
-      const bool no_rank = getenv("BLU_GBY_NO_RANK_FRONT") != nullptr;
+      const bool no_rank = benv("BLU_GBY_NO_RANK_FRONT") != nullptr;
       const uint64_t W = (L.domain + 31) / 32;
       const uint32_t rank_words =
           P->path == BLU_PATH_DIRECT_GLOBAL && !no_rank && L.domain > 0 && W <= base.front_slots ? (uint32_t)W : 0u;
@@ -985,6 +985,7 @@ blu_status_t blu_gby_release_workspace(uint64_t* freed) {
 }
 
 blu_status_t blu_gby_jit_probe(blu_gby_plan_t P, char* log, uint32_t log_cap, int32_t* n_programs) {
+  env_snapshot();
   if (!P) return fail(BLU_E_INVALID, "NULL plan");
   if (log && log_cap) log[0] = 0;
   if (n_programs) *n_programs = 0;
@@ -1033,6 +1034,7 @@ blu_status_t blu_gby_jit_probe(blu_gby_plan_t P, char* log, uint32_t log_cap, in
 
 blu_status_t blu_gby_read_roofline(const void* const* cols, const uint64_t* bytes, int32_t n_cols, void* stream,
                                    uint64_t* dev_out) {
+  env_snapshot();
   if (n_cols < 1 || n_cols > kMaxKeys + kMaxVals || !cols || !bytes || !dev_out)
     return fail(BLU_E_INVALID, "bad read_roofline arguments");
   for (int j = 0; j < n_cols; ++j)
@@ -1046,16 +1048,19 @@ blu_status_t blu_gby_read_roofline(const void* const* cols, const uint64_t* byte
 
 blu_status_t blu_gby_execute(blu_gby_plan_t P, const void* const* key_cols, const void* const* val_cols, uint64_t n_rows,
                              void* stream, blu_gby_result_t* out) {
+  env_snapshot();
   return execute_device(P, key_cols, val_cols, n_rows, (cudaStream_t)stream, false, out);
 }
 
 blu_status_t blu_gby_execute_partial(blu_gby_plan_t P, const void* const* key_cols, const void* const* val_cols,
                                      uint64_t n_rows, void* stream, blu_gby_result_t* out) {
+  env_snapshot();
   return execute_device(P, key_cols, val_cols, n_rows, (cudaStream_t)stream, true, out);
 }
 
 blu_status_t blu_gby_execute_host(blu_gby_plan_t P, const void* const* hkeys, const void* const* hvals, uint64_t n,
                                   void* stream, blu_gby_result_t* out) {
+  env_snapshot();
   if (!P || !out) return fail(BLU_E_INVALID, "NULL plan or out");
   if (n && (!nonnull_cols(hkeys, P->lay.n_keys) || !nonnull_cols(hvals, P->lay.n_vals)))
     return fail(BLU_E_INVALID, "NULL column pointer");
@@ -1209,16 +1214,19 @@ static blu_status_t merge_impl(blu_gby_plan_t P, const blu_gby_result_t* parts, 
 }
 
 blu_status_t blu_gby_merge(blu_gby_plan_t P, const blu_gby_result_t* parts, int32_t np, void* stream, blu_gby_result_t* out) {
+  env_snapshot();
   return merge_impl(P, parts, np, stream, false, out);
 }
 
 blu_status_t blu_gby_merge_partial(blu_gby_plan_t P, const blu_gby_result_t* parts, int32_t np, void* stream,
                                    blu_gby_result_t* out) {
+  env_snapshot();
   return merge_impl(P, parts, np, stream, true, out);
 }
 
 blu_status_t blu_gby_merge_records(blu_gby_plan_t P, const void* records, uint64_t n, void* stream, int32_t partial_out,
                                    blu_gby_result_t* out) {
+  env_snapshot();
   if (!P || !out || (n && !records)) return fail(BLU_E_INVALID, "bad merge_records arguments");
   if (P->lay.has_q) return fail(BLU_E_UNSUPPORTED, "merge_records: 128-bit payloads have no record format");
   cudaStream_t st = (cudaStream_t)stream;
@@ -1237,6 +1245,7 @@ blu_status_t blu_gby_merge_records(blu_gby_plan_t P, const void* records, uint64
 
 blu_status_t blu_gby_execute_dense_state(blu_gby_plan_t P, const void* const* keys, const void* const* vals, uint64_t n,
                                          void* stream, void* const* state_arrays, int32_t init) {
+  env_snapshot();
   if (!P || !state_arrays) return fail(BLU_E_INVALID, "NULL plan or state arrays");
   if (P->path == BLU_PATH_HASH_GLOBAL) return fail(BLU_E_UNSUPPORTED, "dense state needs path a or b'");
   if (n && (!nonnull_cols(keys, P->lay.n_keys) || !nonnull_cols(vals, P->lay.n_vals)))
@@ -1287,6 +1296,7 @@ blu_status_t blu_gby_execute_dense_state(blu_gby_plan_t P, const void* const* ke
 }
 
 blu_status_t blu_gby_finalize_dense_state(blu_gby_plan_t P, void* const* state_arrays, void* stream, blu_gby_result_t* out) {
+  env_snapshot();
   if (!P || !state_arrays || !out) return fail(BLU_E_INVALID, "NULL argument");
   if (P->path == BLU_PATH_HASH_GLOBAL) return fail(BLU_E_UNSUPPORTED, "dense state needs path a or b'");
   cudaStream_t st = (cudaStream_t)stream;
@@ -1307,6 +1317,7 @@ blu_status_t blu_gby_finalize_dense_state(blu_gby_plan_t P, void* const* state_a
 
 blu_status_t blu_gby_execute_records(blu_gby_plan_t P, const void* records, uint64_t n, void* stream, int32_t partial_out,
                                      blu_gby_result_t* out) {
+  env_snapshot();
   if (!P || !out || (n && !records)) return fail(BLU_E_INVALID, "bad execute_records arguments");
   if (P->lay.has_q) return fail(BLU_E_UNSUPPORTED, "execute_records: 128-bit payloads have no record format");
   cudaStream_t st = (cudaStream_t)stream;
@@ -1325,6 +1336,7 @@ blu_status_t blu_gby_execute_records(blu_gby_plan_t P, const void* records, uint
 
 blu_status_t blu_gby_partition_rows(blu_gby_plan_t P, const void* const* key_cols, const void* const* val_cols,
                                     uint64_t n, int32_t n_parts, void* stream, void* send_buf, uint64_t* send_counts) {
+  env_snapshot();
   if (!P || !send_counts || n_parts < 1 || n_parts > 1024) return fail(BLU_E_INVALID, "bad partition_rows arguments");
   if (P->lay.has_q) return fail(BLU_E_UNSUPPORTED, "partition_rows: 128-bit payloads have no record format");
   if (n && (!send_buf || !nonnull_cols(key_cols, P->lay.n_keys) || !nonnull_cols(val_cols, P->lay.n_vals)))
@@ -1354,6 +1366,7 @@ blu_status_t blu_gby_partition_rows(blu_gby_plan_t P, const void* const* key_col
 
 blu_status_t blu_gby_partition(blu_gby_plan_t P, const blu_gby_result_t* partial, int32_t n_parts, void* stream, void* send_buf,
                                uint64_t* send_counts) {
+  env_snapshot();
   if (!P || !partial || !send_counts || n_parts < 1 || n_parts > 1024) return fail(BLU_E_INVALID, "bad partition arguments");
   if (P->lay.has_q) return fail(BLU_E_UNSUPPORTED, "partition: 128-bit payloads have no record format");
   if (!partial->is_partial || partial->is_host) return fail(BLU_E_INVALID, "partition needs a device partial result");
@@ -1380,6 +1393,7 @@ blu_status_t blu_gby_partition(blu_gby_plan_t P, const blu_gby_result_t* partial
 }
 
 blu_status_t blu_gby_init_table(blu_gby_plan_t P, void* dev_table, uint64_t n_slots, void* stream) {
+  env_snapshot();
   if (!P || (n_slots && !dev_table)) return fail(BLU_E_INVALID, "NULL plan or table");
   CK(launch_init_slots(P->lay, dev_table, n_slots, stream), "init slots");
   return BLU_OK;

@@ -112,6 +112,9 @@ void jit_probe_begin(JitProbe* pr);
 void jit_probe_end();
 bool jit_probe_active();
 const void* jit_kernel(const std::string& spec_src, const std::string& entry_src, const char* entry);
+// BLU_* knobs (env.cpp): env_snapshot() at every public entry point, benv() reads the snapshot
+void env_snapshot();
+const char* benv(const char* name);
 std::string jit_spec(const char* name, const Layout& L, uint32_t S, const uint32_t* soff);
 
 // Own LSD radix sort of u64 keys (sort.cu), used by the KMV estimate (kmv.cu)

@@ -141,9 +141,9 @@ std::string spec_source(const char* name, const Layout& L, uint32_t S, const uin
   s += "  static constexpr int SOFF[24] = " + arr(so, L.n_fields, 24) + ";\n";
   s += "  static constexpr int HOTREG = " + std::to_string(jit_hot_reg()) + ";\n";
   // MIN/MAX skip bounds (opt-in): 1 = path (a) dense tables, 2 = also the rank front
-  const char* mb = getenv("BLU_GBY_MMBOUND");
+  const char* mb = benv("BLU_GBY_MMBOUND");
   s += std::string("  static constexpr int MMBOUND = ") + (mb && (mb[0] == '1' || mb[0] == '2') ? mb[0] : '0') + ";\n";
-  const char* dd = getenv("BLU_GBY_DEDUPE");
+  const char* dd = benv("BLU_GBY_DEDUPE");
   s += std::string("  static constexpr int DEDUPE = ") + (dd && dd[0] == '1' ? "1" : "0") + ";\n";
   s += "};\n}  // namespace blu\n";
   return s;
@@ -212,14 +212,14 @@ bool compile(const std::string& src, std::vector<char>& cubin, std::string& log)
 
 // The rank front's 0, 1 or 2 hottest keys summed in registers (BLU_GBY_HOT_REG=0/1/2)
 int jit_hot_reg() {
-  const char* e = getenv("BLU_GBY_HOT_REG");  // read per plan execution (tests switch it)
+  const char* e = benv("BLU_GBY_HOT_REG");  // read per plan execution (tests switch it)
   // default 1: C4 8.91 vs 9.18-9.36 ms (640 threads, one key); two keys measured slower (11.8-12.0 ms)
   const int h = e ? atoi(e) : 1;
   return jit_enabled() ? (h < 0 ? 0 : h > 2 ? 2 : h) : 0;
 }
 
 bool jit_enabled() {
-  const char* e = getenv("BLU_GBY_JIT");
+  const char* e = benv("BLU_GBY_JIT");
   return !(e && e[0] == '0');
 }
 
@@ -233,7 +233,7 @@ bool jit_probe_active() { return t_probe != nullptr; }
 // Experiment switches (benchmarks): BLU_GBY_JIT_DEFS=A,B compiles the kernels with #define A 1 ...
 static std::string jit_defs() {
   std::string out;
-  const char* d = getenv("BLU_GBY_JIT_DEFS");
+  const char* d = benv("BLU_GBY_JIT_DEFS");
   if (!d) return out;
   std::string cur;
   for (const char* c = d;; ++c) {
@@ -268,7 +268,7 @@ static void probe_compile(const std::string& body) {
 
 const void* jit_kernel(const std::string& spec_src, const std::string& entry_src, const char* entry) {
   if (!jit_enabled()) return nullptr;
-  if (const char* dump = getenv("BLU_GBY_JIT_DUMP")) {  // write the program text (SASS inspection offline)
+  if (const char* dump = benv("BLU_GBY_JIT_DUMP")) {  // write the program text (SASS inspection offline)
     std::string fn = std::string(dump) + "/" + entry + ".cu";
     std::string src = std::string(kPreamble) + jit_defs() + kSrc_blu_params_h + "\n" + kSrc_blu_device_cuh + "\n" +
                       spec_src + entry_src;
@@ -315,7 +315,7 @@ const void* jit_kernel(const std::string& spec_src, const std::string& entry_src
     if (cubin.empty()) {
       std::string log;
       if (!compile(src, cubin, log)) {
-        if (getenv("BLU_GBY_JIT_VERBOSE")) fprintf(stderr, "blugby JIT compile failed:\n%s\n", log.c_str());
+        if (benv("BLU_GBY_JIT_VERBOSE")) fprintf(stderr, "blugby JIT compile failed:\n%s\n", log.c_str());
         e.failed = true;
         return nullptr;
       }

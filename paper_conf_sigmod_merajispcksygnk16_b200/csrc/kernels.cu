@@ -30,6 +30,7 @@
 #include <stdio.h>
 #include <string.h>
 #include <string>
+#include <chrono>
 
 namespace blu {
 
@@ -46,55 +47,76 @@ uint64_t launches_total() { return g_launches.load(); }
 static int rows_per_thread(int nv) { return nv <= 4 ? 4 : nv <= 8 ? 2 : 1; }
 // JIT-only tuning knobs (benchmarks): rows per thread of the dense kernel, min CTAs per SM.
 static int jit_env(const char* k, int def) {
-  const char* v = getenv(k);
+  const char* v = benv(k);
   return v && *v ? atoi(v) : def;
 }
 
 // Launch the NVRTC-specialised kernel for this plan's layout, if the JIT is enabled and succeeds.
 static bool launch_jit(const char* body, const char* entry_decl, const AggParams& p, void** args, cudaStream_t st,
                        uint32_t grid, uint32_t block, uint32_t smem, const char* entry, int min_blocks = 1) {
+  static const bool hdbg = benv("BLU_GBY_DEBUG_HOST") != nullptr;
+  auto hnow = [] { return std::chrono::steady_clock::now(); };
+  const auto h0 = hnow();
   if (!p.jit_ok || !jit_enabled()) return false;
   // 1024-thread CTAs (one per SM, wide hot-key front) keep the same 64-register budget
   // (a 768-thread CTA gets 80 registers: __launch_bounds__(768, 1))
   const int maxt = block > 512 ? (int)block : 512, minb = block > 512 ? 1 : jit_env("BLU_GBY_JIT_MINB", min_blocks);
-  std::string src = "extern \"C\" __global__ void __launch_bounds__(" + std::to_string(maxt) + ", " +
-                    std::to_string(minb) + ") ";
-  src += entry_decl;
-  src += " { ";
-  src += body;
-  src += " }\n";
-  // Launch-path cache: (layout bytes, entry source, device, experiment defines) -> kernel handle, so
-  // repeated executes of a plan skip building the spec source and the source-keyed lookup (host
-  // time the GPU would otherwise sit idle for). The layout bytes are compared on a hit.
-  struct Fast {
+  // Launch-path cache: (layout, entry, launch bounds, shared-table shape, device, experiment knobs)
+  // -> kernel handle, so repeated executes of a plan skip building the kernel and spec sources and
+  // the source-keyed lookup (host time the GPU would otherwise sit idle for). The key is a POD
+  // hashed a word at a time and compared whole on a hit.
+  struct Key {
     Layout lay;
-    std::string src;
+    char entry[64];
+    char body[256];
+    char defs[128];
+    int32_t maxt, minb, dev, hot;
+    uint32_t S, soff[kMaxFields];
+  };
+  struct Fast {
+    Key key;
     const void* k;
     uint32_t smem_ok;
   };
   static std::mutex fmu;
   static std::unordered_map<uint64_t, Fast> fast;
   const bool probe = jit_probe_active();
-  int dev = 0;
-  if (!probe) cudaGetDevice(&dev);
-  const char* defs = getenv("BLU_GBY_JIT_DEFS");
-  std::string tag = src + "|" + std::to_string(dev) + "|" + (defs ? defs : "") + "|" + std::to_string(p.S) +
-                    "|hot" + std::to_string(jit_hot_reg());
-  for (int j = 0; j < p.lay.n_fields; ++j) tag += "," + std::to_string(p.soff[j]);
+  thread_local Key key;  // ~2 KB: not on the stack of every launch
+  memset(&key, 0, sizeof key);
+  memcpy(&key.lay, &p.lay, sizeof key.lay);
+  strncpy(key.entry, entry, sizeof key.entry - 1);
+  strncpy(key.body, body, sizeof key.body - 1);
+  if (const char* defs = benv("BLU_GBY_JIT_DEFS")) strncpy(key.defs, defs, sizeof key.defs - 1);
+  key.maxt = maxt;
+  key.minb = minb;
+  if (!probe) cudaGetDevice(&key.dev);
+  key.hot = jit_hot_reg();
+  key.S = p.S;
+  for (int j = 0; j < p.lay.n_fields; ++j) key.soff[j] = p.soff[j];
   uint64_t h = 1469598103934665603ull;
-  for (size_t i = 0; i < sizeof(Layout); ++i) h = (h ^ ((const uint8_t*)&p.lay)[i]) * 1099511628211ull;
-  for (char c : tag) h = (h ^ (uint8_t)c) * 1099511628211ull;
+  {
+    static_assert(sizeof(Key) % 8 == 0, "key hashed by 8-byte words");
+    const uint64_t* w = (const uint64_t*)&key;
+    for (size_t i = 0; i < sizeof(Key) / 8; ++i) h = (h ^ w[i]) * 1099511628211ull;
+  }
+  const auto h1 = hnow();
   const void* k = nullptr;
   uint32_t smem_ok = 0;
   if (!probe) {
     std::lock_guard<std::mutex> lk(fmu);
     auto it = fast.find(h);
-    if (it != fast.end() && it->second.src == tag && memcmp(&it->second.lay, &p.lay, sizeof(Layout)) == 0) {
+    if (it != fast.end() && memcmp(&it->second.key, &key, sizeof key) == 0) {
       k = it->second.k;
       smem_ok = it->second.smem_ok;
     }
   }
   if (!k) {
+    std::string src = "extern \"C\" __global__ void __launch_bounds__(" + std::to_string(maxt) + ", " +
+                      std::to_string(minb) + ") ";
+    src += entry_decl;
+    src += " { ";
+    src += body;
+    src += " }\n";
     k = jit_kernel(jit_spec("JitSpec", p.lay, p.S, p.soff), src, entry);
     if (probe) return true;  // compile-only probe: nothing is launched
     if (!k) return false;
@@ -109,11 +131,20 @@ static bool launch_jit(const char* body, const char* entry_decl, const AggParams
   {
     std::lock_guard<std::mutex> lk(fmu);
     Fast& f = fast[h];
-    if (f.k != k || f.smem_ok < smem_ok || f.src != tag) f = Fast{p.lay, tag, k, smem_ok};
+    if (f.k != k || f.smem_ok < smem_ok || memcmp(&f.key, &key, sizeof key) != 0) f = Fast{key, k, smem_ok};
   }
+  const auto h2 = hnow();
   if (cudaLaunchKernel(k, dim3(grid), dim3(block), args, smem, st) != cudaSuccess) {
     cudaGetLastError();
     return false;
+  }
+  if (hdbg) {
+    const auto h3 = hnow();
+    auto us = [](std::chrono::steady_clock::time_point a, std::chrono::steady_clock::time_point b) {
+      return std::chrono::duration<double, std::micro>(b - a).count();
+    };
+    fprintf(stderr, "[blugby host] launch_jit us: key %.1f | lookup %.1f | cudaLaunchKernel %.1f\n", us(h0, h1),
+            us(h1, h2), us(h2, h3));
   }
   count_launch(1);
   if (strncmp(entry, "blu_jit_scatter", 15) != 0) note_kernel(entry);

@@ -149,6 +149,7 @@ using namespace blu;
 extern "C" blu_status_t blu_gby_estimate_groups(const blu_key_desc_t* keys, int32_t n_keys, const void* const* key_cols,
                                                 uint64_t n_rows, uint32_t k, void* stream, double* est,
                                                 int32_t* exact) {
+  env_snapshot();
   if (!keys || n_keys < 1 || n_keys > kMaxKeys || !est) return fail(BLU_E_INVALID, "bad estimate arguments");
   if (k < 16 || k > kKmvMaxK) return fail(BLU_E_INVALID, "k must be in [16, %u]", kKmvMaxK);
   if (n_rows && !key_cols) return fail(BLU_E_INVALID, "NULL key columns");

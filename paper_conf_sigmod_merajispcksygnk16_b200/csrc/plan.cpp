@@ -150,7 +150,7 @@ static int device_sms() {
 }
 
 static const char* env(const char* k) {
-  const char* v = getenv(k);
+  const char* v = benv(k);
   return (v && *v) ? v : nullptr;
 }
 
@@ -240,6 +240,7 @@ const char* blu_gby_last_error(void) { return g_last_error.c_str(); }
 
 blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64_t n_rows,
                           blu_gby_plan_t* out_plan) {
+  env_snapshot();
   if (!s || !out_plan) return fail(BLU_E_INVALID, "NULL schema or out_plan");
   *out_plan = nullptr;
   if (s->n_keys < 1 || s->n_keys > kMaxKeys || !s->keys)

@@ -833,6 +833,7 @@ extern "C" {
 
 blu_status_t blu_sort_partial_keys(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t word, uint32_t* keys_out,
                                    void* stream) {
+  env_snapshot();
   if (n && (!rows || !keys_out)) return fail(BLU_E_INVALID, "NULL pointer");
   if (W < 4 || W > 1024 || (W & 3) || 4 * word >= W) return fail(BLU_E_INVALID, "bad W %u / word %u", W, word);
   if (!n) return BLU_OK;
@@ -845,6 +846,7 @@ blu_status_t blu_sort_partial_keys(const uint8_t* rows, uint64_t n, uint32_t W, 
 
 blu_status_t blu_sort_pairs(const uint32_t* keys_in, const uint32_t* payload_in, uint64_t n, uint32_t* keys_out,
                             uint32_t* payload_out, void* stream) {
+  env_snapshot();
   if (n && (!keys_in || !payload_in || !keys_out || !payload_out)) return fail(BLU_E_INVALID, "NULL pointer");
   if (n >= (1ull << 32)) return fail(BLU_E_INVALID, "n >= 2^32");
   if (n && ((const void*)keys_out == (const void*)keys_in || (const void*)payload_out == (const void*)payload_in))
@@ -864,6 +866,7 @@ blu_status_t blu_sort_pairs(const uint32_t* keys_in, const uint32_t* payload_in,
 
 blu_status_t blu_sort_dup_ranges(const uint32_t* sorted_keys, uint64_t n, uint64_t* starts, uint64_t* lens, uint64_t cap,
                                  uint64_t* n_ranges, void* stream) {
+  env_snapshot();
   if (!n_ranges || (n && !sorted_keys) || (cap && (!starts || !lens))) return fail(BLU_E_INVALID, "NULL pointer");
   if (n >= (1ull << 32)) return fail(BLU_E_INVALID, "n >= 2^32");
   uint64_t na = 0;
@@ -874,6 +877,7 @@ blu_status_t blu_sort_dup_ranges(const uint32_t* sorted_keys, uint64_t n, uint64
 
 blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t* perm_out, void* stream,
                            blu_sort_stats_t* stats) {
+  env_snapshot();
   if (n && (!rows || !perm_out)) return fail(BLU_E_INVALID, "NULL pointer");
   if (W < 4 || W > 1024 || (W & 3)) return fail(BLU_E_INVALID, "W must be a multiple of 4 in [4, 1024] (got %u)", W);
   if (n >= (1ull << 32)) return fail(BLU_E_INVALID, "n >= 2^32");
@@ -895,10 +899,10 @@ blu_status_t blu_sort_rows(const uint8_t* rows, uint64_t n, uint32_t W, uint32_t
   };
   // workspace: level-0 keys/payload scratch (u32) + level keys (u64 x3) + payload x3 + pos/seg x2;
   // from the block cache (every level ends with a synchronisation, so it is idle on return)
-  static const bool dbg = getenv("BLU_SORT_DEBUG") != nullptr;
-  const bool no_seg = getenv("BLU_SORT_NO_SEG") != nullptr;  // always the batched global radix sort
-  const bool no_warp = getenv("BLU_SORT_NO_WARP") != nullptr;  // window sort even for ranges <= 256
-  const char* sgw = getenv("BLU_SORT_SEG_W");
+  static const bool dbg = benv("BLU_SORT_DEBUG") != nullptr;
+  const bool no_seg = benv("BLU_SORT_NO_SEG") != nullptr;  // always the batched global radix sort
+  const bool no_warp = benv("BLU_SORT_NO_WARP") != nullptr;  // window sort even for ranges <= 256
+  const char* sgw = benv("BLU_SORT_SEG_W");
   const int seg_w = sgw ? atoi(sgw) : 2048;
   auto hnow = [] {
     timespec ts;
