@@ -767,6 +767,8 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
         // Measured 21.1 vs 19.4 ms for C3 against the per-bucket launches below, so opt-in.
         AggParams q = base;
         q.lay = L2;
+        q.gate = d_gate;  // skipped if the first level overflowed
+        q.gate_run_if = 0;
         q.key[0] = kbuf1;
         for (int c = 0; c < L.n_vals; ++c) q.val[c] = vbuf1[c];
         q.vec_ok = 3;  // segments start at multiples of 4096 rows (>= the second level's tile)
@@ -795,6 +797,8 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
           if (!c1) continue;
           AggParams q = base;
           q.lay = L2;
+          q.gate = d_gate;  // skipped if the first level overflowed
+          q.gate_run_if = 0;
           q.key[0] = (const uint8_t*)kbuf1 + b1 * seg_cap1 * 8;
           for (int c = 0; c < L.n_vals; ++c)
             q.val[c] = (const uint8_t*)vbuf1[c] + b1 * seg_cap1 * dtype_bytes(L.val_dtype[c]);
@@ -1349,12 +1353,13 @@ blu_status_t blu_gby_partition_rows(blu_gby_plan_t P, const void* const* key_col
   }
   Work w(st);
   void* tmp = nullptr;
-  CK(w.alloc(&tmp, 16 * (size_t)n_parts + 16), "partition workspace");
-  CK(cudaMemsetAsync(tmp, 0, 16 * (size_t)n_parts + 16, st), "memset");
+  CK(w.alloc(&tmp, 8 * (size_t)n_parts + 16 + partition_scratch_bytes(n, n_parts)), "partition workspace");
   uint64_t* d_counts = (uint64_t*)tmp;
-  uint64_t* d_offs = d_counts + n_parts;
-  uint32_t* d_flags = (uint32_t*)(d_offs + n_parts);
-  CK(launch_partition(P->lay, key_cols, val_cols, n, n_parts, send_buf, d_counts, d_offs, st, d_flags), "partition rows");
+  uint32_t* d_flags = (uint32_t*)(d_counts + n_parts);
+  CK(cudaMemsetAsync(d_flags, 0, 16, st), "memset");
+  CK(launch_partition(P->lay, key_cols, val_cols, n, n_parts, send_buf, d_counts, (uint8_t*)tmp + 8 * (size_t)n_parts + 16,
+                      st, d_flags),
+     "partition rows");
   uint32_t flags = 0;
   CK(cudaMemcpyAsync(send_counts, d_counts, 8 * (size_t)n_parts, cudaMemcpyDeviceToHost, st), "counts D2H");
   CK(cudaMemcpyAsync(&flags, d_flags, 4, cudaMemcpyDeviceToHost, st), "flags D2H");
@@ -1379,12 +1384,10 @@ blu_status_t blu_gby_partition(blu_gby_plan_t P, const blu_gby_result_t* partial
   }
   Work w(st);
   void* tmp = nullptr;
-  CK(w.alloc(&tmp, 16 * (size_t)n_parts), "partition workspace");
-  CK(cudaMemsetAsync(tmp, 0, 16 * (size_t)n_parts, st), "memset");
+  CK(w.alloc(&tmp, 8 * (size_t)n_parts + 16 + partition_scratch_bytes(partial->n_groups, n_parts)), "partition workspace");
   uint64_t* d_counts = (uint64_t*)tmp;
-  uint64_t* d_offs = d_counts + n_parts;
   CK(launch_partition(P->merge_lay, (const void* const*)partial->key_cols, (const void* const*)partial->state_cols,
-                      partial->n_groups, n_parts, send_buf, d_counts, d_offs, st),
+                      partial->n_groups, n_parts, send_buf, d_counts, (uint8_t*)tmp + 8 * (size_t)n_parts + 16, st),
      "partition");
   CK(cudaMemcpyAsync(send_counts, d_counts, 8 * (size_t)n_parts, cudaMemcpyDeviceToHost, st), "counts D2H");
   CK(cudaStreamSynchronize(st), "sync");

@@ -2003,6 +2003,9 @@ constexpr uint32_t kMaxInSeg = 64;  // first-level buckets of a two-level scatte
 template <class SP, int NV, int R, bool PIPE = false, bool SEGIN = false, bool TMAS = false>
 __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterParams& sp) {
   extern __shared__ __align__(16) uint8_t sm[];
+  // second scatter level: skipped once the first level overflowed a bucket (the chunk then takes the
+  // gated one-pass fallback; an overflowed bucket's region may hold unwritten rows)
+  if (p.gate && ((*(volatile const uint32_t*)p.gate != 0) != (p.gate_run_if != 0))) return;
   const Layout& L = p.lay;
   // histogram bins: the buckets one tile can reach (segmented input: the B2 buckets of its first-level
   // bucket, global index bbase + local bin)

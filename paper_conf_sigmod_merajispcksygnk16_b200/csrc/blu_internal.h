@@ -89,9 +89,14 @@ int launch_front_seed(const AggParams& base, uint64_t n, uint32_t S, uint32_t ra
                       const uint64_t** front_out, const uint64_t** hot_out = nullptr);
 int launch_read_roofline(const void* const* cols, const uint64_t* bytes, int n_cols, void* stream, uint64_t* out,
                          int sms);
-int launch_partition(const Layout& lay, const void* const* key_cols, const void* const* state_cols,
-                     uint64_t n, int32_t n_parts, void* send_buf, uint64_t* d_counts, uint64_t* d_offsets,
-                     void* stream, uint32_t* d_flags = nullptr);
+// S10 owner partition (three launches, no host sync): records of owner o land contiguously at
+// [sum of totals[<o], ...); d_totals (n_parts) receives the per-owner record counts; scratch holds
+// partition_scratch_bytes(n, n_parts) bytes.
+uint32_t partition_ctas(uint64_t n);
+uint64_t partition_scratch_bytes(uint64_t n, int32_t n_parts);
+int launch_partition(const Layout& lay, const void* const* key_cols, const void* const* state_cols, uint64_t n,
+                     int32_t n_parts, void* send_buf, uint64_t* d_totals, void* scratch, void* stream,
+                     uint32_t* d_flags = nullptr);
 
 void count_launch(uint64_t n);
 

@@ -720,8 +720,10 @@ struct PartParams {
   const void* st[kMaxFields];
   uint64_t n;
   int32_t n_parts;
-  uint64_t* counts;   // n_parts (histogram, then cursor)
-  uint64_t* offsets;  // n_parts
+  uint64_t chunk;     // rows per CTA (contiguous range [blockIdx.x * chunk, ...))
+  uint32_t ctas;      // grid size of the count and scatter kernels
+  uint64_t* totals;   // n_parts: records per owner (the send counts)
+  uint64_t* cnt;      // n_parts x ctas, owner-major: CTA c's records for owner o at [o * ctas + c]
   uint64_t* out;
   uint32_t words;
   uint32_t* flags;    // rows mode: FLAG_KEY_RANGE if a key code is outside its dictionary (else NULL)
@@ -763,40 +765,93 @@ __device__ __forceinline__ uint64_t pack_row(const PartParams& p, uint64_t i) {
 
 __device__ __forceinline__ uint32_t owner_of(uint64_t key, int32_t P) { return (uint32_t)__umul64hi(fmix64(key), (uint64_t)P); }
 
-__global__ void __launch_bounds__(256) k_partition_hist(PartParams p) {
-  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.n; i += stride) {
-    if (p.flags && row_keys_bad(p, i)) {
+// S10 owner partition, three launches and no host round trip between them (the send counts are
+// read back once at the end). Each CTA owns a contiguous row range: (1) it counts its rows per owner
+// in shared memory (warp-aggregated: lanes with the same owner add once), no global atomics; (2) one
+// CTA scans the owner-major count matrix into each (owner, CTA) output offset and the per-owner
+// totals; (3) each CTA replays its range and writes every record at its owner's next position
+// (shared cursors, warp-aggregated). Records of one owner keep the CTA order; within a CTA's range
+// their order follows the warp aggregation (any order merges to the same result).
+__device__ __forceinline__ bool part_owner(const PartParams& p, uint64_t i, uint32_t& o, uint64_t& key, uint64_t& key1) {
+  if (p.flags && row_keys_bad(p, i)) return false;
+  key1 = 0;
+  if (p.lay.key_words == 2) {
+    pack_row_wide(p, i, key, key1);
+    o = (uint32_t)__umul64hi(hash128(key, key1), (uint64_t)p.n_parts);
+  } else {
+    key = pack_row(p, i);
+    o = owner_of(key, p.n_parts);
+  }
+  return true;
+}
+
+__global__ void __launch_bounds__(256) k_partition_count(PartParams p) {
+  __shared__ uint32_t hist[1024];
+  for (int o = threadIdx.x; o < p.n_parts; o += blockDim.x) hist[o] = 0;
+  __syncthreads();
+  const uint64_t r0 = (uint64_t)blockIdx.x * p.chunk, r1 = min(p.n, r0 + p.chunk);
+  for (uint64_t b = r0; b < r1; b += blockDim.x) {
+    const uint64_t i = b + threadIdx.x;
+    uint32_t o = 0xFFFFFFFFu;
+    uint64_t k0, k1;
+    if (i < r1 && !part_owner(p, i, o, k0, k1)) {
       atomicOr(p.flags, FLAG_KEY_RANGE);
-      continue;
+      o = 0xFFFFFFFFu;
     }
-    uint32_t o;
-    if (p.lay.key_words == 2) {
-      uint64_t w0, w1;
-      pack_row_wide(p, i, w0, w1);
-      o = (uint32_t)__umul64hi(hash128(w0, w1), (uint64_t)p.n_parts);
-    } else {
-      o = owner_of(pack_row(p, i), p.n_parts);
+    const unsigned peers = __match_any_sync(0xffffffffu, o);
+    if (o != 0xFFFFFFFFu && (threadIdx.x & 31) == (unsigned)(__ffs(peers) - 1)) atomicAdd(&hist[o], (uint32_t)__popc(peers));
+  }
+  __syncthreads();
+  for (int o = threadIdx.x; o < p.n_parts; o += blockDim.x) p.cnt[(uint64_t)o * p.ctas + blockIdx.x] = hist[o];
+}
+
+// one CTA: thread o (< n_parts <= 1024) sums owner o's row of the matrix, a block scan gives the
+// owner bases, then the row is rewritten as exclusive offsets
+__global__ void __launch_bounds__(1024) k_partition_scan(PartParams p) {
+  __shared__ uint64_t tot[1024];
+  const int o = threadIdx.x;
+  uint64_t t = 0;
+  if (o < p.n_parts)
+    for (uint32_t c = 0; c < p.ctas; ++c) t += p.cnt[(uint64_t)o * p.ctas + c];
+  tot[o] = t;
+  __syncthreads();
+  for (int d = 1; d < 1024; d <<= 1) {  // inclusive Hillis-Steele scan over the owners
+    const uint64_t x = o >= d ? tot[o - d] : 0;
+    __syncthreads();
+    tot[o] += x;
+    __syncthreads();
+  }
+  if (o < p.n_parts) {
+    p.totals[o] = t;
+    uint64_t run = tot[o] - t;
+    for (uint32_t c = 0; c < p.ctas; ++c) {
+      uint64_t* q = p.cnt + (uint64_t)o * p.ctas + c;
+      const uint64_t x = *q;
+      *q = run;
+      run += x;
     }
-    atomicAdd((unsigned long long*)&p.counts[o], 1ull);
   }
 }
 
 __global__ void __launch_bounds__(256) k_partition_scatter(PartParams p) {
-  uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < p.n; i += stride) {
-    if (p.flags && row_keys_bad(p, i)) continue;
-    const int kw = p.lay.key_words == 2 ? 2 : 1;
+  __shared__ unsigned long long cur[1024];
+  for (int o = threadIdx.x; o < p.n_parts; o += blockDim.x) cur[o] = p.cnt[(uint64_t)o * p.ctas + blockIdx.x];
+  __syncthreads();
+  const int kw = p.lay.key_words == 2 ? 2 : 1;
+  const unsigned lane = threadIdx.x & 31;
+  const uint64_t r0 = (uint64_t)blockIdx.x * p.chunk, r1 = min(p.n, r0 + p.chunk);
+  for (uint64_t b = r0; b < r1; b += blockDim.x) {
+    const uint64_t i = b + threadIdx.x;
+    uint32_t o = 0xFFFFFFFFu;
     uint64_t key = 0, key1 = 0;
-    uint32_t o;
-    if (kw == 2) {
-      pack_row_wide(p, i, key, key1);
-      o = (uint32_t)__umul64hi(hash128(key, key1), (uint64_t)p.n_parts);
-    } else {
-      key = pack_row(p, i);
-      o = owner_of(key, p.n_parts);
-    }
-    uint64_t pos = p.offsets[o] + atomicAdd((unsigned long long*)&p.counts[o], 1ull);
+    if (i < r1 && !part_owner(p, i, o, key, key1)) o = 0xFFFFFFFFu;
+    const unsigned peers = __match_any_sync(0xffffffffu, o);
+    const int leader = __ffs(peers) - 1;
+    unsigned long long base = 0;
+    if (o != 0xFFFFFFFFu && (int)lane == leader) base = atomicAdd(&cur[o], (unsigned long long)__popc(peers));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    if (o == 0xFFFFFFFFu) continue;
+    const uint64_t pos = base + __popc(peers & ((1u << lane) - 1u));
     uint64_t* rec = p.out + pos * p.words;
     rec[0] = key;
     if (kw == 2) rec[1] = key1;
@@ -1262,12 +1317,18 @@ int launch_compact(const CompactParams& p, void* stream, uint32_t* launches) {
   return (int)cudaGetLastError();
 }
 
+uint64_t partition_scratch_bytes(uint64_t n, int32_t n_parts) {
+  return (uint64_t)n_parts * partition_ctas(n) * 8 + 64;
+}
+
+uint32_t partition_ctas(uint64_t n) {
+  const uint64_t by_rows = (n + 4095) / 4096;  // >= 4096 rows per CTA
+  return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(by_rows, 148 * 8));
+}
+
 int launch_partition(const Layout& lay, const void* const* key_cols, const void* const* state_cols, uint64_t n,
-                     int32_t n_parts, void* send_buf, uint64_t* d_counts, uint64_t* d_offsets, void* stream,
+                     int32_t n_parts, void* send_buf, uint64_t* d_totals, void* scratch, void* stream,
                      uint32_t* d_flags) {
-  // two-phase: histogram -> (host) offsets -> scatter. The caller passes d_counts zeroed; this
-  // launcher runs the histogram, copies counts to the host, scans, uploads offsets, re-zeroes the
-  // cursors and scatters.
   cudaStream_t st = (cudaStream_t)stream;
   PartParams p{};
   p.lay = lay;
@@ -1275,25 +1336,17 @@ int launch_partition(const Layout& lay, const void* const* key_cols, const void*
   for (int j = 0; j < lay.n_vals; ++j) p.st[j] = state_cols[j];
   p.n = n;
   p.n_parts = n_parts;
-  p.counts = d_counts;
-  p.offsets = d_offsets;
+  p.ctas = partition_ctas(n);
+  p.chunk = (n + p.ctas - 1) / p.ctas;
+  p.totals = d_totals;
+  p.cnt = (uint64_t*)scratch;
   p.out = (uint64_t*)send_buf;
   p.words = (lay.key_words == 2 ? 2 : 1) + lay.n_vals;
   p.flags = d_flags;
-  int grid = grid_for(n, 256, 148 * 8);
-  k_partition_hist<<<grid, 256, 0, st>>>(p);
-  count_launch(1);
-  uint64_t h_counts[1024];
-  cudaMemcpyAsync(h_counts, d_counts, sizeof(uint64_t) * n_parts, cudaMemcpyDeviceToHost, st);
-  cudaStreamSynchronize(st);
-  uint64_t h_off[1024];
-  uint64_t acc = 0;
-  for (int i = 0; i < n_parts; ++i) { h_off[i] = acc; acc += h_counts[i]; }
-  cudaMemcpyAsync(d_offsets, h_off, sizeof(uint64_t) * n_parts, cudaMemcpyHostToDevice, st);
-  cudaMemsetAsync(d_counts, 0, sizeof(uint64_t) * n_parts, st);
-  k_partition_scatter<<<grid, 256, 0, st>>>(p);
-  count_launch(1);
-  cudaStreamSynchronize(st);
+  k_partition_count<<<p.ctas, 256, 0, st>>>(p);
+  k_partition_scan<<<1, 1024, 0, st>>>(p);
+  k_partition_scatter<<<p.ctas, 256, 0, st>>>(p);
+  count_launch(3);
   return (int)cudaGetLastError();
 }
 

@@ -398,6 +398,48 @@ def test_partition_records_exchange(bg, oracles, name):
                   o, w.schema)
 
 
+def _owner_np(keys: np.ndarray, P: int) -> np.ndarray:
+    """S2 owner = mulhi(fmix64(key), P), uint64 arithmetic in numpy."""
+    h = keys.astype(np.uint64)
+    with np.errstate(over="ignore"):
+        h ^= h >> np.uint64(33)
+        h *= np.uint64(0xff51afd7ed558ccd)
+        h ^= h >> np.uint64(33)
+        h *= np.uint64(0xc4ceb9fe1a85ec53)
+        h ^= h >> np.uint64(33)
+    a = (h >> np.uint64(32)) * np.uint64(P)
+    b = ((h & np.uint64(0xFFFFFFFF)) * np.uint64(P)) >> np.uint64(32)
+    return ((a + b) >> np.uint64(32)).astype(np.int64)
+
+
+@pytest.mark.parametrize("n", [1, 4097, 1_000_003])
+@pytest.mark.parametrize("P", [1, 3, 8, 1024])
+def test_partition_rows_layout(bg, n, P):
+    """S10 owner partition (count / scan / scatter kernels): the send buffer holds owner 0's records,
+    then owner 1's, ...; every record lands in its key's owner bucket (owner computed here in numpy),
+    the counts match, and the records are exactly the input rows (as a multiset)."""
+    rng = np.random.default_rng(n + P)
+    sch = blugen.Schema([(I64, 0)], [I64, F64], [(COUNT, -1), (SUM, 0), (AVG, 1)])
+    k = rng.integers(0, 2**62, n).astype(np.int64)
+    v = [rng.integers(-(2**40), 2**40, n), rng.integers(-(2**20), 2**20, n) / 64.0]
+    plan = bg.plan_for(sch, n, n)
+    words = plan.row_record_bytes // 8
+    assert words == 3
+    dk, dv = _mk([k], v)
+    send = torch.empty(n * words, dtype=torch.int64, device="cuda")
+    counts = bg.blu_gby_partition_rows(plan, dk, dv, P, send)
+    assert len(counts) == P and sum(counts) == n
+    own = _owner_np(k, P)
+    assert np.array_equal(np.bincount(own, minlength=P), np.array(counts))
+    recs = send.cpu().numpy().reshape(n, words)
+    starts = np.concatenate([[0], np.cumsum(counts)])
+    for o in range(P):
+        assert np.all(_owner_np(recs[starts[o]:starts[o + 1], 0], P) == o)
+    got = recs[np.lexsort(recs.T[::-1])]
+    exp = np.stack([k, v[0], v[1].view(np.int64)], axis=1)
+    assert np.array_equal(got, exp[np.lexsort(exp.T[::-1])])
+
+
 @pytest.mark.parametrize("name", ["C1", "C2", "C4"])
 def test_dense_state_accumulate_and_finalize(bg, oracles, name):
     """Path (a)/(b') multi-GPU helpers on one GPU: 3 shards accumulate into one dense state."""
