@@ -1,6 +1,9 @@
 """Phase timing of one config through libblugby (wall clock vs CUDA-event phases). Dev tool."""
 import os, sys, time, json
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+if os.environ.get("OLD"):  # same-run A/B: the package built from an earlier revision under _oldpkg/
+    sys.path.insert(0, os.path.join(ROOT, "_oldpkg"))
 import torch, blugen
 from paper_conf_sigmod_merajispcksygnk16_b200 import blugby as bg
 cfg = sys.argv[1] if len(sys.argv) > 1 else "C3"
