@@ -539,7 +539,8 @@ def test_launch_count_and_timing(bg):
 
 @pytest.mark.parametrize("smem", ["1", "0"])
 @pytest.mark.parametrize("parts,chunk,div", [("8", None, None), ("16", "300000", None), ("64", "1000003", None),
-                                             ("2", None, None), ("256", None, "7"), ("128", "700001", "64")])
+                                             ("2", None, None), ("256", None, "7"), ("128", "700001", "64"),
+                                             ("32", None, "2")])
 def test_partitioned_two_pass(bg, oracles, monkeypatch, parts, chunk, div, smem):
     """Path (b) partitioned mode: scatter into buckets by slot bits, then bucket-by-bucket
     aggregation — in per-CTA shared-memory bucket tables merged once per piece (smem=1; with 2
