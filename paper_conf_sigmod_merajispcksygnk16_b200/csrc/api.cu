@@ -832,6 +832,9 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
     p2.seg_count = d_cursor;
     p2.n_segs = B;
     p2.tile_ctr = benv("BLU_GBY_DYN") && atoi(benv("BLU_GBY_DYN")) == 0 ? nullptr : (uint64_t*)(d_cursor + B + 1);
+    // bucket tables: TMA bulk L2 prefetch of the piece's tile this many tiles ahead (0 = off)
+    p2.prefetch = P->part_smem ? (benv("BLU_GBY_BUCKET_PF") ? (uint32_t)atoi(benv("BLU_GBY_BUCKET_PF")) : 1u)
+                               : (benv("BLU_GBY_SEG_PF") ? (uint32_t)atoi(benv("BLU_GBY_SEG_PF")) : 0u);
     if (const char* g = benv("BLU_GBY_GRAB")) p2.grab = (uint32_t)atoi(g);
     p2.gate = d_gate;
     p2.gate_run_if = 0;

@@ -284,6 +284,32 @@ __device__ __forceinline__ void prefetch_warp_rows_l2(const AggParams& p, uint64
   }
 }
 
+// Bulk L2 prefetch of a contiguous byte range by the TMA unit (one instruction for the whole range):
+// cp.async.bulk.prefetch.L2 needs a 16-byte aligned address and a multiple of 16 bytes.
+__device__ __forceinline__ void bulk_prefetch_l2(const void* p, uint64_t bytes) {
+  const uintptr_t a0 = (uintptr_t)p & ~(uintptr_t)15, a1 = ((uintptr_t)p + bytes + 15) & ~(uintptr_t)15;
+  if (a1 > a0)
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"((uint32_t)(a1 - a0)) : "memory");
+}
+
+// Rows [r0, r1) of every key and value column prefetched into L2 by the TMA unit (JIT kernels).
+template <class SP>
+__device__ __forceinline__ void bulk_prefetch_rows_l2(const AggParams& p, uint64_t r0, uint64_t r1) {
+  if constexpr (SP::kStatic) {
+    if (r0 >= r1) return;
+    sfor<0, SP::NK>([&](auto kc) {
+      constexpr int k = decltype(kc)::v;
+      constexpr uint64_t w = SP::KDT[k] == BLU_I32 ? 4 : 8;
+      bulk_prefetch_l2((const uint8_t*)p.key[k] + r0 * w, (r1 - r0) * w);
+    });
+    sfor<0, SP::NV>([&](auto cc) {
+      constexpr int c = decltype(cc)::v;
+      constexpr uint64_t w = SP::VDT[c] == BLU_I32 ? 4 : 8;
+      bulk_prefetch_l2((const uint8_t*)p.val[c] + r0 * w, (r1 - r0) * w);
+    });
+  }
+}
+
 // Shared-memory table (path (a) and the hot-key front): SoA per field, S entries per field.
 // Encodings: COUNT u32; SUMI as two u32 arrays lo[S], hi[S] — native 32-bit ATOMS with an explicit
 // carry (64-bit shared atomics are CAS loops on sm_100a); SUMF f64 (CAS loop);
@@ -1596,6 +1622,24 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
     chunk_next = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;  // prefetched
     t = chunk * kGrab;
   }
+  // SEG with p.prefetch: lane 0 has the warp's next claimed chunk; its rows (within their bucket)
+  // go DRAM -> L2 by the TMA unit while the current chunk is worked on (BLU_GBY_SEG_PF)
+  auto seg_prefetch = [&](uint64_t cn) {
+    if constexpr (SEG && SP::kStatic) {
+      if (p.prefetch && lane == 0 && cn * kGrab < ntiles) {
+        const uint64_t tt = cn * kGrab;
+        uint32_t lo = 0, hi = p.n_segs - 1;
+        while (lo < hi) {
+          const uint32_t mid = (lo + hi + 1) >> 1;
+          if (tpre[mid] <= tt) lo = mid; else hi = mid - 1;
+        }
+        const uint64_t a = (uint64_t)lo * p.seg_stride + (tt - tpre[lo]) * tile;
+        const uint64_t end = (uint64_t)lo * p.seg_stride + p.seg_count[lo];
+        bulk_prefetch_rows_l2<SP>(p, a, a + (uint64_t)kGrab * tile < end ? a + (uint64_t)kGrab * tile : end);
+      }
+    }
+  };
+  if (dyn) seg_prefetch(chunk_next);
   if constexpr (MODE == 3) {  // software-pipelined row stream (see RawTile)
     const uint64_t n = p.n_rows;
     const unsigned warp = threadIdx.x >> 5;
@@ -1642,6 +1686,7 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
         chunk = __shfl_sync(0xffffffffu, chunk_next, 0);
         t_next = chunk * kGrab;
         chunk_next = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;
+        seg_prefetch(chunk_next);
       }
       const uint32_t fl = *(volatile uint32_t*)p.flags;
       if (t_next < ntiles) {
@@ -1674,6 +1719,7 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
         chunk = __shfl_sync(0xffffffffu, chunk_next, 0);
         t_next = chunk * kGrab;
         chunk_next = lane == 0 ? atomicAdd((unsigned long long*)p.tile_ctr, 1ull) : 0ull;
+        seg_prefetch(chunk_next);
       }
       uint32_t lo = 0, hi = p.n_segs - 1;
       while (lo < hi) {
@@ -1879,6 +1925,20 @@ __device__ __forceinline__ void bucket_body(const AggParams& p) {
       if (r0 < r1) tile_load<SP, R>(p, lane_base<R>(r0, warp, lane), r1, pol, A);
     for (uint64_t row0 = r0; row0 < r1; row0 += tile) {
       const uint64_t row = lane_base<R>(row0, warp, lane);
+      if constexpr (SP::kStatic) {
+        if (p.prefetch && threadIdx.x == 0) {  // the tile p.prefetch tiles ahead: DRAM -> L2 by the TMA unit
+          const uint64_t a = row0 + (uint64_t)p.prefetch * tile;
+          if (a < r1) {
+            const uint64_t m = r1 - a < tile ? r1 - a : tile;
+            bulk_prefetch_l2((const uint64_t*)p.key[0] + a, m * 8);
+            sfor<0, SP::NV>([&](auto cc) {
+              constexpr int c = decltype(cc)::v;
+              constexpr uint64_t w = SP::VDT[c] == BLU_I32 ? 4 : 8;
+              bulk_prefetch_l2((const uint8_t*)p.val[c] + a * w, m * w);
+            });
+          }
+        }
+      }
       uint64_t key[R];
       uint64_t v[NV][R];
       uint32_t valid;
@@ -2077,6 +2137,13 @@ __device__ __forceinline__ void scatter_body(const AggParams& p, const ScatterPa
     if (!PIPE && p.prefetch) {  // a later tile of this CTA: in flight during the sort and the writes below
       const uint64_t nt = t + (uint64_t)gridDim.x * p.prefetch;
       prefetch_rows_l2<SP>(p, nt * TILE, nt * TILE + TILE < n ? nt * TILE + TILE : n);
+    }
+    if (PIPE && p.prefetch > 1 && threadIdx.x == 0) {  // beyond the register-pipelined next tile: TMA L2 prefetch
+      const uint64_t nt = t + (uint64_t)gridDim.x * p.prefetch;
+      if (nt < ntiles) {
+        const uint64_t lim2 = tile_lim(nt);
+        bulk_prefetch_rows_l2<SP>(p, nt * TILE, nt * TILE + TILE < lim2 ? nt * TILE + TILE : lim2);
+      }
     }
     uint32_t bb[R], pos[R];
 #pragma unroll
