@@ -633,7 +633,9 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   // into B / B1 second-level buckets by a second scatter, instead of one B-way scatter (a 2048-way
   // scatter writes ~2 rows per bucket per tile); needs a second set of partition buffers
   const char* tl = benv("BLU_GBY_PART_2LEVEL");
-  const uint32_t B1 = (P->part_smem && !(tl && tl[0] == '0') && B >= 256) ? 32u : 0u;
+  uint32_t B1 = (P->part_smem && !(tl && tl[0] == '0') && B >= 256) ? two_level_b1(B) : 0u;
+  if (const char* b1 = benv("BLU_GBY_PART_B1"))  // experiment: first-level fan-out (power of two < B)
+    if (B1 && atoi(b1) >= 2 && (uint32_t)atoi(b1) < B && !((uint32_t)atoi(b1) & ((uint32_t)atoi(b1) - 1))) B1 = (uint32_t)atoi(b1);
   if (B1) M = std::max<uint64_t>(M / 2, 1ull << 22);
   M = std::min<uint64_t>(n, M);
   if (const char* cr = benv("BLU_GBY_PART_CHUNK")) M = std::min<uint64_t>(n, std::max<uint64_t>(1024, strtoull(cr, 0, 10)));
@@ -785,7 +787,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
         if (le) return (cudaError_t)le;
       } else {
         // second level per first-level bucket: one host read of the B1 counts, then B1 launches
-        uint64_t* hc = B1 <= 32 ? pinned_scratch() : nullptr;  // 256 pinned bytes
+        uint64_t* hc = B1 <= 32 ? pinned_scratch() : nullptr;  // 256 pinned bytes (else pageable)
         std::vector<uint64_t> cnt1(B1);
         if ((e = cudaMemcpyAsync(hc ? (void*)hc : (void*)cnt1.data(), d_cursor1, (size_t)B1 * 8, cudaMemcpyDeviceToHost,
                                  st)))

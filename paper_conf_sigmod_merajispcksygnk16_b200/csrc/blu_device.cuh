@@ -2056,7 +2056,7 @@ __device__ __forceinline__ void block_excl_scan(uint32_t* a, uint32_t* out, uint
   }
 }
 
-constexpr uint32_t kMaxInSeg = 64;  // first-level buckets of a two-level scatter (the planner uses 32)
+constexpr uint32_t kMaxInSeg = 256;  // first-level buckets of a two-level scatter (32 or 128)
 
 // PIPE (NVRTC kernels only): the next tile's rows are loaded into registers as soon as the current
 // tile is staged in shared memory, so those HBM reads are in flight during its write-out phase.

@@ -59,7 +59,7 @@ constexpr uint64_t kRowLockRatio = 16;          // kernel 3 when rows/groups <= 
 constexpr uint32_t kPartBudgetMB = 48;          // L2 slice per bucket (126 MB L2)
 constexpr uint32_t kSmemMax = 232448;           // dynamic shared memory per CTA (227 KB opt-in)
 constexpr uint32_t kMaxBuckets = 4096;          // one-pass scatter fan-out
-constexpr uint32_t kMaxBuckets2 = 16384;        // two-level scatter (32 x 512)
+constexpr uint32_t kMaxBuckets2 = 16384;        // two-level scatter (128 x 128)
 constexpr double kBucketLoad = 0.7;             // mean groups per bucket / bucket table entries
 constexpr uint32_t kMaxSlotBytes = 256;         // AoS slot limit (init template size)
 
@@ -455,14 +455,16 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     };
     // smallest B whose buckets hold <= kBucketLoad * S groups on average, within the scatter's
     // shared memory and <= kMaxBuckets; the records' layout has the same fields as L
-    // two_level: the fan-outs are 32 and b / 32 (api.cu), so b may exceed the one-pass limit
+    // two_level: the fan-outs are two_level_b1(b) and b / two_level_b1(b) (api.cu), so b may exceed the
+    // one-pass limit; widest = the larger histogram of the two levels
+    auto widest = [&](bool two_level, uint64_t b) {
+      return (uint32_t)(two_level && b >= 256 ? std::max<uint64_t>(two_level_b1(b), b / two_level_b1(b)) : b);
+    };
     auto smem_B = [&](bool two_level, bool cap_default = false) {
       const uint64_t max_b = two_level && !cap_default ? kMaxBuckets2 : kMaxBuckets;
       uint64_t b = 2;
       while (b < max_b && (double)P->est_groups > kBucketLoad * S_of((uint32_t)b) * (double)b &&
-             scatter_smem(L.n_vals, (uint32_t)(two_level && b >= 256 ? std::max<uint64_t>(64, 2 * b / 32) : b * 2)) <=
-                 kSmemMax &&
-             b * 2 <= P->cap / 1024)
+             scatter_smem(L.n_vals, widest(two_level, 2 * b)) <= kSmemMax && b * 2 <= P->cap / 1024)
         b <<= 1;
       return b;
     };
@@ -472,9 +474,10 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     if (const char* ps = env("BLU_GBY_PART_SMEM")) {
       smem_mode = !L.lock_off && ps[0] == '1';
     } else if (!L.lock_off && budget && tbytes > budget && !env("BLU_GBY_PARTS") && two_ok) {
-      // default only up to kMaxBuckets: C5 (5*10^7 groups) in 16384 tables behind a 32 x 512 scatter
-      // measured 45.5 ms per 10^9 rows against 36.7 ms in the L2-slice mode (the 512-way second level
-      // and the smaller tables cost more than the L2 atomics they save)
+      // default only up to kMaxBuckets: C5 (5*10^7 groups) in 16384 tables behind a 128 x 128 scatter
+      // measured 147.4 vs 148.1-148.6 ms for 4*10^9 rows in the L2-slice mode (58.9 vs 61.4 ms at
+      // 1.6*10^9; a 32 x 512 scatter made it 74.3 ms): within noise at full size, so C5 keeps the L2
+      // mode and BLU_GBY_PART_SMEM=1 selects the tables
       const uint64_t b = smem_B(true, true);
       smem_mode = b >= 256 && (double)P->est_groups <= kBucketLoad * S_of((uint32_t)b) * (double)b;
     }
@@ -483,8 +486,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     if (smem_mode && ((budget && tbytes > budget) || (forced && atoi(forced) > 1))) {
       B = smem_B(two_ok, !env("BLU_GBY_PART_SMEM"));
       if (forced) B = std::max(2, std::min((int)(two_ok ? kMaxBuckets2 : kMaxBuckets), atoi(forced)));
-      auto widest = [&](uint64_t b) { return (uint32_t)(two_ok && b >= 256 ? std::max<uint64_t>(32, b / 32) : b); };
-      while (B > 2 && scatter_smem(L.n_vals, widest(B)) > kSmemMax) B >>= 1;  // histogram bins per tile
+      while (B > 2 && scatter_smem(L.n_vals, widest(two_ok, B)) > kSmemMax) B >>= 1;  // histogram bins per tile
       P->part_smem = 1;
       P->bucket_S = S_of((uint32_t)B);
       P->bucket_smem = bucket_smem_bytes(L, P->bucket_S, (uint32_t)B);

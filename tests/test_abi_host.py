@@ -104,7 +104,8 @@ def test_planner_paths_for_the_five_configs(bg):
 
 
 def test_planner_partitioned_l2_mode(bg, monkeypatch):
-    """C5's 5*10^7 groups need more than 4096 bucket tables (16384 measured slower than the L2 mode)
+    """C5's 5*10^7 groups need more than 4096 bucket tables (16384 behind a 128 x 128 scatter measured
+    even with the L2 mode at full size, so the default stays there; BLU_GBY_PART_SMEM=1 selects them)
     and K3's 8-field states do not fit either: both keep pass 2 in L2-resident slices of the global
     table, sized at load <= 0.5; BLU_GBY_PART_SMEM=0 forces that mode for C3 too."""
     c5 = _plan(bg, blugen.workload("C5")).info()

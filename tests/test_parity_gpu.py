@@ -637,6 +637,29 @@ def test_host_results_pinned_reuse(bg, oracles):
         assert_parity(gk, ga, o, sch)
 
 
+@pytest.mark.parametrize("one", ["0", "1"])
+def test_partitioned_two_level_128(bg, monkeypatch, one):
+    """More than 4096 bucket tables: the two-level scatter splits 128 x B/128 (8192 buckets = 128 x 64
+    here; C5's forced shared-memory mode is 128 x 128), per-bucket second-level launches or one
+    segmented launch; 40M rows into 4M groups, against the oracle."""
+    w = blugen.workload("C3", n_rows=40_000_003, n_groups=4_000_000)
+    o = oracle.groupby_generated(w)
+    kc, vc = blugen.device_columns(w)
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
+    monkeypatch.setenv("BLU_GBY_PARTS", "8192")
+    monkeypatch.setenv("BLU_GBY_2LEVEL_ONE", one)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    info = plan.info()
+    assert info["part_smem"] == 1 and info["partitions"] == 8192, info
+    bg.blu_gby_set_timing(True)
+    res = bg.blu_gby_execute(plan, kc, vc)
+    t = bg.blu_gby_last_timing()
+    bg.blu_gby_set_timing(False)
+    assert t["part_chunks"] == 1 and t["part_fallbacks"] == 0, t
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
 @pytest.mark.parametrize("two_level", ["0", "1", "1-one"])
 @pytest.mark.parametrize("parts", [None, "4096"])
 def test_partitioned_wide_fanout(bg, monkeypatch, parts, two_level):
