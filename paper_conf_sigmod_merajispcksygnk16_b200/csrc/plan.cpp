@@ -60,6 +60,7 @@ constexpr uint32_t kPartBudgetMB = 48;          // L2 slice per bucket (126 MB L
 constexpr uint32_t kSmemMax = 232448;           // dynamic shared memory per CTA (227 KB opt-in)
 constexpr uint32_t kMaxBuckets = 4096;          // one-pass scatter fan-out
 constexpr uint32_t kMaxBuckets2 = 16384;        // two-level scatter (128 x 128)
+constexpr bool kSmemDefault2 = true;             // bucket tables by default up to kMaxBuckets2 (C5)
 constexpr double kBucketLoad = 0.7;             // mean groups per bucket / bucket table entries
 constexpr uint32_t kMaxSlotBytes = 256;         // AoS slot limit (init template size)
 
@@ -474,17 +475,16 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     if (const char* ps = env("BLU_GBY_PART_SMEM")) {
       smem_mode = !L.lock_off && ps[0] == '1';
     } else if (!L.lock_off && budget && tbytes > budget && !env("BLU_GBY_PARTS") && two_ok) {
-      // default only up to kMaxBuckets: C5 (5*10^7 groups) in 16384 tables behind a 128 x 128 scatter
-      // measured 147.4 vs 148.1-148.6 ms for 4*10^9 rows in the L2-slice mode (58.9 vs 61.4 ms at
-      // 1.6*10^9; a 32 x 512 scatter made it 74.3 ms): within noise at full size, so C5 keeps the L2
-      // mode and BLU_GBY_PART_SMEM=1 selects the tables
-      const uint64_t b = smem_B(true, true);
+      // up to kMaxBuckets2: C5 (5*10^7 groups) in 16384 tables behind a 128 x 128 scatter (second
+      // level over two streams) 57.1 vs 61.4 ms per 1.6*10^9 rows in the L2-slice mode (a 32 x 512
+      // scatter made it 74.3 ms)
+      const uint64_t b = smem_B(true, !kSmemDefault2);
       smem_mode = b >= 256 && (double)P->est_groups <= kBucketLoad * S_of((uint32_t)b) * (double)b;
     }
     uint64_t B = 1;
     const char* forced = env("BLU_GBY_PARTS");
     if (smem_mode && ((budget && tbytes > budget) || (forced && atoi(forced) > 1))) {
-      B = smem_B(two_ok, !env("BLU_GBY_PART_SMEM"));
+      B = smem_B(two_ok, !env("BLU_GBY_PART_SMEM") && !kSmemDefault2);
       if (forced) B = std::max(2, std::min((int)(two_ok ? kMaxBuckets2 : kMaxBuckets), atoi(forced)));
       while (B > 2 && scatter_smem(L.n_vals, widest(two_ok, B)) > kSmemMax) B >>= 1;  // histogram bins per tile
       P->part_smem = 1;

@@ -104,12 +104,12 @@ def test_planner_paths_for_the_five_configs(bg):
 
 
 def test_planner_partitioned_l2_mode(bg, monkeypatch):
-    """C5's 5*10^7 groups need more than 4096 bucket tables (16384 behind a 128 x 128 scatter measured
-    even with the L2 mode at full size, so the default stays there; BLU_GBY_PART_SMEM=1 selects them)
-    and K3's 8-field states do not fit either: both keep pass 2 in L2-resident slices of the global
-    table, sized at load <= 0.5; BLU_GBY_PART_SMEM=0 forces that mode for C3 too."""
+    """K3's 8-field states need more than the 16384 bucket tables a two-level scatter reaches: pass 2
+    in L2-resident slices of the global table, sized at load <= 0.5. C5's 5*10^7 groups fit 16384
+    tables behind a 128 x 128 scatter (the default, 141 vs 148 ms for the L2 mode at 4e9 rows);
+    BLU_GBY_PART_SMEM=0 forces the L2 mode for C5 and C3."""
     c5 = _plan(bg, blugen.workload("C5")).info()
-    assert c5["part_smem"] == 0 and c5["partitions"] >= 64
+    assert c5["part_smem"] == 1 and c5["partitions"] == 16384
     k3 = _plan(bg, blugen.workload("K3")).info()
     assert k3["part_smem"] == 0 and k3["partitions"] > 1
     monkeypatch.setenv("BLU_GBY_PART_SMEM", "0")
