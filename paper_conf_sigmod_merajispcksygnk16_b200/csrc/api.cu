@@ -799,8 +799,14 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
         // per 1.6e9 rows; 3 streams: the same); the host sync above orders them after the first level,
         // and st waits for every auxiliary stream before pass 2
         int ns = benv("BLU_GBY_2LEVEL_STREAMS") ? std::max(1, std::min(4, atoi(benv("BLU_GBY_2LEVEL_STREAMS")))) : 2;
-        thread_local cudaStream_t aux[3] = {nullptr, nullptr, nullptr};
-        thread_local cudaEvent_t aux_ev[3] = {nullptr, nullptr, nullptr};
+        // per thread and device (streams and events belong to the device current at creation)
+        thread_local cudaStream_t aux_all[16][3] = {};
+        thread_local cudaEvent_t aux_ev_all[16][3] = {};
+        int dev_now = 0;
+        cudaGetDevice(&dev_now);
+        if (dev_now < 0 || dev_now >= 16) ns = 1;
+        cudaStream_t* aux = aux_all[dev_now & 15];
+        cudaEvent_t* aux_ev = aux_ev_all[dev_now & 15];
         for (int i = 0; i + 1 < ns; ++i)
           if (!aux[i] && (cudaStreamCreateWithFlags(&aux[i], cudaStreamNonBlocking) != cudaSuccess ||
                           cudaEventCreateWithFlags(&aux_ev[i], cudaEventDisableTiming) != cudaSuccess)) {
