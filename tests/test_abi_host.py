@@ -310,3 +310,25 @@ def test_planner_rejects_slots_over_256_bytes(bg):
     assert e.value.status == bg.BLU_E_UNSUPPORTED
     ok = bg.blu_gby_plan([(I64, 0)], [I128] * 15, [(SUM, c) for c in range(15)], 1000, 10**6).info()
     assert ok["slot_bytes"] == 256
+
+
+def test_env_knobs_follow_the_environment_per_call(bg, monkeypatch):
+    """BLU_* knobs come from a per-API-call snapshot of the environment (csrc/env.cpp): a change is
+    seen by the next call, a removal too, and another thread sees its process environment as well."""
+    import threading
+    w = blugen.workload("C2")
+    monkeypatch.delenv("BLU_GBY_FORCE_PATH", raising=False)
+    assert _plan(bg, w).info()["path"] == bg.BLU_PATH_DENSE_SMEM
+    monkeypatch.setenv("BLU_GBY_FORCE_PATH", "b")
+    assert _plan(bg, w).info()["path"] == bg.BLU_PATH_HASH_GLOBAL
+    monkeypatch.setenv("BLU_GBY_FORCE_PATH", "d")
+    assert _plan(bg, w).info()["path"] == bg.BLU_PATH_DIRECT_GLOBAL
+    out = {}
+    t = threading.Thread(target=lambda: out.setdefault("path", _plan(bg, w).info()["path"]))
+    t.start()
+    t.join()
+    assert out["path"] == bg.BLU_PATH_DIRECT_GLOBAL
+    monkeypatch.setenv("BLU_GBY_FORCE_PATH", "b")
+    assert _plan(bg, w).info()["path"] == bg.BLU_PATH_HASH_GLOBAL
+    monkeypatch.delenv("BLU_GBY_FORCE_PATH")
+    assert _plan(bg, w).info()["path"] == bg.BLU_PATH_DENSE_SMEM
