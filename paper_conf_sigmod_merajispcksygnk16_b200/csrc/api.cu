@@ -605,6 +605,7 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
   const double h0 = now();
   const Layout& L = P->lay;
   const uint32_t B = P->parts;
+  if (!P->part_smem && B > kMaxSegs) return cudaErrorInvalidConfiguration;  // the planner clamps to kMaxSegs
   size_t row_bytes = 8;
   for (int c = 0; c < L.n_vals; ++c) row_bytes += dtype_bytes(L.val_dtype[c]);
   // Chunk rows: decided once per plan from the free memory (cudaMemGetInfo and the pool queries are

@@ -1546,8 +1546,8 @@ __device__ __forceinline__ void global_body(const AggParams& p, const RecSrc& rs
   if (p.gate && ((*(volatile const uint32_t*)p.gate != 0) != (p.gate_run_if != 0))) return;
   const Layout& L = p.lay;
   const uint32_t S = p.S;
-  __shared__ uint64_t tpre[SEG ? 1025 : 1];
-  __shared__ uint64_t tend[MODE == 4 ? 1024 : 1];  // MODE 4: end row of each segment
+  __shared__ uint64_t tpre[SEG ? kMaxSegs + 1 : 1];  // the planner keeps n_segs <= kMaxSegs in this mode
+  __shared__ uint64_t tend[MODE == 4 ? kMaxSegs : 1];  // MODE 4: end row of each segment
   if constexpr (SEG) {  // warp-tile prefix over the buckets (warp 0)
     if (threadIdx.x < 32) {
       const uint64_t tile = 32ull * R;
@@ -1918,6 +1918,12 @@ __device__ __forceinline__ void bucket_body(const AggParams& p) {
     const uint64_t r0 = seg0 + (uint64_t)(item - ppre[lo]) * piece;
     const uint64_t cnt = p.seg_count[lo];
     const uint64_t r1 = seg0 + ((uint64_t)(item - ppre[lo]) * piece + piece < cnt ? (uint64_t)(item - ppre[lo]) * piece + piece : cnt);
+#ifdef BLU_DEBUG_BOUNDS
+    if (threadIdx.x == 0 && (lo >= nb || r1 > seg0 + p.seg_stride || r0 > r1))
+      printf("BOUNDS item %u lo %u nb %u r0 %llu r1 %llu seg0 %llu stride %llu cnt %llu piece %llu\n", item, lo, nb,
+             (unsigned long long)r0, (unsigned long long)r1, (unsigned long long)seg0, (unsigned long long)p.seg_stride,
+             (unsigned long long)cnt, (unsigned long long)piece);
+#endif
     // PIPE (NVRTC kernels): the piece's next tile is loaded into registers before this one is probed
     using Raw = RawTileFor<SP, R, PIPE>;
     Raw A, Bt;
@@ -1988,6 +1994,10 @@ __device__ __forceinline__ void bucket_body(const AggParams& p) {
         if (!__any_sync(0xffffffffu, pending)) break;
       }
       __syncwarp();
+#ifdef BLU_DEBUG_BOUNDS
+      for (int r = 0; r < R; ++r)
+        if ((hit >> r & 1) && e[r] >= S) printf("BOUNDS e %u S %u\n", e[r], S);
+#endif
       smem_apply_rows<SP, NV, R>(p, sm, e, hit, v);
       if (__any_sync(0xffffffffu, pending)) {  // no room in the shared table: global table (S5b)
         uint64_t slot[R];
@@ -2004,6 +2014,10 @@ __device__ __forceinline__ void bucket_body(const AggParams& p) {
           }
         }
         __syncwarp();
+#ifdef BLU_DEBUG_BOUNDS
+        for (int r = 0; r < R; ++r)
+          if ((miss >> r & 1) && slot[r] > p.cap_mask) printf("BOUNDS slot %llu mask %llu\n", (unsigned long long)slot[r], (unsigned long long)p.cap_mask);
+#endif
         global_apply_rows<SP, NV, R, false>(p, slot, miss, v);
       }
     }

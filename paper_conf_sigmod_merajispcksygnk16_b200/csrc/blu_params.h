@@ -19,6 +19,9 @@ constexpr int kMaxKeys = 8;
 constexpr int kMaxVals = 16;
 constexpr int kMaxAggs = 16;
 constexpr int kMaxFields = 24;
+// partitioned pass 2 in the L2-slice mode (global_body SEG): at most this many buckets (per-CTA
+// shared prefix of the buckets' warp tiles)
+constexpr uint32_t kMaxSegs = 1024;
 constexpr uint64_t kEmpty = ~0ull;  // key portion of the mask: M/4 Fs (Table 1)
 
 // State-field kinds. Each aggregate maps to one or two fields (AVG = SUM field + COUNT field);

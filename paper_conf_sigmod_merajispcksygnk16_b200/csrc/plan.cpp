@@ -449,9 +449,11 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     // 19.4 ms, and pass 2 drops from 25.4 to 12.5 ms: 32.5 vs 35.7 ms. So the mode is
     // the default when the estimated groups fit >= 256 buckets of at most kMaxBuckets (two-level
     // scatter); C5's 5*10^7 groups do not fit and keep the L2 mode. BLU_GBY_PART_SMEM=0/1 overrides.
+    // BLU_GBY_BUCKET_S (experiment): cap the entries per bucket table below what shared memory holds
+    const uint32_t s_cap = env("BLU_GBY_BUCKET_S") ? (uint32_t)std::max(64, atoi(env("BLU_GBY_BUCKET_S"))) : 1u << 30;
     auto S_of = [&](uint32_t b) {
       uint32_t S = 16;
-      while (bucket_smem_bytes(L, S + 16, b) <= kSmemMax) S += 16;
+      while (bucket_smem_bytes(L, S + 16, b) <= kSmemMax && S + 16 <= s_cap) S += 16;
       return S;
     };
     // smallest B whose buckets hold <= kBucketLoad * S groups on average, within the scatter's
@@ -492,7 +494,9 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
       P->bucket_smem = bucket_smem_bytes(L, P->bucket_S, (uint32_t)B);
     } else {
       while (budget && B < 1024 && tbytes / B > budget && B < P->cap / 1024) B <<= 1;
-      if (const char* pp = env("BLU_GBY_PARTS")) B = std::max(1, atoi(pp));
+      // a forced count is clamped to what the L2-slice pass 2 indexes (kMaxSegs: 2048 forced buckets
+      // overran its shared prefix array)
+      if (const char* pp = env("BLU_GBY_PARTS")) B = std::max(1, std::min((int)kMaxSegs, atoi(pp)));
       if (B > 1 && !env("BLU_GBY_PARTS")) {
         // partitioned tables live in L2 one bucket at a time: trade HBM footprint for short probes
         uint64_t cap2 = std::max<uint64_t>(kMinCap, next_pow2((uint64_t)((double)P->est_groups / kMaxLoadPart + 0.999999)));

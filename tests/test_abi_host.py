@@ -332,3 +332,16 @@ def test_env_knobs_follow_the_environment_per_call(bg, monkeypatch):
     assert _plan(bg, w).info()["path"] == bg.BLU_PATH_HASH_GLOBAL
     monkeypatch.delenv("BLU_GBY_FORCE_PATH")
     assert _plan(bg, w).info()["path"] == bg.BLU_PATH_DENSE_SMEM
+
+
+def test_planner_clamps_forced_l2_partitions(bg, monkeypatch):
+    """The L2-slice pass 2 indexes at most kMaxSegs = 1024 buckets (its per-CTA prefix of the buckets'
+    warp tiles): a forced BLU_GBY_PARTS above that is clamped (2048 forced buckets once overran the
+    shared array: an illegal address on the GPU)."""
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "0")
+    monkeypatch.setenv("BLU_GBY_PARTS", "2048")
+    info = _plan(bg, blugen.workload("C3")).info()
+    assert info["part_smem"] == 0 and info["partitions"] == 1024
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
+    info = _plan(bg, blugen.workload("C3")).info()
+    assert info["part_smem"] == 1 and info["partitions"] == 2048

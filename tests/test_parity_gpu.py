@@ -637,6 +637,27 @@ def test_host_results_pinned_reuse(bg, oracles):
         assert_parity(gk, ga, o, sch)
 
 
+@pytest.mark.parametrize("parts", ["1024", "4096"])
+def test_partitioned_l2_mode_max_buckets(bg, monkeypatch, parts):
+    """The L2-slice pass 2 at its bucket limit (kMaxSegs = 1024): forced 1024 buckets, and a forced
+    4096 clamped to 1024 by the planner (2048 once overran the pass's shared prefix array)."""
+    w = blugen.workload("C3", n_rows=5_000_011, n_groups=300_000)
+    o = oracle.groupby_generated(w)
+    kc, vc = blugen.device_columns(w)
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "0")
+    monkeypatch.setenv("BLU_GBY_PARTS", parts)
+    plan = bg.plan_for(w.schema, w.est_groups, w.n_rows)
+    info = plan.info()
+    assert info["part_smem"] == 0 and info["partitions"] == 1024, info
+    bg.blu_gby_set_timing(True)
+    res = bg.blu_gby_execute(plan, kc, vc)
+    t = bg.blu_gby_last_timing()
+    bg.blu_gby_set_timing(False)
+    assert t["part_chunks"] == 1, t
+    gk, ga = gpu_sorted(res, w.schema)
+    assert_parity(gk, ga, o, w.schema)
+
+
 @pytest.mark.parametrize("one", ["0", "1"])
 def test_partitioned_two_level_128(bg, monkeypatch, one):
     """More than 4096 bucket tables: the two-level scatter splits 128 x B/128 (8192 buckets = 128 x 64
