@@ -763,7 +763,8 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       le = launch_scatter(p1, s1, st, scatter_grid((uint32_t)P->sms, B1));
       if (le) return (cudaError_t)le;
       const uint32_t B2 = B / B1;
-      const bool one_launch = benv("BLU_GBY_2LEVEL_ONE") && atoi(benv("BLU_GBY_2LEVEL_ONE")) == 1;
+      // (the segmented kernel keeps the first-level bucket ends in a 256-entry shared array, kMaxInSeg)
+      const bool one_launch = benv("BLU_GBY_2LEVEL_ONE") && atoi(benv("BLU_GBY_2LEVEL_ONE")) == 1 && B1 <= 256;
       if (one_launch) {
         // second level as ONE launch over every first-level bucket (segmented input; the first-level
         // counts stay on the device, no host round trip): bucket b1's rows go to [b1 * B2, b1 * B2 + B2).
