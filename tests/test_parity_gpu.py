@@ -477,6 +477,59 @@ def test_execute_host_columns(bg, oracles, monkeypatch, name):
         del res
 
 
+def test_concurrent_executes_on_streams(bg, oracles, monkeypatch):
+    """The header's concurrency promise: host threads running whole queries at the same time on their
+    own streams — host-column queries (partitioned plan: staging, two-level scatter with its second
+    stream, pinned result blocks) next to device-column queries — each equal to the oracle."""
+    import threading
+    w3, o3 = oracles("C3")
+    w5, o5 = oracles("C5")
+    monkeypatch.setenv("BLU_GBY_PARTS", "256")
+    monkeypatch.setenv("BLU_GBY_PART_SMEM", "1")
+    plan3 = bg.plan_for(w3.schema, w3.est_groups, w3.n_rows)
+    assert plan3.info()["partitions"] == 256 and plan3.info()["part_smem"] == 1
+    monkeypatch.delenv("BLU_GBY_PARTS")
+    monkeypatch.delenv("BLU_GBY_PART_SMEM")
+    plan5 = bg.plan_for(w5.schema, w5.est_groups, w5.n_rows)
+    hk, hv = blugen.host_columns(w3)
+    hk = [torch.from_numpy(k).pin_memory() for k in hk]
+    hv = [torch.from_numpy(v).pin_memory() for v in hv]
+    kc5, vc5 = blugen.device_columns(w5)
+    torch.cuda.synchronize()
+    errors = []
+
+    def host_worker():
+        try:
+            s = torch.cuda.Stream()
+            for _ in range(3):
+                res = bg.blu_gby_execute_host(plan3, hk, hv, stream=s)
+                gk, ga = host_sorted(res, w3.schema)
+                assert_parity(gk, ga, o3, w3.schema)
+                del res
+        except Exception as e:  # noqa: BLE001 - reported below
+            errors.append(e)
+
+    def device_worker():
+        try:
+            s = torch.cuda.Stream()
+            for _ in range(3):
+                with torch.cuda.stream(s):
+                    res = bg.blu_gby_execute(plan5, kc5, vc5, stream=s)
+                    gk, ga = gpu_sorted(res, w5.schema)
+                assert_parity(gk, ga, o5, w5.schema)
+                del res
+        except Exception as e:  # noqa: BLE001
+            errors.append(e)
+
+    ts = [threading.Thread(target=host_worker), threading.Thread(target=host_worker),
+          threading.Thread(target=device_worker)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    assert not errors, errors
+
+
 def test_init_table_matches_table1(bg):
     """S4 on the device: every slot equals the Table 1 mask."""
     plan = bg.blu_gby_plan([(I64, 0)], [I64, I64, I32], [(SUM, 0), (MAX, 1), (MIN, 2)], 1000, 10**6)
