@@ -475,7 +475,16 @@ def measure(cfg, args, world, rank, local, torch, dist, bg, bdist, sampler_on):
         rows_per_launch = n / chunks
         levels = info.get("scatter_levels", 2 if (info["part_smem"] == 1 and info["partitions"] >= 256) else 1)
         method_bpr = bpr + rec_bytes * (2 * levels)  # each scatter level writes the records once, the next reads them
-        tr_sc, tr_rows_sc = load_traffic(cfg, "scatter2" if levels == 2 else "scatter")
+        # scatter traffic per launch: the first level's capture scaled to the chunk, plus (two levels)
+        # one second-level launch's capture scaled to the chunk (the second level reads the first
+        # level's output partly from L2)
+        tr_sc, tr_rows_sc = load_traffic(cfg, "scatter")
+        if levels == 2 and tr_sc and tr_rows_sc:
+            tr_sc2, tr_rows_sc2 = load_traffic(cfg, "scatter2")
+            if tr_sc2 and tr_rows_sc2:
+                tr_sc, tr_rows_sc = (tr_sc / tr_rows_sc + tr_sc2 / tr_rows_sc2) * tr_rows_sc, tr_rows_sc
+            else:
+                tr_sc = None
         tr_p2, tr_rows_p2 = load_traffic(cfg, "pass2")
         alg = rows_per_launch * bpr
         phases = {
