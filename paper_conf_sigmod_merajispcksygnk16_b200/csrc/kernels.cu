@@ -1323,7 +1323,9 @@ uint64_t partition_scratch_bytes(uint64_t n, int32_t n_parts) {
 
 uint32_t partition_ctas(uint64_t n) {
   const uint64_t by_rows = (n + 4095) / 4096;  // >= 4096 rows per CTA
-  return (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(by_rows, 148 * 8));
+  // per-CTA shared counts are 32-bit: at most 2^31 rows per CTA
+  const uint64_t min_ctas = (n >> 31) + 1;
+  return (uint32_t)std::max<uint64_t>(min_ctas, std::max<uint64_t>(1, std::min<uint64_t>(by_rows, 148 * 8)));
 }
 
 int launch_partition(const Layout& lay, const void* const* key_cols, const void* const* state_cols, uint64_t n,
