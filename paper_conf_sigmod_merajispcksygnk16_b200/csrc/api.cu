@@ -872,11 +872,12 @@ static cudaError_t partitioned_feed(const blu_gby_plan_s* P, AggParams& base, co
       // bucket-local shared-memory tables: pieces of ~1/div of the mean bucket, whole 4096-row tiles
       // (div 1, one piece per mean bucket: one flush of each group into the global table instead of
       // two; C3 30.4 vs 31.1 ms for div 2, 32.5 for div 4)
+      // piece_rows 0: one work item per bucket (the plan's default, no piece prefix in shared memory)
       const uint64_t div = benv("BLU_GBY_PIECE_DIV") ? std::max(1, atoi(benv("BLU_GBY_PIECE_DIV"))) : 1;
       const uint64_t mean = (m + B - 1) / B;
       uint64_t piece = ((mean + div - 1) / div + 4095) / 4096 * 4096;
       piece = std::min<uint64_t>(std::max<uint64_t>(piece, 4096), 1ull << 30);
-      p2.piece_rows = piece;
+      p2.piece_rows = P->bucket_whole ? 0 : piece;
       p2.aux_off = bucket_table_bytes(L2, P->bucket_S);
       p2.tile_ctr = (uint64_t*)(d_cursor + B + 1);
       p2.vec_ok = 3;  // segments start at multiples of 64 rows of 8-byte-aligned buffers

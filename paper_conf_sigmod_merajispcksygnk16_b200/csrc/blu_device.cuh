@@ -1873,12 +1873,15 @@ __device__ __forceinline__ void bucket_body(const AggParams& p) {
   const Layout& L = p.lay;
   const uint32_t S = p.S;
   const uint32_t nb = p.n_segs;
-  uint32_t* ppre = (uint32_t*)(sm + p.aux_off);  // nb + 1 piece prefix, then 2 scalars
-  volatile uint32_t* s_item = ppre + nb + 1;
+  // piece_rows 0: one work item per bucket, no prefix (aux = 2 scalars); else pieces of piece_rows rows
+  // with the buckets' piece prefix (nb + 1 u32) ahead of the 2 scalars
+  const bool whole = p.piece_rows == 0;
+  uint32_t* ppre = (uint32_t*)(sm + p.aux_off);
+  volatile uint32_t* s_item = whole ? ppre : ppre + nb + 1;
   uint64_t* fk = (uint64_t*)(sm + p.key_off);
-  const uint64_t piece = p.piece_rows;
+  const uint64_t piece = whole ? ~0ull : p.piece_rows;
   // piece prefix over the buckets (warp 0) and the table mask (all threads)
-  if (threadIdx.x < 32) {
+  if (!whole && threadIdx.x < 32) {
     uint32_t carry = 0;
     for (uint32_t b0 = 0; b0 < nb; b0 += 32) {
       const uint32_t b = b0 + threadIdx.x;
@@ -1908,16 +1911,17 @@ __device__ __forceinline__ void bucket_body(const AggParams& p) {
     }
     __syncthreads();
     const uint32_t item = s_item[0];
-    if (item >= ppre[nb] || (s_item[1] & FLAG_OVERFLOW)) break;
-    uint32_t lo = 0, hi = nb - 1;  // bucket of the item: largest b with ppre[b] <= item
+    if (item >= (whole ? nb : ppre[nb]) || (s_item[1] & FLAG_OVERFLOW)) break;
+    uint32_t lo = whole ? item : 0, hi = whole ? item : nb - 1;  // bucket of the item: largest b with ppre[b] <= item
     while (lo < hi) {
       const uint32_t mid = (lo + hi + 1) >> 1;
       if (ppre[mid] <= item) lo = mid; else hi = mid - 1;
     }
     const uint64_t seg0 = (uint64_t)lo * p.seg_stride;
-    const uint64_t r0 = seg0 + (uint64_t)(item - ppre[lo]) * piece;
     const uint64_t cnt = p.seg_count[lo];
-    const uint64_t r1 = seg0 + ((uint64_t)(item - ppre[lo]) * piece + piece < cnt ? (uint64_t)(item - ppre[lo]) * piece + piece : cnt);
+    const uint64_t k = whole ? 0 : (uint64_t)(item - ppre[lo]);  // piece of the bucket
+    const uint64_t r0 = seg0 + k * (whole ? 0 : piece);
+    const uint64_t r1 = whole ? seg0 + cnt : seg0 + (k * piece + piece < cnt ? k * piece + piece : cnt);
 #ifdef BLU_DEBUG_BOUNDS
     if (threadIdx.x == 0 && (lo >= nb || r1 > seg0 + p.seg_stride || r0 > r1))
       printf("BOUNDS item %u lo %u nb %u r0 %llu r1 %llu seg0 %llu stride %llu cnt %llu piece %llu\n", item, lo, nb,

@@ -51,6 +51,7 @@ struct blu_gby_plan_s {
   int32_t part_smem;      // partitioned pass 2: 1 = bucket-local shared-memory tables, 0 = L2-resident slices
   uint32_t bucket_S;      // part_smem: entries of the per-CTA bucket table
   uint32_t bucket_smem;   // part_smem: dynamic shared memory of the bucket kernel
+  int32_t bucket_whole;   // part_smem: 1 = one work item per bucket (no piece prefix in shared memory)
   mutable std::atomic<uint64_t> part_chunk{0};  // rows per partitioned chunk (decided at first execute)
   mutable std::atomic<uint32_t> retries_last{0};
 };
@@ -81,7 +82,7 @@ size_t scatter_smem(int nv, uint32_t B, bool tma = false);
 int launch_bucket(const AggParams& p, void* stream, uint32_t grid, uint32_t smem);
 // bucket table sizing: bytes of an S-entry table (keys + SoA fields) and the kernel's total smem
 uint32_t bucket_table_bytes(const Layout& L, uint32_t S);
-uint32_t bucket_smem_bytes(const Layout& L, uint32_t S, uint32_t B);
+uint32_t bucket_smem_bytes(const Layout& L, uint32_t S, uint32_t B, bool prefix = true);
 blu_status_t fail(blu_status_t s, const char* fmt, ...);
 int launch_init_slots(const Layout& lay, void* table, uint64_t n_slots, void* stream, uint64_t* zero = nullptr,
                       uint32_t n_zero = 0);

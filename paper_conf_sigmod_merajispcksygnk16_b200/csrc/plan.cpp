@@ -192,8 +192,9 @@ uint32_t bucket_table_bytes(const Layout& L, uint32_t S) {
   return o;
 }
 
-uint32_t bucket_smem_bytes(const Layout& L, uint32_t S, uint32_t B) {
-  return bucket_table_bytes(L, S) + ((B + 1 + 2) * 4 + 15) / 16 * 16;
+uint32_t bucket_smem_bytes(const Layout& L, uint32_t S, uint32_t B, bool prefix) {
+  // behind the table: the buckets' piece prefix (B + 1 u32; pieces mode only) and 2 scalars
+  return bucket_table_bytes(L, S) + (((prefix ? B + 1 : 0) + 2) * 4 + 15) / 16 * 16;
 }
 
 void fill_smem_layout(AggParams& p, uint32_t S, bool with_keys) {
@@ -440,6 +441,7 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
   P->part_smem = 0;
   P->bucket_S = 0;
   P->bucket_smem = 0;
+  P->bucket_whole = 0;
   if (path == BLU_PATH_HASH_GLOBAL && L.key_words == 1 && !L.has_q) {
     uint64_t budget = (uint64_t)kPartBudgetMB << 20;
     if (const char* pm = env("BLU_GBY_PART_MB")) budget = (uint64_t)atoi(pm) << 20;
@@ -451,9 +453,13 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
     // scatter); C5's 5*10^7 groups do not fit and keep the L2 mode. BLU_GBY_PART_SMEM=0/1 overrides.
     // BLU_GBY_BUCKET_S (experiment): cap the entries per bucket table below what shared memory holds
     const uint32_t s_cap = env("BLU_GBY_BUCKET_S") ? (uint32_t)std::max(64, atoi(env("BLU_GBY_BUCKET_S"))) : 1u << 30;
+    // work items = whole buckets (default: a bucket is at most its capacity, ~1.1-1.2x the mean, so
+    // one item per bucket balances, and the table gets the shared memory a piece prefix would take:
+    // 64 KB at 16384 buckets), or pieces of ~1/div of the mean bucket with BLU_GBY_PIECE_DIV=div
+    const bool whole = !env("BLU_GBY_PIECE_DIV");
     auto S_of = [&](uint32_t b) {
       uint32_t S = 16;
-      while (bucket_smem_bytes(L, S + 16, b) <= kSmemMax && S + 16 <= s_cap) S += 16;
+      while (bucket_smem_bytes(L, S + 16, b, !whole) <= kSmemMax && S + 16 <= s_cap) S += 16;
       return S;
     };
     // smallest B whose buckets hold <= kBucketLoad * S groups on average, within the scatter's
@@ -491,7 +497,8 @@ blu_status_t blu_gby_plan(const blu_gby_schema_t* s, uint64_t est_groups, uint64
       while (B > 2 && scatter_smem(L.n_vals, widest(two_ok, B)) > kSmemMax) B >>= 1;  // histogram bins per tile
       P->part_smem = 1;
       P->bucket_S = S_of((uint32_t)B);
-      P->bucket_smem = bucket_smem_bytes(L, P->bucket_S, (uint32_t)B);
+      P->bucket_whole = whole ? 1 : 0;
+      P->bucket_smem = bucket_smem_bytes(L, P->bucket_S, (uint32_t)B, !whole);
     } else {
       while (budget && B < 1024 && tbytes / B > budget && B < P->cap / 1024) B <<= 1;
       // a forced count is clamped to what the L2-slice pass 2 indexes (kMaxSegs: 2048 forced buckets
